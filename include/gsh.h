@@ -1,0 +1,239 @@
+/*
+ * gsh.h -- C-ABI of the B200-native GSH (GPU Skew-conscious Hash join) library, libgsh.so.
+ *
+ * Paper: Cai & Chen, "CPU and GPU Hash Joins on Skewed Data", ICDE 2024.
+ * The operation (§III, §IV-B): an inner equi-join of two
+ * GPU-resident tables R and S of (4 B key, 4 B payload) tuples (L49 "joining GPU-resident
+ * data", L55 / L132 "a pair of 4B join key and 4B payload"), computed by GSH's phases
+ *   (1) radix-partition R and S in two passes, count-then-partition (L106)
+ *   (2) detect skewed keys in large partitions after partitioning (L107, L112)
+ *   (3) divide large partitions into per-skewed-key arrays and a normal partition (L114)
+ *   (4) NM-join: one thread block per normal partition pair, shared-memory table (L115)
+ *   (5) skewed-key join spread over many thread blocks (L116).
+ * Result: match count, an order-independent 64-bit checksum, optionally the pairs.
+ *
+ * Semantics:
+ *   M = { (payload_R[i], payload_S[j]) : key_R[i] == key_S[j] }, multiset over row pairs.
+ *   count    = |M|;
+ *   checksum = sum_{(a,b) in M} fmix64(((u64)a << 32 | b) ^ 0x9E3779B97F4A7C15) mod 2^64;
+ *   pairs    = (payload_R, payload_S) per match, unspecified order.
+ *   Keys and payloads are opaque u32 bit patterns; every value (0, 0xFFFFFFFF, ...) is legal.
+ *   n = 0 on either side gives count = checksum = written = 0.
+ *
+ * Conventions for every entry point:
+ *   - Pointers named d_* / device are CUDA device pointers (cudaMalloc / torch CUDA storage);
+ *     pointers named h_* / host are host pointers.  The caller owns all buffers; the library
+ *     never allocates device memory (all scratch comes from the caller's `workspace`).
+ *   - Inputs are read-only and never modified.
+ *   - `stream` is a cudaStream_t passed as void* (NULL = legacy default stream).  All GPU
+ *     work is enqueued on it; entry points that fill a host result synchronise it.
+ *   - Errors are status codes; nothing is thrown across the ABI.  Argument errors are
+ *     reported before any launch (GSH_ERR_INVALID).  After GSH_ERR_CUDA the contents of
+ *     results and outputs are undefined.  gsh_last_error() gives a thread-local message.
+ *   - Reentrant given distinct workspaces and streams.
+ */
+#ifndef GSH_H_
+#define GSH_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#if defined(__GNUC__)
+#define GSH_API __attribute__((visibility("default")))
+#else
+#define GSH_API
+#endif
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+    GSH_OK = 0,
+    GSH_ERR_INVALID = 1,   /* bad argument (NULL with n > 0, workspace too small, ...) */
+    GSH_ERR_NOMEM = 2,     /* host allocation failed */
+    GSH_ERR_CUDA = 3,      /* a CUDA call or kernel failed */
+    GSH_ERR_NCCL = 4,      /* reserved for collective failures (multi-GPU driver) */
+    GSH_ERR_INTERNAL = 5   /* broken internal invariant */
+} gsh_status;
+
+typedef enum {
+    GSH_OUT_COUNT = 0,        /* count + checksum only (output consumed) */
+    GSH_OUT_MATERIALIZE = 1   /* also write (payload_R, payload_S) pairs */
+} gsh_out_mode;
+
+/* A relation in SoA layout: keys[i], payloads[i], i < n.  Device pointers for gsh_join,
+ * host pointers for gsh_join_host.  n must be < 2^32 (payloads are row ids). */
+typedef struct {
+    const uint32_t *keys;
+    const uint32_t *payloads;
+    uint64_t n;
+} gsh_relation;
+
+/* Materialised output: pairs[2i] = payload_R, pairs[2i+1] = payload_S for i < written.
+ * capacity is in pairs.  Device pointer for gsh_join, host pointer for gsh_join_host. */
+typedef struct {
+    uint32_t *pairs;
+    uint64_t capacity;
+} gsh_output;
+
+/* Tuning / test hooks.  Initialise with gsh_config_default(); NULL means defaults. */
+typedef struct {
+    uint32_t capacity;         /* C: max R tuples per NM-join build table and the
+                                  large-partition threshold (L107).  0 = auto
+                                  (max(4096, 2 * mean partition size), <= 8192). */
+    int32_t pass_bits[2];      /* radix bits of pass 1 / pass 2 (L106).  -1 = auto so the
+                                  mean partition holds ~2048 tuples (max 8 + 8 bits). */
+    uint32_t heavy_threshold;  /* T_h: a key of a large partition is skewed iff
+                                  max(cnt_R, cnt_S) >= T_h (L112 reading).  0 = C / 4. */
+    uint32_t route_bits;       /* top bits of fmix32(key) already consumed by multi-GPU
+                                  routing; partition digits start below them. */
+    int32_t force_all_normal;  /* test hook: no skew detection; every key goes through the
+                                  NM-join (chunked when a partition exceeds C). */
+    int32_t force_all_heavy;   /* test hook: every partition is large and every key skewed. */
+    int32_t timing;            /* 1 = record per-phase CUDA events into gsh_result.ms_* */
+    int32_t reserved;
+} gsh_config;
+
+/* Per-call result (host struct). */
+typedef struct {
+    uint64_t count;            /* |M| (all pairs, even on overflow) */
+    uint64_t checksum;         /* sum of pair_hash over M mod 2^64 */
+    uint64_t written;          /* pairs written = min(count, capacity) (MATERIALIZE) */
+    uint64_t normal_count;     /* share of count produced by the NM-join phase */
+    uint64_t normal_checksum;  /* share of checksum produced by the NM-join phase */
+    uint64_t heavy_tuples_r;   /* R tuples routed to skewed-key arrays */
+    uint64_t heavy_tuples_s;   /* S tuples routed to skewed-key arrays */
+    uint64_t skew_pairs;       /* |R_k| * |S_k| summed over skewed keys */
+    uint32_t overflow;         /* 1 iff count > capacity (MATERIALIZE) */
+    uint32_t n_heavy;          /* number of skewed keys detected */
+    uint32_t n_large;          /* number of large partitions */
+    uint32_t detect_overflow;  /* 1 iff the detection table filled (fallback used) */
+    uint32_t pass_bits[2];     /* radix bits actually used */
+    uint32_t capacity;         /* C actually used */
+    uint32_t heavy_threshold;  /* T_h actually used */
+    uint32_t launches;         /* kernels launched by this call */
+    uint32_t reserved;
+    float ms_hist, ms_pass1, ms_pass2, ms_detect, ms_split, ms_nmjoin, ms_skewjoin, ms_total;
+} gsh_result;
+
+/* Fill *cfg with defaults (all auto, no hooks, timing off). */
+GSH_API void gsh_config_default(gsh_config *cfg);
+
+/* Bytes of device workspace gsh_join needs for these sizes (independent of the data).
+ * Roughly 20 B per input tuple plus O(fanout) tables; see DESIGN.md §5. */
+GSH_API size_t gsh_workspace_bytes(uint64_t n_r, uint64_t n_s, const gsh_config *cfg);
+
+/*
+ * gsh_join -- the GSH equi-join of device-resident R and S (§IV-B).
+ *   R, S       : device SoA relations (host structs holding device pointers).
+ *   mode       : GSH_OUT_COUNT or GSH_OUT_MATERIALIZE.
+ *   out        : NULL iff mode == GSH_OUT_COUNT; else device pairs buffer + capacity.
+ *                Exactly min(count, capacity) pairs are written, unspecified order and
+ *                (on overflow) unspecified subset; count/checksum always cover all pairs.
+ *   workspace  : device scratch of >= gsh_workspace_bytes(R->n, S->n, cfg) bytes,
+ *                256-byte aligned.  Contents on entry are ignored.
+ *   cfg        : NULL = defaults.
+ *   stream     : cudaStream_t as void*.
+ *   res        : host result, filled after the stream is synchronised.
+ * Returns GSH_ERR_INVALID for NULL pointers with n > 0, MATERIALIZE without output,
+ * a too-small or misaligned workspace, n >= 2^32, or bad config values.
+ */
+GSH_API gsh_status gsh_join(const gsh_relation *R, const gsh_relation *S, gsh_out_mode mode,
+                    const gsh_output *out, void *workspace, size_t workspace_bytes,
+                    const gsh_config *cfg, void *stream, gsh_result *res);
+
+/* Device workspace for gsh_join_host: gsh_workspace_bytes + device staging for the inputs
+ * (8 B per tuple) and, for MATERIALIZE, for out_capacity pairs (8 B per pair). */
+GSH_API size_t gsh_host_workspace_bytes(uint64_t n_r, uint64_t n_s, gsh_out_mode mode,
+                                uint64_t out_capacity, const gsh_config *cfg);
+
+/*
+ * gsh_join_host -- end-to-end variant: R, S and out hold HOST pointers (pinned memory
+ * gives full PCIe/C2C bandwidth; pageable works but is slower).  The inputs are copied
+ * host->device into the workspace, joined with gsh_join, and (MATERIALIZE) the written
+ * pairs copied device->host, all on `stream`.  res->written pairs land in out->pairs.
+ */
+GSH_API gsh_status gsh_join_host(const gsh_relation *R, const gsh_relation *S, gsh_out_mode mode,
+                         const gsh_output *out, void *workspace, size_t workspace_bytes,
+                         const gsh_config *cfg, void *stream, gsh_result *res);
+
+/* ---------------------------------------------------------------- step entry points --
+ * Individual phases exposed for per-kernel parity tests and the multi-GPU driver.
+ * Each synchronises `stream` before returning when it fills host outputs.             */
+
+/* d_out[i] = fmix32(d_keys[i]) (SURVEY §8 notation h).  Device arrays of length n. */
+GSH_API gsh_status gsh_hash_keys(const uint32_t *d_keys, uint32_t *d_out, uint64_t n, void *stream);
+
+/* Radix histogram, the "count" scan of L106: d_hist[d] += #{i : digit(i) == d} where
+ * digit = bits [32 - hi_bits - nbits, 32 - hi_bits) of fmix32(key).  d_hist is a device
+ * array of 2^nbits u64 that the caller zeroes; nbits <= 16, hi_bits + nbits <= 32. */
+GSH_API gsh_status gsh_radix_histogram(const uint32_t *d_keys, uint64_t n, uint32_t hi_bits,
+                               uint32_t nbits, uint64_t *d_hist, void *workspace,
+                               size_t workspace_bytes, void *stream);
+
+/* Run the partition phase (L106: histogram, scan, pass-1 scatter, pass-2 scatter) and copy
+ * out the final partitioned relations.  d_part_r / d_part_s: device arrays of 2*n u32
+ * receiving AoS (h = fmix32(key), payload) tuples grouped by partition; d_off_r / d_off_s:
+ * device arrays of (2^(b1+b2) + 1) u64 partition start offsets; h_bits[2]: host, receives
+ * (b1, b2).  The order of tuples inside a partition is unspecified. */
+GSH_API gsh_status gsh_partition(const gsh_relation *R, const gsh_relation *S, const gsh_config *cfg,
+                         void *workspace, size_t workspace_bytes, void *stream,
+                         uint32_t *d_part_r, uint32_t *d_part_s, uint64_t *d_off_r,
+                         uint64_t *d_off_s, uint32_t *h_bits);
+
+/* Run partition + classify + skew detection (L107, L112) and copy out the skewed-key side
+ * list H: h_keys[k] = fmix32(key), h_cnt_r[k], h_cnt_s[k] for k < *h_n (host arrays of
+ * `cap` entries; unspecified order).  Returns GSH_ERR_INVALID if more than cap keys. */
+GSH_API gsh_status gsh_detect(const gsh_relation *R, const gsh_relation *S, const gsh_config *cfg,
+                      void *workspace, size_t workspace_bytes, void *stream,
+                      uint32_t *h_keys, uint32_t *h_cnt_r, uint32_t *h_cnt_s, uint64_t cap,
+                      uint64_t *h_n, gsh_result *res);
+
+/* -------------------------------------------------------------- multi-GPU routing --
+ * Hash sharding over G = 2^route_bits ranks: a normal tuple goes to rank
+ * top_route_bits(fmix32(key)); a tuple whose key is in the agreed skewed set goes to the
+ * extra "heavy" bucket G (S stays local, R is all-gathered by the driver).             */
+
+/* d_counts[0..G] (device u64, caller zeroes): tuples per destination, index G = heavy.
+ * d_heavy_keys: device array of n_heavy keys (raw keys, not hashes) sorted ascending. */
+GSH_API gsh_status gsh_route_count(const uint32_t *d_keys, uint64_t n, uint32_t route_bits,
+                           const uint32_t *d_heavy_keys, uint64_t n_heavy,
+                           uint64_t *d_counts, void *stream);
+
+/* Scatter tuples into destination-grouped SoA send buffers.  d_offsets[0..G]: device u64
+ * exclusive scan of gsh_route_count's counts.  d_cursor: device u64[G+1] scratch the
+ * caller zeroes.  Order inside a destination group is unspecified. */
+GSH_API gsh_status gsh_route_scatter(const uint32_t *d_keys, const uint32_t *d_payloads, uint64_t n,
+                             uint32_t route_bits, const uint32_t *d_heavy_keys, uint64_t n_heavy,
+                             const uint64_t *d_offsets, uint64_t *d_cursor,
+                             uint32_t *d_out_keys, uint32_t *d_out_payloads, void *stream);
+
+/* Exact local counts of query keys: d_counts[q] += #{i : d_keys[i] == d_query[q]} for a
+ * device array d_query of m keys sorted ascending (d_counts device u64[m], caller zeroes). */
+GSH_API gsh_status gsh_count_keys(const uint32_t *d_keys, uint64_t n, const uint32_t *d_query,
+                          uint64_t m, uint64_t *d_counts, void *stream);
+
+/* Candidate skewed keys of a shard: keys whose partition (top part_bits of fmix32 below
+ * hi_bits) is flagged in d_large (device u8[2^part_bits]) and whose local count on either
+ * side is >= threshold.  Writes raw keys to d_cand (device, cap entries), count to *h_n. */
+GSH_API gsh_status gsh_local_candidates(const gsh_relation *R, const gsh_relation *S, uint32_t hi_bits,
+                                uint32_t part_bits, const uint8_t *d_large, uint32_t threshold,
+                                void *workspace, size_t workspace_bytes, void *stream,
+                                uint32_t *d_cand, uint64_t cap, uint64_t *h_n);
+
+/* Workspace for gsh_local_candidates. */
+GSH_API size_t gsh_candidates_workspace_bytes(uint64_t n_r, uint64_t n_s);
+
+/* ------------------------------------------------------------------- diagnostics -- */
+GSH_API const char *gsh_status_string(gsh_status s);
+GSH_API const char *gsh_last_error(void);
+/* Library version and the SM architecture it was compiled for (e.g. 100 for sm_100a). */
+GSH_API int gsh_version(void);
+GSH_API int gsh_compiled_arch(void);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* GSH_H_ */

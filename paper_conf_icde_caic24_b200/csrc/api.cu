@@ -1,0 +1,575 @@
+// api.cu -- the C-ABI (include/gsh.h): argument checking, workspace carve-up and the host-side
+// phase sequence of GSH (§IV-B) on one CUDA stream.
+//
+// Host synchronisation points: one after classification (number of large partitions, to size
+// detection) and one after skewed-key selection (number of skewed keys, to size the split and
+// the tile list); the final one fills gsh_result.  When no partition is large (uniform inputs,
+// PAPER.md L166) the detect/split/skew phases are skipped entirely.
+#include <cstdio>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "gsh_device.cuh"
+#include "gsh_internal.h"
+
+namespace gsh {
+// defined in skew.cu
+size_t cand_table_slots(uint64_t nR, uint64_t nS);
+int launch_candidates(const uint32_t* kr, uint64_t nR, const uint32_t* ks, uint64_t nS, uint32_t hi_bits,
+                      uint32_t part_bits, const uint8_t* large, uint32_t threshold, void* ws, uint32_t* out,
+                      uint64_t outcap, unsigned long long* d_nout, cudaStream_t s);
+}  // namespace gsh
+
+using namespace gsh;
+
+namespace {
+
+thread_local std::string g_err;
+
+gsh_status fail(gsh_status s, const std::string& msg) {
+    g_err = msg;
+    return s;
+}
+
+gsh_status cuda_fail(cudaError_t e, const char* where) {
+    g_err = std::string(where) + ": " + cudaGetErrorString(e);
+    return GSH_ERR_CUDA;
+}
+
+int device_sms() {
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess) return 148;
+    static int cached[64] = {0};
+    if (dev >= 0 && dev < 64 && cached[dev]) return cached[dev];
+    int sms = 148;
+    if (cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess) sms = 148;
+    if (dev >= 0 && dev < 64) cached[dev] = sms;
+    return sms;
+}
+
+uint64_t next_pow2_u64(uint64_t x) {
+    uint64_t p = 1;
+    while (p < x) p <<= 1;
+    return p;
+}
+
+size_t align256(size_t x) { return (x + 255) & ~size_t(255); }
+
+struct Carver {
+    unsigned char* base;
+    size_t off = 0;
+    template <class T>
+    T* take(size_t count) {
+        T* p = base ? reinterpret_cast<T*>(base + off) : nullptr;
+        off = align256(off + count * sizeof(T));
+        return p;
+    }
+};
+
+bool validate_rel(const gsh_relation* r) {
+    if (!r) return false;
+    if (r->n >= (1ull << 32)) return false;
+    if (r->n > 0 && (!r->keys || !r->payloads)) return false;
+    return true;
+}
+
+}  // namespace
+
+namespace gsh {
+
+bool plan_build(Plan& p, uint64_t nR, uint64_t nS, const gsh_config* cfg_in, void* ws, int num_sms) {
+    gsh_config cfg;
+    gsh_config_default(&cfg);
+    if (cfg_in) cfg = *cfg_in;
+    p.n[0] = nR;
+    p.n[1] = nS;
+    p.num_sms = num_sms;
+    const uint64_t nmax = nR > nS ? nR : nS;
+    if (cfg.route_bits > 16) return false;
+    p.route_bits = cfg.route_bits;
+    // radix bits: mean partition ~2048 tuples ("shared memory sized partitions")
+    if (cfg.pass_bits[0] >= 0 && cfg.pass_bits[1] >= 0) {
+        if (cfg.pass_bits[0] > kMaxDigitBits || cfg.pass_bits[1] > kMaxDigitBits) return false;
+        p.b1 = (uint32_t)cfg.pass_bits[0];
+        p.b2 = (uint32_t)cfg.pass_bits[1];
+    } else {
+        uint32_t B = 0;
+        while (B < (uint32_t)kMaxPartBits && (nmax >> B) > 2048) ++B;
+        p.b1 = (B + 1) / 2;
+        p.b2 = B / 2;
+    }
+    if (p.route_bits + p.b1 + p.b2 > 32) return false;
+    p.F = 1u << (p.b1 + p.b2);
+    // capacity C (power of two): large-partition threshold and NM build-table size (L107, L115)
+    if (cfg.capacity) {
+        uint64_t c = next_pow2_u64(cfg.capacity);
+        if (c < 64 || c > kMaxCapacity) return false;
+        p.C = (uint32_t)c;
+    } else {
+        uint64_t mean = (nmax + p.F - 1) / p.F;
+        uint64_t c = next_pow2_u64(2 * mean);
+        if (c < 4096) c = 4096;
+        if (c > kMaxCapacity) c = kMaxCapacity;
+        p.C = (uint32_t)c;
+    }
+    p.Th = cfg.heavy_threshold ? cfg.heavy_threshold : p.C / 4;
+    p.force_normal = cfg.force_all_normal;
+    p.force_heavy = cfg.force_all_heavy;
+    p.timing = cfg.timing;
+    if (p.force_normal && p.force_heavy) return false;
+    p.hist_grid = num_sms / 2 > 0 ? num_sms / 2 : 1;
+    for (int s = 0; s < 2; ++s)
+        p.max_tiles[s] = (p.n[s] + kScatterTile - 1) / kScatterTile + (1u << p.b1) + 1;
+    uint64_t t = next_pow2_u64(2 * (nR + nS));
+    if (t < 1024) t = 1024;
+    if (t > (1ull << 25)) t = 1ull << 25;
+    p.gt_cap_alloc = (uint32_t)t;
+    if (p.force_heavy)
+        p.h_max = p.gt_cap_alloc;
+    else {
+        uint64_t hm = (nR + nS) / (p.Th ? p.Th : 1) + 1;
+        p.h_max = hm < p.gt_cap_alloc ? hm : p.gt_cap_alloc;
+    }
+    uint64_t scan_max = p.F + 1 > p.h_max + 1 ? p.F + 1 : p.h_max + 1;
+    p.scan_scratch_elems = scan_max / 4096 + 2;
+
+    Carver c{reinterpret_cast<unsigned char*>(ws)};
+    const size_t F = p.F;
+    p.st = c.take<DevState>(1);
+    uint2* a = c.take<uint2>(nR + nS + 1);
+    uint2* b = c.take<uint2>(nR + nS + 1);
+    uint32_t* hp = c.take<uint32_t>(nR + nS + 1);
+    p.bufA[0] = a;
+    p.bufA[1] = a ? a + nR : nullptr;
+    p.bufB[0] = b;
+    p.bufB[1] = b ? b + nR : nullptr;
+    p.heavy_pay[0] = hp;
+    p.heavy_pay[1] = hp ? hp + nR : nullptr;
+    p.hist_partial = c.take<uint16_t>(size_t(2) * p.hist_grid * (F < 2 ? 2 : F));
+    p.hist_spill = c.take<uint32_t>(2 * F);
+    p.cnt = c.take<uint32_t>(2 * F);
+    p.start = c.take<uint64_t>(2 * (F + 1));
+    p.status = c.take<uint64_t>(size_t(p.max_tiles[0] + p.max_tiles[1]) * 256);
+    p.gt_key = c.take<unsigned long long>(p.gt_cap_alloc);
+    p.gt_cnt = c.take<uint32_t>(size_t(2) * p.gt_cap_alloc);
+    p.gt_hid = c.take<uint32_t>(p.gt_cap_alloc);
+    p.large_list = c.take<uint32_t>(F);
+    p.large_idx = c.take<uint32_t>(F);
+    p.part_heavy = c.take<uint32_t>(2 * F);
+    p.det_prefix = c.take<uint64_t>(F + 1);
+    p.nrm_off = c.take<uint64_t>(2 * (F + 1));
+    p.nrm_cur = c.take<uint32_t>(2 * F);
+    p.H = c.take<HeavyKey>(p.h_max);
+    p.h_off = c.take<uint64_t>(2 * (p.h_max + 1));
+    p.h_tiles = c.take<uint64_t>(p.h_max + 1);
+    p.h_cur = c.take<uint32_t>(2 * p.h_max);
+    p.nm = c.take<NmPart>(F);
+    p.nm_prefix = c.take<uint64_t>(F + 1);
+    p.scan_scratch = c.take<uint64_t>(p.scan_scratch_elems);
+    p.bytes = c.off;
+    return true;
+}
+
+}  // namespace gsh
+
+namespace {
+
+struct Timer {
+    bool on;
+    cudaStream_t s;
+    std::vector<cudaEvent_t> ev;
+    explicit Timer(bool enable, cudaStream_t st) : on(enable), s(st) {}
+    int mark() {
+        if (!on) return -1;
+        cudaEvent_t e;
+        cudaEventCreate(&e);
+        cudaEventRecord(e, s);
+        ev.push_back(e);
+        return (int)ev.size() - 1;
+    }
+    float ms(int a, int b) {
+        if (!on || a < 0 || b < 0) return 0.f;
+        float t = 0.f;
+        cudaEventElapsedTime(&t, ev[a], ev[b]);
+        return t;
+    }
+    ~Timer() {
+        for (auto e : ev) cudaEventDestroy(e);
+    }
+};
+
+gsh_status check_launch(const char* where) {
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return cuda_fail(e, where);
+    return GSH_OK;
+}
+
+// Runs hist + scan + pass 1 + pass 2.  Returns kernels launched, or -1 after setting g_err.
+int run_partition(const Plan& p, const gsh_relation* R, const gsh_relation* S, cudaStream_t s) {
+    int l = 0;
+    l += launch_hist(p, R->keys, S->keys, s);
+    l += launch_hist_reduce_scan(p, s);
+    const uint32_t* keys[2] = {R->keys, S->keys};
+    const uint32_t* pays[2] = {R->payloads, S->payloads};
+    l += launch_scatter(p, 1, keys, pays, s);
+    l += launch_scatter(p, 2, nullptr, nullptr, s);
+    return l;
+}
+
+gsh_status prep(const gsh_relation* R, const gsh_relation* S, void* ws, size_t ws_bytes, const gsh_config* cfg,
+                Plan& p) {
+    if (!validate_rel(R) || !validate_rel(S)) return fail(GSH_ERR_INVALID, "invalid relation (NULL or n >= 2^32)");
+    if (!plan_build(p, R->n, S->n, cfg, nullptr, device_sms()))
+        return fail(GSH_ERR_INVALID, "invalid gsh_config");
+    if (!ws || (reinterpret_cast<uintptr_t>(ws) & 255u)) return fail(GSH_ERR_INVALID, "workspace NULL or not 256-byte aligned");
+    if (ws_bytes < p.bytes) return fail(GSH_ERR_INVALID, "workspace too small");
+    plan_build(p, R->n, S->n, cfg, ws, device_sms());
+    return GSH_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+void gsh_config_default(gsh_config* cfg) {
+    if (!cfg) return;
+    std::memset(cfg, 0, sizeof(*cfg));
+    cfg->pass_bits[0] = -1;
+    cfg->pass_bits[1] = -1;
+}
+
+size_t gsh_workspace_bytes(uint64_t n_r, uint64_t n_s, const gsh_config* cfg) {
+    Plan p;
+    if (!plan_build(p, n_r, n_s, cfg, nullptr, device_sms())) return 0;
+    return p.bytes;
+}
+
+gsh_status gsh_join(const gsh_relation* R, const gsh_relation* S, gsh_out_mode mode, const gsh_output* out,
+                    void* workspace, size_t workspace_bytes, const gsh_config* cfg, void* stream, gsh_result* res) {
+    if (!res) return fail(GSH_ERR_INVALID, "res is NULL");
+    std::memset(res, 0, sizeof(*res));
+    if (mode != GSH_OUT_COUNT && mode != GSH_OUT_MATERIALIZE) return fail(GSH_ERR_INVALID, "bad mode");
+    const bool mat = (mode == GSH_OUT_MATERIALIZE);
+    if (mat && (!out || (!out->pairs && out->capacity > 0)))
+        return fail(GSH_ERR_INVALID, "MATERIALIZE needs an output buffer");
+    Plan p;
+    gsh_status st = prep(R, S, workspace, workspace_bytes, cfg, p);
+    if (st != GSH_OK) return st;
+    cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+    res->pass_bits[0] = p.b1;
+    res->pass_bits[1] = p.b2;
+    res->capacity = p.C;
+    res->heavy_threshold = p.Th;
+    if (R->n == 0 || S->n == 0) return GSH_OK;
+
+    uint32_t* pairs = mat ? out->pairs : nullptr;
+    const uint64_t cap = mat ? out->capacity : 0;
+    Timer tm(p.timing != 0, s);
+    int launches = 0;
+    cudaMemsetAsync(p.st, 0, sizeof(DevState), s);
+    const int e0 = tm.mark();
+    launches += launch_hist(p, R->keys, S->keys, s);
+    launches += launch_hist_reduce_scan(p, s);
+    const int e1 = tm.mark();
+    {
+        const uint32_t* keys[2] = {R->keys, S->keys};
+        const uint32_t* pays[2] = {R->payloads, S->payloads};
+        launches += launch_scatter(p, 1, keys, pays, s);
+    }
+    const int e2 = tm.mark();
+    launches += launch_scatter(p, 2, nullptr, nullptr, s);
+    const int e3 = tm.mark();
+    launches += launch_classify(p, s);
+    if ((st = check_launch("partition")) != GSH_OK) return st;
+
+    DevState hs;
+    cudaError_t ce = cudaMemcpyAsync(&hs, p.st, sizeof(DevState), cudaMemcpyDeviceToHost, s);
+    if (ce == cudaSuccess) ce = cudaStreamSynchronize(s);
+    if (ce != cudaSuccess) return cuda_fail(ce, "classify sync");
+    const uint32_t n_large = hs.n_large;
+    uint32_t n_heavy = 0;
+    int e4 = e3, e5 = e3;
+    if (n_large > 0) {
+        uint64_t gcap = next_pow2_u64(2 * (hs.large_tuples[0] + hs.large_tuples[1]));
+        if (gcap < 1024) gcap = 1024;
+        if (gcap > p.gt_cap_alloc) gcap = p.gt_cap_alloc;
+        launches += launch_detect_prefix(p, n_large, s);
+        launches += launch_detect(p, n_large, (uint32_t)gcap, s);
+        launches += launch_select(p, (uint32_t)gcap, s);
+        e4 = tm.mark();
+        if ((st = check_launch("detect")) != GSH_OK) return st;
+        ce = cudaMemcpyAsync(&hs, p.st, sizeof(DevState), cudaMemcpyDeviceToHost, s);
+        if (ce == cudaSuccess) ce = cudaStreamSynchronize(s);
+        if (ce != cudaSuccess) return cuda_fail(ce, "detect sync");
+        n_heavy = hs.n_heavy;
+        if (n_heavy > p.h_max) return fail(GSH_ERR_INTERNAL, "skewed-key list overflow");
+        launches += launch_heavy_prefix(p, n_heavy, n_large, s);
+        launches += launch_split(p, n_large, (uint32_t)gcap, s);
+        e5 = tm.mark();
+    }
+    launches += launch_nm_setup(p, n_large, s);
+    launches += launch_nmjoin(p, mat ? 1 : 0, pairs, cap, s);
+    const int e6 = tm.mark();
+    launches += launch_skewjoin(p, n_heavy, mat ? 1 : 0, pairs, cap, s);
+    const int e7 = tm.mark();
+    if ((st = check_launch("join")) != GSH_OK) return st;
+    ce = cudaMemcpyAsync(&hs, p.st, sizeof(DevState), cudaMemcpyDeviceToHost, s);
+    if (ce == cudaSuccess) ce = cudaStreamSynchronize(s);
+    if (ce != cudaSuccess) return cuda_fail(ce, "join sync");
+
+    res->count = hs.count + hs.nm_count;
+    res->checksum = hs.checksum + hs.nm_checksum;
+    res->normal_count = hs.nm_count;
+    res->normal_checksum = hs.nm_checksum;
+    res->written = mat ? (hs.cursor < cap ? hs.cursor : cap) : 0;
+    res->overflow = mat ? (hs.cursor > cap ? 1u : 0u) : 0u;
+    res->heavy_tuples_r = hs.heavy_tuples[0];
+    res->heavy_tuples_s = hs.heavy_tuples[1];
+    res->skew_pairs = hs.skew_pairs;
+    res->n_heavy = n_heavy;
+    res->n_large = n_large;
+    res->detect_overflow = hs.detect_overflow;
+    res->launches = (uint32_t)launches;
+    if (p.timing) {
+        res->ms_hist = tm.ms(e0, e1);
+        res->ms_pass1 = tm.ms(e1, e2);
+        res->ms_pass2 = tm.ms(e2, e3);
+        res->ms_detect = n_large ? tm.ms(e3, e4) : 0.f;
+        res->ms_split = n_large ? tm.ms(e4, e5) : 0.f;
+        res->ms_nmjoin = tm.ms(e5, e6);
+        res->ms_skewjoin = tm.ms(e6, e7);
+        res->ms_total = tm.ms(e0, e7);
+    }
+    return GSH_OK;
+}
+
+size_t gsh_host_workspace_bytes(uint64_t n_r, uint64_t n_s, gsh_out_mode mode, uint64_t out_capacity,
+                                const gsh_config* cfg) {
+    size_t w = gsh_workspace_bytes(n_r, n_s, cfg);
+    if (!w) return 0;
+    w = align256(w);
+    w += align256(n_r * 4) * 2 + align256(n_s * 4) * 2;
+    if (mode == GSH_OUT_MATERIALIZE) w += align256(out_capacity * 8);
+    return w;
+}
+
+gsh_status gsh_join_host(const gsh_relation* R, const gsh_relation* S, gsh_out_mode mode, const gsh_output* out,
+                         void* workspace, size_t workspace_bytes, const gsh_config* cfg, void* stream,
+                         gsh_result* res) {
+    if (!res) return fail(GSH_ERR_INVALID, "res is NULL");
+    std::memset(res, 0, sizeof(*res));
+    if (!validate_rel(R) || !validate_rel(S)) return fail(GSH_ERR_INVALID, "invalid relation");
+    const bool mat = (mode == GSH_OUT_MATERIALIZE);
+    if (mat && (!out || (!out->pairs && out->capacity > 0)))
+        return fail(GSH_ERR_INVALID, "MATERIALIZE needs an output buffer");
+    const uint64_t cap = mat ? out->capacity : 0;
+    const size_t need = gsh_host_workspace_bytes(R->n, S->n, mode, cap, cfg);
+    if (!need) return fail(GSH_ERR_INVALID, "invalid gsh_config");
+    if (!workspace || workspace_bytes < need || (reinterpret_cast<uintptr_t>(workspace) & 255u))
+        return fail(GSH_ERR_INVALID, "workspace NULL, misaligned or too small");
+    cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+    const size_t jw = align256(gsh_workspace_bytes(R->n, S->n, cfg));
+    unsigned char* base = reinterpret_cast<unsigned char*>(workspace);
+    size_t off = jw;
+    uint32_t* rk = reinterpret_cast<uint32_t*>(base + off); off += align256(R->n * 4);
+    uint32_t* rp = reinterpret_cast<uint32_t*>(base + off); off += align256(R->n * 4);
+    uint32_t* sk = reinterpret_cast<uint32_t*>(base + off); off += align256(S->n * 4);
+    uint32_t* sp = reinterpret_cast<uint32_t*>(base + off); off += align256(S->n * 4);
+    uint32_t* dp = mat ? reinterpret_cast<uint32_t*>(base + off) : nullptr;
+    cudaError_t ce = cudaSuccess;
+    if (R->n) {
+        ce = cudaMemcpyAsync(rk, R->keys, R->n * 4, cudaMemcpyHostToDevice, s);
+        if (ce == cudaSuccess) ce = cudaMemcpyAsync(rp, R->payloads, R->n * 4, cudaMemcpyHostToDevice, s);
+    }
+    if (ce == cudaSuccess && S->n) {
+        ce = cudaMemcpyAsync(sk, S->keys, S->n * 4, cudaMemcpyHostToDevice, s);
+        if (ce == cudaSuccess) ce = cudaMemcpyAsync(sp, S->payloads, S->n * 4, cudaMemcpyHostToDevice, s);
+    }
+    if (ce != cudaSuccess) return cuda_fail(ce, "H2D");
+    gsh_relation dR{rk, rp, R->n}, dS{sk, sp, S->n};
+    gsh_output dout{dp, cap};
+    gsh_status st = gsh_join(&dR, &dS, mode, mat ? &dout : nullptr, workspace, jw, cfg, stream, res);
+    if (st != GSH_OK) return st;
+    if (mat && res->written) {
+        ce = cudaMemcpyAsync(out->pairs, dp, res->written * 8, cudaMemcpyDeviceToHost, s);
+        if (ce == cudaSuccess) ce = cudaStreamSynchronize(s);
+        if (ce != cudaSuccess) return cuda_fail(ce, "D2H");
+    }
+    return GSH_OK;
+}
+
+gsh_status gsh_hash_keys(const uint32_t* d_keys, uint32_t* d_out, uint64_t n, void* stream) {
+    if (n && (!d_keys || !d_out)) return fail(GSH_ERR_INVALID, "NULL pointer");
+    launch_hash(d_keys, d_out, n, reinterpret_cast<cudaStream_t>(stream));
+    return check_launch("hash");
+}
+
+gsh_status gsh_radix_histogram(const uint32_t* d_keys, uint64_t n, uint32_t hi_bits, uint32_t nbits,
+                               uint64_t* d_hist, void* workspace, size_t workspace_bytes, void* stream) {
+    (void)workspace;
+    (void)workspace_bytes;
+    if (nbits > 16 || hi_bits + nbits > 32) return fail(GSH_ERR_INVALID, "bad bit range");
+    if (n && (!d_keys || !d_hist)) return fail(GSH_ERR_INVALID, "NULL pointer");
+    launch_radix_hist(d_keys, n, hi_bits, nbits, d_hist, reinterpret_cast<cudaStream_t>(stream));
+    return check_launch("radix_histogram");
+}
+
+gsh_status gsh_partition(const gsh_relation* R, const gsh_relation* S, const gsh_config* cfg, void* workspace,
+                         size_t workspace_bytes, void* stream, uint32_t* d_part_r, uint32_t* d_part_s,
+                         uint64_t* d_off_r, uint64_t* d_off_s, uint32_t* h_bits) {
+    Plan p;
+    gsh_status st = prep(R, S, workspace, workspace_bytes, cfg, p);
+    if (st != GSH_OK) return st;
+    if ((R->n && !d_part_r) || (S->n && !d_part_s) || !d_off_r || !d_off_s || !h_bits)
+        return fail(GSH_ERR_INVALID, "NULL output");
+    cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+    cudaMemsetAsync(p.st, 0, sizeof(DevState), s);
+    run_partition(p, R, S, s);
+    if ((st = check_launch("partition")) != GSH_OK) return st;
+    if (R->n) cudaMemcpyAsync(d_part_r, p.bufB[0], R->n * 8, cudaMemcpyDeviceToDevice, s);
+    if (S->n) cudaMemcpyAsync(d_part_s, p.bufB[1], S->n * 8, cudaMemcpyDeviceToDevice, s);
+    cudaMemcpyAsync(d_off_r, p.start, (p.F + 1) * 8, cudaMemcpyDeviceToDevice, s);
+    cudaMemcpyAsync(d_off_s, p.start + (p.F + 1), (p.F + 1) * 8, cudaMemcpyDeviceToDevice, s);
+    cudaError_t ce = cudaStreamSynchronize(s);
+    if (ce != cudaSuccess) return cuda_fail(ce, "partition sync");
+    h_bits[0] = p.b1;
+    h_bits[1] = p.b2;
+    return GSH_OK;
+}
+
+gsh_status gsh_detect(const gsh_relation* R, const gsh_relation* S, const gsh_config* cfg, void* workspace,
+                      size_t workspace_bytes, void* stream, uint32_t* h_keys, uint32_t* h_cnt_r, uint32_t* h_cnt_s,
+                      uint64_t cap, uint64_t* h_n, gsh_result* res) {
+    Plan p;
+    gsh_status st = prep(R, S, workspace, workspace_bytes, cfg, p);
+    if (st != GSH_OK) return st;
+    if (!h_n || (cap && (!h_keys || !h_cnt_r || !h_cnt_s))) return fail(GSH_ERR_INVALID, "NULL output");
+    if (res) std::memset(res, 0, sizeof(*res));
+    *h_n = 0;
+    if (R->n == 0 || S->n == 0) return GSH_OK;
+    cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+    cudaMemsetAsync(p.st, 0, sizeof(DevState), s);
+    run_partition(p, R, S, s);
+    launch_classify(p, s);
+    if ((st = check_launch("partition")) != GSH_OK) return st;
+    DevState hs;
+    cudaError_t ce = cudaMemcpyAsync(&hs, p.st, sizeof(DevState), cudaMemcpyDeviceToHost, s);
+    if (ce == cudaSuccess) ce = cudaStreamSynchronize(s);
+    if (ce != cudaSuccess) return cuda_fail(ce, "classify sync");
+    if (hs.n_large) {
+        uint64_t gcap = next_pow2_u64(2 * (hs.large_tuples[0] + hs.large_tuples[1]));
+        if (gcap < 1024) gcap = 1024;
+        if (gcap > p.gt_cap_alloc) gcap = p.gt_cap_alloc;
+        launch_detect_prefix(p, hs.n_large, s);
+        launch_detect(p, hs.n_large, (uint32_t)gcap, s);
+        launch_select(p, (uint32_t)gcap, s);
+        if ((st = check_launch("detect")) != GSH_OK) return st;
+        ce = cudaMemcpyAsync(&hs, p.st, sizeof(DevState), cudaMemcpyDeviceToHost, s);
+        if (ce == cudaSuccess) ce = cudaStreamSynchronize(s);
+        if (ce != cudaSuccess) return cuda_fail(ce, "detect sync");
+    }
+    if (res) {
+        res->n_large = hs.n_large;
+        res->n_heavy = hs.n_heavy;
+        res->detect_overflow = hs.detect_overflow;
+        res->pass_bits[0] = p.b1;
+        res->pass_bits[1] = p.b2;
+        res->capacity = p.C;
+        res->heavy_threshold = p.Th;
+        res->heavy_tuples_r = hs.heavy_tuples[0];
+        res->heavy_tuples_s = hs.heavy_tuples[1];
+        res->skew_pairs = hs.skew_pairs;
+    }
+    *h_n = hs.n_heavy;
+    if (hs.n_heavy > cap) return fail(GSH_ERR_INVALID, "h_keys capacity too small");
+    if (hs.n_heavy) {
+        std::vector<HeavyKey> hk(hs.n_heavy);
+        ce = cudaMemcpyAsync(hk.data(), p.H, hs.n_heavy * sizeof(HeavyKey), cudaMemcpyDeviceToHost, s);
+        if (ce == cudaSuccess) ce = cudaStreamSynchronize(s);
+        if (ce != cudaSuccess) return cuda_fail(ce, "heavy copy");
+        for (uint32_t i = 0; i < hs.n_heavy; ++i) {
+            h_keys[i] = hk[i].h;
+            h_cnt_r[i] = hk[i].cnt_r;
+            h_cnt_s[i] = hk[i].cnt_s;
+        }
+    }
+    return GSH_OK;
+}
+
+gsh_status gsh_route_count(const uint32_t* d_keys, uint64_t n, uint32_t route_bits, const uint32_t* d_heavy_keys,
+                           uint64_t n_heavy, uint64_t* d_counts, void* stream) {
+    if (route_bits > 8) return fail(GSH_ERR_INVALID, "route_bits > 8");
+    if ((n && !d_keys) || !d_counts || (n_heavy && !d_heavy_keys)) return fail(GSH_ERR_INVALID, "NULL pointer");
+    launch_route_count(d_keys, n, route_bits, d_heavy_keys, n_heavy, d_counts, reinterpret_cast<cudaStream_t>(stream));
+    return check_launch("route_count");
+}
+
+gsh_status gsh_route_scatter(const uint32_t* d_keys, const uint32_t* d_payloads, uint64_t n, uint32_t route_bits,
+                             const uint32_t* d_heavy_keys, uint64_t n_heavy, const uint64_t* d_offsets,
+                             uint64_t* d_cursor, uint32_t* d_out_keys, uint32_t* d_out_payloads, void* stream) {
+    if (route_bits > 8) return fail(GSH_ERR_INVALID, "route_bits > 8");
+    if (n && (!d_keys || !d_payloads || !d_offsets || !d_cursor || !d_out_keys || !d_out_payloads))
+        return fail(GSH_ERR_INVALID, "NULL pointer");
+    if (n_heavy && !d_heavy_keys) return fail(GSH_ERR_INVALID, "NULL heavy keys");
+    launch_route_scatter(d_keys, d_payloads, n, route_bits, d_heavy_keys, n_heavy, d_offsets, d_cursor, d_out_keys,
+                         d_out_payloads, reinterpret_cast<cudaStream_t>(stream));
+    return check_launch("route_scatter");
+}
+
+gsh_status gsh_count_keys(const uint32_t* d_keys, uint64_t n, const uint32_t* d_query, uint64_t m, uint64_t* d_counts,
+                          void* stream) {
+    if ((n && !d_keys) || (m && (!d_query || !d_counts))) return fail(GSH_ERR_INVALID, "NULL pointer");
+    launch_count_keys(d_keys, n, d_query, m, d_counts, reinterpret_cast<cudaStream_t>(stream));
+    return check_launch("count_keys");
+}
+
+size_t gsh_candidates_workspace_bytes(uint64_t n_r, uint64_t n_s) {
+    return align256(cand_table_slots(n_r, n_s) * 16 + 16) + 256;
+}
+
+gsh_status gsh_local_candidates(const gsh_relation* R, const gsh_relation* S, uint32_t hi_bits, uint32_t part_bits,
+                                const uint8_t* d_large, uint32_t threshold, void* workspace, size_t workspace_bytes,
+                                void* stream, uint32_t* d_cand, uint64_t cap, uint64_t* h_n) {
+    if (!validate_rel(R) || !validate_rel(S)) return fail(GSH_ERR_INVALID, "invalid relation");
+    if (part_bits > 16 || hi_bits + part_bits > 32 || !d_large || !h_n || (cap && !d_cand))
+        return fail(GSH_ERR_INVALID, "bad argument");
+    const size_t need = gsh_candidates_workspace_bytes(R->n, S->n);
+    if (!workspace || workspace_bytes < need || (reinterpret_cast<uintptr_t>(workspace) & 255u))
+        return fail(GSH_ERR_INVALID, "workspace NULL, misaligned or too small");
+    cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+    unsigned long long* d_nout =
+        reinterpret_cast<unsigned long long*>(reinterpret_cast<unsigned char*>(workspace) + need - 256);
+    cudaMemsetAsync(d_nout, 0, 8, s);
+    launch_candidates(R->keys, R->n, S->keys, S->n, hi_bits, part_bits, d_large, threshold ? threshold : 1, workspace,
+                      d_cand, cap, d_nout, s);
+    gsh_status st = check_launch("candidates");
+    if (st != GSH_OK) return st;
+    unsigned long long nout = 0;
+    cudaError_t ce = cudaMemcpyAsync(&nout, d_nout, 8, cudaMemcpyDeviceToHost, s);
+    if (ce == cudaSuccess) ce = cudaStreamSynchronize(s);
+    if (ce != cudaSuccess) return cuda_fail(ce, "candidates sync");
+    *h_n = nout;
+    if (nout > cap) return fail(GSH_ERR_INVALID, "candidate capacity too small");
+    return GSH_OK;
+}
+
+const char* gsh_status_string(gsh_status s) {
+    switch (s) {
+        case GSH_OK: return "GSH_OK";
+        case GSH_ERR_INVALID: return "GSH_ERR_INVALID";
+        case GSH_ERR_NOMEM: return "GSH_ERR_NOMEM";
+        case GSH_ERR_CUDA: return "GSH_ERR_CUDA";
+        case GSH_ERR_NCCL: return "GSH_ERR_NCCL";
+        case GSH_ERR_INTERNAL: return "GSH_ERR_INTERNAL";
+    }
+    return "GSH_UNKNOWN";
+}
+
+const char* gsh_last_error(void) { return g_err.c_str(); }
+
+int gsh_version(void) { return 1; }
+
+int gsh_compiled_arch(void) { return 100; }
+
+}  // extern "C"

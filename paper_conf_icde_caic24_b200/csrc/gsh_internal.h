@@ -1,0 +1,131 @@
+// gsh_internal.h -- host-side plan, workspace layout and kernel launchers (not part of the ABI).
+#pragma once
+#include <cstddef>
+#include <cstdint>
+#include <cuda_runtime.h>
+
+#include "../../include/gsh.h"
+
+namespace gsh {
+
+// ----------------------------------------------------------------- fixed shapes --
+constexpr int kScatterBlock = 512;              // threads per partition-scatter CTA
+constexpr int kScatterIpt = 16;                 // tuples per thread per tile
+constexpr int kScatterTile = kScatterBlock * kScatterIpt;  // 8192 tuples per tile
+constexpr int kMaxDigitBits = 8;                // radix bits per pass (256 buckets)
+constexpr int kMaxPartBits = 16;                // b1 + b2 <= 16 (65536 partitions)
+constexpr int kHistBlock = 1024;
+constexpr int kNmBlock = 256;                   // NM-join CTA
+constexpr uint32_t kMaxCapacity = 8192;         // largest NM build table (tuples)
+constexpr uint32_t kNmSlice = 8192;             // S tuples probed per NM work item
+constexpr int kSkewBlock = 256;                 // skewed-key join CTA
+constexpr int kSkewSpt = 4;                     // S payloads per thread (registers)
+constexpr int kSkewTileS = kSkewBlock * kSkewSpt;  // 1024
+constexpr int kSkewTileR = 64;                  // R payloads per tile (shared memory)
+constexpr uint32_t kDetectChunk = 4096;         // tuples per detect / split work item
+constexpr uint32_t kNoHeavy = 0xffffffffu;
+constexpr int kDetectMaxProbe = 4096;
+
+// Device-resident counters and accumulators, zeroed once per call.
+struct DevState {
+    unsigned long long count, checksum, cursor;    // result accumulators (all phases)
+    unsigned long long nm_count, nm_checksum;      // NM-join share
+    unsigned long long large_tuples[2];            // tuples in large partitions (R, S)
+    unsigned long long heavy_tuples[2];            // tuples of skewed keys (R, S)
+    unsigned long long skew_pairs;                 // sum |R_k| |S_k|
+    unsigned long long skew_tiles;                 // total dense tiles
+    unsigned long long nm_items;                   // NM work items
+    unsigned long long skew_claim;                 // tile claim counter
+    unsigned int n_large, n_heavy, detect_overflow, nm_claim;
+    unsigned int claim[8];                         // per-kernel work claim counters
+};
+
+// Skewed-key side list entry H[k].
+struct HeavyKey {
+    uint32_t h, cnt_r, cnt_s, part;
+};
+
+// NM-join descriptor of one partition pair after the split (normal tuples only).
+struct NmPart {
+    const uint2* r;
+    const uint2* s;
+    uint32_t rlen, slen;
+};
+
+struct Plan {
+    // sizes and parameters
+    uint64_t n[2] = {0, 0};
+    uint32_t b1 = 0, b2 = 0, route_bits = 0;
+    uint32_t C = 4096, Th = 1024;
+    uint32_t F = 1;                 // 1 << (b1 + b2)
+    int force_normal = 0, force_heavy = 0, timing = 0;
+    int num_sms = 148;
+    int hist_grid = 74;             // CTAs per side in the histogram kernel
+    uint64_t max_tiles[2] = {0, 0}; // look-back status rows per side
+    uint32_t gt_cap_alloc = 0;      // detection table slots allocated
+    uint64_t h_max = 0;             // skewed-key list capacity
+    uint64_t scan_scratch_elems = 0;
+
+    // workspace carve-up (device pointers)
+    uint2* bufA[2] = {nullptr, nullptr};      // pass-1 output, later normal remainders
+    uint2* bufB[2] = {nullptr, nullptr};      // final partitions
+    uint32_t* heavy_pay[2] = {nullptr, nullptr};  // skewed-key payload arrays
+    uint16_t* hist_partial = nullptr;         // [2][hist_grid][F]
+    uint32_t* hist_spill = nullptr;           // [2][F]
+    uint32_t* cnt = nullptr;                  // [2][F]
+    uint64_t* start = nullptr;                // [2][F + 1]
+    uint64_t* status = nullptr;               // [2][max_tiles][256]
+    DevState* st = nullptr;
+    unsigned long long* gt_key = nullptr;     // [gt_cap_alloc]  (1 << 32 | h), 0 = empty
+    uint32_t* gt_cnt = nullptr;               // [2][gt_cap_alloc]
+    uint32_t* gt_hid = nullptr;               // [gt_cap_alloc]
+    uint32_t* large_list = nullptr;           // [F]
+    uint32_t* large_idx = nullptr;            // [F] partition -> large index or kNoHeavy
+    uint32_t* part_heavy = nullptr;           // [2][F]  skewed tuples per partition
+    uint64_t* det_prefix = nullptr;           // [F + 1] detect/split items per large partition
+    uint64_t* nrm_off = nullptr;              // [2][F + 1] normal remainder offsets (large idx)
+    HeavyKey* H = nullptr;                    // [h_max]
+    uint64_t* h_off = nullptr;                // [2][h_max + 1]
+    uint64_t* h_tiles = nullptr;              // [h_max + 1]
+    uint32_t* h_cur = nullptr;                // [2][h_max] split cursors
+    uint32_t* nrm_cur = nullptr;              // [2][F]     split cursors (normal)
+    NmPart* nm = nullptr;                     // [F]
+    uint64_t* nm_prefix = nullptr;            // [F + 1]
+    uint64_t* scan_scratch = nullptr;         // block sums for the generic scan
+    size_t bytes = 0;
+};
+
+// Computes parameters and carves `ws` (may be nullptr to only size it).  Returns false on
+// invalid configuration.
+bool plan_build(Plan& p, uint64_t nR, uint64_t nS, const gsh_config* cfg, void* ws, int num_sms);
+
+// ------------------------------------------------------------------ launchers --
+// Every launcher enqueues on `s` and returns the number of kernels it launched.
+int launch_hash(const uint32_t* keys, uint32_t* out, uint64_t n, cudaStream_t s);
+int launch_hist(const Plan& p, const uint32_t* k0, const uint32_t* k1, cudaStream_t s);
+int launch_hist_reduce_scan(const Plan& p, cudaStream_t s);
+int launch_scatter(const Plan& p, int pass, const uint32_t* const keys[2], const uint32_t* const pays[2],
+                   cudaStream_t s);
+int launch_classify(const Plan& p, cudaStream_t s);
+int launch_detect_prefix(const Plan& p, uint32_t n_large, cudaStream_t s);
+int launch_detect(const Plan& p, uint32_t n_large, uint32_t gt_cap, cudaStream_t s);
+int launch_select(const Plan& p, uint32_t gt_cap, cudaStream_t s);
+int launch_heavy_prefix(const Plan& p, uint32_t n_heavy, uint32_t n_large, cudaStream_t s);
+int launch_split(const Plan& p, uint32_t n_large, uint32_t gt_cap, cudaStream_t s);
+int launch_nm_setup(const Plan& p, uint32_t n_large, cudaStream_t s);
+int launch_nmjoin(const Plan& p, int materialize, uint32_t* pairs, uint64_t cap, cudaStream_t s);
+int launch_skewjoin(const Plan& p, uint32_t n_heavy, int materialize, uint32_t* pairs, uint64_t cap,
+                    cudaStream_t s);
+
+// Routing (multi-GPU)
+int launch_route_count(const uint32_t* keys, uint64_t n, uint32_t rb, const uint32_t* hk, uint64_t nh,
+                       uint64_t* counts, cudaStream_t s);
+int launch_route_scatter(const uint32_t* keys, const uint32_t* pays, uint64_t n, uint32_t rb,
+                         const uint32_t* hk, uint64_t nh, const uint64_t* off, uint64_t* cur,
+                         uint32_t* ok, uint32_t* op, cudaStream_t s);
+int launch_count_keys(const uint32_t* keys, uint64_t n, const uint32_t* q, uint64_t m, uint64_t* counts,
+                      cudaStream_t s);
+int launch_radix_hist(const uint32_t* keys, uint64_t n, uint32_t hi_bits, uint32_t nbits, uint64_t* hist,
+                      cudaStream_t s);
+
+}  // namespace gsh

@@ -1,0 +1,454 @@
+// skew.cu -- GSH phases (2) and (3) (§IV-B), SURVEY.md §8(a) rows a5-a7.
+//
+//   a5 k_classify : "identify normal vs. large partitions by comparing the partition size with
+//                   a pre-defined threshold" (L107).  large(p) <=> |R_p| > C or |S_p| > C
+//                   (and both sides non-empty: a partition with an empty side yields nothing).
+//   a6 k_detect   : exact per-key counts of every key of every large partition, both sides.
+//                   Warp aggregation with __match_any_sync collapses a skewed key's tuples to
+//                   one update per warp; counts live in an open-addressing table keyed by
+//                   h = fmix32(key) (the paper's "linear probing based hash table", L107/L112,
+//                   fed with all tuples instead of a 1 % sample -- DESIGN.md §3 reading R3).
+//      k_select   : threshold pass compacting skewed keys into the side list H (L112 top-k,
+//                   reading R4: max(cnt_R, cnt_S) >= T_h inside a large partition).
+//   a7 k_split    : "checks each R tuple against the skewed keys.  If the tuple is skewed, it
+//                   is appended to an array allocated for the associated skewed key ...
+//                   Otherwise ... appends the tuple to a normal partition" (L114); same for S.
+//                   Skewed arrays hold payloads only (every tuple of R_k has key k).
+#include "gsh_device.cuh"
+#include "gsh_internal.h"
+#include "gsh_scan.cuh"
+
+namespace gsh {
+
+__device__ __forceinline__ uint32_t part_of(uint32_t h, uint32_t shift, uint32_t mask) {
+    return (h >> shift) & mask;
+}
+
+// ------------------------------------------------------------------ a5: classify --
+__global__ void k_classify(const uint32_t* __restrict__ cnt, uint32_t F, uint32_t C, int force_normal,
+                           int force_heavy, uint32_t* __restrict__ large_list, uint32_t* __restrict__ large_idx,
+                           uint32_t* __restrict__ part_heavy, DevState* st) {
+    for (uint32_t p = blockIdx.x * blockDim.x + threadIdx.x; p < F; p += gridDim.x * blockDim.x) {
+        const uint32_t cr = cnt[p], cs = cnt[F + p];
+        part_heavy[p] = 0;
+        part_heavy[F + p] = 0;
+        const bool large = (cr > 0 && cs > 0) && !force_normal && (force_heavy || cr > C || cs > C);
+        uint32_t idx = kNoHeavy;
+        if (large) {
+            idx = atomicAdd(&st->n_large, 1u);
+            large_list[idx] = p;
+            atomicAdd(&st->large_tuples[0], (unsigned long long)cr);
+            atomicAdd(&st->large_tuples[1], (unsigned long long)cs);
+        }
+        large_idx[p] = idx;
+    }
+}
+
+int launch_classify(const Plan& p, cudaStream_t s) {
+    unsigned grid = (p.F + 255) / 256;
+    k_classify<<<grid, 256, 0, s>>>(p.cnt, p.F, p.C, p.force_normal, p.force_heavy, p.large_list, p.large_idx,
+                                    p.part_heavy, p.st);
+    return 1;
+}
+
+// Items of detect / split: ceil((|R_p| + |S_p|) / kDetectChunk) per large partition.
+struct DetectItems {
+    const uint32_t* cnt;
+    const uint32_t* large_list;
+    uint32_t F;
+    __device__ uint64_t operator()(uint64_t i) const {
+        uint32_t p = large_list[i];
+        uint64_t t = uint64_t(cnt[p]) + cnt[F + p];
+        return (t + kDetectChunk - 1) / kDetectChunk;
+    }
+};
+
+int launch_detect_prefix(const Plan& p, uint32_t n_large, cudaStream_t s) {
+    return launch_scan(DetectItems{p.cnt, p.large_list, p.F}, n_large, p.det_prefix, p.scan_scratch, s);
+}
+
+// Locate item `it` among large partitions: returns large index li and chunk c.
+__device__ __forceinline__ uint32_t find_prefix(const uint64_t* prefix, uint32_t n, uint64_t it) {
+    // largest i with prefix[i] <= it, i < n
+    uint32_t lo = 0, hi = n;
+    while (hi - lo > 1) {
+        uint32_t mid = (lo + hi) >> 1;
+        if (prefix[mid] <= it) lo = mid; else hi = mid;
+    }
+    return lo;
+}
+
+struct LargeView {
+    const uint2* part[2];     // final partitions (bufB)
+    const uint64_t* start;    // [2][F + 1]
+    const uint32_t* cnt;      // [2][F]
+    const uint32_t* large_list;
+    const uint64_t* det_prefix;
+    uint32_t F, n_large;
+};
+
+// The element range of one item: tuples [e0, e1) of the concatenation R_p ++ S_p.
+struct ItemRange {
+    uint32_t li, p, cr, cs;
+    uint64_t e0, e1;
+};
+
+__device__ __forceinline__ ItemRange item_range(const LargeView& v, uint64_t it) {
+    ItemRange r;
+    r.li = find_prefix(v.det_prefix, v.n_large, it);
+    r.p = v.large_list[r.li];
+    r.cr = v.cnt[r.p];
+    r.cs = v.cnt[v.F + r.p];
+    uint64_t c = it - v.det_prefix[r.li];
+    r.e0 = c * kDetectChunk;
+    r.e1 = umin64(r.e0 + kDetectChunk, uint64_t(r.cr) + r.cs);
+    return r;
+}
+
+__device__ __forceinline__ uint2 item_tuple(const LargeView& v, const ItemRange& r, uint64_t e, int& side) {
+    side = e >= r.cr;
+    uint64_t off = side ? (e - r.cr) : e;
+    return v.part[side][v.start[size_t(side) * (v.F + 1) + r.p] + off];
+}
+
+__device__ __forceinline__ uint32_t gt_slot0(uint32_t h, uint32_t logcap) {
+    return (h * 0x9E3779B1u) >> (32 - logcap);
+}
+
+// Insert-or-find h; returns slot or kNoHeavy when the probe budget is exhausted.
+__device__ __forceinline__ uint32_t gt_insert(unsigned long long* keys, uint32_t h, uint32_t logcap) {
+    const unsigned long long tag = (1ull << 32) | h;
+    const uint32_t mask = (1u << logcap) - 1;
+    uint32_t slot = gt_slot0(h, logcap);
+    for (int probe = 0; probe < kDetectMaxProbe; ++probe) {
+        unsigned long long cur = keys[slot];
+        if (cur == tag) return slot;
+        if (cur == 0) {
+            unsigned long long prev = atomicCAS(&keys[slot], 0ull, tag);
+            if (prev == 0 || prev == tag) return slot;
+        }
+        slot = (slot + 1) & mask;
+    }
+    return kNoHeavy;
+}
+
+__device__ __forceinline__ uint32_t gt_find(const unsigned long long* keys, uint32_t h, uint32_t logcap) {
+    const unsigned long long tag = (1ull << 32) | h;
+    const uint32_t mask = (1u << logcap) - 1;
+    uint32_t slot = gt_slot0(h, logcap);
+    for (int probe = 0; probe < kDetectMaxProbe; ++probe) {
+        unsigned long long cur = keys[slot];
+        if (cur == tag) return slot;
+        if (cur == 0) return kNoHeavy;
+        slot = (slot + 1) & mask;
+    }
+    return kNoHeavy;
+}
+
+// ------------------------------------------------------------------- a6: detect --
+constexpr int kDetBlock = 256;
+
+__global__ void __launch_bounds__(kDetBlock) k_detect(LargeView v, unsigned long long* gt_key, uint32_t* gt_cnt,
+                                                     uint32_t cap_alloc, uint32_t logcap, DevState* st,
+                                                     unsigned int* claim) {
+    __shared__ unsigned int s_it;
+    const uint64_t total = v.det_prefix[v.n_large];
+    for (;;) {
+        if (threadIdx.x == 0) s_it = atomicAdd(claim, 1u);
+        __syncthreads();
+        const uint64_t it = s_it;
+        __syncthreads();
+        if (it >= total) break;
+        const ItemRange r = item_range(v, it);
+        for (uint64_t base = r.e0; base < r.e1; base += kDetBlock) {
+            const uint64_t e = base + threadIdx.x;
+            const bool valid = e < r.e1;
+            int side = 0;
+            uint32_t h = 0;
+            if (valid) h = item_tuple(v, r, e, side).x;
+            const unsigned long long key = valid ? ((uint64_t(side) << 32) | h) : ((2ull << 32) | lane_id());
+            const uint32_t peers = __match_any_sync(kFull, key);
+            if (valid && (peers & lanemask_lt()) == 0) {
+                uint32_t slot = gt_insert(gt_key, h, logcap);
+                if (slot == kNoHeavy) {
+                    st->detect_overflow = 1;
+                } else {
+                    atomicAdd(&gt_cnt[size_t(side) * cap_alloc + slot], (uint32_t)__popc(peers));
+                }
+            }
+        }
+    }
+}
+
+int launch_detect(const Plan& p, uint32_t n_large, uint32_t gt_cap, cudaStream_t s) {
+    if (n_large == 0) return 0;
+    uint32_t logcap = 0;
+    while ((1u << logcap) < gt_cap) ++logcap;
+    cudaMemsetAsync(p.gt_key, 0, size_t(gt_cap) * sizeof(unsigned long long), s);
+    cudaMemsetAsync(p.gt_cnt, 0, size_t(gt_cap) * sizeof(uint32_t), s);
+    cudaMemsetAsync(p.gt_cnt + p.gt_cap_alloc, 0, size_t(gt_cap) * sizeof(uint32_t), s);
+    LargeView v{{p.bufB[0], p.bufB[1]}, p.start, p.cnt, p.large_list, p.det_prefix, p.F, n_large};
+    k_detect<<<p.num_sms * 8, kDetBlock, 0, s>>>(v, p.gt_key, p.gt_cnt, p.gt_cap_alloc, logcap, p.st,
+                                                 &p.st->claim[2]);
+    return 1;
+}
+
+// ------------------------------------------------------------------- a6: select --
+__global__ void k_select(const unsigned long long* __restrict__ gt_key, const uint32_t* __restrict__ gt_cnt,
+                         uint32_t* __restrict__ gt_hid, uint32_t cap, uint32_t cap_alloc, uint32_t Th,
+                         int force_heavy, uint32_t pshift, uint32_t pmask, uint32_t F, HeavyKey* __restrict__ H,
+                         uint32_t* __restrict__ part_heavy, DevState* st) {
+    for (uint32_t slot = blockIdx.x * blockDim.x + threadIdx.x; slot < cap; slot += gridDim.x * blockDim.x) {
+        const unsigned long long kw = gt_key[slot];
+        if (kw == 0) continue;
+        const uint32_t h = (uint32_t)kw;
+        const uint32_t cr = gt_cnt[slot], cs = gt_cnt[cap_alloc + slot];
+        const bool heavy = force_heavy || max(cr, cs) >= Th;
+        uint32_t hid = kNoHeavy;
+        if (heavy) {
+            const uint32_t p = part_of(h, pshift, pmask);
+            hid = atomicAdd(&st->n_heavy, 1u);
+            H[hid] = HeavyKey{h, cr, cs, p};
+            if (cr) atomicAdd(&part_heavy[p], cr);
+            if (cs) atomicAdd(&part_heavy[F + p], cs);
+            atomicAdd(&st->heavy_tuples[0], (unsigned long long)cr);
+            atomicAdd(&st->heavy_tuples[1], (unsigned long long)cs);
+            atomicAdd(&st->skew_pairs, (unsigned long long)cr * cs);
+        }
+        gt_hid[slot] = hid;
+    }
+}
+
+int launch_select(const Plan& p, uint32_t gt_cap, cudaStream_t s) {
+    const uint32_t B = p.b1 + p.b2;
+    const uint32_t pshift = B ? (32 - p.route_bits - B) : 0;
+    unsigned grid = (unsigned)umin64((gt_cap + 255) / 256, uint64_t(p.num_sms) * 16);
+    k_select<<<grid, 256, 0, s>>>(p.gt_key, p.gt_cnt, p.gt_hid, gt_cap, p.gt_cap_alloc, p.Th, p.force_heavy, pshift,
+                                  p.F - 1, p.F, p.H, p.part_heavy, p.st);
+    return 1;
+}
+
+// ------------------------------------------------------------- offsets of H / normal --
+struct HeavyCount {
+    const HeavyKey* H;
+    int side;
+    __device__ uint64_t operator()(uint64_t k) const { return side ? H[k].cnt_s : H[k].cnt_r; }
+};
+struct HeavyTiles {
+    const HeavyKey* H;
+    __device__ uint64_t operator()(uint64_t k) const {
+        uint64_t tr = (H[k].cnt_r + kSkewTileR - 1) / kSkewTileR;
+        uint64_t ts = (H[k].cnt_s + kSkewTileS - 1) / kSkewTileS;
+        return tr * ts;
+    }
+};
+struct NormalRemainder {
+    const uint32_t* cnt;
+    const uint32_t* part_heavy;
+    const uint32_t* large_list;
+    uint32_t F;
+    int side;
+    __device__ uint64_t operator()(uint64_t li) const {
+        uint32_t p = large_list[li];
+        return uint64_t(cnt[side * F + p]) - part_heavy[side * F + p];
+    }
+};
+
+int launch_heavy_prefix(const Plan& p, uint32_t n_heavy, uint32_t n_large, cudaStream_t s) {
+    int l = 0;
+    l += launch_scan(HeavyCount{p.H, 0}, n_heavy, p.h_off, p.scan_scratch, s);
+    l += launch_scan(HeavyCount{p.H, 1}, n_heavy, p.h_off + (p.h_max + 1), p.scan_scratch, s);
+    l += launch_scan(HeavyTiles{p.H}, n_heavy, p.h_tiles, p.scan_scratch, s);
+    l += launch_scan(NormalRemainder{p.cnt, p.part_heavy, p.large_list, p.F, 0}, n_large, p.nrm_off,
+                     p.scan_scratch, s);
+    l += launch_scan(NormalRemainder{p.cnt, p.part_heavy, p.large_list, p.F, 1}, n_large, p.nrm_off + (p.F + 1),
+                     p.scan_scratch, s);
+    cudaMemsetAsync(p.h_cur, 0, size_t(2) * p.h_max * sizeof(uint32_t), s);
+    cudaMemsetAsync(p.nrm_cur, 0, size_t(2) * p.F * sizeof(uint32_t), s);
+    return l;
+}
+
+// -------------------------------------------------------------------- a7: split --
+__global__ void __launch_bounds__(kDetBlock) k_split(LargeView v, const unsigned long long* gt_key,
+                                                    const uint32_t* gt_hid, uint32_t logcap,
+                                                    const uint64_t* h_off, uint64_t h_stride, uint32_t* h_cur,
+                                                    uint32_t h_max, uint32_t* heavy_pay_r, uint32_t* heavy_pay_s,
+                                                    const uint64_t* nrm_off, uint32_t* nrm_cur, uint2* out_r,
+                                                    uint2* out_s, unsigned int* claim) {
+    __shared__ unsigned int s_it;
+    const uint64_t total = v.det_prefix[v.n_large];
+    const uint32_t lane = lane_id();
+    const uint32_t ltm = lanemask_lt();
+    for (;;) {
+        if (threadIdx.x == 0) s_it = atomicAdd(claim, 1u);
+        __syncthreads();
+        const uint64_t it = s_it;
+        __syncthreads();
+        if (it >= total) break;
+        const ItemRange r = item_range(v, it);
+        for (uint64_t base = r.e0; base < r.e1; base += kDetBlock) {
+            const uint64_t e = base + threadIdx.x;
+            const bool valid = e < r.e1;
+            int side = 0;
+            uint2 t = make_uint2(0, 0);
+            if (valid) t = item_tuple(v, r, e, side);
+            // one table lookup per distinct key in the warp
+            const unsigned long long key = valid ? ((uint64_t(side) << 32) | t.x) : ((2ull << 32) | lane);
+            const uint32_t peers = __match_any_sync(kFull, key);
+            const uint32_t leader = __ffs(peers) - 1;
+            uint32_t hid = kNoHeavy;
+            if (valid && lane == leader) {
+                uint32_t slot = gt_find(gt_key, t.x, logcap);
+                hid = (slot == kNoHeavy) ? kNoHeavy : gt_hid[slot];
+            }
+            hid = __shfl_sync(kFull, hid, leader);
+            // heavy: append payload to its key array (warp-aggregated cursor per (side, key))
+            const bool heavy = valid && hid != kNoHeavy;
+            uint32_t pos = 0;
+            if (heavy && lane == leader) pos = atomicAdd(&h_cur[size_t(side) * h_max + hid], (uint32_t)__popc(peers));
+            pos = __shfl_sync(kFull, pos, leader) + __popc(peers & ltm);
+            if (heavy) {
+                uint32_t* dst = side ? heavy_pay_s : heavy_pay_r;
+                dst[h_off[size_t(side) * h_stride + hid] + pos] = t.y;
+            }
+            // normal: compact into the normal remainder of this large partition
+            const bool normal = valid && hid == kNoHeavy;
+#pragma unroll
+            for (int sd = 0; sd < 2; ++sd) {
+                const uint32_t m = __ballot_sync(kFull, normal && side == sd);
+                if (m == 0) continue;
+                const uint32_t lead = __ffs(m) - 1;
+                uint32_t b = 0;
+                if (lane == lead) b = atomicAdd(&nrm_cur[size_t(sd) * v.F + r.li], (uint32_t)__popc(m));
+                b = __shfl_sync(kFull, b, lead);
+                if (normal && side == sd) {
+                    uint2* dst = sd ? out_s : out_r;
+                    dst[nrm_off[size_t(sd) * (v.F + 1) + r.li] + b + __popc(m & ltm)] = t;
+                }
+            }
+        }
+    }
+}
+
+int launch_split(const Plan& p, uint32_t n_large, uint32_t gt_cap, cudaStream_t s) {
+    if (n_large == 0) return 0;
+    uint32_t logcap = 0;
+    while ((1u << logcap) < gt_cap) ++logcap;
+    LargeView v{{p.bufB[0], p.bufB[1]}, p.start, p.cnt, p.large_list, p.det_prefix, p.F, n_large};
+    k_split<<<p.num_sms * 8, kDetBlock, 0, s>>>(v, p.gt_key, p.gt_hid, logcap, p.h_off, p.h_max + 1, p.h_cur,
+                                                (uint32_t)p.h_max, p.heavy_pay[0], p.heavy_pay[1], p.nrm_off,
+                                                p.nrm_cur, p.bufA[0], p.bufA[1], &p.st->claim[3]);
+    return 1;
+}
+
+// --------------------------------------------------------------- NM descriptors --
+__global__ void k_nm_setup(const uint2* bufB0, const uint2* bufB1, const uint2* bufA0, const uint2* bufA1,
+                           const uint64_t* start, const uint32_t* cnt, const uint32_t* large_idx,
+                           const uint32_t* part_heavy, const uint64_t* nrm_off, uint32_t F, NmPart* nm) {
+    for (uint32_t p = blockIdx.x * blockDim.x + threadIdx.x; p < F; p += gridDim.x * blockDim.x) {
+        NmPart d;
+        const uint32_t li = large_idx[p];
+        if (li == kNoHeavy) {
+            d.r = bufB0 + start[p];
+            d.s = bufB1 + start[F + 1 + p];
+            d.rlen = cnt[p];
+            d.slen = cnt[F + p];
+        } else {
+            d.r = bufA0 + nrm_off[li];
+            d.s = bufA1 + nrm_off[F + 1 + li];
+            d.rlen = cnt[p] - part_heavy[p];
+            d.slen = cnt[F + p] - part_heavy[F + p];
+        }
+        nm[p] = d;
+    }
+}
+
+struct NmItems {
+    const NmPart* nm;
+    uint32_t C;
+    __device__ uint64_t operator()(uint64_t p) const {
+        const NmPart d = nm[p];
+        if (d.rlen == 0 || d.slen == 0) return 0;
+        return uint64_t((d.rlen + C - 1) / C) * ((d.slen + kNmSlice - 1) / kNmSlice);
+    }
+};
+
+int launch_nm_setup(const Plan& p, uint32_t n_large, cudaStream_t s) {
+    (void)n_large;
+    unsigned grid = (p.F + 255) / 256;
+    k_nm_setup<<<grid, 256, 0, s>>>(p.bufB[0], p.bufB[1], p.bufA[0], p.bufA[1], p.start, p.cnt, p.large_idx,
+                                    p.part_heavy, p.nrm_off, p.F, p.nm);
+    return 1 + launch_scan(NmItems{p.nm, p.C}, p.F, p.nm_prefix, p.scan_scratch, s);
+}
+
+}  // namespace gsh
+
+namespace gsh {
+
+// ----------------------------------------------- multi-GPU: local skew candidates --
+// Exact local counts of every key whose partition is flagged large (globally agreed flags),
+// then keys with local max(cnt_R, cnt_S) >= threshold are emitted as candidates (by hash h).
+__global__ void k_cand_count(const uint32_t* __restrict__ keys, uint64_t n, int side, uint32_t pshift,
+                             uint32_t pmask, const uint8_t* __restrict__ large, unsigned long long* gt_key,
+                             uint32_t* gt_cnt, uint32_t cap, uint32_t logcap, unsigned int* overflow) {
+    for (uint64_t i = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; i - threadIdx.x < n;
+         i += uint64_t(gridDim.x) * blockDim.x) {
+        bool v = i < n;
+        uint32_t h = v ? hash32(keys[i]) : 0u;
+        v = v && large[part_of(h, pshift, pmask)];
+        const unsigned long long key = v ? h : ((1ull << 32) | lane_id());
+        const uint32_t peers = __match_any_sync(kFull, key);
+        if (v && (peers & lanemask_lt()) == 0) {
+            uint32_t slot = gt_insert(gt_key, h, logcap);
+            if (slot == kNoHeavy) *overflow = 1;
+            else atomicAdd(&gt_cnt[size_t(side) * cap + slot], (uint32_t)__popc(peers));
+        }
+    }
+}
+
+__global__ void k_cand_select(const unsigned long long* __restrict__ gt_key, const uint32_t* __restrict__ gt_cnt,
+                              uint32_t cap, uint32_t threshold, uint32_t* out, unsigned long long outcap,
+                              unsigned long long* nout) {
+    for (uint32_t slot = blockIdx.x * blockDim.x + threadIdx.x; slot < cap; slot += gridDim.x * blockDim.x) {
+        const unsigned long long kw = gt_key[slot];
+        if (kw == 0) continue;
+        if (max(gt_cnt[slot], gt_cnt[cap + slot]) >= threshold) {
+            unsigned long long i = atomicAdd(nout, 1ull);
+            if (i < outcap) out[i] = (uint32_t)kw;
+        }
+    }
+}
+
+size_t cand_table_slots(uint64_t nR, uint64_t nS) {
+    uint64_t t = 2 * (nR + nS);
+    uint64_t c = 1024;
+    while (c < t && c < (1ull << 26)) c <<= 1;
+    return (size_t)c;
+}
+
+int launch_candidates(const uint32_t* kr, uint64_t nR, const uint32_t* ks, uint64_t nS, uint32_t hi_bits,
+                      uint32_t part_bits, const uint8_t* large, uint32_t threshold, void* ws, uint32_t* out,
+                      uint64_t outcap, unsigned long long* d_nout, cudaStream_t s) {
+    const uint32_t cap = (uint32_t)cand_table_slots(nR, nS);
+    uint32_t logcap = 0;
+    while ((1u << logcap) < cap) ++logcap;
+    unsigned long long* gt_key = reinterpret_cast<unsigned long long*>(ws);
+    uint32_t* gt_cnt = reinterpret_cast<uint32_t*>(gt_key + cap);
+    unsigned int* overflow = gt_cnt + 2 * size_t(cap);
+    cudaMemsetAsync(ws, 0, size_t(cap) * 16 + 16, s);
+    const uint32_t pshift = part_bits ? (32 - hi_bits - part_bits) : 0;
+    const uint32_t pmask = (1u << part_bits) - 1;
+    int l = 0;
+    if (nR) {
+        k_cand_count<<<148 * 8, 512, 0, s>>>(kr, nR, 0, pshift, pmask, large, gt_key, gt_cnt, cap, logcap, overflow);
+        ++l;
+    }
+    if (nS) {
+        k_cand_count<<<148 * 8, 512, 0, s>>>(ks, nS, 1, pshift, pmask, large, gt_key, gt_cnt, cap, logcap, overflow);
+        ++l;
+    }
+    k_cand_select<<<148 * 4, 256, 0, s>>>(gt_key, gt_cnt, cap, threshold, out, outcap, d_nout);
+    return l + 1;
+}
+
+}  // namespace gsh

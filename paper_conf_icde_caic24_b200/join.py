@@ -1,0 +1,252 @@
+"""Python API of the B200 GSH join: thin marshalling over the C-ABI (include/gsh.h).
+
+Every step of the join runs in libgsh.so's CUDA kernels; PyTorch only provides device
+memory (the workspace and outputs come from torch's caching allocator) and the stream.
+Inputs are CUDA tensors of dtype int32 (or uint32) holding u32 bit patterns.  There is
+no CPU path: calling with CPU tensors raises.
+"""
+from __future__ import annotations
+
+import ctypes
+from dataclasses import dataclass, field
+
+import torch
+
+from . import _lib
+from ._lib import GshConfig, GshOutput, GshRelation, GshResult, check, load
+
+
+def make_config(capacity: int = 0, pass_bits=None, heavy_threshold: int = 0, route_bits: int = 0,
+                force_all_normal: bool = False, force_all_heavy: bool = False, timing: bool = False) -> GshConfig:
+    """Build a gsh_config (see include/gsh.h for each field's meaning)."""
+    cfg = _lib.default_config()
+    cfg.capacity = int(capacity)
+    if pass_bits is not None:
+        cfg.pass_bits[0] = int(pass_bits[0])
+        cfg.pass_bits[1] = int(pass_bits[1])
+    cfg.heavy_threshold = int(heavy_threshold)
+    cfg.route_bits = int(route_bits)
+    cfg.force_all_normal = int(bool(force_all_normal))
+    cfg.force_all_heavy = int(bool(force_all_heavy))
+    cfg.timing = int(bool(timing))
+    return cfg
+
+
+@dataclass
+class JoinResult:
+    count: int
+    checksum: int
+    written: int = 0
+    overflow: bool = False
+    pairs: torch.Tensor | None = None   # (written, 2) int32 view of (payload_R, payload_S)
+    stats: dict = field(default_factory=dict)
+
+
+def _check_dev(t: torch.Tensor, name: str) -> torch.Tensor:
+    if not isinstance(t, torch.Tensor):
+        raise TypeError(f"{name} must be a torch.Tensor")
+    if not t.is_cuda:
+        raise ValueError(f"{name} must be a CUDA tensor (the GSH join has no CPU path)")
+    if t.dtype not in (torch.int32, torch.uint32):
+        raise TypeError(f"{name} must be int32/uint32, got {t.dtype}")
+    if t.dim() != 1:
+        raise ValueError(f"{name} must be 1-D")
+    return t.contiguous()
+
+
+def _rel(keys: torch.Tensor, pays: torch.Tensor, side: str) -> GshRelation:
+    if keys.numel() != pays.numel():
+        raise ValueError(f"{side}: keys and payloads differ in length")
+    return GshRelation(keys.data_ptr() if keys.numel() else None, pays.data_ptr() if pays.numel() else None,
+                       keys.numel())
+
+
+def _stream_handle(stream) -> int | None:
+    if stream is None:
+        return torch.cuda.current_stream().cuda_stream
+    if isinstance(stream, torch.cuda.Stream):
+        return stream.cuda_stream
+    return int(stream)
+
+
+class Workspace:
+    """Grow-only device scratch buffer (torch caching allocator), one per device."""
+
+    def __init__(self):
+        self._buf: dict[int, torch.Tensor] = {}
+
+    def get(self, nbytes: int, device: torch.device) -> torch.Tensor:
+        idx = device.index if device.index is not None else torch.cuda.current_device()
+        b = self._buf.get(idx)
+        if b is None or b.numel() < nbytes:
+            self._buf.pop(idx, None)
+            b = torch.empty(max(nbytes, 256), dtype=torch.uint8, device=torch.device("cuda", idx))
+            self._buf[idx] = b
+        return b
+
+
+_default_ws = Workspace()
+
+
+def workspace_bytes(n_r: int, n_s: int, config: GshConfig | None = None) -> int:
+    lib = load()
+    nb = lib.gsh_workspace_bytes(n_r, n_s, ctypes.byref(config) if config is not None else None)
+    if nb == 0:
+        raise ValueError("invalid gsh_config")
+    return int(nb)
+
+
+def join(r_keys: torch.Tensor, r_payloads: torch.Tensor, s_keys: torch.Tensor, s_payloads: torch.Tensor,
+         mode: str = "count", out: torch.Tensor | None = None, out_capacity: int | None = None,
+         config: GshConfig | None = None, stream=None, workspace: torch.Tensor | None = None) -> JoinResult:
+    """GSH equi-join of device-resident R and S (gsh_join, include/gsh.h).
+
+    mode: "count" (count + checksum) or "materialize" (also (payload_R, payload_S) pairs into
+    `out`, an int32 CUDA tensor of shape (capacity, 2), or a fresh one of out_capacity rows).
+    """
+    lib = load()
+    rk, rp = _check_dev(r_keys, "r_keys"), _check_dev(r_payloads, "r_payloads")
+    sk, sp = _check_dev(s_keys, "s_keys"), _check_dev(s_payloads, "s_payloads")
+    dev = rk.device
+    R, S = _rel(rk, rp, "R"), _rel(sk, sp, "S")
+    mat = mode == "materialize"
+    if mode not in ("count", "materialize"):
+        raise ValueError("mode must be 'count' or 'materialize'")
+    outp = None
+    if mat:
+        if out is None:
+            if out_capacity is None:
+                raise ValueError("materialize needs out or out_capacity")
+            out = torch.empty((int(out_capacity), 2), dtype=torch.int32, device=dev)
+        if not out.is_cuda or out.dtype not in (torch.int32, torch.uint32) or out.dim() != 2 or out.shape[1] != 2:
+            raise ValueError("out must be a CUDA int32 tensor of shape (capacity, 2)")
+        if not out.is_contiguous():
+            raise ValueError("out must be contiguous")
+        outp = GshOutput(out.data_ptr() if out.numel() else None, out.shape[0])
+    nb = workspace_bytes(R.n, S.n, config)
+    ws = workspace if workspace is not None else _default_ws.get(nb, dev)
+    if ws.numel() < nb:
+        raise ValueError(f"workspace too small ({ws.numel()} < {nb} bytes)")
+    res = GshResult()
+    with torch.cuda.device(dev):
+        st = lib.gsh_join(ctypes.byref(R), ctypes.byref(S), _lib.GSH_OUT_MATERIALIZE if mat else _lib.GSH_OUT_COUNT,
+                          ctypes.byref(outp) if outp is not None else None, ws.data_ptr(), ws.numel(),
+                          ctypes.byref(config) if config is not None else None, _stream_handle(stream),
+                          ctypes.byref(res))
+    check(st, "gsh_join")
+    d = res.as_dict()
+    return JoinResult(count=int(res.count), checksum=int(res.checksum), written=int(res.written),
+                      overflow=bool(res.overflow), pairs=(out[: res.written] if mat else None), stats=d)
+
+
+def join_host(r_keys, r_payloads, s_keys, s_payloads, mode: str = "count", out=None, out_capacity=None,
+              config: GshConfig | None = None, device=None, stream=None,
+              workspace: torch.Tensor | None = None) -> JoinResult:
+    """End-to-end join of HOST tensors (gsh_join_host): H2D copy, join, D2H of the pairs.
+
+    Inputs are CPU int32 tensors (pin_memory() for full bandwidth).  The device workspace is
+    allocated on `device` (default: current CUDA device)."""
+    lib = load()
+    t = [r_keys, r_payloads, s_keys, s_payloads]
+    for x in t:
+        if not isinstance(x, torch.Tensor) or x.is_cuda or x.dtype not in (torch.int32, torch.uint32):
+            raise TypeError("join_host takes CPU int32 tensors")
+    rk, rp, sk, sp = (x.contiguous() for x in t)
+    R, S = _rel(rk, rp, "R"), _rel(sk, sp, "S")
+    mat = mode == "materialize"
+    dev = torch.device("cuda", torch.cuda.current_device()) if device is None else torch.device(device)
+    outp = None
+    cap = 0
+    if mat:
+        if out is None:
+            out = torch.empty((int(out_capacity), 2), dtype=torch.int32, pin_memory=True)
+        cap = out.shape[0]
+        outp = GshOutput(out.data_ptr() if out.numel() else None, cap)
+    nb = lib.gsh_host_workspace_bytes(R.n, S.n, 1 if mat else 0, cap,
+                                      ctypes.byref(config) if config is not None else None)
+    if nb == 0:
+        raise ValueError("invalid gsh_config")
+    ws = workspace if workspace is not None else _default_ws.get(int(nb), dev)
+    res = GshResult()
+    with torch.cuda.device(dev):
+        st = lib.gsh_join_host(ctypes.byref(R), ctypes.byref(S), 1 if mat else 0,
+                               ctypes.byref(outp) if outp is not None else None, ws.data_ptr(), ws.numel(),
+                               ctypes.byref(config) if config is not None else None, _stream_handle(stream),
+                               ctypes.byref(res))
+    check(st, "gsh_join_host")
+    return JoinResult(count=int(res.count), checksum=int(res.checksum), written=int(res.written),
+                      overflow=bool(res.overflow), pairs=(out[: res.written] if mat else None), stats=res.as_dict())
+
+
+# ------------------------------------------------------------------ step entry points
+def hash_keys(keys: torch.Tensor, stream=None) -> torch.Tensor:
+    """fmix32 of every key (gsh_hash_keys) -> int32 CUDA tensor."""
+    lib = load()
+    k = _check_dev(keys, "keys")
+    out = torch.empty_like(k, dtype=torch.int32)
+    with torch.cuda.device(k.device):
+        check(lib.gsh_hash_keys(k.data_ptr() if k.numel() else None, out.data_ptr() if k.numel() else None,
+                                k.numel(), _stream_handle(stream)), "gsh_hash_keys")
+    return out
+
+
+def radix_histogram(keys: torch.Tensor, hi_bits: int, nbits: int, stream=None) -> torch.Tensor:
+    """Histogram of radix digits of fmix32(key) (gsh_radix_histogram) -> int64 tensor."""
+    lib = load()
+    k = _check_dev(keys, "keys")
+    hist = torch.zeros(1 << nbits, dtype=torch.int64, device=k.device)
+    with torch.cuda.device(k.device):
+        check(lib.gsh_radix_histogram(k.data_ptr() if k.numel() else None, k.numel(), hi_bits, nbits,
+                                      hist.data_ptr(), None, 0, _stream_handle(stream)), "gsh_radix_histogram")
+    return hist
+
+
+def partition(r_keys, r_payloads, s_keys, s_payloads, config: GshConfig | None = None, stream=None):
+    """Partition phase only (gsh_partition).  Returns (part_r, part_s, off_r, off_s, (b1, b2)) where
+    part_* are (n, 2) int32 tensors of (h, payload) grouped by partition and off_* int64 starts."""
+    lib = load()
+    rk, rp = _check_dev(r_keys, "r_keys"), _check_dev(r_payloads, "r_payloads")
+    sk, sp = _check_dev(s_keys, "s_keys"), _check_dev(s_payloads, "s_payloads")
+    dev = rk.device
+    R, S = _rel(rk, rp, "R"), _rel(sk, sp, "S")
+    nb = workspace_bytes(R.n, S.n, config)
+    ws = _default_ws.get(nb, dev)
+    # F is only known inside the library: size the offsets for the maximum fanout
+    off_r = torch.zeros((1 << 16) + 1, dtype=torch.int64, device=dev)
+    off_s = torch.zeros((1 << 16) + 1, dtype=torch.int64, device=dev)
+    part_r = torch.empty((max(R.n, 1), 2), dtype=torch.int32, device=dev)
+    part_s = torch.empty((max(S.n, 1), 2), dtype=torch.int32, device=dev)
+    bits = (ctypes.c_uint32 * 2)()
+    with torch.cuda.device(dev):
+        check(lib.gsh_partition(ctypes.byref(R), ctypes.byref(S), ctypes.byref(config) if config is not None else None,
+                                ws.data_ptr(), ws.numel(), _stream_handle(stream), part_r.data_ptr(),
+                                part_s.data_ptr(), off_r.data_ptr(), off_s.data_ptr(), bits), "gsh_partition")
+    F = 1 << (bits[0] + bits[1])
+    return part_r[: R.n], part_s[: S.n], off_r[: F + 1], off_s[: F + 1], (int(bits[0]), int(bits[1]))
+
+
+def detect(r_keys, r_payloads, s_keys, s_payloads, config: GshConfig | None = None, stream=None, cap: int = 1 << 22):
+    """Partition + skew detection (gsh_detect).  Returns (h, cnt_r, cnt_s, stats) as int64 CPU
+    tensors sorted by h (h = fmix32 of each skewed key, as u32 values)."""
+    lib = load()
+    rk, rp = _check_dev(r_keys, "r_keys"), _check_dev(r_payloads, "r_payloads")
+    sk, sp = _check_dev(s_keys, "s_keys"), _check_dev(s_payloads, "s_payloads")
+    dev = rk.device
+    R, S = _rel(rk, rp, "R"), _rel(sk, sp, "S")
+    nb = workspace_bytes(R.n, S.n, config)
+    ws = _default_ws.get(nb, dev)
+    hk = (ctypes.c_uint32 * cap)()
+    cr = (ctypes.c_uint32 * cap)()
+    cs = (ctypes.c_uint32 * cap)()
+    n = ctypes.c_uint64(0)
+    res = GshResult()
+    with torch.cuda.device(dev):
+        check(lib.gsh_detect(ctypes.byref(R), ctypes.byref(S), ctypes.byref(config) if config is not None else None,
+                             ws.data_ptr(), ws.numel(), _stream_handle(stream), hk, cr, cs, cap, ctypes.byref(n),
+                             ctypes.byref(res)), "gsh_detect")
+    m = int(n.value)
+    h = torch.tensor(list(hk[:m]), dtype=torch.int64)
+    a = torch.tensor(list(cr[:m]), dtype=torch.int64)
+    b = torch.tensor(list(cs[:m]), dtype=torch.int64)
+    order = torch.argsort(h)
+    return h[order], a[order], b[order], res.as_dict()

@@ -1,0 +1,93 @@
+"""CPU checks of the C-ABI boundary: libgsh.so loads, exports every symbol include/gsh.h
+declares, reports argument errors before any launch, and the Python binding mirrors the
+header's structs.  No compute calls (no GPU here)."""
+import ctypes
+import re
+
+import pytest
+
+import paper_conf_icde_caic24_b200 as gsh
+from paper_conf_icde_caic24_b200 import _lib
+
+
+def header_functions():
+    txt = open(_lib.HEADER_PATH).read()
+    return sorted(set(re.findall(r"GSH_API\s+[\w\s\*]*?\b(gsh_\w+)\s*\(", txt)))
+
+
+def test_library_exports_every_header_symbol():
+    lib = _lib.load()
+    names = header_functions()
+    assert len(names) >= 15
+    for n in names:
+        assert hasattr(lib, n), n
+    assert sorted(_lib.EXPORTED) == names
+
+
+def test_compiled_for_sm100a():
+    lib = _lib.load()
+    assert lib.gsh_compiled_arch() == 100
+    assert lib.gsh_version() >= 1
+    import subprocess
+    out = subprocess.run(["/usr/local/cuda/bin/cuobjdump", "--list-elf", _lib.LIB_PATH], capture_output=True,
+                         text=True).stdout
+    assert "sm_100a" in out
+
+
+def test_status_strings_and_struct_sizes():
+    lib = _lib.load()
+    assert lib.gsh_status_string(0) == b"GSH_OK"
+    assert lib.gsh_status_string(1) == b"GSH_ERR_INVALID"
+    # gsh_result: 8 u64 + 10 u32 + 8 floats
+    assert ctypes.sizeof(_lib.GshResult) == 8 * 8 + 10 * 4 + 8 * 4
+    assert ctypes.sizeof(_lib.GshConfig) == 9 * 4
+    cfg = _lib.default_config()
+    assert list(cfg.pass_bits) == [-1, -1] and cfg.capacity == 0
+
+
+def test_workspace_sizing_is_monotone_and_rejects_bad_config():
+    a = gsh.workspace_bytes(1 << 10, 1 << 10)
+    b = gsh.workspace_bytes(1 << 20, 1 << 20)
+    assert 0 < a < b
+    # ~20 B per tuple plus tables
+    assert b >= 20 * (2 << 20)
+    with pytest.raises(ValueError):
+        gsh.workspace_bytes(100, 100, gsh.make_config(pass_bits=(9, 1)))
+    with pytest.raises(ValueError):
+        gsh.workspace_bytes(100, 100, gsh.make_config(force_all_heavy=True, force_all_normal=True))
+
+
+def test_argument_errors_before_any_launch():
+    lib = _lib.load()
+    res = _lib.GshResult()
+    R = _lib.GshRelation(None, None, 10)  # NULL with n > 0
+    S = _lib.GshRelation(None, None, 0)
+    st = lib.gsh_join(ctypes.byref(R), ctypes.byref(S), 0, None, None, 0, None, None, ctypes.byref(res))
+    assert st == _lib.GSH_ERR_INVALID
+    assert b"invalid relation" in lib.gsh_last_error()
+    R = _lib.GshRelation(None, None, 0)
+    st = lib.gsh_join(ctypes.byref(R), ctypes.byref(S), 1, None, None, 0, None, None, ctypes.byref(res))
+    assert st == _lib.GSH_ERR_INVALID  # MATERIALIZE without output
+    st = lib.gsh_join(ctypes.byref(R), ctypes.byref(S), 0, None, None, 0, None, None, None)
+    assert st == _lib.GSH_ERR_INVALID  # res NULL
+    R = _lib.GshRelation(None, None, 1 << 32)
+    st = lib.gsh_join(ctypes.byref(R), ctypes.byref(S), 0, None, None, 0, None, None, ctypes.byref(res))
+    assert st == _lib.GSH_ERR_INVALID  # n >= 2^32
+
+
+def test_product_path_refuses_cpu_tensors():
+    import torch
+    k = torch.zeros(4, dtype=torch.int32)
+    with pytest.raises(ValueError, match="CUDA"):
+        gsh.join(k, k, k, k)
+
+
+def test_product_does_not_import_oracle():
+    import os
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    pkg = os.path.join(root, "paper_conf_icde_caic24_b200")
+    for dirpath, _, files in os.walk(pkg):
+        for f in files:
+            if f.endswith((".py", ".cu", ".cuh", ".h", ".cpp")):
+                txt = open(os.path.join(dirpath, f)).read()
+                assert "import oracle" not in txt and "from oracle" not in txt and "join_oracle" not in txt, f

@@ -1,0 +1,197 @@
+"""GPU parity of the CUDA path (through the C-ABI) against the CPU oracle, element by element,
+on seeded synthetic inputs shaped like the paper's workloads (DESIGN.md §4 recipe).
+
+Integer-only method -> the bar is bit-exact: count, checksum, and the sorted pair multiset."""
+import numpy as np
+import pytest
+import torch
+
+import datagen
+import oracle
+import paper_conf_icde_caic24_b200 as gsh
+
+pytestmark = pytest.mark.gpu
+DEV = "cuda"
+
+
+def _np(t):
+    return t.cpu().numpy().view(np.uint32)
+
+
+def _dev(*ts):
+    return [t.to(DEV) for t in ts]
+
+
+def _oracle(rk, rp, sk, sp, pairs=False):
+    if pairs:
+        return oracle.join_sorted_pairs(_np(rk), _np(rp), _np(sk), _np(sp))
+    n, c, _ = oracle.join(_np(rk), _np(rp), _np(sk), _np(sp))
+    return n, c, None
+
+
+def _sorted_pairs(p):
+    a = p.cpu().numpy().view(np.uint32).reshape(-1, 2)
+    return a[np.lexsort((a[:, 1], a[:, 0]))]
+
+
+# ---------------------------------------------------------------------- single phases
+@pytest.mark.parametrize("n", [0, 1, 5, 1000, (1 << 16) + 3])
+def test_hash_keys_bit_exact(n):
+    k = torch.randint(-(1 << 31), (1 << 31) - 1, (n,), dtype=torch.int32)
+    if n >= 2:
+        k[0] = 0
+        k[1] = -1
+    got = gsh.hash_keys(k.to(DEV))
+    assert np.array_equal(_np(got), oracle.fmix32(_np(k)))
+
+
+@pytest.mark.parametrize("hi,nb", [(0, 0), (0, 8), (0, 16), (3, 5), (8, 8)])
+def test_radix_histogram_bit_exact(hi, nb):
+    rk, _, _, _ = datagen.zipf_pair(200_003, 10, 1.0, seed=1)
+    got = gsh.radix_histogram(rk.to(DEV), hi, nb).cpu().numpy()
+    assert np.array_equal(got, oracle.radix_histogram(_np(rk), hi, nb))
+
+
+@pytest.mark.parametrize("kind,n,theta", [("uniform", 100_000, 0.0), ("zipf", 300_001, 1.0),
+                                          ("zipf", 1 << 18, 1.5), ("pkfk", 50_000, 0.0), ("uniform", 5, 0.0)])
+def test_partition_phase(kind, n, theta):
+    """Histogram + scan + pass-1 + pass-2 scatter: offsets equal the oracle's
+    exclusive scan of the digit histogram, every partition holds exactly the tuples whose
+    digits select it, and each side is a permutation of (fmix32(key), payload)."""
+    rk, rp, sk, sp = datagen.make_workload(kind, n, theta, seed=7)
+    part_r, part_s, off_r, off_s, (b1, b2) = gsh.partition(*_dev(rk, rp, sk, sp))
+    B = b1 + b2
+    for keys, pays, part, off in ((rk, rp, part_r, off_r), (sk, sp, part_s, off_s)):
+        hist = oracle.radix_histogram(_np(keys), 0, B)
+        assert np.array_equal(off.cpu().numpy(), np.concatenate([[0], np.cumsum(hist)]))
+        pr = part.cpu().numpy().view(np.uint32)
+        digits = (pr[:, 0].astype(np.int64) >> (32 - B)) if B else np.zeros(pr.shape[0], np.int64)
+        expect_digit = np.repeat(np.arange(1 << B), hist)
+        assert np.array_equal(digits, expect_digit)
+        # permutation of (h, payload)
+        h = oracle.fmix32(_np(keys))
+        a = np.stack([h, _np(pays)], 1)
+        assert np.array_equal(a[np.lexsort((a[:, 1], a[:, 0]))], pr[np.lexsort((pr[:, 1], pr[:, 0]))])
+
+
+@pytest.mark.parametrize("theta,n,cfg", [(1.0, 1 << 18, {}), (1.5, 1 << 17, {}), (0.75, 1 << 18, {}),
+                                         (1.0, 1 << 16, {"capacity": 512, "heavy_threshold": 16}),
+                                         (0.5, 1 << 17, {"capacity": 256, "heavy_threshold": 4})])
+def test_skew_detection_matches_exact_rule(theta, n, cfg):
+    """Skewed keys (PAPER.md L107/L112 with exact counts, DESIGN.md §3 R3/R4) equal the oracle's
+    heavy_rule on the same partition bits, capacity and threshold."""
+    rk, rp, sk, sp = datagen.zipf_pair(n, n, theta, seed=3)
+    config = gsh.make_config(**cfg)
+    h, cr, cs, st = gsh.detect(*_dev(rk, rp, sk, sp), config=config)
+    B = st["pass_bits"][0] + st["pass_bits"][1]
+    oh, ocr, ocs = oracle.heavy_rule(_np(rk), _np(sk), B, st["capacity"], st["heavy_threshold"])
+    assert st["detect_overflow"] == 0
+    assert np.array_equal(h.numpy().astype(np.uint32), oh)
+    assert np.array_equal(cr.numpy(), ocr) and np.array_equal(cs.numpy(), ocs)
+    if theta >= 1.0:
+        assert len(oh) > 0
+
+
+# ------------------------------------------------------------------- full join parity
+LADDER = [
+    ("uniform", 0, 0.0), ("uniform", 1, 0.0), ("uniform", 7, 0.0), ("uniform", 1000, 0.0),
+    ("pkfk", (1 << 14) + 3, 0.0), ("uniform", 1 << 18, 0.0), ("pkfk", 1 << 20, 0.0),
+    ("zipf", (1 << 14) + 3, 0.5), ("zipf", 1 << 18, 0.5), ("zipf", 1 << 18, 0.75),
+    ("zipf", (1 << 14) + 3, 1.0), ("zipf", 1 << 18, 1.0), ("zipf", 1 << 20, 1.0),
+    ("zipf", 1 << 16, 1.25), ("zipf", 1 << 17, 1.5), ("graph", 1 << 18, 0.909),
+]
+
+
+@pytest.mark.parametrize("kind,n,theta", LADDER)
+def test_join_count_checksum_ladder(kind, n, theta):
+    rk, rp, sk, sp = datagen.make_workload(kind, n, theta, seed=11)
+    r = gsh.join(*_dev(rk, rp, sk, sp))
+    on, oc, _ = _oracle(rk, rp, sk, sp)
+    assert (r.count, r.checksum) == (on, oc)
+    assert r.stats["count"] == r.count
+
+
+@pytest.mark.parametrize("kind,n,theta", [("uniform", 1000, 0.0), ("pkfk", 100_003, 0.0), ("zipf", 40_000, 1.0),
+                                          ("zipf", 1 << 16, 0.75), ("zipf", 20_000, 1.5), ("graph", 1 << 16, 0.909)])
+def test_join_materialize_pairs_exact(kind, n, theta):
+    rk, rp, sk, sp = datagen.make_workload(kind, n, theta, seed=5)
+    on, oc, op = _oracle(rk, rp, sk, sp, pairs=True)
+    r = gsh.join(*_dev(rk, rp, sk, sp), mode="materialize", out_capacity=on + 10)
+    assert (r.count, r.checksum, r.written, r.overflow) == (on, oc, on, False)
+    assert np.array_equal(_sorted_pairs(r.pairs), op)
+
+
+def test_join_materialize_overflow_subset():
+    rk, rp, sk, sp = datagen.zipf_pair(30_000, 30_000, 1.0, seed=8)
+    on, oc, op = _oracle(rk, rp, sk, sp, pairs=True)
+    cap = on // 3
+    r = gsh.join(*_dev(rk, rp, sk, sp), mode="materialize", out_capacity=cap)
+    assert (r.count, r.checksum, r.written, r.overflow) == (on, oc, cap, True)
+    got = _sorted_pairs(r.pairs)
+    # every written pair is a real match (payload = rid): R.key[a] == S.key[b]; no duplicates beyond M
+    rkn, skn = _np(rk), _np(sk)
+    assert np.all(rkn[got[:, 0]] == skn[got[:, 1]])
+    assert np.unique(got, axis=0).shape[0] == got.shape[0]  # payloads are rids -> pairs unique
+
+
+@pytest.mark.parametrize("cfg", [{"force_all_normal": True}, {"force_all_heavy": True}, {"capacity": 256},
+                                 {"capacity": 8192}, {"pass_bits": (3, 2)}, {"pass_bits": (8, 8)},
+                                 {"pass_bits": (0, 0)}, {"heavy_threshold": 2}, {"capacity": 128, "heavy_threshold": 1000000}])
+def test_join_invariant_under_config(cfg):
+    """Skew classification, fanout and capacity change performance only:
+    results must be identical under every configuration (metamorphic pin P4)."""
+    rk, rp, sk, sp = datagen.zipf_pair(1 << 15, 1 << 15, 1.0, seed=21)
+    on, oc, _ = _oracle(rk, rp, sk, sp)
+    r = gsh.join(*_dev(rk, rp, sk, sp), config=gsh.make_config(**cfg))
+    assert (r.count, r.checksum) == (on, oc)
+
+
+def test_join_edge_cases():
+    # all keys equal (one giant skewed key), extremes of the key range, no matches, empty sides
+    z = torch.zeros
+    cases = []
+    cases.append((z(3000, dtype=torch.int32), torch.arange(3000, dtype=torch.int32),
+                  z(2000, dtype=torch.int32), torch.arange(2000, dtype=torch.int32)))
+    cases.append((torch.full((5000,), -1, dtype=torch.int32), torch.arange(5000, dtype=torch.int32),
+                  torch.tensor([-1, 0, 5, -1], dtype=torch.int32), torch.arange(4, dtype=torch.int32)))
+    cases.append((torch.arange(0, 10000, 2, dtype=torch.int32), torch.arange(5000, dtype=torch.int32),
+                  torch.arange(1, 10001, 2, dtype=torch.int32), torch.arange(5000, dtype=torch.int32)))
+    cases.append((z(0, dtype=torch.int32), z(0, dtype=torch.int32), torch.arange(10, dtype=torch.int32),
+                  torch.arange(10, dtype=torch.int32)))
+    cases.append((torch.arange(10, dtype=torch.int32), torch.arange(10, dtype=torch.int32), z(0, dtype=torch.int32),
+                  z(0, dtype=torch.int32)))
+    # duplicate payloads (pair multiset)
+    cases.append((torch.tensor([1, 1, 2, 2], dtype=torch.int32), torch.tensor([7, 7, 7, 7], dtype=torch.int32),
+                  torch.tensor([1, 2, 2], dtype=torch.int32), torch.tensor([9, 9, 9], dtype=torch.int32)))
+    for rk, rp, sk, sp in cases:
+        on, oc, op = _oracle(rk, rp, sk, sp, pairs=True)
+        r = gsh.join(*_dev(rk, rp, sk, sp), mode="materialize", out_capacity=on + 1)
+        assert (r.count, r.checksum, r.written) == (on, oc, on)
+        assert np.array_equal(_sorted_pairs(r.pairs), op)
+
+
+def test_join_unaligned_views():
+    """Input pointers need not be 16-byte aligned (sliced views)."""
+    rk, rp, sk, sp = datagen.zipf_pair(50_001, 50_003, 1.0, seed=2)
+    rk, rp, sk, sp = _dev(rk, rp, sk, sp)
+    r = gsh.join(rk[1:], rp[1:], sk[3:], sp[3:])
+    on, oc, _ = _oracle(rk[1:], rp[1:], sk[3:], sp[3:])
+    assert (r.count, r.checksum) == (on, oc)
+
+
+def test_join_host_end_to_end():
+    rk, rp, sk, sp = datagen.zipf_pair(70_000, 60_000, 1.0, seed=4)
+    on, oc, op = _oracle(rk, rp, sk, sp, pairs=True)
+    r = gsh.join_host(rk.pin_memory(), rp.pin_memory(), sk.pin_memory(), sp.pin_memory(), mode="materialize",
+                      out_capacity=on)
+    assert (r.count, r.checksum, r.written) == (on, oc, on)
+    assert np.array_equal(_sorted_pairs(r.pairs), op)
+    r2 = gsh.join_host(rk, rp, sk, sp)
+    assert (r2.count, r2.checksum) == (on, oc)
+
+
+def test_repeatable_bit_exact():
+    rk, rp, sk, sp = _dev(*datagen.zipf_pair(1 << 18, 1 << 18, 1.25, seed=9))
+    a = gsh.join(rk, rp, sk, sp)
+    b = gsh.join(rk, rp, sk, sp)
+    assert (a.count, a.checksum) == (b.count, b.checksum)
