@@ -420,21 +420,30 @@ int launch_scatter(const Plan& p, int pass, const uint32_t* const keys[2], const
 }
 
 // ----------------------------------------------- standalone radix histogram (ABI) --
+// Shared-memory bins for up to 2^14 digits; wider histograms aggregate per warp and go
+// straight to global atomics.
 __global__ void k_radix_hist(const uint32_t* __restrict__ keys, uint64_t n, uint32_t shift, uint32_t mask,
-                             unsigned long long* __restrict__ hist) {
+                             unsigned long long* __restrict__ hist, int use_smem) {
     extern __shared__ uint32_t hs[];
-    for (uint32_t i = threadIdx.x; i <= mask; i += blockDim.x) hs[i] = 0;
-    __syncthreads();
+    if (use_smem) {
+        for (uint32_t i = threadIdx.x; i <= mask; i += blockDim.x) hs[i] = 0;
+        __syncthreads();
+    }
     for (uint64_t i = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; i - threadIdx.x < n;
          i += uint64_t(gridDim.x) * blockDim.x) {
         bool v = i < n;
         uint32_t bin = v ? ((hash32(keys[i]) >> shift) & mask) : (0x80000000u | lane_id());
         uint32_t peers = __match_any_sync(kFull, bin);
-        if (v && (peers & lanemask_lt()) == 0) atomicAdd(&hs[bin], (uint32_t)__popc(peers));
+        if (v && (peers & lanemask_lt()) == 0) {
+            if (use_smem) atomicAdd(&hs[bin], (uint32_t)__popc(peers));
+            else atomicAdd(&hist[bin], (unsigned long long)__popc(peers));
+        }
     }
-    __syncthreads();
-    for (uint32_t i = threadIdx.x; i <= mask; i += blockDim.x)
-        if (hs[i]) atomicAdd(&hist[i], (unsigned long long)hs[i]);
+    if (use_smem) {
+        __syncthreads();
+        for (uint32_t i = threadIdx.x; i <= mask; i += blockDim.x)
+            if (hs[i]) atomicAdd(&hist[i], (unsigned long long)hs[i]);
+    }
 }
 
 int launch_radix_hist(const uint32_t* keys, uint64_t n, uint32_t hi_bits, uint32_t nbits, uint64_t* hist,
@@ -442,14 +451,16 @@ int launch_radix_hist(const uint32_t* keys, uint64_t n, uint32_t hi_bits, uint32
     if (n == 0) return 0;
     const uint32_t F = 1u << nbits;
     const uint32_t shift = nbits ? (32 - hi_bits - nbits) : 0;
-    size_t smem = size_t(F) * 4;
+    const int use_smem = nbits <= 14;
+    size_t smem = use_smem ? size_t(F) * 4 : 0;
     static bool attr_set = false;
     if (!attr_set) {
-        cudaFuncSetAttribute(k_radix_hist, cudaFuncAttributeMaxDynamicSharedMemorySize, 256 * 1024 - 1024);
+        cudaFuncSetAttribute(k_radix_hist, cudaFuncAttributeMaxDynamicSharedMemorySize, 64 * 1024);
         attr_set = true;
     }
     unsigned grid = (unsigned)umin64((n + 1023) / 1024, 148);
-    k_radix_hist<<<grid, 1024, smem, s>>>(keys, n, shift, F - 1, reinterpret_cast<unsigned long long*>(hist));
+    k_radix_hist<<<grid, 1024, smem, s>>>(keys, n, shift, F - 1, reinterpret_cast<unsigned long long*>(hist),
+                                          use_smem);
     return 1;
 }
 
