@@ -118,7 +118,7 @@ bool plan_build(Plan& p, uint64_t nR, uint64_t nS, const gsh_config* cfg_in, voi
     p.force_heavy = cfg.force_all_heavy;
     p.timing = cfg.timing;
     if (p.force_normal && p.force_heavy) return false;
-    p.hist_grid = num_sms / 2 > 0 ? num_sms / 2 : 1;
+    p.hist_grid = num_sms >= 2 ? (num_sms & ~1) : 2;  // even: CTA pairs share a chunk when F > 2^15
     for (int s = 0; s < 2; ++s)
         p.max_tiles[s] = (p.n[s] + kScatterTile - 1) / kScatterTile + (1u << p.b1) + 1;
     uint64_t t = next_pow2_u64(2 * (nR + nS));
@@ -146,8 +146,7 @@ bool plan_build(Plan& p, uint64_t nR, uint64_t nS, const gsh_config* cfg_in, voi
     p.bufB[1] = b ? b + nR : nullptr;
     p.heavy_pay[0] = hp;
     p.heavy_pay[1] = hp ? hp + nR : nullptr;
-    p.hist_partial = c.take<uint16_t>(size_t(2) * p.hist_grid * (F < 2 ? 2 : F));
-    p.hist_spill = c.take<uint32_t>(2 * F);
+    p.hist_partial = c.take<uint32_t>(size_t(2) * p.hist_grid * F);
     p.cnt = c.take<uint32_t>(2 * F);
     p.start = c.take<uint64_t>(2 * (F + 1));
     p.status = c.take<uint64_t>(size_t(p.max_tiles[0] + p.max_tiles[1]) * 256);

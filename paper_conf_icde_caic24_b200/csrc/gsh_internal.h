@@ -15,7 +15,7 @@ constexpr int kScatterTile = kScatterBlock * kScatterIpt;  // 8192 tuples per ti
 constexpr int kMaxDigitBits = 8;                // radix bits per pass (256 buckets)
 constexpr int kMaxPartBits = 16;                // b1 + b2 <= 16 (65536 partitions)
 constexpr int kHistBlock = 1024;
-constexpr int kNmBlock = 256;                   // NM-join CTA
+constexpr int kNmBlock = 512;                   // NM-join CTA
 constexpr uint32_t kMaxCapacity = 8192;         // largest NM build table (tuples)
 constexpr uint32_t kNmSlice = 8192;             // S tuples probed per NM work item
 constexpr int kSkewBlock = 256;                 // skewed-key join CTA
@@ -60,7 +60,7 @@ struct Plan {
     uint32_t F = 1;                 // 1 << (b1 + b2)
     int force_normal = 0, force_heavy = 0, timing = 0;
     int num_sms = 148;
-    int hist_grid = 74;             // CTAs per side in the histogram kernel
+    int hist_grid = 148;            // histogram CTAs (1 per SM)
     uint64_t max_tiles[2] = {0, 0}; // look-back status rows per side
     uint32_t gt_cap_alloc = 0;      // detection table slots allocated
     uint64_t h_max = 0;             // skewed-key list capacity
@@ -70,8 +70,7 @@ struct Plan {
     uint2* bufA[2] = {nullptr, nullptr};      // pass-1 output, later normal remainders
     uint2* bufB[2] = {nullptr, nullptr};      // final partitions
     uint32_t* heavy_pay[2] = {nullptr, nullptr};  // skewed-key payload arrays
-    uint16_t* hist_partial = nullptr;         // [2][hist_grid][F]
-    uint32_t* hist_spill = nullptr;           // [2][F]
+    uint32_t* hist_partial = nullptr;         // [2][chunks][F]
     uint32_t* cnt = nullptr;                  // [2][F]
     uint64_t* start = nullptr;                // [2][F + 1]
     uint64_t* status = nullptr;               // [2][max_tiles][256]

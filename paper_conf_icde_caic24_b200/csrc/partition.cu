@@ -34,120 +34,92 @@ int launch_hash(const uint32_t* keys, uint32_t* out, uint64_t n, cudaStream_t s)
 }
 
 // ------------------------------------------------------------------- a1: histogram --
-// Packed u16 counters: word w holds bins 2w (low half) and 2w+1 (high half).  When a half
-// crosses 0x8000 the crossing warp moves 0x8000 to the global spill counter, so a half never
-// exceeds 0x8000 + (adds in flight) < 0x10000 and never carries into its neighbour.
-__device__ __forceinline__ void hist_add(uint32_t* cnt, uint32_t bin, uint32_t c, uint32_t* spill) {
-    const uint32_t sh = (bin & 1u) * 16u;
-    uint32_t old = atomicAdd(&cnt[bin >> 1], c << sh);
-    uint32_t ov = (old >> sh) & 0xffffu;
-    if (ov < 0x8000u && ov + c >= 0x8000u) {
-        atomicSub(&cnt[bin >> 1], 0x8000u << sh);
-        atomicAdd(&spill[bin], 0x8000u);
-    }
+// One read of the keys yields the (d1, d2) histogram of BOTH partition passes.  Counters are
+// u32 in shared memory incremented with atomicAdd(.., 1), which sm_100a executes as a
+// warp-aggregated ATOMS.POPC.INC: lanes hitting the same bin are combined in hardware, so
+// skewed digits cost no more than spread ones (measured: ~1 SM-cycle per warp-op either way,
+// while __match_any_sync costs ~64 -- scripts/microbench_warp_ops.cu, profiles/).
+// 2^16 u32 bins do not fit one CTA (256 KB), so for F > 2^15 two CTAs read the same chunk
+// (the second read is served by L2) and each counts one half of the bins in 128 KB.
+__device__ __forceinline__ void hist_one(uint32_t* cnt, uint32_t key, uint32_t shift, uint32_t mask, uint32_t lo,
+                                         uint32_t nb) {
+    const uint32_t bin = ((hash32(key) >> shift) & mask) - lo;
+    if (bin < nb) atomicAdd(&cnt[bin], 1u);
 }
 
-__device__ __forceinline__ void hist_key(uint32_t* cnt, uint32_t* spill, uint32_t key, bool valid,
-                                         uint32_t shift, uint32_t mask) {
-    uint32_t bin = valid ? ((hash32(key) >> shift) & mask) : (0x80000000u | lane_id());
-    uint32_t peers = __match_any_sync(kFull, bin);
-    if (valid && (peers & lanemask_lt()) == 0) hist_add(cnt, bin, __popc(peers), spill);
-}
-
-// grid = (hist_grid, 2): blockIdx.y = side.  Writes this CTA's counters to partial[side][bx][*].
 __global__ void __launch_bounds__(kHistBlock, 1)
 k_hist2d(const uint32_t* __restrict__ k0, uint64_t n0, const uint32_t* __restrict__ k1, uint64_t n1,
-         uint32_t shift, uint32_t nbits, uint16_t* __restrict__ partial, uint32_t* __restrict__ spill) {
+         uint32_t shift, uint32_t nbits, uint32_t* __restrict__ partial) {
     extern __shared__ uint32_t cnt[];
-    const int side = blockIdx.y;
-    const uint32_t* keys = side ? k1 : k0;
-    const uint64_t n = side ? n1 : n0;
     const uint32_t F = 1u << nbits;
-    const uint32_t words = (F + 1) / 2;
     const uint32_t mask = F - 1;
-    uint32_t* sp = spill + size_t(side) * F;
-    for (uint32_t w = threadIdx.x; w < words; w += blockDim.x) cnt[w] = 0;
-    __syncthreads();
-
-    // contiguous chunk per CTA, in units of 4 keys (uint4) when the pointer is 16 B aligned
-    const uint64_t G = gridDim.x;
-    const bool vec = ((reinterpret_cast<uintptr_t>(keys) & 15u) == 0);
-    if (vec) {
-        const uint64_t nv = n / 4;
-        const uint64_t b = nv * blockIdx.x / G, e = nv * (blockIdx.x + 1) / G;
+    const bool split = F > (1u << 15);
+    const uint32_t nchunks = split ? gridDim.x / 2 : gridDim.x;
+    const uint32_t chunk = split ? blockIdx.x >> 1 : blockIdx.x;
+    const uint32_t nb = split ? F / 2 : F;
+    const uint32_t lo = split ? (blockIdx.x & 1) * nb : 0;
+    for (int side = 0; side < 2; ++side) {
+        const uint32_t* keys = side ? k1 : k0;
+        const uint64_t n = side ? n1 : n0;
+        for (uint32_t w = threadIdx.x; w < nb; w += blockDim.x) cnt[w] = 0;
+        __syncthreads();
+        const bool vec = ((reinterpret_cast<uintptr_t>(keys) & 15u) == 0);
+        const uint64_t nv = vec ? n / 4 : 0;
+        const uint64_t b = nv * chunk / nchunks, e = nv * (chunk + 1) / nchunks;
         const uint4* kv = reinterpret_cast<const uint4*>(keys);
-        // block-uniform loop bounds (full-warp __match_any_sync below)
-        uint64_t base = b;
-        for (; base + 2ull * blockDim.x <= e; base += 2ull * blockDim.x) {
-            const uint64_t i = base + threadIdx.x;
-            uint4 a = ld_stream_u4(kv + i);
-            uint4 c = ld_stream_u4(kv + i + blockDim.x);
-            hist_key(cnt, sp, a.x, true, shift, mask);
-            hist_key(cnt, sp, a.y, true, shift, mask);
-            hist_key(cnt, sp, a.z, true, shift, mask);
-            hist_key(cnt, sp, a.w, true, shift, mask);
-            hist_key(cnt, sp, c.x, true, shift, mask);
-            hist_key(cnt, sp, c.y, true, shift, mask);
-            hist_key(cnt, sp, c.z, true, shift, mask);
-            hist_key(cnt, sp, c.w, true, shift, mask);
-        }
-        for (; base < e; base += blockDim.x) {
-            const uint64_t i = base + threadIdx.x;
-            bool v = i < e;
-            uint4 a = v ? ld_stream_u4(kv + i) : make_uint4(0, 0, 0, 0);
-            hist_key(cnt, sp, a.x, v, shift, mask);
-            hist_key(cnt, sp, a.y, v, shift, mask);
-            hist_key(cnt, sp, a.z, v, shift, mask);
-            hist_key(cnt, sp, a.w, v, shift, mask);
-        }
-        // scalar tail (n % 4 keys) handled by the last CTA
-        if (blockIdx.x == G - 1) {
-            uint64_t t0 = nv * 4;
-            uint64_t j = t0 + threadIdx.x;
-            if (j - threadIdx.x < n) {
-                bool v = j < n;
-                hist_key(cnt, sp, v ? keys[j] : 0u, v, shift, mask);
+        uint64_t i = b + threadIdx.x;
+        for (; i + 3ull * blockDim.x < e; i += 4ull * blockDim.x) {
+            uint4 v[4];
+#pragma unroll
+            for (int u = 0; u < 4; ++u) v[u] = ld_stream_u4(kv + i + u * blockDim.x);
+#pragma unroll
+            for (int u = 0; u < 4; ++u) {
+                hist_one(cnt, v[u].x, shift, mask, lo, nb);
+                hist_one(cnt, v[u].y, shift, mask, lo, nb);
+                hist_one(cnt, v[u].z, shift, mask, lo, nb);
+                hist_one(cnt, v[u].w, shift, mask, lo, nb);
             }
         }
-    } else {
-        const uint64_t b = n * blockIdx.x / G, e = n * (blockIdx.x + 1) / G;
-        for (uint64_t i = b + threadIdx.x; i - threadIdx.x < e; i += blockDim.x) {
-            bool v = i < e;
-            hist_key(cnt, sp, v ? keys[i] : 0u, v, shift, mask);
+        for (; i < e; i += blockDim.x) {
+            uint4 v = ld_stream_u4(kv + i);
+            hist_one(cnt, v.x, shift, mask, lo, nb);
+            hist_one(cnt, v.y, shift, mask, lo, nb);
+            hist_one(cnt, v.z, shift, mask, lo, nb);
+            hist_one(cnt, v.w, shift, mask, lo, nb);
         }
+        // scalar remainder (all keys when unaligned, else the n % 4 tail) -> chunk 0
+        if (chunk == 0)
+            for (uint64_t j = nv * 4 + threadIdx.x; j < n; j += blockDim.x) hist_one(cnt, keys[j], shift, mask, lo, nb);
+        __syncthreads();
+        uint32_t* row = partial + (size_t(side) * nchunks + chunk) * F + lo;
+        for (uint32_t w = threadIdx.x; w < nb; w += blockDim.x) row[w] = cnt[w];
+        __syncthreads();
     }
-    __syncthreads();
-    uint32_t* row = reinterpret_cast<uint32_t*>(partial + (size_t(side) * G + blockIdx.x) * (F < 2 ? 2 : F));
-    for (uint32_t w = threadIdx.x; w < words; w += blockDim.x) row[w] = cnt[w];
 }
 
 int launch_hist(const Plan& p, const uint32_t* k0, const uint32_t* k1, cudaStream_t s) {
     const uint32_t nbits = p.b1 + p.b2;
-    const uint32_t shift = (32 - p.route_bits - nbits) & 31;
+    const uint32_t shift = nbits ? (32 - p.route_bits - nbits) : 0;
     const uint32_t F = 1u << nbits;
-    size_t smem = size_t((F + 1) / 2) * 4;
+    const size_t smem = size_t(F > (1u << 15) ? F / 2 : F) * 4;
     static bool attr_set = false;
     if (!attr_set) {
         cudaFuncSetAttribute(k_hist2d, cudaFuncAttributeMaxDynamicSharedMemorySize, 128 * 1024);
         attr_set = true;
     }
-    cudaMemsetAsync(p.hist_spill, 0, size_t(2) * F * sizeof(uint32_t), s);
-    dim3 grid(p.hist_grid, 2);
-    k_hist2d<<<grid, kHistBlock, smem, s>>>(k0, p.n[0], k1, p.n[1], nbits ? shift : 0, nbits, p.hist_partial,
-                                            p.hist_spill);
+    k_hist2d<<<p.hist_grid, kHistBlock, smem, s>>>(k0, p.n[0], k1, p.n[1], shift, nbits, p.hist_partial);
     return 1;
 }
 
 // --------------------------------------------------- a2: reduce partials + prefix scan --
-// cnt[side][bin] = sum_g partial[side][g][bin] + spill[side][bin]
-__global__ void k_hist_reduce(const uint16_t* __restrict__ partial, const uint32_t* __restrict__ spill,
-                              uint32_t* __restrict__ cnt, uint32_t F, uint32_t G) {
-    const uint32_t rowlen = F < 2 ? 2 : F;
+// cnt[side][bin] = sum over chunks of partial[side][chunk][bin]
+__global__ void k_hist_reduce(const uint32_t* __restrict__ partial, uint32_t* __restrict__ cnt, uint32_t F,
+                              uint32_t nchunks) {
     for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < 2 * F; i += gridDim.x * blockDim.x) {
         const uint32_t side = i / F, bin = i % F;
-        const uint16_t* base = partial + size_t(side) * G * rowlen + bin;
-        uint32_t s = spill[i];
-        for (uint32_t g = 0; g < G; ++g) s += base[size_t(g) * rowlen];
+        const uint32_t* base = partial + size_t(side) * nchunks * F + bin;
+        uint32_t s = 0;
+        for (uint32_t g = 0; g < nchunks; ++g) s += base[size_t(g) * F];
         cnt[i] = s;
     }
 }
@@ -186,8 +158,9 @@ __global__ void __launch_bounds__(1024) k_part_scan(const uint32_t* __restrict__
 
 int launch_hist_reduce_scan(const Plan& p, cudaStream_t s) {
     const uint32_t F = p.F;
+    const uint32_t nchunks = F > (1u << 15) ? p.hist_grid / 2 : p.hist_grid;
     unsigned grid = (2 * F + 255) / 256;
-    k_hist_reduce<<<grid, 256, 0, s>>>(p.hist_partial, p.hist_spill, p.cnt, F, p.hist_grid);
+    k_hist_reduce<<<grid, 256, 0, s>>>(p.hist_partial, p.cnt, F, nchunks);
     k_part_scan<<<2, 1024, 0, s>>>(p.cnt, p.start, F);
     return 2;
 }
@@ -211,7 +184,7 @@ constexpr uint64_t kValMask = (1ull << 62) - 1;
 constexpr int kWarps = kScatterBlock / 32;
 
 struct ScatterSmem {
-    uint16_t wc[kWarps][256];           // per-warp bucket counters -> per-warp exclusive prefix
+    uint32_t bcnt[256];                 // per-tile bucket counters (ATOMS.POPC.INC ranks)
     uint32_t local_start[256];          // bucket start inside the tile
     unsigned long long gbase[256];      // global index of tile element 0 of bucket b
     uint32_t segtiles[2][257];          // tile prefix over segments per side
@@ -224,7 +197,7 @@ __global__ void __launch_bounds__(kScatterBlock, 2) k_scatter(ScatterArgs a) {
     ScatterSmem& S = *reinterpret_cast<ScatterSmem*>(smem_raw);
     uint2* stage = reinterpret_cast<uint2*>(smem_raw + ((sizeof(ScatterSmem) + 15) & ~size_t(15)));
 
-    const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const uint32_t tid = threadIdx.x;
     const bool p1 = (a.pass == 1);
     const uint32_t bits = p1 ? a.b1 : a.b2;
     const uint32_t nb = 1u << bits;
@@ -279,10 +252,11 @@ __global__ void __launch_bounds__(kScatterBlock, 2) k_scatter(ScatterArgs a) {
         const uint64_t begin = seg_b + uint64_t(tile_in_seg) * kScatterTile;
         const uint32_t len = (uint32_t)umin64(kScatterTile, seg_e - begin);
 
-        for (uint32_t i = tid; i < kWarps * 256 / 2; i += kScatterBlock) reinterpret_cast<uint32_t*>(S.wc)[i] = 0;
+        if (tid < 256) S.bcnt[tid] = 0;
         __syncthreads();
 
-        // load + rank within warp
+        // load + rank: atomicAdd(.., 1) on a per-tile bucket counter returns a unique rank
+        // (hardware-aggregated for lanes of the same bucket, so skew does not serialise)
         uint32_t hv[kScatterIpt], pv[kScatterIpt], rk[kScatterIpt / 2];  // ranks packed 2 x u16
         if (p1) {
             const uint32_t* kp = a.keys[side] + begin;
@@ -306,33 +280,17 @@ __global__ void __launch_bounds__(kScatterBlock, 2) k_scatter(ScatterArgs a) {
                 pv[j] = e.y;
             }
         }
-        const uint32_t lt_mask = lanemask_lt();
 #pragma unroll
         for (int j = 0; j < kScatterIpt; ++j) {
             uint32_t i = j * kScatterBlock + tid;
-            bool v = i < len;
-            uint32_t d = (hv[j] >> dshift) & dmask;
-            uint32_t key = v ? d : (0x100u | lane);
-            uint32_t peers = __match_any_sync(kFull, key);
-            uint32_t before = v ? S.wc[warp][d] : 0u;
-            __syncwarp();
-            uint32_t r = before + __popc(peers & lt_mask);
-            if (v && (peers & lt_mask) == 0) S.wc[warp][d] = (uint16_t)(before + __popc(peers));
-            __syncwarp();
+            uint32_t r = 0;
+            if (i < len) r = atomicAdd(&S.bcnt[(hv[j] >> dshift) & dmask], 1u);
             if (j & 1) rk[j >> 1] |= r << 16; else rk[j >> 1] = r;
         }
         __syncthreads();
 
-        // per-bucket: exclusive prefix over warps, bucket totals, block scan -> local starts
-        uint32_t tot = 0;
-        if (tid < nb) {
-#pragma unroll
-            for (int w = 0; w < kWarps; ++w) {
-                uint32_t c = S.wc[w][tid];
-                S.wc[w][tid] = (uint16_t)tot;
-                tot += c;
-            }
-        }
+        // bucket totals -> block scan -> local starts
+        const uint32_t tot = (tid < nb) ? S.bcnt[tid] : 0u;
         uint32_t all;
         uint32_t lstart = block_excl_scan_u32<kScatterBlock>(tid < nb ? tot : 0u, &all, S.scan_tmp);
         if (tid < nb) S.local_start[tid] = lstart;
@@ -366,7 +324,7 @@ __global__ void __launch_bounds__(kScatterBlock, 2) k_scatter(ScatterArgs a) {
             if (i < len) {
                 uint32_t d = (hv[j] >> dshift) & dmask;
                 uint32_t r = (j & 1) ? (rk[j >> 1] >> 16) : (rk[j >> 1] & 0xffffu);
-                uint32_t pos = S.local_start[d] + S.wc[warp][d] + r;
+                uint32_t pos = S.local_start[d] + r;
                 stage[pos] = make_uint2(hv[j], pv[j]);
             }
         }
