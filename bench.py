@@ -190,7 +190,7 @@ def main():
         dist.init_process_group("nccl", device_id=dev)
     rk, rp, sk, sp = make_data(kind, n, theta, args.seed, dev, rank)
     torch.cuda.synchronize()
-    cfg = gsh.make_config(timing=True)
+    cfg = gsh.make_config(timing=True, **json.loads(os.environ.get("GSH_BENCH_CFG", "{}")))  # experiments only
     if world > 1:
         from paper_conf_icde_caic24_b200 import sharded
 

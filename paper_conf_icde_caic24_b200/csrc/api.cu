@@ -14,6 +14,8 @@
 #include "gsh_internal.h"
 
 namespace gsh {
+// defined in join.cu
+uint32_t nm_table_slots(uint32_t rl);
 // defined in skew.cu
 size_t cand_table_slots(uint64_t nR, uint64_t nS);
 int launch_candidates(const uint32_t* kr, uint64_t nR, const uint32_t* ks, uint64_t nS, uint32_t hi_bits,
@@ -120,7 +122,7 @@ bool plan_build(Plan& p, uint64_t nR, uint64_t nS, const gsh_config* cfg_in, voi
     if (p.force_normal && p.force_heavy) return false;
     p.hist_grid = num_sms >= 2 ? (num_sms & ~1) : 2;  // even: CTA pairs share a chunk when F > 2^15
     for (int s = 0; s < 2; ++s)
-        p.max_tiles[s] = (p.n[s] + kScatterTile - 1) / kScatterTile + (1u << p.b1) + 1;
+        p.max_chunks[s] = (p.n[s] + kScatterChunk - 1) / kScatterChunk + (1u << p.b1) + 1;
     uint64_t t = next_pow2_u64(2 * (nR + nS));
     if (t < 1024) t = 1024;
     if (t > (1ull << 25)) t = 1ull << 25;
@@ -137,19 +139,21 @@ bool plan_build(Plan& p, uint64_t nR, uint64_t nS, const gsh_config* cfg_in, voi
     Carver c{reinterpret_cast<unsigned char*>(ws)};
     const size_t F = p.F;
     p.st = c.take<DevState>(1);
-    uint2* a = c.take<uint2>(nR + nS + 1);
-    uint2* b = c.take<uint2>(nR + nS + 1);
+    // side S starts 256-byte aligned so sector alignment of partition writes is index alignment
+    const uint64_t nRp = (nR + 31) & ~uint64_t(31);
+    uint2* a = c.take<uint2>(nRp + nS + 32);
+    uint2* b = c.take<uint2>(nRp + nS + 32);
     uint32_t* hp = c.take<uint32_t>(nR + nS + 1);
     p.bufA[0] = a;
-    p.bufA[1] = a ? a + nR : nullptr;
+    p.bufA[1] = a ? a + nRp : nullptr;
     p.bufB[0] = b;
-    p.bufB[1] = b ? b + nR : nullptr;
+    p.bufB[1] = b ? b + nRp : nullptr;
     p.heavy_pay[0] = hp;
     p.heavy_pay[1] = hp ? hp + nR : nullptr;
     p.hist_partial = c.take<uint32_t>(size_t(2) * p.hist_grid * F);
     p.cnt = c.take<uint32_t>(2 * F);
     p.start = c.take<uint64_t>(2 * (F + 1));
-    p.status = c.take<uint64_t>(size_t(p.max_tiles[0] + p.max_tiles[1]) * 256);
+    p.status = c.take<uint64_t>(size_t(p.max_chunks[0] + p.max_chunks[1]) * 256);
     p.gt_key = c.take<unsigned long long>(p.gt_cap_alloc);
     p.gt_cnt = c.take<uint32_t>(size_t(2) * p.gt_cap_alloc);
     p.gt_hid = c.take<uint32_t>(p.gt_cap_alloc);
@@ -288,6 +292,7 @@ gsh_status gsh_join(const gsh_relation* R, const gsh_relation* S, gsh_out_mode m
     if (ce != cudaSuccess) return cuda_fail(ce, "classify sync");
     const uint32_t n_large = hs.n_large;
     uint32_t n_heavy = 0;
+    p.nm_slots = nm_table_slots(hs.max_rlen < p.C ? (hs.max_rlen ? hs.max_rlen : 1) : p.C);
     int e4 = e3, e5 = e3;
     if (n_large > 0) {
         uint64_t gcap = next_pow2_u64(2 * (hs.large_tuples[0] + hs.large_tuples[1]));

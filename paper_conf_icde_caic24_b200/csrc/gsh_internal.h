@@ -10,12 +10,13 @@ namespace gsh {
 
 // ----------------------------------------------------------------- fixed shapes --
 constexpr int kScatterBlock = 512;              // threads per partition-scatter CTA
-constexpr int kScatterIpt = 16;                 // tuples per thread per tile
-constexpr int kScatterTile = kScatterBlock * kScatterIpt;  // 8192 tuples per tile
+constexpr int kScatterIpt = 8;                  // tuples per thread per tile
+constexpr int kScatterTile = kScatterBlock * kScatterIpt;  // 4096 tuples per tile
+constexpr int kScatterChunk = 4 * kScatterTile;  // 16384 tuples per look-back unit
 constexpr int kMaxDigitBits = 8;                // radix bits per pass (256 buckets)
 constexpr int kMaxPartBits = 16;                // b1 + b2 <= 16 (65536 partitions)
 constexpr int kHistBlock = 1024;
-constexpr int kNmBlock = 512;                   // NM-join CTA
+constexpr int kNmBlock = 256;                   // NM-join CTA
 constexpr uint32_t kMaxCapacity = 8192;         // largest NM build table (tuples)
 constexpr uint32_t kNmSlice = 8192;             // S tuples probed per NM work item
 constexpr int kSkewBlock = 256;                 // skewed-key join CTA
@@ -36,7 +37,7 @@ struct DevState {
     unsigned long long skew_tiles;                 // total dense tiles
     unsigned long long nm_items;                   // NM work items
     unsigned long long skew_claim;                 // tile claim counter
-    unsigned int n_large, n_heavy, detect_overflow, nm_claim;
+    unsigned int n_large, n_heavy, detect_overflow, max_rlen;  // max_rlen: largest |R_p| with |S_p| > 0
     unsigned int claim[8];                         // per-kernel work claim counters
 };
 
@@ -57,11 +58,12 @@ struct Plan {
     uint64_t n[2] = {0, 0};
     uint32_t b1 = 0, b2 = 0, route_bits = 0;
     uint32_t C = 4096, Th = 1024;
+    uint32_t nm_slots = 0;          // NM build-table slots (set after classification; 0 = from C)
     uint32_t F = 1;                 // 1 << (b1 + b2)
     int force_normal = 0, force_heavy = 0, timing = 0;
     int num_sms = 148;
     int hist_grid = 148;            // histogram CTAs (1 per SM)
-    uint64_t max_tiles[2] = {0, 0}; // look-back status rows per side
+    uint64_t max_chunks[2] = {0, 0};  // look-back status rows per side
     uint32_t gt_cap_alloc = 0;      // detection table slots allocated
     uint64_t h_max = 0;             // skewed-key list capacity
     uint64_t scan_scratch_elems = 0;
@@ -73,7 +75,7 @@ struct Plan {
     uint32_t* hist_partial = nullptr;         // [2][chunks][F]
     uint32_t* cnt = nullptr;                  // [2][F]
     uint64_t* start = nullptr;                // [2][F + 1]
-    uint64_t* status = nullptr;               // [2][max_tiles][256]
+    uint64_t* status = nullptr;               // [2][max_chunks][256]
     DevState* st = nullptr;
     unsigned long long* gt_key = nullptr;     // [gt_cap_alloc]  (1 << 32 | h), 0 = empty
     uint32_t* gt_cnt = nullptr;               // [2][gt_cap_alloc]

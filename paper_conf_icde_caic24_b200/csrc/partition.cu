@@ -12,6 +12,7 @@
 //                        runs (coalesced 8 B AoS stores).  16 B/tuple per pass.  Pass-2 tiles
 //                        never cross a pass-1 partition; the look-back chain restarts there.
 #include <cstdio>
+#include <cstdlib>
 
 #include "gsh_device.cuh"
 #include "gsh_internal.h"
@@ -172,30 +173,148 @@ struct ScatterArgs {
     const uint2* in[2];        // pass 2 input (AoS)
     uint2* out[2];
     const uint64_t* start[2];  // partition start offsets [F + 1] per side
-    uint64_t* status[2];       // look-back words [tiles][256] per side
+    void* status[2];           // look-back words [tiles][256] per side (u32 or u64)
     uint64_t n[2];
     uint32_t pass, b1, b2, route_bits;
     unsigned int* tile_ctr;
+    uint32_t dbg;              // experiment switches (GSH_SCATTER_DEBUG), 0 in production
 };
 
-constexpr uint64_t kFlagAgg = 1ull << 62;
-constexpr uint64_t kFlagInc = 2ull << 62;
-constexpr uint64_t kValMask = (1ull << 62) - 1;
-constexpr int kWarps = kScatterBlock / 32;
+// Look-back status word: 2 flag bits (0 = not ready, 1 = tile aggregate, 2 = inclusive prefix)
+// above the value.  u32 words (30-bit values) unless a side holds >= 2^30 tuples.
+template <typename W>
+struct LB {
+    static constexpr int kShift = sizeof(W) * 8 - 2;
+    static constexpr W kAgg = W(1) << kShift;
+    static constexpr W kInc = W(2) << kShift;
+    static constexpr W kMask = (W(1) << kShift) - 1;
+    __device__ static W load(const W* p) {
+        if constexpr (sizeof(W) == 8) {
+            return ld_volatile_u64(reinterpret_cast<const uint64_t*>(p));
+        } else {
+            W v;
+            asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+            return v;
+        }
+    }
+    __device__ static void store(W* p, W v) {
+        if constexpr (sizeof(W) == 8) {
+            st_volatile_u64(reinterpret_cast<uint64_t*>(p), v);
+        } else {
+            asm volatile("st.relaxed.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+        }
+    }
+};
 
+// Work unit = a CHUNK of kScatterChunk tuples inside one segment (the whole side in pass 1, one
+// pass-1 partition in pass 2).  A CTA first COUNTS its chunk (TMA tiles, bucket counts only),
+// publishes the chunk's bucket aggregates and looks back over preceding chunks (decoupled
+// look-back at chunk granularity: 8x fewer, 8x longer-lived units than tiles, so the look-back
+// depth stays short), then re-streams the chunk (from L2) and SCATTERS it tile by tile with
+// per-CTA running bucket offsets -- no cross-CTA dependency per tile.
 struct ScatterSmem {
-    uint32_t bcnt[256];                 // per-tile bucket counters (ATOMS.POPC.INC ranks)
+    uint32_t cnt[256];                  // chunk bucket counts (count phase)
+    uint32_t tcnt[256];                 // tile bucket counters -> ranks (scatter phase)
     uint32_t local_start[256];          // bucket start inside the tile
-    unsigned long long gbase[256];      // global index of tile element 0 of bucket b
-    uint32_t segtiles[2][257];          // tile prefix over segments per side
-    uint32_t scan_tmp[kWarps + 1];
+    unsigned long long run[256];        // next global index of bucket b for this chunk
+    unsigned long long wpos[256];       // first index of bucket b not yet written to memory
+    unsigned long long gbase[256];      // global index of stage position 0 of bucket b
+    unsigned long long endw[256];       // write-out limit of bucket b for the current tile
+    uint2 cbuf[256][4];                 // carry: < 4 tuples (one 32 B sector) per bucket
+    uint32_t carry[256];                // tuples in cbuf[b]
+    uint32_t segch[2][257];             // chunk prefix over segments per side
+    uint32_t scan_tmp[33];
     uint32_t claim;
+    uint64_t mbar[2];                   // TMA completion, one per tile buffer
 };
 
-__global__ void __launch_bounds__(kScatterBlock, 2) k_scatter(ScatterArgs a) {
-    extern __shared__ __align__(16) unsigned char smem_raw[];
+struct ChunkInfo {
+    int side;
+    uint32_t lc, seg, first_chunk, chunk_in_seg, len;
+    uint64_t begin;
+};
+
+__device__ __forceinline__ ChunkInfo chunk_info(const ScatterArgs& a, const ScatterSmem& S, uint32_t t,
+                                                uint32_t chunks0, uint32_t nseg, bool p1) {
+    ChunkInfo ci;
+    ci.side = (t >= chunks0) ? 1 : 0;
+    ci.lc = t - (ci.side ? chunks0 : 0);
+    uint32_t lo = 0, hi = nseg;  // largest s with segch[s] <= lc
+    while (hi - lo > 1) {
+        const uint32_t mid = (lo + hi) >> 1;
+        if (S.segch[ci.side][mid] <= ci.lc) lo = mid; else hi = mid;
+    }
+    ci.seg = lo;
+    ci.first_chunk = S.segch[ci.side][lo];
+    ci.chunk_in_seg = ci.lc - ci.first_chunk;
+    const uint64_t seg_b = p1 ? 0 : a.start[ci.side][uint64_t(lo) << a.b2];
+    const uint64_t seg_e = p1 ? a.n[ci.side] : a.start[ci.side][uint64_t(lo + 1) << a.b2];
+    ci.begin = seg_b + uint64_t(ci.chunk_in_seg) * kScatterChunk;
+    ci.len = (uint32_t)umin64(kScatterChunk, seg_e - ci.begin);
+    return ci;
+}
+
+// Which tile elements arrive by TMA bulk copy: [head, head + nbulk); element i lives at shared
+// index i + shift (keeps the bulk destination 16-byte aligned).  The rest (an unaligned first
+// AoS tuple, a tail that is not a multiple of 16 bytes, or everything when the SoA inputs are
+// not 16-byte aligned) is loaded by its owning thread with ordinary loads.
+struct LoadPlan {
+    uint32_t head, nbulk, shift;
+};
+
+__device__ __forceinline__ LoadPlan load_plan(const ScatterArgs& a, int side, uint64_t begin, uint32_t len, bool p1) {
+    LoadPlan lp;
+    if (p1) {
+        const uintptr_t k = reinterpret_cast<uintptr_t>(a.keys[side] + begin);
+        const uintptr_t q = reinterpret_cast<uintptr_t>(a.pays[side] + begin);
+        const bool al = ((k | q) & 15u) == 0;
+        lp.head = al ? 0 : len;
+        lp.nbulk = al ? (len & ~3u) : 0;
+        lp.shift = 0;
+    } else {
+        const uintptr_t ip = reinterpret_cast<uintptr_t>(a.in[side] + begin);
+        lp.head = umin32((ip & 15u) ? 1u : 0u, len);
+        lp.nbulk = (len - lp.head) & ~1u;
+        lp.shift = lp.head ? 1u : 0u;
+    }
+    return lp;
+}
+
+// Thread 0: arm `bar` and issue the bulk copies of tile [begin, begin + len).  keys_only: pass-1
+// count phase (payloads not needed).  kdst/pdst: pass-1 key / payload buffers; adst: pass-2 AoS.
+__device__ __forceinline__ void tile_issue(const ScatterArgs& a, int side, uint64_t begin, uint32_t len, bool p1,
+                                           bool keys_only, uint32_t* kdst, uint32_t* pdst, uint2* adst,
+                                           uint64_t* bar) {
+    // count phase (keys_only): the chunk is re-read by the scatter phase -> keep it in L2;
+    // scatter phase: last use -> evict first.  (Pass-1 payloads are only read once.)
+    const uint64_t pol = keys_only ? policy_evict_last() : policy_evict_first();
+    const LoadPlan lp = load_plan(a, side, begin, len, p1);
+    if (p1) {
+        const uint32_t bytes = lp.nbulk * 4;
+        mbar_arrive_expect_tx(bar, keys_only ? bytes : 2 * bytes);
+        if (bytes) {
+            bulk_g2s_hint(kdst, a.keys[side] + begin, bytes, bar, pol);
+            if (!keys_only) bulk_g2s_hint(pdst, a.pays[side] + begin, bytes, bar, pol);
+        }
+    } else {
+        const uint32_t bytes = lp.nbulk * 8;
+        mbar_arrive_expect_tx(bar, bytes);
+        if (bytes) bulk_g2s_hint(adst + lp.head + lp.shift, a.in[side] + begin + lp.head, bytes, bar, pol);
+    }
+}
+
+template <typename W, int BLOCK, int IPT>
+__global__ void __launch_bounds__(BLOCK) k_scatter(ScatterArgs a) {
+    constexpr int TILE = BLOCK * IPT;
+    extern __shared__ __align__(128) unsigned char smem_raw[];
     ScatterSmem& S = *reinterpret_cast<ScatterSmem*>(smem_raw);
-    uint2* stage = reinterpret_cast<uint2*>(smem_raw + ((sizeof(ScatterSmem) + 15) & ~size_t(15)));
+    unsigned char* buf0 = smem_raw + ((sizeof(ScatterSmem) + 127) & ~size_t(127));
+    unsigned char* buf1 = buf0 + (size_t(TILE) + 4) * 8;
+    // scatter phase: buf0 = input tile ("orig"), buf1 = bucket-ordered staging
+    uint32_t* ok = reinterpret_cast<uint32_t*>(buf0);   // pass 1: keys -> h
+    uint32_t* op = ok + TILE + 4;               // pass 1: payloads
+    uint2* o2 = reinterpret_cast<uint2*>(buf0);         // pass 2: (h, payload)
+    uint2* stage = reinterpret_cast<uint2*>(buf1);
 
     const uint32_t tid = threadIdx.x;
     const bool p1 = (a.pass == 1);
@@ -206,148 +325,257 @@ __global__ void __launch_bounds__(kScatterBlock, 2) k_scatter(ScatterArgs a) {
     const uint32_t nseg = p1 ? 1 : (1u << a.b1);
     const uint32_t lowbits = p1 ? a.b2 : 0;
 
-    // tile prefix over segments (pass 1: one segment per side)
+    // chunk prefix over segments (pass 1: one segment per side)
     for (int side = 0; side < 2; ++side) {
         if (p1) {
             if (tid == 0) {
-                S.segtiles[side][0] = 0;
-                S.segtiles[side][1] = (uint32_t)((a.n[side] + kScatterTile - 1) / kScatterTile);
+                S.segch[side][0] = 0;
+                S.segch[side][1] = (uint32_t)((a.n[side] + kScatterChunk - 1) / kScatterChunk);
             }
         } else {
-            // thread t < nseg computes tiles of segment t; serial scan by warp 0 below
             uint32_t v = 0;
             if (tid < nseg) {
-                uint64_t b = a.start[side][uint64_t(tid) << a.b2];
-                uint64_t e = a.start[side][uint64_t(tid + 1) << a.b2];
-                v = (uint32_t)((e - b + kScatterTile - 1) / kScatterTile);
+                const uint64_t b = a.start[side][uint64_t(tid) << a.b2];
+                const uint64_t e = a.start[side][uint64_t(tid + 1) << a.b2];
+                v = (uint32_t)((e - b + kScatterChunk - 1) / kScatterChunk);
             }
             uint32_t tot;
-            uint32_t ex = block_excl_scan_u32<kScatterBlock>(v, &tot, S.scan_tmp);
-            if (tid < nseg) S.segtiles[side][tid] = ex;
-            if (tid == 0) S.segtiles[side][nseg] = tot;
+            const uint32_t ex = block_excl_scan_u32<BLOCK>(v, &tot, S.scan_tmp);
+            if (tid < nseg) S.segch[side][tid] = ex;
+            if (tid == 0) S.segch[side][nseg] = tot;
         }
     }
+    if (tid == 0) {
+        mbar_init(&S.mbar[0], 1);
+        mbar_init(&S.mbar[1], 1);
+        S.claim = atomicAdd(a.tile_ctr, 1u);
+    }
+    if (tid < 256) S.tcnt[tid] = 0;
     __syncthreads();
-    const uint32_t tiles0 = S.segtiles[0][nseg];
-    const uint32_t total = tiles0 + S.segtiles[1][nseg];
+    const uint32_t chunks0 = S.segch[0][nseg];
+    const uint32_t total = chunks0 + S.segch[1][nseg];
+    uint32_t par0 = 0, par1 = 0;
 
-    for (;;) {
-        if (tid == 0) S.claim = atomicAdd(a.tile_ctr, 1u);
-        __syncthreads();
-        const uint32_t t = S.claim;
-        if (t >= total) break;
-        const int side = (t >= tiles0) ? 1 : 0;
-        const uint32_t lt = t - (side ? tiles0 : 0);
-        // segment: largest s with segtiles[s] <= lt
-        uint32_t lo = 0, hi = nseg;
-        while (hi - lo > 1) {
-            uint32_t mid = (lo + hi) >> 1;
-            if (S.segtiles[side][mid] <= lt) lo = mid; else hi = mid;
+    for (uint32_t t = S.claim; t < total;) {
+        const ChunkInfo ci = chunk_info(a, S, t, chunks0, nseg, p1);
+        const uint32_t ntile = (ci.len + TILE - 1) / TILE;
+
+        // ------------------------------------------------ count phase (double-buffered TMA)
+        if (tid < 256) S.cnt[tid] = 0;
+        const uint32_t ncount = (a.dbg & 1) ? 0 : ntile;
+        if (tid == 0 && ncount) {
+            fence_proxy_async_smem();
+            tile_issue(a, ci.side, ci.begin, umin32(TILE, ci.len), p1, true, ok, nullptr, o2, &S.mbar[0]);
         }
-        const uint32_t seg = lo;
-        const uint32_t first_tile = S.segtiles[side][seg];
-        const uint32_t tile_in_seg = lt - first_tile;
-        const uint64_t seg_b = p1 ? 0 : a.start[side][uint64_t(seg) << a.b2];
-        const uint64_t seg_e = p1 ? a.n[side] : a.start[side][uint64_t(seg + 1) << a.b2];
-        const uint64_t begin = seg_b + uint64_t(tile_in_seg) * kScatterTile;
-        const uint32_t len = (uint32_t)umin64(kScatterTile, seg_e - begin);
-
-        if (tid < 256) S.bcnt[tid] = 0;
         __syncthreads();
-
-        // load + rank: atomicAdd(.., 1) on a per-tile bucket counter returns a unique rank
-        // (hardware-aggregated for lanes of the same bucket, so skew does not serialise)
-        uint32_t hv[kScatterIpt], pv[kScatterIpt], rk[kScatterIpt / 2];  // ranks packed 2 x u16
-        if (p1) {
-            const uint32_t* kp = a.keys[side] + begin;
-            const uint32_t* pp = a.pays[side] + begin;
-#pragma unroll
-            for (int j = 0; j < kScatterIpt; ++j) {
-                uint32_t i = j * kScatterBlock + tid;
-                bool v = i < len;
-                hv[j] = v ? ld_stream_u32(kp + i) : 0u;
-                pv[j] = v ? ld_stream_u32(pp + i) : 0u;
+        for (uint32_t q = 0; q < ncount; ++q) {
+            const uint32_t qb = q * TILE;
+            const uint32_t ql = umin32(TILE, ci.len - qb);
+            unsigned char* cur = (q & 1) ? buf1 : buf0;
+            if (tid == 0 && q + 1 < ncount) {
+                unsigned char* nxt = (q & 1) ? buf0 : buf1;
+                tile_issue(a, ci.side, ci.begin + qb + TILE, umin32(TILE, ci.len - qb - TILE), p1,
+                           true, reinterpret_cast<uint32_t*>(nxt), nullptr, reinterpret_cast<uint2*>(nxt),
+                           &S.mbar[(q + 1) & 1]);
             }
-#pragma unroll
-            for (int j = 0; j < kScatterIpt; ++j) hv[j] = hash32(hv[j]);
-        } else {
-            const uint2* ip = a.in[side] + begin;
-#pragma unroll
-            for (int j = 0; j < kScatterIpt; ++j) {
-                uint32_t i = j * kScatterBlock + tid;
-                uint2 e = (i < len) ? ld_stream_u2(ip + i) : make_uint2(0, 0);
-                hv[j] = e.x;
-                pv[j] = e.y;
-            }
-        }
-#pragma unroll
-        for (int j = 0; j < kScatterIpt; ++j) {
-            uint32_t i = j * kScatterBlock + tid;
-            uint32_t r = 0;
-            if (i < len) r = atomicAdd(&S.bcnt[(hv[j] >> dshift) & dmask], 1u);
-            if (j & 1) rk[j >> 1] |= r << 16; else rk[j >> 1] = r;
-        }
-        __syncthreads();
-
-        // bucket totals -> block scan -> local starts
-        const uint32_t tot = (tid < nb) ? S.bcnt[tid] : 0u;
-        uint32_t all;
-        uint32_t lstart = block_excl_scan_u32<kScatterBlock>(tid < nb ? tot : 0u, &all, S.scan_tmp);
-        if (tid < nb) S.local_start[tid] = lstart;
-
-        // decoupled look-back, one bucket per thread
-        if (tid < nb) {
-            uint64_t* st = a.status[side];
-            const size_t me = size_t(lt) * 256 + tid;
-            uint64_t excl = 0;
-            if (tile_in_seg == 0) {
-                st_volatile_u64(st + me, kFlagInc | tot);
-            } else {
-                st_volatile_u64(st + me, kFlagAgg | tot);
-                for (int64_t j = int64_t(lt) - 1; j >= int64_t(first_tile); --j) {
-                    uint64_t v;
-                    do { v = ld_volatile_u64(st + size_t(j) * 256 + tid); } while ((v >> 62) == 0);
-                    excl += v & kValMask;
-                    if ((v >> 62) == 2) break;
-                }
-                st_volatile_u64(st + me, kFlagInc | (excl + tot));
-            }
-            const uint64_t pidx = ((uint64_t(seg) << bits) | tid) << lowbits;
-            S.gbase[tid] = a.start[side][pidx] + excl - lstart;
-        }
-        __syncthreads();
-
-        // scatter into shared staging in bucket order
-#pragma unroll
-        for (int j = 0; j < kScatterIpt; ++j) {
-            uint32_t i = j * kScatterBlock + tid;
-            if (i < len) {
-                uint32_t d = (hv[j] >> dshift) & dmask;
-                uint32_t r = (j & 1) ? (rk[j >> 1] >> 16) : (rk[j >> 1] & 0xffffu);
-                uint32_t pos = S.local_start[d] + r;
-                stage[pos] = make_uint2(hv[j], pv[j]);
-            }
-        }
-        __syncthreads();
-
-        // write out contiguous bucket runs
-        uint2* out = a.out[side];
+            if (q & 1) { mbar_wait(&S.mbar[1], par1); par1 ^= 1; } else { mbar_wait(&S.mbar[0], par0); par0 ^= 1; }
+            const LoadPlan lp = load_plan(a, ci.side, ci.begin + qb, ql, p1);
 #pragma unroll 4
-        for (uint32_t i = tid; i < len; i += kScatterBlock) {
-            uint2 e = stage[i];
-            uint32_t d = (e.x >> dshift) & dmask;
-            out[S.gbase[d] + i] = e;
+            for (uint32_t i = tid; i < ql; i += BLOCK) {
+                const bool bulk = (i - lp.head) < lp.nbulk;
+                uint32_t h;
+                if (p1) h = hash32(bulk ? reinterpret_cast<const uint32_t*>(cur)[i] : a.keys[ci.side][ci.begin + qb + i]);
+                else h = bulk ? reinterpret_cast<const uint2*>(cur)[i + lp.shift].x : a.in[ci.side][ci.begin + qb + i].x;
+                atomicAdd(&S.cnt[(h >> dshift) & dmask], 1u);
+            }
+            fence_proxy_async_smem();
+            __syncthreads();
         }
-        __syncthreads();
+        // first scatter tile: its TMA overlaps the look-back below
+        if (tid == 0)
+            tile_issue(a, ci.side, ci.begin, umin32(TILE, ci.len), p1, false, ok, op, o2, &S.mbar[0]);
+
+        // --------------------------------------- chunk-level decoupled look-back, one bucket/thread
+        if (tid < nb) {
+            const uint32_t tot = S.cnt[tid];
+            W* st = reinterpret_cast<W*>(a.status[ci.side]);
+            const size_t me = size_t(ci.lc) * 256 + tid;
+            uint64_t excl = 0;
+            if (ci.chunk_in_seg == 0) {
+                LB<W>::store(st + me, LB<W>::kInc | W(tot));
+            } else {
+                LB<W>::store(st + me, LB<W>::kAgg | W(tot));
+                // walk back in windows of 4 predecessors (independent loads in flight)
+                int64_t j = int64_t(ci.lc) - 1;
+                const int64_t stop = int64_t(ci.first_chunk);
+                bool done = false;
+                while (!done) {
+                    W v[4];
+#pragma unroll
+                    for (int u = 0; u < 4; ++u) v[u] = (j - u >= stop) ? LB<W>::load(st + size_t(j - u) * 256 + tid) : W(0);
+#pragma unroll
+                    for (int u = 0; u < 4; ++u) {
+                        if (done || j - u < stop) continue;
+                        W x = v[u];
+                        while ((x >> LB<W>::kShift) == 0) x = LB<W>::load(st + size_t(j - u) * 256 + tid);
+                        excl += x & LB<W>::kMask;
+                        if ((x >> LB<W>::kShift) == 2) done = true;
+                    }
+                    j -= 4;
+                    if (j < stop) done = true;
+                }
+                LB<W>::store(st + me, LB<W>::kInc | W(excl + tot));
+            }
+            const uint64_t pidx = ((uint64_t(ci.seg) << bits) | tid) << lowbits;
+            S.run[tid] = a.start[ci.side][pidx] + excl;
+            S.wpos[tid] = S.run[tid];
+            S.carry[tid] = 0;
+        }
+        // (the first sync of the tile loop below orders run[] before its use)
+
+        // ------------------------------------------------------------------ scatter phase
+        if (a.dbg & 4) {
+            if (tid == 0) { mbar_wait(&S.mbar[0], par0); S.claim = atomicAdd(a.tile_ctr, 1u); }
+            par0 ^= 1;
+            __syncthreads();
+            t = S.claim;
+            __syncthreads();
+            continue;
+        }
+        for (uint32_t q = 0; q < ntile; ++q) {
+            const uint32_t qb = q * TILE;
+            const uint32_t ql = umin32(TILE, ci.len - qb);
+            const uint64_t tb = ci.begin + qb;
+            const LoadPlan lp = load_plan(a, ci.side, tb, ql, p1);
+            mbar_wait(&S.mbar[0], par0);
+            par0 ^= 1;
+            uint32_t rk[IPT / 2];  // ranks, packed 2 x u16
+#pragma unroll
+            for (int jj = 0; jj < IPT; ++jj) {
+                const uint32_t i = jj * BLOCK + tid;
+                uint32_t r = 0;
+                if (i < ql) {
+                    const bool bulk = (i - lp.head) < lp.nbulk;
+                    uint32_t h;
+                    if (p1) {
+                        uint32_t k;
+                        if (bulk) {
+                            k = ok[i];
+                        } else {
+                            k = a.keys[ci.side][tb + i];
+                            op[i] = a.pays[ci.side][tb + i];
+                        }
+                        h = hash32(k);
+                        ok[i] = h;
+                    } else {
+                        if (bulk) {
+                            h = o2[i + lp.shift].x;
+                        } else {
+                            const uint2 e = a.in[ci.side][tb + i];
+                            o2[i + lp.shift] = e;
+                            h = e.x;
+                        }
+                    }
+                    r = atomicAdd(&S.tcnt[(h >> dshift) & dmask], 1u);
+                }
+                if (jj & 1) rk[jj >> 1] |= r << 16; else rk[jj >> 1] = r;
+            }
+            __syncthreads();
+            // Write combining: bucket b's staged run = [carry from the previous tile | this tile's
+            // tuples]; only whole 32-byte sectors are written (partial-sector writes cost ~1.7x,
+            // scripts/microbench_scatter_ceiling.cu), the < 4-tuple remainder carries over.
+            const uint32_t tc = (tid < nb) ? S.tcnt[tid] : 0u;
+            const uint32_t cin = (tid < nb) ? S.carry[tid] : 0u;
+            uint32_t all;
+            const uint32_t lstart = block_excl_scan_u32<BLOCK>(tc + cin, &all, S.scan_tmp);
+            if (tid < nb) {
+                const unsigned long long nxt = S.run[tid] + tc;
+                const unsigned long long w0 = S.wpos[tid];
+                unsigned long long ew = (q + 1 == ntile) ? nxt : (nxt & ~3ull);
+                if (ew < w0) ew = w0;
+                S.local_start[tid] = lstart + cin;
+                S.gbase[tid] = w0 - lstart;
+                S.endw[tid] = ew;
+                for (uint32_t k = 0; k < cin; ++k) stage[lstart + k] = S.cbuf[tid][k];
+                S.wpos[tid] = ew;
+                S.run[tid] = nxt;
+                S.carry[tid] = (uint32_t)(nxt - ew);
+                S.tcnt[tid] = 0;
+            }
+            __syncthreads();
+#pragma unroll
+            for (int jj = 0; jj < IPT; ++jj) {
+                const uint32_t i = jj * BLOCK + tid;
+                if (i < ql) {
+                    const uint2 e = p1 ? make_uint2(ok[i], op[i]) : o2[i + lp.shift];
+                    const uint32_t r = (jj & 1) ? (rk[jj >> 1] >> 16) : (rk[jj >> 1] & 0xffffu);
+                    stage[S.local_start[(e.x >> dshift) & dmask] + r] = e;
+                }
+            }
+            if (tid == 0 && q + 1 == ntile) S.claim = atomicAdd(a.tile_ctr, 1u);
+            fence_proxy_async_smem();  // reads of the input tile precede the next TMA writes
+            __syncthreads();
+            if (tid == 0 && q + 1 < ntile)
+                tile_issue(a, ci.side, tb + TILE, umin32(TILE, ci.len - qb - TILE), p1, false,
+                           ok, op, o2, &S.mbar[0]);
+            uint2* out = a.out[ci.side];
+            const uint64_t wpol = policy_evict_first();
+#pragma unroll 4
+            for (uint32_t i = tid; i < all; i += BLOCK) {
+                const uint2 e = stage[i];
+                const uint32_t d = (e.x >> dshift) & dmask;
+                const unsigned long long g = S.gbase[d] + i;
+                const unsigned long long ew = S.endw[d];
+                if (g < ew) { if (!(a.dbg & 2)) st_stream_u2(out + g, e, wpol); }
+                else S.cbuf[d][g - ew] = e;
+            }
+            __syncthreads();
+        }
+        t = S.claim;
     }
 }
 
-size_t scatter_smem_bytes() {
-    return ((sizeof(ScatterSmem) + 15) & ~size_t(15)) + size_t(kScatterTile) * sizeof(uint2);
+size_t scatter_smem_bytes(int tile) {
+    // buf0: input tile (+4 slack); buf1: staging = tile + up to 3 carried tuples per bucket
+    return ((sizeof(ScatterSmem) + 127) & ~size_t(127)) + (size_t(tile) + 4) * 8 + (size_t(tile) + 3 * 256 + 4) * 8;
+}
+
+bool scatter_wide_status(const Plan& p) { return p.n[0] >= (1ull << 30) || p.n[1] >= (1ull << 30); }
+
+template <typename W, int BLOCK, int IPT>
+int launch_scatter_cfg(const Plan& p, const ScatterArgs& a, cudaStream_t s) {
+    const size_t smem = scatter_smem_bytes(BLOCK * IPT);
+    static bool attr_set = false;
+    if (!attr_set) {
+        cudaFuncSetAttribute(k_scatter<W, BLOCK, IPT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        attr_set = true;
+    }
+    int occ = 0;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_scatter<W, BLOCK, IPT>, BLOCK, smem);
+    if (occ < 1) occ = 1;
+    k_scatter<W, BLOCK, IPT><<<(unsigned)(p.num_sms * occ), BLOCK, smem, s>>>(a);
+    return 1;
+}
+
+template <typename W>
+int launch_scatter_w(const Plan& p, const ScatterArgs& a, cudaStream_t s) {
+    static int cfg = -1;
+    if (cfg < 0) {
+        const char* e = getenv("GSH_SCATTER_CFG");
+        cfg = e ? atoi(e) : 1;
+    }
+    switch (cfg) {
+        case 0: return launch_scatter_cfg<W, 256, 8>(p, a, s);
+        case 2: return launch_scatter_cfg<W, 256, 16>(p, a, s);
+        case 3: return launch_scatter_cfg<W, 1024, 8>(p, a, s);
+        default: return launch_scatter_cfg<W, 512, 8>(p, a, s);
+    }
 }
 
 int launch_scatter(const Plan& p, int pass, const uint32_t* const keys[2], const uint32_t* const pays[2],
                    cudaStream_t s) {
+    const bool wide = scatter_wide_status(p);
+    const size_t wbytes = wide ? 8 : 4;
     ScatterArgs a;
     for (int side = 0; side < 2; ++side) {
         a.keys[side] = keys ? keys[side] : nullptr;
@@ -355,26 +583,22 @@ int launch_scatter(const Plan& p, int pass, const uint32_t* const keys[2], const
         a.in[side] = (pass == 2) ? p.bufA[side] : nullptr;
         a.out[side] = (pass == 1) ? p.bufA[side] : p.bufB[side];
         a.start[side] = p.start + size_t(side) * (p.F + 1);
-        a.status[side] = p.status + size_t(side) * p.max_tiles[0] * 256;
         a.n[side] = p.n[side];
     }
-    a.status[1] = p.status + size_t(p.max_tiles[0]) * 256;
+    a.status[0] = p.status;
+    a.status[1] = reinterpret_cast<unsigned char*>(p.status) + size_t(p.max_chunks[0]) * 256 * wbytes;
     a.pass = pass;
     a.b1 = p.b1;
     a.b2 = p.b2;
     a.route_bits = p.route_bits;
     a.tile_ctr = &p.st->claim[pass - 1];
-    const size_t smem = scatter_smem_bytes();
-    static bool attr_set = false;
-    if (!attr_set) {
-        cudaFuncSetAttribute(k_scatter, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-        attr_set = true;
+    {
+        const char* e = getenv("GSH_SCATTER_DEBUG");
+        a.dbg = e ? (uint32_t)atoi(e) : 0u;
     }
     // status words must be zero before the pass
-    cudaMemsetAsync(p.status, 0, size_t(p.max_tiles[0] + p.max_tiles[1]) * 256 * sizeof(uint64_t), s);
-    unsigned grid = (unsigned)p.num_sms * 2;
-    k_scatter<<<grid, kScatterBlock, smem, s>>>(a);
-    return 1;
+    cudaMemsetAsync(p.status, 0, size_t(p.max_chunks[0] + p.max_chunks[1]) * 256 * wbytes, s);
+    return wide ? launch_scatter_w<unsigned long long>(p, a, s) : launch_scatter_w<uint32_t>(p, a, s);
 }
 
 // ----------------------------------------------- standalone radix histogram (ABI) --

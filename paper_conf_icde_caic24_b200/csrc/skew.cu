@@ -32,6 +32,7 @@ __global__ void k_classify(const uint32_t* __restrict__ cnt, uint32_t F, uint32_
         const uint32_t cr = cnt[p], cs = cnt[F + p];
         part_heavy[p] = 0;
         part_heavy[F + p] = 0;
+        if (cs > 0 && cr > 0) atomicMax(&st->max_rlen, cr);
         const bool large = (cr > 0 && cs > 0) && !force_normal && (force_heavy || cr > C || cs > C);
         uint32_t idx = kNoHeavy;
         if (large) {
