@@ -79,20 +79,21 @@ typedef struct {
 
 /* Tuning / test hooks.  Initialise with gsh_config_default(); NULL means defaults. */
 typedef struct {
-    uint32_t capacity;         /* C: max R tuples per NM-join build table and the
-                                  large-partition threshold (L107).  0 = auto
+    uint32_t capacity;         /* C: max R tuples per NM-join build table (L115).  0 = auto
                                   (max(4096, 2 * mean partition size), <= 8192). */
     int32_t pass_bits[2];      /* radix bits of pass 1 / pass 2 (L106).  -1 = auto so the
                                   mean partition holds ~2048 tuples (max 8 + 8 bits). */
     uint32_t heavy_threshold;  /* T_h: a key of a large partition is skewed iff
-                                  max(cnt_R, cnt_S) >= T_h (L112 reading).  0 = C / 4. */
+                                  max(cnt_R, cnt_S) >= T_h (L112 reading).  0 = 64. */
     uint32_t route_bits;       /* top bits of fmix32(key) already consumed by multi-GPU
                                   routing; partition digits start below them. */
     int32_t force_all_normal;  /* test hook: no skew detection; every key goes through the
                                   NM-join (chunked when a partition exceeds C). */
     int32_t force_all_heavy;   /* test hook: every partition is large and every key skewed. */
     int32_t timing;            /* 1 = record per-phase CUDA events into gsh_result.ms_* */
-    int32_t reserved;
+    uint32_t large_threshold;  /* L: a partition is large iff |R_p| > L or |S_p| > L (L107's
+                                  "pre-defined threshold").  0 = auto: mean + 8 sqrt(mean),
+                                  i.e. far beyond the binomial spread of a skew-free partition. */
 } gsh_config;
 
 /* Per-call result (host struct). */
@@ -113,7 +114,7 @@ typedef struct {
     uint32_t capacity;         /* C actually used */
     uint32_t heavy_threshold;  /* T_h actually used */
     uint32_t launches;         /* kernels launched by this call */
-    uint32_t reserved;
+    uint32_t large_threshold;  /* L actually used */
     float ms_hist, ms_pass1, ms_pass2, ms_detect, ms_split, ms_nmjoin, ms_skewjoin, ms_total;
 } gsh_result;
 

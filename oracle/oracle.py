@@ -170,12 +170,12 @@ def radix_histogram(keys, hi_bits: int, nbits: int) -> np.ndarray:
     return np.bincount(d, minlength=1 << nbits).astype(np.int64)
 
 
-def heavy_rule(rk, sk, part_bits: int, capacity: int, threshold: int, route_bits: int = 0):
+def heavy_rule(rk, sk, part_bits: int, large_threshold: int, threshold: int, route_bits: int = 0):
     """Skew detection after partitioning (§IV-B(2)), with the
     readings of DESIGN.md §3 (exact counts replace the 1 % sample, north star):
 
       partition p = top `part_bits` bits of h below `route_bits` (final partitions);
-      large(p)  <=>  |R_p| > capacity  or  |S_p| > capacity          (L107 threshold)
+      large(p)  <=>  |R_p| > L  or  |S_p| > L,  L = large_threshold   (L107 threshold)
       heavy(k)  <=>  k lies in a large partition and
                      max(cnt_R(k), cnt_S(k)) >= threshold            (L112 'top-k')
 
@@ -189,7 +189,7 @@ def heavy_rule(rk, sk, part_bits: int, capacity: int, threshold: int, route_bits
     nparts = 1 << part_bits
     szr = np.bincount(pr, minlength=nparts)
     szs = np.bincount(ps, minlength=nparts)
-    large = (szr > capacity) | (szs > capacity)
+    large = (szr > large_threshold) | (szs > large_threshold)
     ur, cr = np.unique(hr[large[pr]], return_counts=True)
     us, cs = np.unique(hs[large[ps]], return_counts=True)
     allk = np.union1d(ur, us).astype(np.uint32)

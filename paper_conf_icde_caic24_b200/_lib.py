@@ -41,7 +41,7 @@ class GshConfig(ctypes.Structure):
         ("force_all_normal", i32),
         ("force_all_heavy", i32),
         ("timing", i32),
-        ("reserved", i32),
+        ("large_threshold", u32),
     ]
 
 
@@ -63,7 +63,7 @@ class GshResult(ctypes.Structure):
         ("capacity", u32),
         ("heavy_threshold", u32),
         ("launches", u32),
-        ("reserved", u32),
+        ("large_threshold", u32),
         ("ms_hist", ctypes.c_float),
         ("ms_pass1", ctypes.c_float),
         ("ms_pass2", ctypes.c_float),

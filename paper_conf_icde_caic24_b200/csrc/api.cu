@@ -5,6 +5,7 @@
 // detection) and one after skewed-key selection (number of skewed keys, to size the split and
 // the tile list); the final one fills gsh_result.  When no partition is large (uniform inputs,
 // PAPER.md L166) the detect/split/skew phases are skipped entirely.
+#include <cmath>
 #include <cstdio>
 #include <cstring>
 #include <string>
@@ -115,7 +116,14 @@ bool plan_build(Plan& p, uint64_t nR, uint64_t nS, const gsh_config* cfg_in, voi
         if (c > kMaxCapacity) c = kMaxCapacity;
         p.C = (uint32_t)c;
     }
-    p.Th = cfg.heavy_threshold ? cfg.heavy_threshold : p.C / 4;
+    p.Th = cfg.heavy_threshold ? cfg.heavy_threshold : 64;
+    if (cfg.large_threshold) {
+        p.L = cfg.large_threshold;
+    } else {
+        const double mean = double(nmax) / double(p.F);
+        uint64_t l = uint64_t(mean + 8.0 * std::sqrt(mean > 1.0 ? mean : 1.0)) + 1;
+        p.L = (uint32_t)(l < 64 ? 64 : l);
+    }
     p.force_normal = cfg.force_all_normal;
     p.force_heavy = cfg.force_all_heavy;
     p.timing = cfg.timing;
@@ -264,6 +272,7 @@ gsh_status gsh_join(const gsh_relation* R, const gsh_relation* S, gsh_out_mode m
     res->pass_bits[1] = p.b2;
     res->capacity = p.C;
     res->heavy_threshold = p.Th;
+    res->large_threshold = p.L;
     if (R->n == 0 || S->n == 0) return GSH_OK;
 
     uint32_t* pairs = mat ? out->pairs : nullptr;
@@ -481,6 +490,7 @@ gsh_status gsh_detect(const gsh_relation* R, const gsh_relation* S, const gsh_co
         res->pass_bits[1] = p.b2;
         res->capacity = p.C;
         res->heavy_threshold = p.Th;
+        res->large_threshold = p.L;
         res->heavy_tuples_r = hs.heavy_tuples[0];
         res->heavy_tuples_s = hs.heavy_tuples[1];
         res->skew_pairs = hs.skew_pairs;

@@ -25,7 +25,7 @@ constexpr int kSkewTileS = kSkewBlock * kSkewSpt;  // 1024
 constexpr int kSkewTileR = 64;                  // R payloads per tile (shared memory)
 constexpr uint32_t kDetectChunk = 4096;         // tuples per detect / split work item
 constexpr uint32_t kNoHeavy = 0xffffffffu;
-constexpr int kDetectMaxProbe = 4096;
+constexpr int kDetectMaxProbe = 64;   // a full table degrades to "normal", never to a long probe
 
 // Device-resident counters and accumulators, zeroed once per call.
 struct DevState {
@@ -57,7 +57,7 @@ struct Plan {
     // sizes and parameters
     uint64_t n[2] = {0, 0};
     uint32_t b1 = 0, b2 = 0, route_bits = 0;
-    uint32_t C = 4096, Th = 1024;
+    uint32_t C = 4096, Th = 64, L = 4096;  // NM capacity, skew-key threshold, large-partition threshold
     uint32_t nm_slots = 0;          // NM build-table slots (set after classification; 0 = from C)
     uint32_t F = 1;                 // 1 << (b1 + b2)
     int force_normal = 0, force_heavy = 0, timing = 0;

@@ -1,7 +1,7 @@
 // skew.cu -- GSH phases (2) and (3) (§IV-B), SURVEY.md §8(a) rows a5-a7.
 //
 //   a5 k_classify : "identify normal vs. large partitions by comparing the partition size with
-//                   a pre-defined threshold" (L107).  large(p) <=> |R_p| > C or |S_p| > C
+//                   a pre-defined threshold" (L107).  large(p) <=> |R_p| > L or |S_p| > L
 //                   (and both sides non-empty: a partition with an empty side yields nothing).
 //   a6 k_detect   : exact per-key counts of every key of every large partition, both sides.
 //                   Warp aggregation with __match_any_sync collapses a skewed key's tuples to
@@ -25,7 +25,7 @@ __device__ __forceinline__ uint32_t part_of(uint32_t h, uint32_t shift, uint32_t
 }
 
 // ------------------------------------------------------------------ a5: classify --
-__global__ void k_classify(const uint32_t* __restrict__ cnt, uint32_t F, uint32_t C, int force_normal,
+__global__ void k_classify(const uint32_t* __restrict__ cnt, uint32_t F, uint32_t L, int force_normal,
                            int force_heavy, uint32_t* __restrict__ large_list, uint32_t* __restrict__ large_idx,
                            uint32_t* __restrict__ part_heavy, DevState* st) {
     for (uint32_t p = blockIdx.x * blockDim.x + threadIdx.x; p < F; p += gridDim.x * blockDim.x) {
@@ -33,7 +33,7 @@ __global__ void k_classify(const uint32_t* __restrict__ cnt, uint32_t F, uint32_
         part_heavy[p] = 0;
         part_heavy[F + p] = 0;
         if (cs > 0 && cr > 0) atomicMax(&st->max_rlen, cr);
-        const bool large = (cr > 0 && cs > 0) && !force_normal && (force_heavy || cr > C || cs > C);
+        const bool large = (cr > 0 && cs > 0) && !force_normal && (force_heavy || cr > L || cs > L);
         uint32_t idx = kNoHeavy;
         if (large) {
             idx = atomicAdd(&st->n_large, 1u);
@@ -47,7 +47,7 @@ __global__ void k_classify(const uint32_t* __restrict__ cnt, uint32_t F, uint32_
 
 int launch_classify(const Plan& p, cudaStream_t s) {
     unsigned grid = (p.F + 255) / 256;
-    k_classify<<<grid, 256, 0, s>>>(p.cnt, p.F, p.C, p.force_normal, p.force_heavy, p.large_list, p.large_idx,
+    k_classify<<<grid, 256, 0, s>>>(p.cnt, p.F, p.L, p.force_normal, p.force_heavy, p.large_list, p.large_idx,
                                     p.part_heavy, p.st);
     return 1;
 }

@@ -36,7 +36,8 @@ M64 = (1 << 64) - 1
 
 
 def _cfg_params(n_global: int, config) -> tuple[int, int, int]:
-    """(B, C, T_h) exactly as plan_build() derives them (api.cu) for n = max side size."""
+    """(B, L, T_h) exactly as plan_build() derives them (api.cu) for n = max side size:
+    radix bits, large-partition threshold, skewed-key threshold."""
     if config is not None and config.pass_bits[0] >= 0 and config.pass_bits[1] >= 0:
         B = int(config.pass_bits[0]) + int(config.pass_bits[1])
     else:
@@ -44,14 +45,13 @@ def _cfg_params(n_global: int, config) -> tuple[int, int, int]:
         while B < 16 and (n_global >> B) > 2048:
             B += 1
     F = 1 << B
-    if config is not None and config.capacity:
-        C = 1 << max(0, math.ceil(math.log2(config.capacity)))
+    if config is not None and config.large_threshold:
+        L = int(config.large_threshold)
     else:
-        mean = (n_global + F - 1) // F
-        C = 1 << max(0, math.ceil(math.log2(max(2 * mean, 1))))
-        C = min(max(C, 4096), 8192)
-    Th = int(config.heavy_threshold) if (config is not None and config.heavy_threshold) else C // 4
-    return B, C, Th
+        mean = float(n_global) / float(F)
+        L = max(64, int(mean + 8.0 * math.sqrt(max(mean, 1.0))) + 1)
+    Th = int(config.heavy_threshold) if (config is not None and config.heavy_threshold) else 64
+    return B, L, Th
 
 
 class CudaOps:
@@ -138,29 +138,29 @@ def agree_heavy(rk, rp, sk, sp, config=None, group=None, ops=None):
     n = torch.tensor([rk.numel(), sk.numel()], dtype=torch.int64, device=dev)
     dist.all_reduce(n, group=group)
     n_r, n_s = int(n[0]), int(n[1])
-    B, C, Th = _cfg_params(max(n_r, n_s), config)
+    B, L, Th = _cfg_params(max(n_r, n_s), config)
     hr = ops.radix_histogram(rk, 0, B)
     hs = ops.radix_histogram(sk, 0, B)
     h = torch.stack([hr, hs])
     dist.all_reduce(h, group=group)
-    large = ((h[0] > C) | (h[1] > C)) & (h[0] > 0) & (h[1] > 0)
+    large = ((h[0] > L) | (h[1] > L)) & (h[0] > 0) & (h[1] > 0)
     if config is not None and config.force_all_normal:
         large[:] = False
     G = dist.get_world_size(group)
     empty = torch.zeros(0, dtype=torch.int32, device=dev)
     if not bool(large.any()):
-        return empty, (B, C, Th, n_r, n_s)
+        return empty, (B, L, Th, n_r, n_s)
     tau = max(1, -(-Th // G))
     cand = ops.local_candidates(rk, rp, sk, sp, B, large.to(torch.uint8), tau)
     allc = _allgather_var(cand, group)
     q = torch.unique(allc)  # sorted int64 u32 values
     if q.numel() == 0:
-        return empty, (B, C, Th, n_r, n_s)
+        return empty, (B, L, Th, n_r, n_s)
     q32 = _to_i32_sorted(q)
     cnt = torch.stack([ops.count_keys(rk, q32), ops.count_keys(sk, q32)])
     dist.all_reduce(cnt, group=group)
     heavy = q[torch.maximum(cnt[0], cnt[1]) >= Th]
-    return _to_i32_sorted(heavy), (B, C, Th, n_r, n_s)
+    return _to_i32_sorted(heavy), (B, L, Th, n_r, n_s)
 
 
 def _exchange_normal(keys, pays, counts, G, group):
@@ -217,7 +217,7 @@ def join_sharded(rk, rp, sk, sp, config=None, group=None, ops=None):
     if G & (G - 1):
         raise ValueError("world size must be a power of two (route bits)")
     rb = G.bit_length() - 1
-    heavy, (B, C, Th, n_r, n_s) = agree_heavy(rk, rp, sk, sp, config, group, ops)
+    heavy, (B, L, Th, n_r, n_s) = agree_heavy(rk, rp, sk, sp, config, group, ops)
     rks, rps, rc = ops.route(rk, rp, rb, heavy)
     sks, sps, sc = ops.route(sk, sp, rb, heavy)
     rk_n, rp_n = _exchange_normal(rks, rps, rc, G, group)

@@ -75,16 +75,17 @@ def test_partition_phase(kind, n, theta):
 
 
 @pytest.mark.parametrize("theta,n,cfg", [(1.0, 1 << 18, {}), (1.5, 1 << 17, {}), (0.75, 1 << 18, {}),
-                                         (1.0, 1 << 16, {"capacity": 512, "heavy_threshold": 16}),
-                                         (0.5, 1 << 17, {"capacity": 256, "heavy_threshold": 4})])
+                                         (1.0, 1 << 16, {"large_threshold": 512, "heavy_threshold": 16}),
+                                         (0.5, 1 << 17, {"large_threshold": 256, "heavy_threshold": 4}),
+                                         (1.0, 1 << 18, {"capacity": 256})])
 def test_skew_detection_matches_exact_rule(theta, n, cfg):
     """Skewed keys (PAPER.md L107/L112 with exact counts, DESIGN.md §3 R3/R4) equal the oracle's
-    heavy_rule on the same partition bits, capacity and threshold."""
+    heavy_rule on the same partition bits, large-partition threshold and key threshold."""
     rk, rp, sk, sp = datagen.zipf_pair(n, n, theta, seed=3)
     config = gsh.make_config(**cfg)
     h, cr, cs, st = gsh.detect(*_dev(rk, rp, sk, sp), config=config)
     B = st["pass_bits"][0] + st["pass_bits"][1]
-    oh, ocr, ocs = oracle.heavy_rule(_np(rk), _np(sk), B, st["capacity"], st["heavy_threshold"])
+    oh, ocr, ocs = oracle.heavy_rule(_np(rk), _np(sk), B, st["large_threshold"], st["heavy_threshold"])
     assert st["detect_overflow"] == 0
     assert np.array_equal(h.numpy().astype(np.uint32), oh)
     assert np.array_equal(cr.numpy(), ocr) and np.array_equal(cs.numpy(), ocs)
@@ -136,7 +137,8 @@ def test_join_materialize_overflow_subset():
 
 @pytest.mark.parametrize("cfg", [{"force_all_normal": True}, {"force_all_heavy": True}, {"capacity": 256},
                                  {"capacity": 8192}, {"pass_bits": (3, 2)}, {"pass_bits": (8, 8)},
-                                 {"pass_bits": (0, 0)}, {"heavy_threshold": 2}, {"capacity": 128, "heavy_threshold": 1000000}])
+                                 {"pass_bits": (0, 0)}, {"heavy_threshold": 2}, {"capacity": 128, "heavy_threshold": 1000000},
+                                 {"large_threshold": 1}, {"large_threshold": 100000}, {"heavy_threshold": 100000}])
 def test_join_invariant_under_config(cfg):
     """Skew classification, fanout and capacity change performance only:
     results must be identical under every configuration (metamorphic pin P4)."""

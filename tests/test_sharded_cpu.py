@@ -70,7 +70,7 @@ def _worker(rank, world, port, kind, n, theta, q):
     dist.init_process_group("gloo", rank=rank, world_size=world)
     try:
         from paper_conf_icde_caic24_b200 import make_config, sharded
-        cfg = make_config(capacity=512, heavy_threshold=64)
+        cfg = make_config(large_threshold=512, heavy_threshold=64)
         rk, rp, sk, sp = datagen.make_workload(kind, n, theta, seed=17)
         lo_r, hi_r = rank * rk.numel() // world, (rank + 1) * rk.numel() // world
         lo_s, hi_s = rank * sk.numel() // world, (rank + 1) * sk.numel() // world
@@ -109,8 +109,8 @@ def test_sharded_matches_oracle(world, kind, n, theta):
     on, oc, _ = oracle.join(_u32(rk), _u32(rp), _u32(sk), _u32(sp))
     heavy_sets = {tuple(o[3]) for o in out}
     assert len(heavy_sets) == 1  # all ranks agree
-    B, C, Th, _, _ = out[0][4]
-    oh, _, _ = oracle.heavy_rule(_u32(rk), _u32(sk), B, C, Th)
+    B, L, Th, _, _ = out[0][4]
+    oh, _, _ = oracle.heavy_rule(_u32(rk), _u32(sk), B, L, Th)
     assert list(heavy_sets.pop()) == oh.tolist()
     for o in out:
         assert (o[1], o[2]) == (on, oc)
