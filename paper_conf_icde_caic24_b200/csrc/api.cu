@@ -141,7 +141,10 @@ bool plan_build(Plan& p, uint64_t nR, uint64_t nS, const gsh_config* cfg_in, voi
         uint64_t hm = (nR + nS) / (p.Th ? p.Th : 1) + 1;
         p.h_max = hm < p.gt_cap_alloc ? hm : p.gt_cap_alloc;
     }
+    for (int s = 0; s < 2; ++s) p.nch1[s] = (uint32_t)((p.n[s] + kScatterChunk - 1) / kScatterChunk);
     uint64_t scan_max = p.F + 1 > p.h_max + 1 ? p.F + 1 : p.h_max + 1;
+    for (int s = 0; s < 2; ++s)
+        if (uint64_t(p.nch1[s]) * 256 + 1 > scan_max) scan_max = uint64_t(p.nch1[s]) * 256 + 1;
     p.scan_scratch_elems = scan_max / 4096 + 2;
 
     Carver c{reinterpret_cast<unsigned char*>(ws)};
@@ -159,6 +162,8 @@ bool plan_build(Plan& p, uint64_t nR, uint64_t nS, const gsh_config* cfg_in, voi
     p.heavy_pay[0] = hp;
     p.heavy_pay[1] = hp ? hp + nR : nullptr;
     p.hist_partial = c.take<uint32_t>(size_t(2) * p.hist_grid * F);
+    p.c1cnt = c.take<uint32_t>((size_t(p.nch1[0]) + p.nch1[1]) * 256 + 1);
+    p.off1 = c.take<uint64_t>((size_t(p.nch1[0]) + p.nch1[1]) * 256 + 2);
     p.cnt = c.take<uint32_t>(2 * F);
     p.start = c.take<uint64_t>(2 * (F + 1));
     p.status = c.take<uint64_t>(size_t(p.max_chunks[0] + p.max_chunks[1]) * 256);

@@ -73,6 +73,9 @@ struct Plan {
     uint2* bufB[2] = {nullptr, nullptr};      // final partitions
     uint32_t* heavy_pay[2] = {nullptr, nullptr};  // skewed-key payload arrays
     uint32_t* hist_partial = nullptr;         // [2][chunks][F]
+    uint32_t nch1[2] = {0, 0};                // pass-1 chunks per side
+    uint32_t* c1cnt = nullptr;                // [nch1[0] + nch1[1]][256] pass-1 digit counts per chunk
+    uint64_t* off1 = nullptr;                 // per side [256 * nch1 + 1] chunk/bucket output offsets
     uint32_t* cnt = nullptr;                  // [2][F]
     uint64_t* start = nullptr;                // [2][F + 1]
     uint64_t* status = nullptr;               // [2][max_chunks][256]

@@ -5,7 +5,7 @@
 //   a1 k_hist2d        : h = fmix32(key); joint (d1,d2) histogram of BOTH passes from one read
 //                        of the keys (4 B/tuple).  Per-CTA packed-u16 shared-memory counters with
 //                        warp aggregation (__match_any_sync) so skewed digits do not serialise.
-//   a2 k_hist_reduce / k_part_scan : per-partition counts and start offsets.
+//   a2 k_hist_reduce + scans : per-partition counts and start offsets, pass-1 chunk offsets.
 //   a3/a4 k_scatter    : Onesweep-style scatter -- dynamic tile ids, per-tile bucket ranks via
 //                        __match_any_sync, decoupled look-back across tiles per bucket, tiles
 //                        staged in shared memory in bucket order, then written as contiguous
@@ -48,51 +48,86 @@ __device__ __forceinline__ void hist_one(uint32_t* cnt, uint32_t key, uint32_t s
     if (bin < nb) atomicAdd(&cnt[bin], 1u);
 }
 
+// The same read also yields, per pass-1 chunk (kScatterChunk consecutive tuples), the chunk's
+// pass-1 digit counts: "count then partition" at chunk granularity, so pass 1
+// needs neither a second read nor a cross-CTA look-back (its offsets come from one scan).
 __global__ void __launch_bounds__(kHistBlock, 1)
 k_hist2d(const uint32_t* __restrict__ k0, uint64_t n0, const uint32_t* __restrict__ k1, uint64_t n1,
-         uint32_t shift, uint32_t nbits, uint32_t* __restrict__ partial) {
+         uint32_t shift, uint32_t nbits, uint32_t b2, uint32_t* __restrict__ partial, uint32_t* __restrict__ c1cnt,
+         uint32_t nch0, uint32_t nch1) {
     extern __shared__ uint32_t cnt[];
+    __shared__ uint32_t c1[256];
     const uint32_t F = 1u << nbits;
     const uint32_t mask = F - 1;
     const bool split = F > (1u << 15);
-    const uint32_t nchunks = split ? gridDim.x / 2 : gridDim.x;
-    const uint32_t chunk = split ? blockIdx.x >> 1 : blockIdx.x;
+    const uint32_t groups = split ? gridDim.x / 2 : gridDim.x;
+    const uint32_t g = split ? blockIdx.x >> 1 : blockIdx.x;
     const uint32_t nb = split ? F / 2 : F;
     const uint32_t lo = split ? (blockIdx.x & 1) * nb : 0;
+    const uint32_t d1lo = lo >> b2, d1n = (nb >> b2) ? (nb >> b2) : 1;
     for (int side = 0; side < 2; ++side) {
         const uint32_t* keys = side ? k1 : k0;
         const uint64_t n = side ? n1 : n0;
+        const uint32_t nch = side ? nch1 : nch0;
+        uint32_t* c1out = c1cnt + (side ? size_t(nch0) * 256 : 0);
         for (uint32_t w = threadIdx.x; w < nb; w += blockDim.x) cnt[w] = 0;
+        if (threadIdx.x < 256) c1[threadIdx.x] = 0;
         __syncthreads();
         const bool vec = ((reinterpret_cast<uintptr_t>(keys) & 15u) == 0);
-        const uint64_t nv = vec ? n / 4 : 0;
-        const uint64_t b = nv * chunk / nchunks, e = nv * (chunk + 1) / nchunks;
-        const uint4* kv = reinterpret_cast<const uint4*>(keys);
-        uint64_t i = b + threadIdx.x;
-        for (; i + 3ull * blockDim.x < e; i += 4ull * blockDim.x) {
-            uint4 v[4];
+        for (uint32_t c = g; c < nch; c += groups) {
+            const uint64_t cb = uint64_t(c) * kScatterChunk;
+            const uint64_t ce = umin64(cb + kScatterChunk, n);
+            uint64_t done = cb;
+            if (vec) {
+                const uint4* kv = reinterpret_cast<const uint4*>(keys + cb);
+                const uint64_t nv = (ce - cb) / 4;
+                uint64_t i = threadIdx.x;
+                for (; i + 3ull * blockDim.x < nv; i += 4ull * blockDim.x) {
+                    uint4 v[4];
 #pragma unroll
-            for (int u = 0; u < 4; ++u) v[u] = ld_stream_u4(kv + i + u * blockDim.x);
+                    for (int u = 0; u < 4; ++u) v[u] = ld_stream_u4(kv + i + u * blockDim.x);
 #pragma unroll
-            for (int u = 0; u < 4; ++u) {
-                hist_one(cnt, v[u].x, shift, mask, lo, nb);
-                hist_one(cnt, v[u].y, shift, mask, lo, nb);
-                hist_one(cnt, v[u].z, shift, mask, lo, nb);
-                hist_one(cnt, v[u].w, shift, mask, lo, nb);
+                    for (int u = 0; u < 4; ++u) {
+                        const uint32_t kk[4] = {v[u].x, v[u].y, v[u].z, v[u].w};
+#pragma unroll
+                        for (int q = 0; q < 4; ++q) {
+                            const uint32_t bin = (hash32(kk[q]) >> shift) & mask;
+                            if (bin - lo < nb) {
+                                atomicAdd(&cnt[bin - lo], 1u);
+                                atomicAdd(&c1[bin >> b2], 1u);
+                            }
+                        }
+                    }
+                }
+                for (; i < nv; i += blockDim.x) {
+                    const uint4 v = ld_stream_u4(kv + i);
+                    const uint32_t kk[4] = {v.x, v.y, v.z, v.w};
+#pragma unroll
+                    for (int q = 0; q < 4; ++q) {
+                        const uint32_t bin = (hash32(kk[q]) >> shift) & mask;
+                        if (bin - lo < nb) {
+                            atomicAdd(&cnt[bin - lo], 1u);
+                            atomicAdd(&c1[bin >> b2], 1u);
+                        }
+                    }
+                }
+                done = cb + nv * 4;
             }
+            for (uint64_t j = done + threadIdx.x; j < ce; j += blockDim.x) {
+                const uint32_t bin = (hash32(keys[j]) >> shift) & mask;
+                if (bin - lo < nb) {
+                    atomicAdd(&cnt[bin - lo], 1u);
+                    atomicAdd(&c1[bin >> b2], 1u);
+                }
+            }
+            __syncthreads();
+            if (threadIdx.x < d1n) {
+                c1out[size_t(d1lo + threadIdx.x) * nch + c] = c1[d1lo + threadIdx.x];
+                c1[d1lo + threadIdx.x] = 0;
+            }
+            __syncthreads();
         }
-        for (; i < e; i += blockDim.x) {
-            uint4 v = ld_stream_u4(kv + i);
-            hist_one(cnt, v.x, shift, mask, lo, nb);
-            hist_one(cnt, v.y, shift, mask, lo, nb);
-            hist_one(cnt, v.z, shift, mask, lo, nb);
-            hist_one(cnt, v.w, shift, mask, lo, nb);
-        }
-        // scalar remainder (all keys when unaligned, else the n % 4 tail) -> chunk 0
-        if (chunk == 0)
-            for (uint64_t j = nv * 4 + threadIdx.x; j < n; j += blockDim.x) hist_one(cnt, keys[j], shift, mask, lo, nb);
-        __syncthreads();
-        uint32_t* row = partial + (size_t(side) * nchunks + chunk) * F + lo;
+        uint32_t* row = partial + (size_t(side) * groups + g) * F + lo;
         for (uint32_t w = threadIdx.x; w < nb; w += blockDim.x) row[w] = cnt[w];
         __syncthreads();
     }
@@ -108,62 +143,53 @@ int launch_hist(const Plan& p, const uint32_t* k0, const uint32_t* k1, cudaStrea
         cudaFuncSetAttribute(k_hist2d, cudaFuncAttributeMaxDynamicSharedMemorySize, 128 * 1024);
         attr_set = true;
     }
-    k_hist2d<<<p.hist_grid, kHistBlock, smem, s>>>(k0, p.n[0], k1, p.n[1], shift, nbits, p.hist_partial);
+    k_hist2d<<<p.hist_grid, kHistBlock, smem, s>>>(k0, p.n[0], k1, p.n[1], shift, nbits, p.b2, p.hist_partial,
+                                                   p.c1cnt, p.nch1[0], p.nch1[1]);
     return 1;
 }
 
-// --------------------------------------------------- a2: reduce partials + prefix scan --
-// cnt[side][bin] = sum over chunks of partial[side][chunk][bin]
+// --------------------------------------------------- a2: reduce partials + prefix scans --
+// cnt[side][bin] = sum over chunk groups of partial[side][group][bin]
 __global__ void k_hist_reduce(const uint32_t* __restrict__ partial, uint32_t* __restrict__ cnt, uint32_t F,
-                              uint32_t nchunks) {
+                              uint32_t groups) {
     for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < 2 * F; i += gridDim.x * blockDim.x) {
         const uint32_t side = i / F, bin = i % F;
-        const uint32_t* base = partial + size_t(side) * nchunks * F + bin;
+        const uint32_t* base = partial + size_t(side) * groups * F + bin;
         uint32_t s = 0;
-        for (uint32_t g = 0; g < nchunks; ++g) s += base[size_t(g) * F];
+        for (uint32_t g = 0; g < groups; ++g) s += base[size_t(g) * F];
         cnt[i] = s;
     }
 }
 
-// One CTA per side: start[side][0..F] = exclusive scan of cnt[side][*].
-__global__ void __launch_bounds__(1024) k_part_scan(const uint32_t* __restrict__ cnt, uint64_t* __restrict__ start,
-                                                    uint32_t F) {
-    __shared__ uint64_t wsum[33];
-    const uint32_t side = blockIdx.x;
-    const uint32_t* c = cnt + size_t(side) * F;
-    uint64_t* o = start + size_t(side) * (F + 1);
-    const uint32_t per = (F + 1023) / 1024;
-    const uint32_t b = threadIdx.x * per;
-    uint64_t local = 0;
-    for (uint32_t j = 0; j < per; ++j)
-        if (b + j < F) local += c[b + j];
-    const uint32_t lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-    uint64_t incl = warp_incl_scan_u64(local);
-    if (lane == 31) wsum[w] = incl;
-    __syncthreads();
-    if (w == 0) {
-        uint64_t v = wsum[lane];
-        uint64_t t = warp_incl_scan_u64(v);
-        wsum[lane] = t - v;
-        if (lane == 31) wsum[32] = t;
-    }
-    __syncthreads();
-    uint64_t run = wsum[w] + incl - local;
-    for (uint32_t j = 0; j < per; ++j)
-        if (b + j < F) {
-            o[b + j] = run;
-            run += c[b + j];
-        }
-    if (threadIdx.x == 0) o[F] = wsum[32];
-}
+struct CountAt {
+    const uint32_t* c;
+    __device__ uint64_t operator()(uint64_t i) const { return c[i]; }
+};
+
+// Pass-1 chunk counts, read in (digit, chunk) order: the exclusive scan in that order IS the
+// output offset of chunk c's bucket-d run (start of bucket d + runs of d in earlier chunks).
+struct ChunkDigit {
+    const uint32_t* c1;   // [256][nch] digit-major
+    __device__ uint64_t operator()(uint64_t i) const { return c1[i]; }
+};
 
 int launch_hist_reduce_scan(const Plan& p, cudaStream_t s) {
     const uint32_t F = p.F;
-    const uint32_t nchunks = F > (1u << 15) ? p.hist_grid / 2 : p.hist_grid;
+    const uint32_t groups = F > (1u << 15) ? p.hist_grid / 2 : p.hist_grid;
     unsigned grid = (2 * F + 255) / 256;
-    k_hist_reduce<<<grid, 256, 0, s>>>(p.hist_partial, p.cnt, F, nchunks);
-    k_part_scan<<<2, 1024, 0, s>>>(p.cnt, p.start, F);
-    return 2;
+    k_hist_reduce<<<grid, 256, 0, s>>>(p.hist_partial, p.cnt, F, groups);
+    int l = 1;
+    for (int side = 0; side < 2; ++side)
+        l += launch_scan(CountAt{p.cnt + size_t(side) * F}, F, p.start + size_t(side) * (F + 1), p.scan_scratch, s);
+    uint64_t off = 0;
+    for (int side = 0; side < 2; ++side) {
+        const uint64_t m = uint64_t(p.nch1[side]) * 256;
+        if (m)
+            l += launch_scan(ChunkDigit{p.c1cnt + (side ? size_t(p.nch1[0]) * 256 : 0)}, m,
+                             p.off1 + off, p.scan_scratch, s);
+        off += m + 1;
+    }
+    return l;
 }
 
 // ------------------------------------------------------------- a3/a4: tile scatter --
@@ -177,6 +203,8 @@ struct ScatterArgs {
     uint64_t n[2];
     uint32_t pass, b1, b2, route_bits;
     unsigned int* tile_ctr;
+    const uint64_t* off1[2];   // pass 1: [256][nch] chunk/bucket output offsets (no count phase)
+    uint32_t nch1[2];
     uint32_t dbg;              // experiment switches (GSH_SCATTER_DEBUG), 0 in production
 };
 
@@ -362,7 +390,9 @@ __global__ void __launch_bounds__(BLOCK) k_scatter(ScatterArgs a) {
 
         // ------------------------------------------------ count phase (double-buffered TMA)
         if (tid < 256) S.cnt[tid] = 0;
-        const uint32_t ncount = (a.dbg & 1) ? 0 : ntile;
+        // pass 1 gets its chunk offsets from the histogram pass: no count phase, no look-back
+        const bool stat = p1 && a.off1[ci.side] != nullptr;
+        const uint32_t ncount = (stat || (a.dbg & 1)) ? 0 : ntile;
         if (tid == 0 && ncount) {
             fence_proxy_async_smem();
             tile_issue(a, ci.side, ci.begin, umin32(TILE, ci.len), p1, true, ok, nullptr, o2, &S.mbar[0]);
@@ -396,7 +426,13 @@ __global__ void __launch_bounds__(BLOCK) k_scatter(ScatterArgs a) {
             tile_issue(a, ci.side, ci.begin, umin32(TILE, ci.len), p1, false, ok, op, o2, &S.mbar[0]);
 
         // --------------------------------------- chunk-level decoupled look-back, one bucket/thread
-        if (tid < nb) {
+        if (stat) {
+            if (tid < nb) {
+                S.run[tid] = a.off1[ci.side][size_t(tid) * a.nch1[ci.side] + ci.lc];
+                S.wpos[tid] = S.run[tid];
+                S.carry[tid] = 0;
+            }
+        } else if (tid < nb) {
             const uint32_t tot = S.cnt[tid];
             W* st = reinterpret_cast<W*>(a.status[ci.side]);
             const size_t me = size_t(ci.lc) * 256 + tid;
@@ -592,6 +628,10 @@ int launch_scatter(const Plan& p, int pass, const uint32_t* const keys[2], const
     a.b2 = p.b2;
     a.route_bits = p.route_bits;
     a.tile_ctr = &p.st->claim[pass - 1];
+    for (int side = 0; side < 2; ++side) {
+        a.off1[side] = (pass == 1) ? p.off1 + (side ? uint64_t(p.nch1[0]) * 256 + 1 : 0) : nullptr;
+        a.nch1[side] = p.nch1[side];
+    }
     {
         const char* e = getenv("GSH_SCATTER_DEBUG");
         a.dbg = e ? (uint32_t)atoi(e) : 0u;
