@@ -143,6 +143,9 @@ int launch_hist(const Plan& p, const uint32_t* k0, const uint32_t* k1, cudaStrea
         cudaFuncSetAttribute(k_hist2d, cudaFuncAttributeMaxDynamicSharedMemorySize, 128 * 1024);
         attr_set = true;
     }
+    // (A cluster-pair variant that hashes each key once and increments the partner's half
+    // through DSMEM atomics measured 3.6 ms vs 0.5 ms here: remote shared-memory atomics are
+    // far slower than re-hashing an L2-resident chunk.)
     k_hist2d<<<p.hist_grid, kHistBlock, smem, s>>>(k0, p.n[0], k1, p.n[1], shift, nbits, p.b2, p.hist_partial,
                                                    p.c1cnt, p.nch1[0], p.nch1[1]);
     return 1;
