@@ -24,6 +24,16 @@ __device__ __forceinline__ uint32_t hash32(uint32_t x) {
     return x;
 }
 
+// fmix32 without its final xor-shift: identical to hash32 in bits 16..31 (the last step
+// h ^= h >> 16 only changes the low half); used where only high digits are needed.
+__device__ __forceinline__ uint32_t hash32_top(uint32_t x) {
+    x ^= x >> 16;
+    x *= 0x85ebca6bu;
+    x ^= x >> 13;
+    x *= 0xc2b2ae35u;
+    return x;
+}
+
 // Checksum term of one join result tuple (a = payload_R, b = payload_S), SURVEY.md §8(c)
 // reading #2: mix64(((u64)a << 32 | b) ^ 0x9E3779B97F4A7C15), mix64 = MurmurHash3 fmix64.
 __device__ __forceinline__ uint64_t mix64(uint64_t k) {

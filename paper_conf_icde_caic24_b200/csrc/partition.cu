@@ -60,6 +60,8 @@ k_hist2d(const uint32_t* __restrict__ k0, uint64_t n0, const uint32_t* __restric
     const uint32_t F = 1u << nbits;
     const uint32_t mask = F - 1;
     const bool split = F > (1u << 15);
+    // digits above bit 16 do not see fmix32's last xor-shift (it only changes the low half)
+    const bool top16 = shift >= 16;
     const uint32_t groups = split ? gridDim.x / 2 : gridDim.x;
     const uint32_t g = split ? blockIdx.x >> 1 : blockIdx.x;
     const uint32_t nb = split ? F / 2 : F;
@@ -91,7 +93,7 @@ k_hist2d(const uint32_t* __restrict__ k0, uint64_t n0, const uint32_t* __restric
                         const uint32_t kk[4] = {v[u].x, v[u].y, v[u].z, v[u].w};
 #pragma unroll
                         for (int q = 0; q < 4; ++q) {
-                            const uint32_t bin = (hash32(kk[q]) >> shift) & mask;
+                            const uint32_t bin = ((top16 ? hash32_top(kk[q]) : hash32(kk[q])) >> shift) & mask;
                             if (bin - lo < nb) {
                                 atomicAdd(&cnt[bin - lo], 1u);
                                 atomicAdd(&c1[bin >> b2], 1u);
@@ -104,7 +106,7 @@ k_hist2d(const uint32_t* __restrict__ k0, uint64_t n0, const uint32_t* __restric
                     const uint32_t kk[4] = {v.x, v.y, v.z, v.w};
 #pragma unroll
                     for (int q = 0; q < 4; ++q) {
-                        const uint32_t bin = (hash32(kk[q]) >> shift) & mask;
+                        const uint32_t bin = ((top16 ? hash32_top(kk[q]) : hash32(kk[q])) >> shift) & mask;
                         if (bin - lo < nb) {
                             atomicAdd(&cnt[bin - lo], 1u);
                             atomicAdd(&c1[bin >> b2], 1u);
@@ -114,7 +116,7 @@ k_hist2d(const uint32_t* __restrict__ k0, uint64_t n0, const uint32_t* __restric
                 done = cb + nv * 4;
             }
             for (uint64_t j = done + threadIdx.x; j < ce; j += blockDim.x) {
-                const uint32_t bin = (hash32(keys[j]) >> shift) & mask;
+                const uint32_t bin = ((top16 ? hash32_top(keys[j]) : hash32(keys[j])) >> shift) & mask;
                 if (bin - lo < nb) {
                     atomicAdd(&cnt[bin - lo], 1u);
                     atomicAdd(&c1[bin >> b2], 1u);
