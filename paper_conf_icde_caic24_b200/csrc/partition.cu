@@ -249,10 +249,11 @@ struct ScatterSmem {
     uint32_t cnt[256];                  // chunk bucket counts (count phase)
     uint32_t tcnt[256];                 // tile bucket counters -> ranks (scatter phase)
     uint32_t local_start[256];          // bucket start inside the tile
-    unsigned long long run[256];        // next global index of bucket b for this chunk
-    unsigned long long wpos[256];       // first index of bucket b not yet written to memory
-    unsigned long long gbase[256];      // global index of stage position 0 of bucket b
-    unsigned long long endw[256];       // write-out limit of bucket b for the current tile
+    uint32_t run[256];                  // next output index of bucket b for this chunk
+    uint32_t wpos[256];                 // first index of bucket b not yet written to memory
+    uint32_t gbase[256];                // output index of stage position 0 of bucket b (mod 2^32)
+    uint32_t endw[256];                 // write-out limit of bucket b for the current tile
+    uint32_t tailpos[256];              // stage position of bucket b's carried tail
     uint2 cbuf[256][4];                 // carry: < 4 tuples (one 32 B sector) per bucket
     uint32_t carry[256];                // tuples in cbuf[b]
     uint32_t segch[2][257];             // chunk prefix over segments per side
@@ -388,6 +389,7 @@ __global__ void __launch_bounds__(BLOCK) k_scatter(ScatterArgs a) {
     const uint32_t chunks0 = S.segch[0][nseg];
     const uint32_t total = chunks0 + S.segch[1][nseg];
     uint32_t par0 = 0, par1 = 0;
+    const uint64_t wpol = policy_evict_first();
 
     for (uint32_t t = S.claim; t < total;) {
         const ChunkInfo ci = chunk_info(a, S, t, chunks0, nseg, p1);
@@ -433,7 +435,7 @@ __global__ void __launch_bounds__(BLOCK) k_scatter(ScatterArgs a) {
         // --------------------------------------- chunk-level decoupled look-back, one bucket/thread
         if (stat) {
             if (tid < nb) {
-                S.run[tid] = a.off1[ci.side][size_t(tid) * a.nch1[ci.side] + ci.lc];
+                S.run[tid] = (uint32_t)a.off1[ci.side][size_t(tid) * a.nch1[ci.side] + ci.lc];
                 S.wpos[tid] = S.run[tid];
                 S.carry[tid] = 0;
             }
@@ -468,7 +470,7 @@ __global__ void __launch_bounds__(BLOCK) k_scatter(ScatterArgs a) {
                 LB<W>::store(st + me, LB<W>::kInc | W(excl + tot));
             }
             const uint64_t pidx = ((uint64_t(ci.seg) << bits) | tid) << lowbits;
-            S.run[tid] = a.start[ci.side][pidx] + excl;
+            S.run[tid] = (uint32_t)(a.start[ci.side][pidx] + excl);
             S.wpos[tid] = S.run[tid];
             S.carry[tid] = 0;
         }
@@ -488,69 +490,98 @@ __global__ void __launch_bounds__(BLOCK) k_scatter(ScatterArgs a) {
             const uint32_t ql = umin32(TILE, ci.len - qb);
             const uint64_t tb = ci.begin + qb;
             const LoadPlan lp = load_plan(a, ci.side, tb, ql, p1);
+            const bool full = (ql == TILE) && lp.head == 0 && lp.nbulk == TILE;
             mbar_wait(&S.mbar[0], par0);
             par0 ^= 1;
             uint32_t rk[IPT / 2];  // ranks, packed 2 x u16
+            if (full) {            // whole tile arrived by TMA: no bounds or straggler checks
 #pragma unroll
-            for (int jj = 0; jj < IPT; ++jj) {
-                const uint32_t i = jj * BLOCK + tid;
-                uint32_t r = 0;
-                if (i < ql) {
-                    const bool bulk = (i - lp.head) < lp.nbulk;
+                for (int jj = 0; jj < IPT; ++jj) {
+                    const uint32_t i = jj * BLOCK + tid;
                     uint32_t h;
                     if (p1) {
-                        uint32_t k;
-                        if (bulk) {
-                            k = ok[i];
-                        } else {
-                            k = a.keys[ci.side][tb + i];
-                            op[i] = a.pays[ci.side][tb + i];
-                        }
-                        h = hash32(k);
+                        h = hash32(ok[i]);
                         ok[i] = h;
                     } else {
-                        if (bulk) {
-                            h = o2[i + lp.shift].x;
-                        } else {
-                            const uint2 e = a.in[ci.side][tb + i];
-                            o2[i + lp.shift] = e;
-                            h = e.x;
-                        }
+                        h = o2[i + lp.shift].x;
                     }
-                    r = atomicAdd(&S.tcnt[(h >> dshift) & dmask], 1u);
+                    const uint32_t r = atomicAdd(&S.tcnt[(h >> dshift) & dmask], 1u);
+                    if (jj & 1) rk[jj >> 1] |= r << 16; else rk[jj >> 1] = r;
                 }
-                if (jj & 1) rk[jj >> 1] |= r << 16; else rk[jj >> 1] = r;
+            } else {
+#pragma unroll
+                for (int jj = 0; jj < IPT; ++jj) {
+                    const uint32_t i = jj * BLOCK + tid;
+                    uint32_t r = 0;
+                    if (i < ql) {
+                        const bool bulk = (i - lp.head) < lp.nbulk;
+                        uint32_t h;
+                        if (p1) {
+                            uint32_t k;
+                            if (bulk) {
+                                k = ok[i];
+                            } else {
+                                k = a.keys[ci.side][tb + i];
+                                op[i] = a.pays[ci.side][tb + i];
+                            }
+                            h = hash32(k);
+                            ok[i] = h;
+                        } else {
+                            if (bulk) {
+                                h = o2[i + lp.shift].x;
+                            } else {
+                                const uint2 e = a.in[ci.side][tb + i];
+                                o2[i + lp.shift] = e;
+                                h = e.x;
+                            }
+                        }
+                        r = atomicAdd(&S.tcnt[(h >> dshift) & dmask], 1u);
+                    }
+                    if (jj & 1) rk[jj >> 1] |= r << 16; else rk[jj >> 1] = r;
+                }
             }
             __syncthreads();
             // Write combining: bucket b's staged run = [carry from the previous tile | this tile's
             // tuples]; only whole 32-byte sectors are written (partial-sector writes cost ~1.7x,
             // scripts/microbench_scatter_ceiling.cu), the < 4-tuple remainder carries over.
+            // Positions are u32 offsets into the side's output (n < 2^32).
             const uint32_t tc = (tid < nb) ? S.tcnt[tid] : 0u;
             const uint32_t cin = (tid < nb) ? S.carry[tid] : 0u;
             uint32_t all;
             const uint32_t lstart = block_excl_scan_u32<BLOCK>(tc + cin, &all, S.scan_tmp);
             if (tid < nb) {
-                const unsigned long long nxt = S.run[tid] + tc;
-                const unsigned long long w0 = S.wpos[tid];
-                unsigned long long ew = (q + 1 == ntile) ? nxt : (nxt & ~3ull);
+                const uint32_t nxt = S.run[tid] + tc;
+                const uint32_t w0 = S.wpos[tid];
+                uint32_t ew = (q + 1 == ntile) ? nxt : (nxt & ~3u);
                 if (ew < w0) ew = w0;
                 S.local_start[tid] = lstart + cin;
                 S.gbase[tid] = w0 - lstart;
                 S.endw[tid] = ew;
+                S.tailpos[tid] = lstart + (ew - w0);
                 for (uint32_t k = 0; k < cin; ++k) stage[lstart + k] = S.cbuf[tid][k];
                 S.wpos[tid] = ew;
                 S.run[tid] = nxt;
-                S.carry[tid] = (uint32_t)(nxt - ew);
+                S.carry[tid] = nxt - ew;
                 S.tcnt[tid] = 0;
             }
             __syncthreads();
+            if (full) {
 #pragma unroll
-            for (int jj = 0; jj < IPT; ++jj) {
-                const uint32_t i = jj * BLOCK + tid;
-                if (i < ql) {
+                for (int jj = 0; jj < IPT; ++jj) {
+                    const uint32_t i = jj * BLOCK + tid;
                     const uint2 e = p1 ? make_uint2(ok[i], op[i]) : o2[i + lp.shift];
                     const uint32_t r = (jj & 1) ? (rk[jj >> 1] >> 16) : (rk[jj >> 1] & 0xffffu);
                     stage[S.local_start[(e.x >> dshift) & dmask] + r] = e;
+                }
+            } else {
+#pragma unroll
+                for (int jj = 0; jj < IPT; ++jj) {
+                    const uint32_t i = jj * BLOCK + tid;
+                    if (i < ql) {
+                        const uint2 e = p1 ? make_uint2(ok[i], op[i]) : o2[i + lp.shift];
+                        const uint32_t r = (jj & 1) ? (rk[jj >> 1] >> 16) : (rk[jj >> 1] & 0xffffu);
+                        stage[S.local_start[(e.x >> dshift) & dmask] + r] = e;
+                    }
                 }
             }
             if (tid == 0 && q + 1 == ntile) S.claim = atomicAdd(a.tile_ctr, 1u);
@@ -559,16 +590,16 @@ __global__ void __launch_bounds__(BLOCK) k_scatter(ScatterArgs a) {
             if (tid == 0 && q + 1 < ntile)
                 tile_issue(a, ci.side, tb + TILE, umin32(TILE, ci.len - qb - TILE), p1, false,
                            ok, op, o2, &S.mbar[0]);
+            // the < 4-tuple tail of each bucket moves to its carry slot; whole sectors go out
+            if (tid < nb)
+                for (uint32_t k = 0; k < S.carry[tid]; ++k) S.cbuf[tid][k] = stage[S.tailpos[tid] + k];
             uint2* out = a.out[ci.side];
-            const uint64_t wpol = policy_evict_first();
 #pragma unroll 4
             for (uint32_t i = tid; i < all; i += BLOCK) {
                 const uint2 e = stage[i];
                 const uint32_t d = (e.x >> dshift) & dmask;
-                const unsigned long long g = S.gbase[d] + i;
-                const unsigned long long ew = S.endw[d];
-                if (g < ew) { if (!(a.dbg & 2)) st_stream_u2(out + g, e, wpol); }
-                else S.cbuf[d][g - ew] = e;
+                const uint32_t g = S.gbase[d] + i;
+                if (g < S.endw[d]) st_stream_u2(out + g, e, wpol);
             }
             __syncthreads();
         }
