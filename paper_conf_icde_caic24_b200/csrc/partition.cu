@@ -494,19 +494,29 @@ __global__ void __launch_bounds__(BLOCK) k_scatter(ScatterArgs a) {
             mbar_wait(&S.mbar[0], par0);
             par0 ^= 1;
             uint32_t rk[IPT / 2];  // ranks, packed 2 x u16
-            if (full) {            // whole tile arrived by TMA: no bounds or straggler checks
+            if (full) {  // whole tile arrived by TMA: vector shared loads, no bounds checks
+                if (p1) {    // uint4 = 4 keys; slot jj = 4 * v + c of element 4 * (v * BLOCK + tid) + c
 #pragma unroll
-                for (int jj = 0; jj < IPT; ++jj) {
-                    const uint32_t i = jj * BLOCK + tid;
-                    uint32_t h;
-                    if (p1) {
-                        h = hash32(ok[i]);
-                        ok[i] = h;
-                    } else {
-                        h = o2[i + lp.shift].x;
+                    for (int v = 0; v < IPT / 4; ++v) {
+                        uint4* k4 = reinterpret_cast<uint4*>(ok) + v * BLOCK + tid;
+                        uint4 x = *k4;
+                        x.x = hash32(x.x); x.y = hash32(x.y); x.z = hash32(x.z); x.w = hash32(x.w);
+                        *k4 = x;
+                        const uint32_t r0 = atomicAdd(&S.tcnt[(x.x >> dshift) & dmask], 1u);
+                        const uint32_t r1 = atomicAdd(&S.tcnt[(x.y >> dshift) & dmask], 1u);
+                        const uint32_t r2 = atomicAdd(&S.tcnt[(x.z >> dshift) & dmask], 1u);
+                        const uint32_t r3 = atomicAdd(&S.tcnt[(x.w >> dshift) & dmask], 1u);
+                        rk[2 * v] = r0 | (r1 << 16);
+                        rk[2 * v + 1] = r2 | (r3 << 16);
                     }
-                    const uint32_t r = atomicAdd(&S.tcnt[(h >> dshift) & dmask], 1u);
-                    if (jj & 1) rk[jj >> 1] |= r << 16; else rk[jj >> 1] = r;
+                } else {     // uint4 = 2 AoS tuples; slot jj = 2 * v + c
+#pragma unroll
+                    for (int v = 0; v < IPT / 2; ++v) {
+                        const uint4 x = reinterpret_cast<const uint4*>(o2)[v * BLOCK + tid];
+                        const uint32_t r0 = atomicAdd(&S.tcnt[(x.x >> dshift) & dmask], 1u);
+                        const uint32_t r1 = atomicAdd(&S.tcnt[(x.z >> dshift) & dmask], 1u);
+                        rk[v] = r0 | (r1 << 16);
+                    }
                 }
             } else {
 #pragma unroll
@@ -566,12 +576,25 @@ __global__ void __launch_bounds__(BLOCK) k_scatter(ScatterArgs a) {
             }
             __syncthreads();
             if (full) {
+                if (p1) {
 #pragma unroll
-                for (int jj = 0; jj < IPT; ++jj) {
-                    const uint32_t i = jj * BLOCK + tid;
-                    const uint2 e = p1 ? make_uint2(ok[i], op[i]) : o2[i + lp.shift];
-                    const uint32_t r = (jj & 1) ? (rk[jj >> 1] >> 16) : (rk[jj >> 1] & 0xffffu);
-                    stage[S.local_start[(e.x >> dshift) & dmask] + r] = e;
+                    for (int v = 0; v < IPT / 4; ++v) {
+                        const uint4 h4 = reinterpret_cast<const uint4*>(ok)[v * BLOCK + tid];
+                        const uint4 p4 = reinterpret_cast<const uint4*>(op)[v * BLOCK + tid];
+                        stage[S.local_start[(h4.x >> dshift) & dmask] + (rk[2 * v] & 0xffffu)] = make_uint2(h4.x, p4.x);
+                        stage[S.local_start[(h4.y >> dshift) & dmask] + (rk[2 * v] >> 16)] = make_uint2(h4.y, p4.y);
+                        stage[S.local_start[(h4.z >> dshift) & dmask] + (rk[2 * v + 1] & 0xffffu)] =
+                            make_uint2(h4.z, p4.z);
+                        stage[S.local_start[(h4.w >> dshift) & dmask] + (rk[2 * v + 1] >> 16)] =
+                            make_uint2(h4.w, p4.w);
+                    }
+                } else {
+#pragma unroll
+                    for (int v = 0; v < IPT / 2; ++v) {
+                        const uint4 x = reinterpret_cast<const uint4*>(o2)[v * BLOCK + tid];
+                        stage[S.local_start[(x.x >> dshift) & dmask] + (rk[v] & 0xffffu)] = make_uint2(x.x, x.y);
+                        stage[S.local_start[(x.z >> dshift) & dmask] + (rk[v] >> 16)] = make_uint2(x.z, x.w);
+                    }
                 }
             } else {
 #pragma unroll
