@@ -129,8 +129,6 @@ bool plan_build(Plan& p, uint64_t nR, uint64_t nS, const gsh_config* cfg_in, voi
     p.timing = cfg.timing;
     if (p.force_normal && p.force_heavy) return false;
     p.hist_grid = num_sms >= 2 ? (num_sms & ~1) : 2;  // even: CTA pairs share a chunk when F > 2^15
-    for (int s = 0; s < 2; ++s)
-        p.max_chunks[s] = (p.n[s] + kScatterChunk - 1) / kScatterChunk + (1u << p.b1) + 1;
     uint64_t t = next_pow2_u64(2 * (nR + nS));
     if (t < 1024) t = 1024;
     if (t > (1ull << 25)) t = 1ull << 25;
@@ -141,7 +139,10 @@ bool plan_build(Plan& p, uint64_t nR, uint64_t nS, const gsh_config* cfg_in, voi
         uint64_t hm = (nR + nS) / (p.Th ? p.Th : 1) + 1;
         p.h_max = hm < p.gt_cap_alloc ? hm : p.gt_cap_alloc;
     }
-    for (int s = 0; s < 2; ++s) p.nch1[s] = (uint32_t)((p.n[s] + kScatterChunk - 1) / kScatterChunk);
+    for (int s = 0; s < 2; ++s) {
+        p.nch1[s] = (uint32_t)((p.n[s] + kScatterChunk - 1) / kScatterChunk);
+        p.ngroups[s] = (p.nch1[s] + kGroupChunks - 1) / kGroupChunks;
+    }
     uint64_t scan_max = p.F + 1 > p.h_max + 1 ? p.F + 1 : p.h_max + 1;
     for (int s = 0; s < 2; ++s)
         if (uint64_t(p.nch1[s]) * 256 + 1 > scan_max) scan_max = uint64_t(p.nch1[s]) * 256 + 1;
@@ -161,12 +162,13 @@ bool plan_build(Plan& p, uint64_t nR, uint64_t nS, const gsh_config* cfg_in, voi
     p.bufB[1] = b ? b + nRp : nullptr;
     p.heavy_pay[0] = hp;
     p.heavy_pay[1] = hp ? hp + nR : nullptr;
-    p.hist_partial = c.take<uint32_t>(size_t(2) * p.hist_grid * F);
+    const size_t nslices = (p.nch1[0] + kSliceChunks - 1) / kSliceChunks + (p.nch1[1] + kSliceChunks - 1) / kSliceChunks;
+    p.hist_partial = c.take<uint32_t>((nslices + 1) * F);
+    p.off2 = c.take<uint32_t>((size_t(p.ngroups[0]) + p.ngroups[1] + 1) * F);
     p.c1cnt = c.take<uint32_t>((size_t(p.nch1[0]) + p.nch1[1]) * 256 + 1);
     p.off1 = c.take<uint64_t>((size_t(p.nch1[0]) + p.nch1[1]) * 256 + 2);
     p.cnt = c.take<uint32_t>(2 * F);
     p.start = c.take<uint64_t>(2 * (F + 1));
-    p.status = c.take<uint64_t>(size_t(p.max_chunks[0] + p.max_chunks[1]) * 256);
     p.gt_key = c.take<unsigned long long>(p.gt_cap_alloc);
     p.gt_cnt = c.take<uint32_t>(size_t(2) * p.gt_cap_alloc);
     p.gt_hid = c.take<uint32_t>(p.gt_cap_alloc);

@@ -12,7 +12,10 @@ namespace gsh {
 constexpr int kScatterBlock = 512;              // threads per partition-scatter CTA
 constexpr int kScatterIpt = 8;                  // tuples per thread per tile
 constexpr int kScatterTile = kScatterBlock * kScatterIpt;  // 4096 tuples per tile
-constexpr int kScatterChunk = 4 * kScatterTile;  // 16384 tuples per look-back unit
+constexpr int kScatterChunk = 4 * kScatterTile;  // 16384 input tuples per pass-1 work unit
+constexpr uint32_t kSliceChunks = 32;             // pass-1 chunks per joint-histogram slice
+constexpr uint32_t kGroupSlices = 8;              // slices per pass-2 chunk group
+constexpr uint32_t kGroupChunks = kSliceChunks * kGroupSlices;  // 256 chunks = 4M tuples
 constexpr int kMaxDigitBits = 8;                // radix bits per pass (256 buckets)
 constexpr int kMaxPartBits = 16;                // b1 + b2 <= 16 (65536 partitions)
 constexpr int kHistBlock = 1024;
@@ -63,7 +66,7 @@ struct Plan {
     int force_normal = 0, force_heavy = 0, timing = 0;
     int num_sms = 148;
     int hist_grid = 148;            // histogram CTAs (1 per SM)
-    uint64_t max_chunks[2] = {0, 0};  // look-back status rows per side
+    uint32_t ngroups[2] = {0, 0};   // pass-2 chunk groups per side
     uint32_t gt_cap_alloc = 0;      // detection table slots allocated
     uint64_t h_max = 0;             // skewed-key list capacity
     uint64_t scan_scratch_elems = 0;
@@ -72,13 +75,13 @@ struct Plan {
     uint2* bufA[2] = {nullptr, nullptr};      // pass-1 output, later normal remainders
     uint2* bufB[2] = {nullptr, nullptr};      // final partitions
     uint32_t* heavy_pay[2] = {nullptr, nullptr};  // skewed-key payload arrays
-    uint32_t* hist_partial = nullptr;         // [2][chunks][F]
+    uint32_t* hist_partial = nullptr;         // [slices side0 + side1][F] joint counts per slice
     uint32_t nch1[2] = {0, 0};                // pass-1 chunks per side
     uint32_t* c1cnt = nullptr;                // [nch1[0] + nch1[1]][256] pass-1 digit counts per chunk
     uint64_t* off1 = nullptr;                 // per side [256 * nch1 + 1] chunk/bucket output offsets
     uint32_t* cnt = nullptr;                  // [2][F]
     uint64_t* start = nullptr;                // [2][F + 1]
-    uint64_t* status = nullptr;               // [2][max_chunks][256]
+    uint32_t* off2 = nullptr;                 // per side [ngroups][F] pass-2 unit offsets
     DevState* st = nullptr;
     unsigned long long* gt_key = nullptr;     // [gt_cap_alloc]  (1 << 32 | h), 0 = empty
     uint32_t* gt_cnt = nullptr;               // [2][gt_cap_alloc]
