@@ -38,6 +38,9 @@ WORKLOADS = {
     "cfg1": ("zipf", 1 << 20, 1.0, "cfg1: |R|=|S|=2^20 Zipf theta=1.0 both sides, COUNT"),
     "zipf05": ("zipf", 1 << 27, 0.5, "cfg3 point: |R|=|S|=2^27 Zipf theta=0.5 both sides, COUNT"),
     "zipf075": ("zipf", 1 << 27, 0.75, "cfg3 point: |R|=|S|=2^27 Zipf theta=0.75 both sides, COUNT"),
+    "zipf10s": ("zipf", 1 << 24, 1.0, "cfg3-shaped (scaled): |R|=|S|=2^24 Zipf theta=1.0 both sides, COUNT"),
+    "zipf15s": ("zipf", 1 << 22, 1.5, "cfg3-shaped (scaled): |R|=|S|=2^22 Zipf theta=1.5 both sides, COUNT"),
+    "graph": ("graph", 1 << 26, 0.909, "cfg4-shaped (scaled): 2^26-edge power-law graph self-join (dst, src), COUNT"),
 }
 
 

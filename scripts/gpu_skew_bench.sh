@@ -1,5 +1,5 @@
 #!/bin/bash
-for w in cfg1 zipf05 zipf075; do
+for w in ${WL:-cfg1 zipf05 zipf075 zipf10s zipf15s graph}; do
   timeout 600 python bench.py --workload $w --steps 3 --warmup 3 --no-cpu-baseline --no-e2e > gpurun_out/skew_$w.json 2>gpurun_out/skew_$w.err
   python -c "
 import json; d=json.load(open('gpurun_out/skew_$w.json')); p=d['phases_ms']; s=d['stats']
