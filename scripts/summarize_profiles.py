@@ -62,23 +62,20 @@ lines.append(f"Kernels of other libraries in the run (data generation by torch):
              f"{len(launches) - len(ours)} launches, not part of the timed join.")
 open(os.path.join(out_dir, f"{tag}_launches.md"), "w").write("\n".join(lines) + "\n")
 
-# scatter launches alternate pass 1 / pass 2 in launch order
+# traffic per roofline kernel: from the --set full capture below (one capture per kernel, the
+# contract's definition); the launch-list DRAM columns are a fallback when present
 traffic = {}
 scat = [x for x in ours if short(x["name"]) == "k_scatter"]
 for i, key in ((0, "ms_pass1"), (1, "ms_pass2")):
     xs = scat[i::2]
-    if xs:
-        traffic[key] = sum(x.get("dram__bytes_read.sum", 0) + x.get("dram__bytes_write.sum", 0) for x in xs) / len(xs)
+    v = sum(x.get("dram__bytes_read.sum", 0) + x.get("dram__bytes_write.sum", 0) for x in xs) / max(len(xs), 1)
+    if v:
+        traffic[key] = v
 for kname, key in (("k_nmjoin", "ms_nmjoin"), ("k_hist2d", "ms_hist")):
     xs = [x for x in ours if short(x["name"]) == kname]
-    if xs:
-        traffic[key] = sum(x.get("dram__bytes_read.sum", 0) + x.get("dram__bytes_write.sum", 0) for x in xs) / len(xs)
-tpath = os.path.join(out_dir, "ncu_traffic.json")
-tj = json.load(open(tpath)) if os.path.exists(tpath) else {}
-tj[workload] = {k: v / 1e9 for k, v in traffic.items()}
-tj["_unit"] = "GB per launch (dram__bytes_read.sum + dram__bytes_write.sum), from profiles/*_launches.md runs"
-tj["_source"] = f"{tag}"
-json.dump(tj, open(tpath, "w"), indent=1)
+    v = sum(x.get("dram__bytes_read.sum", 0) + x.get("dram__bytes_write.sum", 0) for x in xs) / max(len(xs), 1)
+    if v:
+        traffic[key] = v
 
 # ------------------------------------------------------------------ full capture
 rep = os.path.join(ROOT, "gpurun_out", f"prof_{tag}.ncu-rep")
@@ -124,4 +121,23 @@ if os.path.exists(rep):
         out.append("- busiest pipes: " + ", ".join(f"{n} {v:.0f}%" for v, n in sorted(pipes, reverse=True)[:5]))
         out.append("")
     open(os.path.join(out_dir, f"{tag}_ncu_full.md"), "w").write("\n".join(out) + "\n")
+    nscat = 0
+    for r in rows[2:]:
+        k = short(r[col["Kernel Name"]])
+        b = float(r[col["dram__bytes_read.sum"]].replace(",", "")) * (1e9 if units[col["dram__bytes_read.sum"]] == "Gbyte" else 1e6 if units[col["dram__bytes_read.sum"]] == "Mbyte" else 1) + \
+            float(r[col["dram__bytes_write.sum"]].replace(",", "")) * (1e9 if units[col["dram__bytes_write.sum"]] == "Gbyte" else 1e6 if units[col["dram__bytes_write.sum"]] == "Mbyte" else 1)
+        if k == "k_scatter":
+            traffic["ms_pass1" if nscat % 2 == 0 else "ms_pass2"] = b
+            nscat += 1
+        elif k == "k_nmjoin":
+            traffic["ms_nmjoin"] = b
+        elif k == "k_hist2d":
+            traffic["ms_hist"] = b
+tpath = os.path.join(out_dir, "ncu_traffic.json")
+tj = json.load(open(tpath)) if os.path.exists(tpath) else {}
+if traffic:
+    tj[workload] = {k: v / 1e9 for k, v in traffic.items()}
+    tj["_unit"] = "GB per launch (dram__bytes_read.sum + dram__bytes_write.sum)"
+    tj["_source"] = f"profiles/{tag}_ncu_full.md (ncu --set full) / {tag}_launches.md"
+json.dump(tj, open(tpath, "w"), indent=1)
 print("wrote", [f for f in os.listdir(out_dir) if f.startswith(tag)], "traffic", tj.get(workload))
