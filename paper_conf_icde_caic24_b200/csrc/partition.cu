@@ -574,7 +574,17 @@ int launch_scatter(const Plan& p, int pass, const uint32_t* const keys[2], const
     a.b2 = p.b2;
     a.route_bits = p.route_bits;
     a.unit_ctr = &p.st->claim[pass - 1];
-    return launch_scatter_cfg<kScatterBlock, kScatterIpt>(p, a, s);
+    static int cfg = -1;
+    if (cfg < 0) {
+        const char* e = getenv("GSH_SCATTER_CFG");  // experiments only
+        cfg = e ? atoi(e) : 0;
+    }
+    switch (cfg) {
+        case 1: return launch_scatter_cfg<384, 8>(p, a, s);
+        case 2: return launch_scatter_cfg<256, 12>(p, a, s);
+        case 3: return launch_scatter_cfg<256, 16>(p, a, s);
+        default: return launch_scatter_cfg<kScatterBlock, kScatterIpt>(p, a, s);
+    }
 }
 
 // ----------------------------------------------- standalone radix histogram (ABI) --
