@@ -1,0 +1,89 @@
+"""Parity at BASELINE.json's full sizes, in bench.py's launch configuration (default config).
+
+The oracle cannot enumerate these joins in seconds, so the checks are properties that fix the
+result exactly:
+  * cfg2 (|R| = |S| = 2^27, 1:1 PK-FK): every S row matches exactly the R row whose key it copied,
+    so count = n_S and checksum = sum_j pair_hash(row_R(j), j) -- computed with the oracle's
+    pair_hash over the generator's own row map (no CUDA-path value involved);
+  * MATERIALIZE at full size: written == count, every written pair is a real match (payload =
+    row id, so R.key[a] == S.key[b]), no pair repeats, and the oracle's checksum over the written
+    pairs equals the returned checksum -- together these prove the pair multiset is M;
+  * Zipf (both sides skewed) at 2^24: count equals the closed form sum_k cnt_R(k) * cnt_S(k) from
+    exact key histograms (np.unique), and (count, checksum) are identical under configurations
+    that route the work through different phases (invariance, P4).
+"""
+import numpy as np
+import pytest
+import torch
+
+import datagen
+import oracle
+import paper_conf_icde_caic24_b200 as gsh
+
+pytestmark = pytest.mark.gpu
+
+N2 = 1 << 27
+
+
+@pytest.fixture(scope="module")
+def cfg2():
+    rk, rp, sk, sp = datagen.pkfk_pair(N2, N2, seed=0x6A5, device="cuda")
+    return rk, rp, sk, sp
+
+
+def _pkfk_expected(n_r, n_s, seed):
+    """Row of R copied by each S row (the generator's own draw, recomputed on the CPU)."""
+    idx = datagen.rand_u63(seed, 1, n_s) % n_r
+    return idx.numpy().astype(np.uint32)
+
+
+def test_cfg2_count_checksum_fullsize(cfg2):
+    rk, rp, sk, sp = cfg2
+    r = gsh.join(rk, rp, sk, sp)
+    assert r.count == N2
+    rows = _pkfk_expected(N2, N2, 0x6A5)
+    expect = 0
+    step = 1 << 24
+    for b in range(0, N2, step):
+        expect += int(np.sum(oracle.pair_hash(rows[b:b + step], np.arange(b, min(b + step, N2), dtype=np.uint32)),
+                             dtype=np.uint64))
+    assert r.checksum == expect & ((1 << 64) - 1)
+    assert r.stats["n_large"] == 0  # uniform keys never trigger detection
+
+
+def test_cfg2_materialize_fullsize(cfg2):
+    rk, rp, sk, sp = cfg2
+    r = gsh.join(rk, rp, sk, sp, mode="materialize", out_capacity=N2 + 16)
+    assert (r.count, r.written, r.overflow) == (N2, N2, False)
+    p = r.pairs.long() & 0xFFFFFFFF
+    a, b = p[:, 0], p[:, 1]
+    assert bool((rk[a] == sk[b]).all())                       # every pair matches (payload = rid)
+    packed = (a << 32) | b
+    assert torch.unique(packed).numel() == N2                 # no pair repeats
+    pc = r.pairs.cpu().numpy().view(np.uint32)
+    chk = 0
+    for s in range(0, N2, 1 << 24):
+        chk += int(np.sum(oracle.pair_hash(pc[s:s + (1 << 24), 0], pc[s:s + (1 << 24), 1]), dtype=np.uint64))
+    assert chk & ((1 << 64) - 1) == r.checksum
+
+
+def _closed_form(rk, sk):
+    ur, cr = np.unique(rk.cpu().numpy().view(np.uint32), return_counts=True)
+    us, cs = np.unique(sk.cpu().numpy().view(np.uint32), return_counts=True)
+    _, ir, is_ = np.intersect1d(ur, us, assume_unique=True, return_indices=True)
+    return int(np.sum(cr[ir].astype(np.int64) * cs[is_].astype(np.int64)))
+
+
+@pytest.mark.parametrize("theta", [0.75, 1.0])
+def test_zipf_2e24_closed_form_and_invariance(theta):
+    n = 1 << 24 if theta < 1.0 else 1 << 22
+    rk, rp, sk, sp = datagen.zipf_pair(n, n, theta, seed=31, device="cuda")
+    r = gsh.join(rk, rp, sk, sp)
+    assert r.count == _closed_form(rk, sk)
+    assert r.stats["n_heavy"] > 0
+    # every skewed key's |R_k| |S_k| goes through the dense phase; the same pairs through the
+    # NM-join (no detection) must give the identical checksum
+    r2 = gsh.join(rk, rp, sk, sp, config=gsh.make_config(force_all_normal=True))
+    assert (r2.count, r2.checksum) == (r.count, r.checksum)
+    r3 = gsh.join(rk, rp, sk, sp, config=gsh.make_config(large_threshold=1, heavy_threshold=2))
+    assert (r3.count, r3.checksum) == (r.count, r.checksum)
