@@ -261,24 +261,38 @@ def main():
     out_per_s = r.count * args.steps / (ms / 1e3)
     phases = {k: v / args.steps for k, v in phases.items()}
 
-    # roofline of the dominant kernel (pass-1 / pass-2 scatter, or the NM-join)
+    # roofline of the dominant kernel: the phase with the largest share of the step
     peak, peak_src = hbm_peak()
+    clocks = clk.summary()
     n_tot = 2 * n
-    algo = {"ms_pass1": 16 * n_tot, "ms_pass2": 16 * n_tot, "ms_nmjoin": 8 * n_tot, "ms_hist": 4 * n_tot}
-    dom = max(algo, key=lambda k: phases.get(k, 0.0))
-    achieved = algo[dom] / (phases[dom] / 1e3) / 1e9 if phases.get(dom) else None
+    st = r.stats
+    heavy_t = st.get("heavy_tuples_r", 0) + st.get("heavy_tuples_s", 0)
+    # algorithmic bytes per launch: hist 4 B, each pass 16 B, NM 8 B per normal tuple
+    algo = {"ms_hist": 4 * n_tot, "ms_pass1": 16 * n_tot, "ms_pass2": 16 * n_tot, "ms_nmjoin": 8 * (n_tot - heavy_t)}
+    kernels = {"ms_pass1": "k_scatter (pass 1)", "ms_pass2": "k_scatter (pass 2)", "ms_nmjoin": "k_nmjoin",
+               "ms_hist": "k_hist2d", "ms_skewjoin": "k_skewjoin"}
+    dom = max(list(algo) + ["ms_skewjoin"], key=lambda k: phases.get(k, 0.0))
     traffic = None
     try:
         prof = json.load(open(PROFILE_SUMMARY))
         traffic = prof.get(args.workload, {}).get(dom)
     except Exception:
         pass
-    roofline = {"bound": "hbm", "kernel": {"ms_pass1": "k_scatter (pass 1)", "ms_pass2": "k_scatter (pass 2)",
-                                             "ms_nmjoin": "k_nmjoin", "ms_hist": "k_hist2d"}[dom],
-                "achieved": achieved, "peak": peak, "peak_source": peak_src, "unit": "GB/s",
-                "frac": (achieved / peak) if achieved else None, "traffic": traffic,
-                "algorithmic_bytes_per_launch": algo[dom]}
-    clocks = clk.summary()
+    if dom == "ms_skewjoin":
+        # ALU roofline of the dense skewed-key tiles: 8 IMAD-pipe ops per pair (SASS), the IMAD
+        # pipe retires 64 lanes/clk/SM -> 8 pairs/clk/SM x 148 SMs x max SM clock
+        mhz = clocks.get("sm_max_mhz") or 1965.0
+        alu_peak = 8 * 148 * mhz * 1e6 / 1e9
+        achieved = st.get("skew_pairs", 0) / (phases[dom] / 1e3) / 1e9 if phases.get(dom) else None
+        roofline = {"bound": "alu", "kernel": kernels[dom], "achieved": achieved, "peak": alu_peak,
+                    "peak_source": "derived: 8 pairs/clk/SM (IMAD pipe) x 148 SMs x max SM clock",
+                    "unit": "Gpairs/s", "frac": (achieved / alu_peak) if achieved else None, "traffic": traffic,
+                    "algorithmic_pairs_per_launch": st.get("skew_pairs", 0)}
+    else:
+        achieved = algo[dom] / (phases[dom] / 1e3) / 1e9 if phases.get(dom) else None
+        roofline = {"bound": "hbm", "kernel": kernels[dom], "achieved": achieved, "peak": peak,
+                    "peak_source": peak_src, "unit": "GB/s", "frac": (achieved / peak) if achieved else None,
+                    "traffic": traffic, "algorithmic_bytes_per_launch": algo[dom]}
 
     # end-to-end through the public API with host buffers (H2D inside the timed region)
     e2e = None
