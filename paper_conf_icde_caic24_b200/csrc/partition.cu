@@ -52,6 +52,10 @@ __device__ __forceinline__ void hist_one(uint32_t* cnt, uint32_t key, uint32_t s
 // pass-1 digit counts, and per slice of kSliceChunks chunks the joint (d1, d2) counts: "count
 // then partition" at chunk granularity, so neither partition pass needs a
 // second read or a cross-CTA look-back -- their offsets come from scans of these counts.
+// FAST16: the 2^27..2^28-tuple shape (16 partition bits, no route bits, 8 + 8 split): bin = h >> 16,
+// the CTA's half is the top bit, the pass-1 digit h >> 24 -- a few ALU ops less per key on the
+// ALU-bound pair path.
+template <bool FAST16>
 __global__ void __launch_bounds__(kHistBlock, 1)
 k_hist2d(const uint32_t* __restrict__ k0, uint64_t n0, const uint32_t* __restrict__ k1, uint64_t n1,
          uint32_t shift, uint32_t nbits, uint32_t b2, uint32_t* __restrict__ partial, uint32_t* __restrict__ c1cnt,
@@ -69,6 +73,22 @@ k_hist2d(const uint32_t* __restrict__ k0, uint64_t n0, const uint32_t* __restric
     const uint32_t lo = split ? (blockIdx.x & 1) * nb : 0;
     const uint32_t d1lo = lo >> b2, d1n = (nb >> b2) ? (nb >> b2) : 1;
     const uint32_t ns0 = (nch0 + kSliceChunks - 1) / kSliceChunks, ns1 = (nch1 + kSliceChunks - 1) / kSliceChunks;
+    const uint32_t half = blockIdx.x & 1;
+    auto count_key = [&](uint32_t key) {
+        if (FAST16) {
+            const uint32_t h = hash32_top(key);
+            if ((h >> 31) == half) {
+                atomicAdd(&cnt[(h >> 16) & 0x7fffu], 1u);
+                atomicAdd(&c1[h >> 24], 1u);
+            }
+        } else {
+            const uint32_t bin = ((top16 ? hash32_top(key) : hash32(key)) >> shift) & mask;
+            if (bin - lo < nb) {
+                atomicAdd(&cnt[bin - lo], 1u);
+                atomicAdd(&c1[bin >> b2], 1u);
+            }
+        }
+    };
     for (uint32_t w = threadIdx.x; w < nb; w += blockDim.x) cnt[w] = 0;
     if (threadIdx.x < 256) c1[threadIdx.x] = 0;
     __syncthreads();
@@ -97,36 +117,18 @@ k_hist2d(const uint32_t* __restrict__ k0, uint64_t n0, const uint32_t* __restric
                     for (int u = 0; u < 4; ++u) {
                         const uint32_t kk[4] = {v[u].x, v[u].y, v[u].z, v[u].w};
 #pragma unroll
-                        for (int q = 0; q < 4; ++q) {
-                            const uint32_t bin = ((top16 ? hash32_top(kk[q]) : hash32(kk[q])) >> shift) & mask;
-                            if (bin - lo < nb) {
-                                atomicAdd(&cnt[bin - lo], 1u);
-                                atomicAdd(&c1[bin >> b2], 1u);
-                            }
-                        }
+                        for (int q = 0; q < 4; ++q) count_key(kk[q]);
                     }
                 }
                 for (; i < nv; i += blockDim.x) {
                     const uint4 v = ld_stream_u4(kv + i);
                     const uint32_t kk[4] = {v.x, v.y, v.z, v.w};
 #pragma unroll
-                    for (int q = 0; q < 4; ++q) {
-                        const uint32_t bin = ((top16 ? hash32_top(kk[q]) : hash32(kk[q])) >> shift) & mask;
-                        if (bin - lo < nb) {
-                            atomicAdd(&cnt[bin - lo], 1u);
-                            atomicAdd(&c1[bin >> b2], 1u);
-                        }
-                    }
+                    for (int q = 0; q < 4; ++q) count_key(kk[q]);
                 }
                 done = cb + nv * 4;
             }
-            for (uint64_t j = done + threadIdx.x; j < ce; j += blockDim.x) {
-                const uint32_t bin = ((top16 ? hash32_top(keys[j]) : hash32(keys[j])) >> shift) & mask;
-                if (bin - lo < nb) {
-                    atomicAdd(&cnt[bin - lo], 1u);
-                    atomicAdd(&c1[bin >> b2], 1u);
-                }
-            }
+            for (uint64_t j = done + threadIdx.x; j < ce; j += blockDim.x) count_key(keys[j]);
             __syncthreads();
             if (threadIdx.x < d1n) {
                 c1out[size_t(d1lo + threadIdx.x) * nch + c] = c1[d1lo + threadIdx.x];
@@ -151,14 +153,20 @@ int launch_hist(const Plan& p, const uint32_t* k0, const uint32_t* k1, cudaStrea
     const size_t smem = size_t(F > (1u << 15) ? F / 2 : F) * 4;
     static bool attr_set = false;
     if (!attr_set) {
-        cudaFuncSetAttribute(k_hist2d, cudaFuncAttributeMaxDynamicSharedMemorySize, 128 * 1024);
+        cudaFuncSetAttribute(k_hist2d<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, 128 * 1024);
+        cudaFuncSetAttribute(k_hist2d<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, 128 * 1024);
         attr_set = true;
     }
+    const bool fast16 = nbits == 16 && p.route_bits == 0 && p.b2 == 8;
     // (A cluster-pair variant that hashes each key once and increments the partner's half
     // through DSMEM atomics measured 3.6 ms vs 0.5 ms here: remote shared-memory atomics are
     // far slower than re-hashing an L2-resident chunk.)
-    k_hist2d<<<p.hist_grid, kHistBlock, smem, s>>>(k0, p.n[0], k1, p.n[1], shift, nbits, p.b2, p.hist_partial,
-                                                   p.c1cnt, p.nch1[0], p.nch1[1]);
+    if (fast16)
+        k_hist2d<true><<<p.hist_grid, kHistBlock, smem, s>>>(k0, p.n[0], k1, p.n[1], shift, nbits, p.b2,
+                                                             p.hist_partial, p.c1cnt, p.nch1[0], p.nch1[1]);
+    else
+        k_hist2d<false><<<p.hist_grid, kHistBlock, smem, s>>>(k0, p.n[0], k1, p.n[1], shift, nbits, p.b2,
+                                                              p.hist_partial, p.c1cnt, p.nch1[0], p.nch1[1]);
     return 1;
 }
 
