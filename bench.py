@@ -52,6 +52,8 @@ def parse():
     ap.add_argument("--impl", default="gsh", choices=["gsh", "reference"])
     ap.add_argument("--workload", default="cfg2", choices=sorted(WORKLOADS))
     ap.add_argument("--seed", type=int, default=0x6A5)
+    ap.add_argument("--mode", default="count", choices=["count", "materialize"])
+    ap.add_argument("--out-cap", type=int, default=1 << 30, help="MATERIALIZE output capacity (pairs)")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     return ap.parse_args()
@@ -225,9 +227,10 @@ def main():
             return sharded.join_sharded(rk, rp, sk, sp, config=cfg)
     else:
         ws = torch.empty(gsh.workspace_bytes(n, n, cfg), dtype=torch.uint8, device=dev)
+        out = torch.empty((args.out_cap, 2), dtype=torch.int32, device=dev) if args.mode == "materialize" else None
 
         def step():
-            return gsh.join(rk, rp, sk, sp, config=cfg, workspace=ws)
+            return gsh.join(rk, rp, sk, sp, mode=args.mode, out=out, config=cfg, workspace=ws)
 
     for _ in range(max(3, args.warmup)):
         r = step()
@@ -327,7 +330,7 @@ def main():
             "steps": args.steps, "warmup": max(3, args.warmup), "ms_per_step": ms / args.steps,
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32",
             "data": "synthetic (datagen, seeded)",
-            "config": {"workload": desc, "n_r": n * world, "n_s": n * world, "mode": "count",
+            "config": {"workload": desc, "n_r": n * world, "n_s": n * world, "mode": args.mode,
                        "parallelism": f"hash-sharded x{world}" if world > 1 else "single GPU",
                        "l2": "inputs 2 GiB per GPU > 126 MB L2: no flush needed", "seed": args.seed},
             "output_tuples_per_s": out_per_s, "count": r.count, "checksum": f"{r.checksum:#018x}",
