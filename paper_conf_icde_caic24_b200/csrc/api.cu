@@ -128,7 +128,7 @@ bool plan_build(Plan& p, uint64_t nR, uint64_t nS, const gsh_config* cfg_in, voi
     p.force_heavy = cfg.force_all_heavy;
     p.timing = cfg.timing;
     if (p.force_normal && p.force_heavy) return false;
-    p.hist_grid = num_sms >= 2 ? (num_sms & ~1) : 2;  // even: CTA pairs share a chunk when F > 2^15
+    p.hist_grid = num_sms;  // one 1024-thread CTA (128 KB of counters) per SM
     uint64_t t = next_pow2_u64(2 * (nR + nS));
     if (t < 1024) t = 1024;
     if (t > (1ull << 25)) t = 1ull << 25;
@@ -343,7 +343,7 @@ gsh_status gsh_join(const gsh_relation* R, const gsh_relation* S, gsh_out_mode m
     res->normal_count = hs.nm_count;
     res->normal_checksum = hs.nm_checksum;
     res->written = mat ? (hs.cursor < cap ? hs.cursor : cap) : 0;
-    res->overflow = mat ? (hs.cursor > cap ? 1u : 0u) : 0u;
+    res->overflow = mat ? (res->count > cap ? 1u : 0u) : 0u;  // items skip reserving once full
     res->heavy_tuples_r = hs.heavy_tuples[0];
     res->heavy_tuples_s = hs.heavy_tuples[1];
     res->skew_pairs = hs.skew_pairs;

@@ -3,14 +3,15 @@
 //
 // SURVEY.md §8(a) rows a1-a4:
 //   a1 k_hist2d        : h = fmix32(key); joint (d1,d2) histogram of BOTH passes from one read
-//                        of the keys (4 B/tuple).  Per-CTA packed-u16 shared-memory counters with
-//                        warp aggregation (__match_any_sync) so skewed digits do not serialise.
+//                        of the keys (4 B/tuple).  Per-CTA shared-memory counters (packed u16 with
+//                        exact wrap accounting above 2^15 bins) updated by shared-memory atomics.
 //   a2 k_hist_reduce + scans : per-partition counts and start offsets, pass-1 chunk offsets.
-//   a3/a4 k_scatter    : Onesweep-style scatter -- dynamic tile ids, per-tile bucket ranks via
-//                        __match_any_sync, decoupled look-back across tiles per bucket, tiles
-//                        staged in shared memory in bucket order, then written as contiguous
-//                        runs (coalesced 8 B AoS stores).  16 B/tuple per pass.  Pass-2 tiles
-//                        never cross a pass-1 partition; the look-back chain restarts there.
+//   a3/a4 k_scatter    : static-offset scatter -- every unit's (pass-1 chunk / pass-2 (digit,
+//                        group)) bucket offsets come from scans of the histogram, so there is no
+//                        look-back.  Tiles arrive by TMA, ranks come from ATOMS.POPC.INC, tuples
+//                        are staged in shared memory in bucket order and written as whole 32 B
+//                        sectors (a carry holds each bucket's partial sector).  16 B/tuple per
+//                        pass; pass-2 units never cross a pass-1 partition.
 #include <cstdio>
 #include <cstdlib>
 
@@ -35,26 +36,21 @@ int launch_hash(const uint32_t* keys, uint32_t* out, uint64_t n, cudaStream_t s)
 }
 
 // ------------------------------------------------------------------- a1: histogram --
-// One read of the keys yields the (d1, d2) histogram of BOTH partition passes.  Counters are
-// u32 in shared memory incremented with atomicAdd(.., 1), which sm_100a executes as a
-// warp-aggregated ATOMS.POPC.INC: lanes hitting the same bin are combined in hardware, so
-// skewed digits cost no more than spread ones (measured: ~1 SM-cycle per warp-op either way,
-// while __match_any_sync costs ~64 -- scripts/microbench_warp_ops.cu, profiles/).
-// 2^16 u32 bins do not fit one CTA (256 KB), so for F > 2^15 two CTAs read the same chunk
-// (the second read is served by L2) and each counts one half of the bins in 128 KB.
-__device__ __forceinline__ void hist_one(uint32_t* cnt, uint32_t key, uint32_t shift, uint32_t mask, uint32_t lo,
-                                         uint32_t nb) {
-    const uint32_t bin = ((hash32(key) >> shift) & mask) - lo;
-    if (bin < nb) atomicAdd(&cnt[bin], 1u);
-}
+// One read of the keys yields the (d1, d2) histogram of BOTH partition passes.
+// F <= 2^15: u32 counters in shared memory, atomicAdd(.., 1) = hardware-aggregated
+// ATOMS.POPC.INC (skewed digits cost no more than spread ones; __match_any_sync costs ~64
+// cycles -- scripts/microbench_warp_ops.cu).
+// F > 2^15 (up to 2^16 bins): packed u16 counters, two bins per 32-bit word, so ONE CTA holds
+// all bins in 128 KB and every key is hashed once.  A slice (kSliceChunks chunks, <= 2^19
+// tuples) can wrap a u16; wraps are exact to account for because all updates of a word are
+// serialised atomics whose return value shows the old word:
+//   * the lane whose increment takes a half from 0xffff to 0 sees old half == 0xffff;
+//   * a low-half wrap carries +1 into the high half -- recorded as a -1 correction of the high
+//     bin, and if that carry itself wrapped the high half (old high == 0xffff) as a high wrap.
+// true(low) = low + 65536 * wraps(low); true(high) = high + 65536 * wraps(high) - carries.
+// The (bin, delta) events of a slice (at most ~3 * 2^19 / 2^16) are applied at its flush.
+constexpr uint32_t kHistMaxEvents = 64;
 
-// The same read also yields, per pass-1 chunk (kScatterChunk consecutive tuples), the chunk's
-// pass-1 digit counts, and per slice of kSliceChunks chunks the joint (d1, d2) counts: "count
-// then partition" at chunk granularity, so neither partition pass needs a
-// second read or a cross-CTA look-back -- their offsets come from scans of these counts.
-// FAST16: the 2^27..2^28-tuple shape (16 partition bits, no route bits, 8 + 8 split): bin = h >> 16,
-// the CTA's half is the top bit, the pass-1 digit h >> 24 -- a few ALU ops less per key on the
-// ALU-bound pair path.
 template <bool FAST16>
 __global__ void __launch_bounds__(kHistBlock, 1)
 k_hist2d(const uint32_t* __restrict__ k0, uint64_t n0, const uint32_t* __restrict__ k1, uint64_t n1,
@@ -62,37 +58,51 @@ k_hist2d(const uint32_t* __restrict__ k0, uint64_t n0, const uint32_t* __restric
          uint32_t nch0, uint32_t nch1) {
     extern __shared__ uint32_t cnt[];
     __shared__ uint32_t c1[256];
+    __shared__ uint32_t ev_bin[kHistMaxEvents];
+    __shared__ int32_t ev_delta[kHistMaxEvents];
+    __shared__ uint32_t n_ev;
     const uint32_t F = 1u << nbits;
     const uint32_t mask = F - 1;
-    const bool split = F > (1u << 15);
+    const bool packed = F > (1u << 15);
     // digits above bit 16 do not see fmix32's last xor-shift (it only changes the low half)
     const bool top16 = shift >= 16;
-    const uint32_t groups = split ? gridDim.x / 2 : gridDim.x;
-    const uint32_t g = split ? blockIdx.x >> 1 : blockIdx.x;
-    const uint32_t nb = split ? F / 2 : F;
-    const uint32_t lo = split ? (blockIdx.x & 1) * nb : 0;
-    const uint32_t d1lo = lo >> b2, d1n = (nb >> b2) ? (nb >> b2) : 1;
+    const uint32_t nwords = packed ? F / 2 : F;
+    const uint32_t d1n = (F >> b2) ? (F >> b2) : 1;
     const uint32_t ns0 = (nch0 + kSliceChunks - 1) / kSliceChunks, ns1 = (nch1 + kSliceChunks - 1) / kSliceChunks;
-    const uint32_t half = blockIdx.x & 1;
-    auto count_key = [&](uint32_t key) {
-        if (FAST16) {
-            const uint32_t h = hash32_top(key);
-            if ((h >> 31) == half) {
-                atomicAdd(&cnt[(h >> 16) & 0x7fffu], 1u);
-                atomicAdd(&c1[h >> 24], 1u);
-            }
-        } else {
-            const uint32_t bin = ((top16 ? hash32_top(key) : hash32(key)) >> shift) & mask;
-            if (bin - lo < nb) {
-                atomicAdd(&cnt[bin - lo], 1u);
-                atomicAdd(&c1[bin >> b2], 1u);
+    auto event = [&](uint32_t bin, int32_t d) {
+        const uint32_t e = atomicAdd(&n_ev, 1u);
+        if (e < kHistMaxEvents) {
+            ev_bin[e] = bin;
+            ev_delta[e] = d;
+        }
+    };
+    auto count_packed = [&](uint32_t bin) {
+        const uint32_t s16 = (bin & 1u) << 4;
+        const uint32_t old = atomicAdd(&cnt[bin >> 1], 1u << s16);
+        if (((old >> s16) & 0xffffu) == 0xffffu) {  // rare: a u16 wrapped
+            event(bin, 65536);
+            if (s16 == 0) {
+                event(bin | 1u, -1);
+                if ((old >> 16) == 0xffffu) event(bin | 1u, 65536);
             }
         }
     };
-    for (uint32_t w = threadIdx.x; w < nb; w += blockDim.x) cnt[w] = 0;
+    auto count_key = [&](uint32_t key) {
+        if (FAST16) {
+            const uint32_t h = hash32_top(key);
+            count_packed(h >> 16);
+            atomicAdd(&c1[h >> 24], 1u);
+        } else {
+            const uint32_t bin = ((top16 ? hash32_top(key) : hash32(key)) >> shift) & mask;
+            if (packed) count_packed(bin); else atomicAdd(&cnt[bin], 1u);
+            atomicAdd(&c1[bin >> b2], 1u);
+        }
+    };
+    for (uint32_t w = threadIdx.x; w < nwords; w += blockDim.x) cnt[w] = 0;
     if (threadIdx.x < 256) c1[threadIdx.x] = 0;
+    if (threadIdx.x == 0) n_ev = 0;
     __syncthreads();
-    for (uint32_t it = g; it < ns0 + ns1; it += groups) {
+    for (uint32_t it = blockIdx.x; it < ns0 + ns1; it += gridDim.x) {
         const int side = it >= ns0;
         const uint32_t sl = it - (side ? ns0 : 0);
         const uint32_t* keys = side ? k1 : k0;
@@ -131,16 +141,29 @@ k_hist2d(const uint32_t* __restrict__ k0, uint64_t n0, const uint32_t* __restric
             for (uint64_t j = done + threadIdx.x; j < ce; j += blockDim.x) count_key(keys[j]);
             __syncthreads();
             if (threadIdx.x < d1n) {
-                c1out[size_t(d1lo + threadIdx.x) * nch + c] = c1[d1lo + threadIdx.x];
-                c1[d1lo + threadIdx.x] = 0;
+                c1out[size_t(threadIdx.x) * nch + c] = c1[threadIdx.x];
+                c1[threadIdx.x] = 0;
             }
             __syncthreads();
         }
-        // flush this slice's joint counts (my half of the bins) and reset
-        uint32_t* row = partial + (size_t(side ? ns0 : 0) + sl) * F + lo;
-        for (uint32_t w = threadIdx.x; w < nb; w += blockDim.x) {
-            row[w] = cnt[w];
-            cnt[w] = 0;
+        // flush this slice's joint counts and reset
+        uint32_t* row = partial + (size_t(side ? ns0 : 0) + sl) * F;
+        if (packed) {
+            for (uint32_t w = threadIdx.x; w < nwords; w += blockDim.x) {
+                const uint32_t v = cnt[w];
+                reinterpret_cast<uint2*>(row)[w] = make_uint2(v & 0xffffu, v >> 16);
+                cnt[w] = 0;
+            }
+            __syncthreads();
+            if (threadIdx.x == 0) {  // wrap corrections (rare; sequential so repeated bins add up)
+                for (uint32_t e = 0; e < umin32(n_ev, kHistMaxEvents); ++e) row[ev_bin[e]] += ev_delta[e];
+                n_ev = 0;
+            }
+        } else {
+            for (uint32_t w = threadIdx.x; w < nwords; w += blockDim.x) {
+                row[w] = cnt[w];
+                cnt[w] = 0;
+            }
         }
         __syncthreads();
     }
@@ -158,9 +181,9 @@ int launch_hist(const Plan& p, const uint32_t* k0, const uint32_t* k1, cudaStrea
         attr_set = true;
     }
     const bool fast16 = nbits == 16 && p.route_bits == 0 && p.b2 == 8;
-    // (A cluster-pair variant that hashes each key once and increments the partner's half
-    // through DSMEM atomics measured 3.6 ms vs 0.5 ms here: remote shared-memory atomics are
-    // far slower than re-hashing an L2-resident chunk.)
+    // (Rejected, kept in history: CTA pairs each counting one half of 2^16 u32 bins -- every key
+    // hashed twice, ALU-bound at 0.76 ms for 2^28 keys; a cluster pair exchanging bins through
+    // DSMEM atomics, 3.6 ms, or DSMEM loads, 1.0 ms.)
     if (fast16)
         k_hist2d<true><<<p.hist_grid, kHistBlock, smem, s>>>(k0, p.n[0], k1, p.n[1], shift, nbits, p.b2,
                                                              p.hist_partial, p.c1cnt, p.nch1[0], p.nch1[1]);

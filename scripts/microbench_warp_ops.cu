@@ -52,6 +52,21 @@ __global__ void __launch_bounds__(1024) k(uint32_t iters, uint32_t* out, uint32_
             acc += v;
         } else if (MODE == 8) {  // ATOMS.ADD no return, warp-uniform address
             atomicAdd(&sh[__shfl_sync(0xffffffffu, v, 0)], 1u);
+        } else if (MODE == 9) {  // packed u16 counters (2 bins per word), with return (wrap check)
+            const uint32_t vv = (x >> 8) & (2 * bins_mask + 1);
+            const uint32_t sh16 = (vv & 1) << 4;
+            const uint32_t old = atomicAdd(&sh[vv >> 1], 1u << sh16);
+            acc += ((old >> sh16) & 0xffffu) == 0xffffu;
+        } else if (MODE == 10) {  // packed u16, colliding (8 bins)
+            const uint32_t vv = (x >> 20) & 7;
+            const uint32_t sh16 = (vv & 1) << 4;
+            const uint32_t old = atomicAdd(&sh[vv >> 1], 1u << sh16);
+            acc += ((old >> sh16) & 0xffffu) == 0xffffu;
+        } else if (MODE == 11) {  // packed u16, all lanes one bin
+            const uint32_t old = atomicAdd(&sh[3], 1u << 16);
+            acc += (old >> 16) == 0xffffu;
+        } else if (MODE == 12) {  // u32, all lanes one bin, +1 no return
+            atomicAdd(&sh[3], 1u);
         }
     }
     __syncthreads();
@@ -68,10 +83,10 @@ int main() {
     cudaMalloc(&out, 4096 * 4);
     const char* names[] = {"match.any(16b)", "ballot-match 16b", "ballot-match 8b", "atoms.add spread",
                            "atoms.add ret spread", "atoms.add collide(8 addr)", "match+leader atom", "alu baseline",
-                           "atoms uniform addr"};
-    void (*fns[])(uint32_t, uint32_t*, uint32_t) = {k<0>, k<1>, k<2>, k<3>, k<4>, k<5>, k<6>, k<7>, k<8>};
+                           "atoms uniform addr", "packed16 ret spread", "packed16 ret collide8", "packed16 ret one bin", "atoms +1 one bin"};
+    void (*fns[])(uint32_t, uint32_t*, uint32_t) = {k<0>, k<1>, k<2>, k<3>, k<4>, k<5>, k<6>, k<7>, k<8>, k<9>, k<10>, k<11>, k<12>};
     const uint32_t iters = 4096;
-    for (int m = 0; m < 9; ++m) {
+    for (int m = 3; m < 13; ++m) {
         for (uint32_t mask : {0xffffu >> 1, 0xffu}) {
             size_t smem = size_t(mask + 1) * 4;
             cudaFuncSetAttribute(fns[m], cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);

@@ -74,6 +74,44 @@ def test_partition_phase(kind, n, theta):
         assert np.array_equal(a[np.lexsort((a[:, 1], a[:, 0]))], pr[np.lexsort((pr[:, 1], pr[:, 0]))])
 
 
+def _keys_in_bins(bins, hi, nbits):
+    """One key per requested partition digit (bits below the top `hi` of fmix32), found by scan."""
+    cand = np.arange(1, 1 << 22, dtype=np.uint32)
+    d = (oracle.fmix32(cand) << np.uint32(hi)) >> np.uint32(32 - nbits)
+    return [int(cand[np.nonzero(d == b)[0][0]]) for b in bins]
+
+
+@pytest.mark.parametrize("route_bits", [0, 1])
+def test_partition_histogram_u16_wraps(route_bits):
+    """2^16 partitions use packed u16 counters per histogram slice: digits that
+    receive >= 2^16 keys of one 2^19-tuple slice wrap, both halves of one counter word wrap, and a
+    low-half carry can wrap the high half -- offsets must still equal the oracle's exact scan."""
+    pass_bits, B = (8, 8), 16
+    ka, kb, kc = _keys_in_bins([0x1234, 0x1235, 0x7777], route_bits, B)   # ka, kb share a counter word
+    n = (1 << 20) + 77
+    g = np.random.default_rng(5)
+    keys = g.integers(0, 1 << 32, n, dtype=np.uint64).astype(np.uint32)
+    pos = g.permutation(n)
+    keys[pos[:300_000]] = ka          # > 4 wraps of the even bin
+    keys[pos[300_000:560_000]] = kb   # ~4 wraps of the odd bin, interleaved with the carries
+    keys[pos[560_000:626_000]] = kc
+    keys[: 1 << 17] = ka              # the first slice almost all one digit
+    rk = torch.from_numpy(keys.view(np.int32).copy())
+    rp = torch.arange(n, dtype=torch.int32)
+    sk, sp = rk.flip(0).contiguous(), rp.clone()
+    cfg = gsh.make_config(pass_bits=pass_bits, route_bits=route_bits)
+    part_r, part_s, off_r, off_s, bits = gsh.partition(*_dev(rk, rp, sk, sp), config=cfg)
+    assert bits == pass_bits
+    for k, off in ((rk, off_r), (sk, off_s)):
+        hist = oracle.radix_histogram(_np(k), route_bits, B)
+        assert np.array_equal(off.cpu().numpy(), np.concatenate([[0], np.cumsum(hist)]))
+    if route_bits == 0:  # the whole join over the same wrapped histogram
+        sk2 = torch.tensor(np.array([ka, kb, kc, ka, 12345, kb, 7], dtype=np.uint32).view(np.int32))
+        sp2 = torch.arange(7, dtype=torch.int32)
+        r = gsh.join(*_dev(rk, rp, sk2, sp2), config=cfg)
+        assert (r.count, r.checksum) == _oracle(rk, rp, sk2, sp2)[:2]
+
+
 @pytest.mark.parametrize("theta,n,cfg", [(1.0, 1 << 18, {}), (1.5, 1 << 17, {}), (0.75, 1 << 18, {}),
                                          (1.0, 1 << 16, {"large_threshold": 512, "heavy_threshold": 16}),
                                          (0.5, 1 << 17, {"large_threshold": 256, "heavy_threshold": 4}),
