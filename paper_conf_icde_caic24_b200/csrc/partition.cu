@@ -42,14 +42,22 @@ int launch_hash(const uint32_t* keys, uint32_t* out, uint64_t n, cudaStream_t s)
 // cycles -- scripts/microbench_warp_ops.cu).
 // F > 2^15 (up to 2^16 bins): packed u16 counters, two bins per 32-bit word, so ONE CTA holds
 // all bins in 128 KB and every key is hashed once.  A slice (kSliceChunks chunks, <= 2^19
-// tuples) can wrap a u16; wraps are exact to account for because all updates of a word are
-// serialised atomics whose return value shows the old word:
+// tuples) can wrap a u16 only if one pass-1 digit receives >= 2^16 of its keys (a joint bin
+// never holds more than its digit).  The exact per-chunk digit counts come with the same pass,
+// so a slice is counted with plain no-return atomics first; only a slice in which some digit
+// reached 2^16 (heavy skew) is recounted in exact mode, where wraps are accounted for from the
+// atomics' return values (all updates of a word are serialised, each returns the old word):
 //   * the lane whose increment takes a half from 0xffff to 0 sees old half == 0xffff;
 //   * a low-half wrap carries +1 into the high half -- recorded as a -1 correction of the high
 //     bin, and if that carry itself wrapped the high half (old high == 0xffff) as a high wrap.
 // true(low) = low + 65536 * wraps(low); true(high) = high + 65536 * wraps(high) - carries.
 // The (bin, delta) events of a slice (at most ~3 * 2^19 / 2^16) are applied at its flush.
 constexpr uint32_t kHistMaxEvents = 64;
+static_assert(kScatterChunk == 16 * kHistBlock, "a full chunk is 4 uint4 per histogram thread");
+template <bool V>
+struct BoolTag {
+    static constexpr bool value = V;
+};
 
 template <bool FAST16>
 __global__ void __launch_bounds__(kHistBlock, 1)
@@ -57,10 +65,10 @@ k_hist2d(const uint32_t* __restrict__ k0, uint64_t n0, const uint32_t* __restric
          uint32_t shift, uint32_t nbits, uint32_t b2, uint32_t* __restrict__ partial, uint32_t* __restrict__ c1cnt,
          uint32_t nch0, uint32_t nch1) {
     extern __shared__ uint32_t cnt[];
-    __shared__ uint32_t c1[256];
+    __shared__ uint32_t c1[2][256];
     __shared__ uint32_t ev_bin[kHistMaxEvents];
     __shared__ int32_t ev_delta[kHistMaxEvents];
-    __shared__ uint32_t n_ev;
+    __shared__ uint32_t n_ev, s_redo;
     const uint32_t F = 1u << nbits;
     const uint32_t mask = F - 1;
     const bool packed = F > (1u << 15);
@@ -76,10 +84,10 @@ k_hist2d(const uint32_t* __restrict__ k0, uint64_t n0, const uint32_t* __restric
             ev_delta[e] = d;
         }
     };
-    auto count_packed = [&](uint32_t bin) {
+    auto count_exact = [&](uint32_t bin) {
         const uint32_t s16 = (bin & 1u) << 4;
         const uint32_t old = atomicAdd(&cnt[bin >> 1], 1u << s16);
-        if (((old >> s16) & 0xffffu) == 0xffffu) {  // rare: a u16 wrapped
+        if (((old >> s16) & 0xffffu) == 0xffffu) {  // a u16 wrapped
             event(bin, 65536);
             if (s16 == 0) {
                 event(bin | 1u, -1);
@@ -87,20 +95,31 @@ k_hist2d(const uint32_t* __restrict__ k0, uint64_t n0, const uint32_t* __restric
             }
         }
     };
-    auto count_key = [&](uint32_t key) {
+    uint32_t* c1b = c1[0];
+    // EXACT: recount pass of a heavy slice (wrap accounting, no digit counts)
+    auto count_key = [&](uint32_t key, auto ex) {
+        constexpr bool EXACT = decltype(ex)::value;
         if (FAST16) {
             const uint32_t h = hash32_top(key);
-            count_packed(h >> 16);
-            atomicAdd(&c1[h >> 24], 1u);
+            if (EXACT) {
+                count_exact(h >> 16);
+            } else {
+                atomicAdd(&cnt[h >> 17], 1u << ((h >> 12) & 16u));
+                atomicAdd(&c1b[h >> 24], 1u);
+            }
         } else {
             const uint32_t bin = ((top16 ? hash32_top(key) : hash32(key)) >> shift) & mask;
-            if (packed) count_packed(bin); else atomicAdd(&cnt[bin], 1u);
-            atomicAdd(&c1[bin >> b2], 1u);
+            if (EXACT) {
+                count_exact(bin);
+            } else {
+                if (packed) atomicAdd(&cnt[bin >> 1], 1u << ((bin & 1u) << 4)); else atomicAdd(&cnt[bin], 1u);
+                atomicAdd(&c1b[bin >> b2], 1u);
+            }
         }
     };
     for (uint32_t w = threadIdx.x; w < nwords; w += blockDim.x) cnt[w] = 0;
-    if (threadIdx.x < 256) c1[threadIdx.x] = 0;
-    if (threadIdx.x == 0) n_ev = 0;
+    if (threadIdx.x < 512) c1[threadIdx.x >> 8][threadIdx.x & 255] = 0;
+    if (threadIdx.x == 0) n_ev = s_redo = 0;
     __syncthreads();
     for (uint32_t it = blockIdx.x; it < ns0 + ns1; it += gridDim.x) {
         const int side = it >= ns0;
@@ -110,42 +129,73 @@ k_hist2d(const uint32_t* __restrict__ k0, uint64_t n0, const uint32_t* __restric
         const uint32_t nch = side ? nch1 : nch0;
         uint32_t* c1out = c1cnt + (side ? size_t(nch0) * 256 : 0);
         const bool vec = ((reinterpret_cast<uintptr_t>(keys) & 15u) == 0);
-        const uint32_t cend = umin32((sl + 1) * kSliceChunks, nch);
-        for (uint32_t c = sl * kSliceChunks; c < cend; ++c) {
-            const uint64_t cb = uint64_t(c) * kScatterChunk;
-            const uint64_t ce = umin64(cb + kScatterChunk, n);
-            uint64_t done = cb;
-            if (vec) {
-                const uint4* kv = reinterpret_cast<const uint4*>(keys + cb);
-                const uint64_t nv = (ce - cb) / 4;
-                uint64_t i = threadIdx.x;
-                for (; i + 3ull * blockDim.x < nv; i += 4ull * blockDim.x) {
-                    uint4 v[4];
+        const uint32_t c0 = sl * kSliceChunks, cend = umin32((sl + 1) * kSliceChunks, nch);
+        uint32_t dtot = 0;  // thread d < d1n: keys of digit d in this slice
+        // Full chunks are loaded one chunk ahead (16 keys per thread in registers), so the
+        // loads of chunk c+1 are in flight while chunk c is counted and its pass-1 digit counts
+        // flushed; the two c1 buffers alternate so one barrier per chunk suffices.
+        auto run_slice = [&](auto ex) {
+            constexpr bool EXACT = decltype(ex)::value;
+            uint4 v[4];
+            auto load_chunk = [&](uint32_t c) {
+                const uint4* kv = reinterpret_cast<const uint4*>(keys + uint64_t(c) * kScatterChunk);
 #pragma unroll
-                    for (int u = 0; u < 4; ++u) v[u] = ld_stream_u4(kv + i + u * blockDim.x);
+                for (int u = 0; u < 4; ++u) v[u] = ld_stream_u4(kv + threadIdx.x + u * kHistBlock);
+            };
+            auto chunk_full = [&](uint32_t c) { return vec && uint64_t(c + 1) * kScatterChunk <= n; };
+            if (c0 < cend && chunk_full(c0)) load_chunk(c0);
+            for (uint32_t c = c0; c < cend; ++c) {
+                const uint64_t cb = uint64_t(c) * kScatterChunk;
+                const uint64_t ce = umin64(cb + kScatterChunk, n);
+                c1b = c1[c & 1];
+                if (chunk_full(c)) {
+                    uint4 cur[4];
+#pragma unroll
+                    for (int u = 0; u < 4; ++u) cur[u] = v[u];
+                    if (c + 1 < cend && chunk_full(c + 1)) load_chunk(c + 1);
 #pragma unroll
                     for (int u = 0; u < 4; ++u) {
-                        const uint32_t kk[4] = {v[u].x, v[u].y, v[u].z, v[u].w};
+                        const uint32_t kk[4] = {cur[u].x, cur[u].y, cur[u].z, cur[u].w};
 #pragma unroll
-                        for (int q = 0; q < 4; ++q) count_key(kk[q]);
+                        for (int q = 0; q < 4; ++q) count_key(kk[q], ex);
+                    }
+                } else {  // the ragged last chunk, or keys not 16-byte aligned
+                    uint64_t done = cb;
+                    if (vec) {
+                        const uint4* kv = reinterpret_cast<const uint4*>(keys + cb);
+                        const uint64_t nv = (ce - cb) / 4;
+                        for (uint64_t i = threadIdx.x; i < nv; i += blockDim.x) {
+                            const uint4 w = ld_stream_u4(kv + i);
+                            const uint32_t kk[4] = {w.x, w.y, w.z, w.w};
+#pragma unroll
+                            for (int q = 0; q < 4; ++q) count_key(kk[q], ex);
+                        }
+                        done = cb + nv * 4;
+                    }
+                    for (uint64_t j = done + threadIdx.x; j < ce; j += blockDim.x) count_key(keys[j], ex);
+                }
+                if (!EXACT) {
+                    __syncthreads();
+                    if (threadIdx.x < d1n) {
+                        const uint32_t x = c1b[threadIdx.x];
+                        c1out[size_t(threadIdx.x) * nch + c] = x;
+                        c1b[threadIdx.x] = 0;
+                        dtot += x;
                     }
                 }
-                for (; i < nv; i += blockDim.x) {
-                    const uint4 v = ld_stream_u4(kv + i);
-                    const uint32_t kk[4] = {v.x, v.y, v.z, v.w};
-#pragma unroll
-                    for (int q = 0; q < 4; ++q) count_key(kk[q]);
-                }
-                done = cb + nv * 4;
             }
-            for (uint64_t j = done + threadIdx.x; j < ce; j += blockDim.x) count_key(keys[j]);
+        };
+        run_slice(BoolTag<false>{});
+        if (packed) {
+            if (threadIdx.x < d1n && dtot >= 65536u) s_redo = 1;
             __syncthreads();
-            if (threadIdx.x < d1n) {
-                c1out[size_t(threadIdx.x) * nch + c] = c1[threadIdx.x];
-                c1[threadIdx.x] = 0;
+            if (s_redo) {  // some u16 may have wrapped: recount the slice exactly (rare, skew only)
+                for (uint32_t w = threadIdx.x; w < nwords; w += blockDim.x) cnt[w] = 0;
+                __syncthreads();
+                run_slice(BoolTag<true>{});
             }
-            __syncthreads();
         }
+        __syncthreads();
         // flush this slice's joint counts and reset
         uint32_t* row = partial + (size_t(side ? ns0 : 0) + sl) * F;
         if (packed) {
@@ -155,9 +205,10 @@ k_hist2d(const uint32_t* __restrict__ k0, uint64_t n0, const uint32_t* __restric
                 cnt[w] = 0;
             }
             __syncthreads();
-            if (threadIdx.x == 0) {  // wrap corrections (rare; sequential so repeated bins add up)
+            if (threadIdx.x == 0) {  // wrap corrections (sequential so repeated bins add up)
                 for (uint32_t e = 0; e < umin32(n_ev, kHistMaxEvents); ++e) row[ev_bin[e]] += ev_delta[e];
                 n_ev = 0;
+                s_redo = 0;
             }
         } else {
             for (uint32_t w = threadIdx.x; w < nwords; w += blockDim.x) {
@@ -354,7 +405,7 @@ __device__ __forceinline__ void tile_issue(const ScatterArgs& a, int side, uint6
     }
 }
 
-template <int BLOCK, int IPT>
+template <int BLOCK, int IPT, int PASS>
 __global__ void __launch_bounds__(BLOCK) k_scatter(ScatterArgs a) {
     constexpr int TILE = BLOCK * IPT;
     extern __shared__ __align__(128) unsigned char smem_raw[];
@@ -366,7 +417,7 @@ __global__ void __launch_bounds__(BLOCK) k_scatter(ScatterArgs a) {
     uint2* stage = reinterpret_cast<uint2*>(buf0 + (size_t(TILE) + 4) * 8);
 
     const uint32_t tid = threadIdx.x;
-    const bool p1 = (a.pass == 1);
+    constexpr bool p1 = (PASS == 1);
     const uint32_t bits = p1 ? a.b1 : a.b2;
     const uint32_t nb = 1u << bits;
     const uint32_t dmask = nb - 1;
@@ -414,17 +465,36 @@ __global__ void __launch_bounds__(BLOCK) k_scatter(ScatterArgs a) {
             const uint64_t tb = ui.begin + qb;
             const LoadPlan lp = load_plan(a, ui.side, tb, ql, p1);
             const bool full = (ql == TILE) && lp.head == 0 && lp.nbulk == TILE;
+            const bool last = (q + 1 == ntile);
+            if (tid == 0 && last) S.claim = atomicAdd(a.unit_ctr, 1u);
+            // TMA-prefetch the next tile (of this unit, or the first of the next unit) into the
+            // input buffer once this tile's input has been consumed
+            auto issue_next = [&]() {
+                if (tid == 0) {
+                    if (!last) {
+                        tile_issue(a, ui.side, tb + TILE, umin32(TILE, ui.len - qb - TILE), p1, ok, op, o2, &S.mbar,
+                                   rpol);
+                    } else if (un < total) {
+                        const UnitInfo nx = unit_info(a, un, units0, p1);
+                        if (nx.len) tile_issue(a, nx.side, nx.begin, umin32(TILE, nx.len), p1, ok, op, o2, &S.mbar, rpol);
+                    }
+                }
+            };
             mbar_wait(&S.mbar, par);
             par ^= 1;
             uint32_t rk[IPT / 2];  // ranks, packed 2 x u16
+            // full tile: the input stays in registers from the ranking to the staging step, so
+            // the input buffer is free (and the next tile's TMA issued) after the first barrier
+            constexpr int NV = p1 ? IPT / 4 : IPT / 2;
+            uint4 xa[NV], xb[p1 ? NV : 1];
             if (full) {  // whole tile arrived by TMA: vector shared loads, no bounds checks
                 if (p1) {    // uint4 = 4 keys; slot 4 * v + c of element 4 * (v * BLOCK + tid) + c
 #pragma unroll
-                    for (int v = 0; v < IPT / 4; ++v) {
-                        uint4* k4 = reinterpret_cast<uint4*>(ok) + v * BLOCK + tid;
-                        uint4 x = *k4;
+                    for (int v = 0; v < NV; ++v) {
+                        uint4 x = reinterpret_cast<const uint4*>(ok)[v * BLOCK + tid];
+                        xb[v] = reinterpret_cast<const uint4*>(op)[v * BLOCK + tid];
                         x.x = hash32(x.x); x.y = hash32(x.y); x.z = hash32(x.z); x.w = hash32(x.w);
-                        *k4 = x;
+                        xa[v] = x;
                         const uint32_t r0 = atomicAdd(&S.tcnt[(x.x >> dshift) & dmask], 1u);
                         const uint32_t r1 = atomicAdd(&S.tcnt[(x.y >> dshift) & dmask], 1u);
                         const uint32_t r2 = atomicAdd(&S.tcnt[(x.z >> dshift) & dmask], 1u);
@@ -434,13 +504,15 @@ __global__ void __launch_bounds__(BLOCK) k_scatter(ScatterArgs a) {
                     }
                 } else {     // uint4 = 2 AoS tuples; slot 2 * v + c
 #pragma unroll
-                    for (int v = 0; v < IPT / 2; ++v) {
+                    for (int v = 0; v < NV; ++v) {
                         const uint4 x = reinterpret_cast<const uint4*>(o2)[v * BLOCK + tid];
+                        xa[v] = x;
                         const uint32_t r0 = atomicAdd(&S.tcnt[(x.x >> dshift) & dmask], 1u);
                         const uint32_t r1 = atomicAdd(&S.tcnt[(x.z >> dshift) & dmask], 1u);
                         rk[v] = r0 | (r1 << 16);
                     }
                 }
+                fence_proxy_async_smem();  // reads of the input tile precede the next TMA writes
             } else {
 #pragma unroll
                 for (int jj = 0; jj < IPT; ++jj) {
@@ -474,6 +546,8 @@ __global__ void __launch_bounds__(BLOCK) k_scatter(ScatterArgs a) {
                 }
             }
             __syncthreads();
+            if (last) un = S.claim;
+            if (full) issue_next();
             // Write combining: bucket b's staged run = [carry from the previous tile | this tile's
             // tuples]; only whole 32-byte sectors are written, the < 4-tuple remainder carries
             // over (the unit's last tile flushes everything).  u32 offsets (n < 2^32).
@@ -484,7 +558,7 @@ __global__ void __launch_bounds__(BLOCK) k_scatter(ScatterArgs a) {
             if (tid < nb) {
                 const uint32_t nxt = S.run[tid] + tc;
                 const uint32_t w0 = S.wpos[tid];
-                uint32_t ew = (q + 1 == ntile) ? nxt : (nxt & ~3u);
+                uint32_t ew = last ? nxt : (nxt & ~3u);
                 if (ew < w0) ew = w0;
                 S.local_start[tid] = lstart + cin;
                 S.gbase[tid] = w0 - lstart;
@@ -500,9 +574,8 @@ __global__ void __launch_bounds__(BLOCK) k_scatter(ScatterArgs a) {
             if (full) {
                 if (p1) {
 #pragma unroll
-                    for (int v = 0; v < IPT / 4; ++v) {
-                        const uint4 h4 = reinterpret_cast<const uint4*>(ok)[v * BLOCK + tid];
-                        const uint4 p4 = reinterpret_cast<const uint4*>(op)[v * BLOCK + tid];
+                    for (int v = 0; v < NV; ++v) {
+                        const uint4 h4 = xa[v], p4 = xb[v];
                         stage[S.local_start[(h4.x >> dshift) & dmask] + (rk[2 * v] & 0xffffu)] = make_uint2(h4.x, p4.x);
                         stage[S.local_start[(h4.y >> dshift) & dmask] + (rk[2 * v] >> 16)] = make_uint2(h4.y, p4.y);
                         stage[S.local_start[(h4.z >> dshift) & dmask] + (rk[2 * v + 1] & 0xffffu)] =
@@ -512,8 +585,8 @@ __global__ void __launch_bounds__(BLOCK) k_scatter(ScatterArgs a) {
                     }
                 } else {
 #pragma unroll
-                    for (int v = 0; v < IPT / 2; ++v) {
-                        const uint4 x = reinterpret_cast<const uint4*>(o2)[v * BLOCK + tid];
+                    for (int v = 0; v < NV; ++v) {
+                        const uint4 x = xa[v];
                         stage[S.local_start[(x.x >> dshift) & dmask] + (rk[v] & 0xffffu)] = make_uint2(x.x, x.y);
                         stage[S.local_start[(x.z >> dshift) & dmask] + (rk[v] >> 16)] = make_uint2(x.z, x.w);
                     }
@@ -528,22 +601,10 @@ __global__ void __launch_bounds__(BLOCK) k_scatter(ScatterArgs a) {
                         stage[S.local_start[(e.x >> dshift) & dmask] + r] = e;
                     }
                 }
+                fence_proxy_async_smem();  // reads of the input tile precede the next TMA writes
             }
-            const bool last = (q + 1 == ntile);
-            if (tid == 0 && last) S.claim = atomicAdd(a.unit_ctr, 1u);
-            fence_proxy_async_smem();  // reads of the input tile precede the next TMA writes
             __syncthreads();
-            // TMA-prefetch the next tile (of this unit, or the first of the next unit) into the
-            // input buffer while this tile is written out from the staging buffer
-            if (last) un = S.claim;
-            if (tid == 0) {
-                if (!last) {
-                    tile_issue(a, ui.side, tb + TILE, umin32(TILE, ui.len - qb - TILE), p1, ok, op, o2, &S.mbar, rpol);
-                } else if (un < total) {
-                    const UnitInfo nx = unit_info(a, un, units0, p1);
-                    if (nx.len) tile_issue(a, nx.side, nx.begin, umin32(TILE, nx.len), p1, ok, op, o2, &S.mbar, rpol);
-                }
-            }
+            if (!full) issue_next();
             // the < 4-tuple tail of each bucket moves to its carry slot; whole sectors go out
             if (tid < nb)
                 for (uint32_t k = 0; k < S.carry[tid]; ++k) S.cbuf[tid][k] = stage[S.tailpos[tid] + k];
@@ -568,19 +629,23 @@ size_t scatter_smem_bytes(int tile) {
     return ((sizeof(ScatterSmem) + 127) & ~size_t(127)) + (size_t(tile) + 4) * 8 + (size_t(tile) + 3 * 256 + 4) * 8;
 }
 
-template <int BLOCK, int IPT>
-int launch_scatter_cfg(const Plan& p, const ScatterArgs& a, cudaStream_t s) {
+template <int BLOCK, int IPT, int PASS>
+int launch_scatter_pass(const Plan& p, const ScatterArgs& a, cudaStream_t s) {
     const size_t smem = scatter_smem_bytes(BLOCK * IPT);
     static bool attr_set = false;
     if (!attr_set) {
-        cudaFuncSetAttribute(k_scatter<BLOCK, IPT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        cudaFuncSetAttribute(k_scatter<BLOCK, IPT, PASS>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         attr_set = true;
     }
     int occ = 0;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_scatter<BLOCK, IPT>, BLOCK, smem);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_scatter<BLOCK, IPT, PASS>, BLOCK, smem);
     if (occ < 1) occ = 1;
-    k_scatter<BLOCK, IPT><<<(unsigned)(p.num_sms * occ), BLOCK, smem, s>>>(a);
+    k_scatter<BLOCK, IPT, PASS><<<(unsigned)(p.num_sms * occ), BLOCK, smem, s>>>(a);
     return 1;
+}
+template <int BLOCK, int IPT>
+int launch_scatter_cfg(const Plan& p, const ScatterArgs& a, cudaStream_t s) {
+    return a.pass == 1 ? launch_scatter_pass<BLOCK, IPT, 1>(p, a, s) : launch_scatter_pass<BLOCK, IPT, 2>(p, a, s);
 }
 
 int launch_scatter(const Plan& p, int pass, const uint32_t* const keys[2], const uint32_t* const pays[2],
