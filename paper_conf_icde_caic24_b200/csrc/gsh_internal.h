@@ -22,6 +22,21 @@ constexpr int kHistBlock = 1024;
 constexpr int kNmBlock = 256;                   // NM-join CTA
 constexpr uint32_t kMaxCapacity = 8192;         // largest NM build table (tuples)
 constexpr uint32_t kNmSlice = 8192;             // S tuples probed per NM work item
+// Streamed NM-join (nm_ring.cu): one producer warp + kRingGroups consumer groups of
+// kRingGroupWarps warps; partition pairs staged by TMA in a shared-memory byte ring.
+constexpr int kRingGroups = 2;
+constexpr int kRingGroupWarps = 15;
+constexpr int kRingThreads = 32 + kRingGroups * kRingGroupWarps * 32;
+constexpr uint32_t kRingMaxR = 4096;            // largest staged R side = most CSR buckets
+constexpr uint32_t kRingSeBytes = kRingGroups * 2 * kRingMaxR * 4;  // bucket (start, end) tables
+constexpr uint32_t kRingBytes = (kRingGroups == 1 ? 192u : 160u) * 1024u;
+// An item (R_p and S_p spans, 16-byte aligned) must fit the empty ring (every resident item is
+// being joined or queued behind one that is, so the producer only ever waits for progress);
+// half the ring keeps at least two in flight.
+constexpr uint32_t kRingItemMax = kRingBytes / 2;
+__host__ __device__ __forceinline__ bool ring_eligible(uint32_t rl, uint32_t sl) {
+    return rl > 0 && sl > 0 && rl <= kRingMaxR && (uint64_t(rl) + sl) * 8 + 32 <= kRingItemMax;
+}
 constexpr int kSkewBlock = 256;                 // skewed-key join CTA
 constexpr int kSkewSpt = 4;                     // S payloads per thread (registers)
 constexpr int kSkewTileS = kSkewBlock * kSkewSpt;  // 1024
@@ -121,6 +136,7 @@ int launch_heavy_prefix(const Plan& p, uint32_t n_heavy, uint32_t n_large, cudaS
 int launch_split(const Plan& p, uint32_t n_large, uint32_t gt_cap, cudaStream_t s);
 int launch_nm_setup(const Plan& p, uint32_t n_large, cudaStream_t s);
 int launch_nmjoin(const Plan& p, int materialize, uint32_t* pairs, uint64_t cap, cudaStream_t s);
+int launch_nmjoin_ring(const Plan& p, int materialize, uint32_t* pairs, uint64_t cap, cudaStream_t s);
 int launch_skewjoin(const Plan& p, uint32_t n_heavy, int materialize, uint32_t* pairs, uint64_t cap,
                     cudaStream_t s);
 

@@ -370,7 +370,7 @@ struct NmItems {
     __device__ uint64_t operator()(uint64_t p) const {
         const NmPart d = nm[p];
         if (d.rlen == 0 || d.slen == 0) return 0;
-        if (d.rlen <= C && d.slen <= kNmSlice) return 0;  // single item: claimed by partition id
+        if (ring_eligible(d.rlen, d.slen)) return 0;  // streamed kernel (nm_ring.cu)
         return uint64_t((d.rlen + C - 1) / C) * ((d.slen + kNmSlice - 1) / kNmSlice);
     }
 };
