@@ -94,6 +94,11 @@ typedef struct {
     uint32_t large_threshold;  /* L: a partition is large iff |R_p| > L or |S_p| > L (L107's
                                   "pre-defined threshold").  0 = auto: mean + 8 sqrt(mean),
                                   i.e. far beyond the binomial spread of a skew-free partition. */
+    int32_t nm_table;          /* NM-join shared-memory table (L115: "chained hash table").
+                                  0 = auto: chained when no partition is large and the partition
+                                  digits cover the top 16 bits of fmix32(key), else bucketized
+                                  CSR;  1 = always CSR;  2 = chained wherever possible.  The
+                                  result never depends on it. */
 } gsh_config;
 
 /* Per-call result (host struct). */
@@ -115,6 +120,7 @@ typedef struct {
     uint32_t heavy_threshold;  /* T_h actually used */
     uint32_t launches;         /* kernels launched by this call */
     uint32_t large_threshold;  /* L actually used */
+    int32_t nm_table;          /* NM-join table used by the streamed kernel: 1 = CSR, 2 = chained */
     float ms_hist, ms_pass1, ms_pass2, ms_detect, ms_split, ms_nmjoin, ms_skewjoin, ms_total;
 } gsh_result;
 

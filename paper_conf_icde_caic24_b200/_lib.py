@@ -42,6 +42,7 @@ class GshConfig(ctypes.Structure):
         ("force_all_heavy", i32),
         ("timing", i32),
         ("large_threshold", u32),
+        ("nm_table", i32),
     ]
 
 
@@ -64,6 +65,7 @@ class GshResult(ctypes.Structure):
         ("heavy_threshold", u32),
         ("launches", u32),
         ("large_threshold", u32),
+        ("nm_table", i32),
         ("ms_hist", ctypes.c_float),
         ("ms_pass1", ctypes.c_float),
         ("ms_pass2", ctypes.c_float),

@@ -127,6 +127,8 @@ bool plan_build(Plan& p, uint64_t nR, uint64_t nS, const gsh_config* cfg_in, voi
     p.force_normal = cfg.force_all_normal;
     p.force_heavy = cfg.force_all_heavy;
     p.timing = cfg.timing;
+    if (cfg.nm_table < 0 || cfg.nm_table > 2) return false;
+    p.nm_table = cfg.nm_table;
     if (p.force_normal && p.force_heavy) return false;
     p.hist_grid = num_sms;  // one 1024-thread CTA (128 KB of counters) per SM
     uint64_t t = next_pow2_u64(2 * (nR + nS));
@@ -328,6 +330,11 @@ gsh_status gsh_join(const gsh_relation* R, const gsh_relation* S, gsh_out_mode m
         launches += launch_split(p, n_large, (uint32_t)gcap, s);
         e5 = tm.mark();
     }
+    // Chained NM table (L115) when the partition digits fix the top 16 bits of h (the chain link
+    // then lives there) and, in auto mode, no partition is large (no duplicated keys that would
+    // serialise a chain walk; the CSR table flattens those across the warp).
+    p.nm_chain = (p.route_bits + p.b1 + p.b2 >= 16) && p.nm_table != 1 && (p.nm_table == 2 || n_large == 0);
+    res->nm_table = p.nm_chain ? 2 : 1;
     launches += launch_nm_setup(p, n_large, s);
     launches += launch_nmjoin(p, mat ? 1 : 0, pairs, cap, s);
     const int e6 = tm.mark();

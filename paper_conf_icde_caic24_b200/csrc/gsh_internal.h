@@ -79,6 +79,8 @@ struct Plan {
     uint32_t nm_slots = 0;          // NM build-table slots (set after classification; 0 = from C)
     uint32_t F = 1;                 // 1 << (b1 + b2)
     int force_normal = 0, force_heavy = 0, timing = 0;
+    int nm_table = 0;               // config: 0 auto, 1 CSR, 2 chained where possible
+    int nm_chain = 0;               // chosen for this call (nm_ring.cu)
     int num_sms = 148;
     int hist_grid = 148;            // histogram CTAs (1 per SM)
     uint32_t ngroups[2] = {0, 0};   // pass-2 chunk groups per side

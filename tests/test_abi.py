@@ -2,12 +2,17 @@
 declares, reports argument errors before any launch, and the Python binding mirrors the
 header's structs.  No compute calls (no GPU here)."""
 import ctypes
+import os
 import re
+import subprocess
+import tempfile
 
 import pytest
 
 import paper_conf_icde_caic24_b200 as gsh
 from paper_conf_icde_caic24_b200 import _lib
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 
 def header_functions():
@@ -38,9 +43,23 @@ def test_status_strings_and_struct_sizes():
     lib = _lib.load()
     assert lib.gsh_status_string(0) == b"GSH_OK"
     assert lib.gsh_status_string(1) == b"GSH_ERR_INVALID"
-    # gsh_result: 8 u64 + 10 u32 + 8 floats
-    assert ctypes.sizeof(_lib.GshResult) == 8 * 8 + 10 * 4 + 8 * 4
-    assert ctypes.sizeof(_lib.GshConfig) == 9 * 4
+    # the ctypes mirrors match the C compiler's layout of include/gsh.h field by field
+    src = "#include <stdio.h>\n#include <stddef.h>\n#include \"gsh.h\"\nint main(void){\n"
+    for cname, cls in (("gsh_config", _lib.GshConfig), ("gsh_result", _lib.GshResult)):
+        src += f'printf("%zu\\n", sizeof({cname}));\n'
+        for f, _ in cls._fields_:
+            src += f'printf("%zu\\n", offsetof({cname}, {f}));\n'
+    src += "return 0;}\n"
+    with tempfile.TemporaryDirectory() as d:
+        c, exe = os.path.join(d, "sz.c"), os.path.join(d, "sz")
+        open(c, "w").write(src)
+        subprocess.check_call(["gcc", "-std=c11", "-I", os.path.join(ROOT, "include"), c, "-o", exe])
+        got = [int(x) for x in subprocess.check_output([exe]).split()]
+    want = []
+    for cls in (_lib.GshConfig, _lib.GshResult):
+        want.append(ctypes.sizeof(cls))
+        want += [getattr(cls, f).offset for f, _ in cls._fields_]
+    assert got == want
     cfg = _lib.default_config()
     assert list(cfg.pass_bits) == [-1, -1] and cfg.capacity == 0
 

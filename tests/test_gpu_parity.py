@@ -235,3 +235,23 @@ def test_repeatable_bit_exact():
     a = gsh.join(rk, rp, sk, sp)
     b = gsh.join(rk, rp, sk, sp)
     assert (a.count, a.checksum) == (b.count, b.checksum)
+
+
+@pytest.mark.parametrize("kind,n,theta", [("pkfk", 1 << 20, 0.0), ("uniform", (1 << 22) + 5, 0.0),
+                                          ("zipf", 1 << 18, 0.5), ("zipf", 1 << 17, 1.0), ("graph", 1 << 17, 0.909)])
+@pytest.mark.parametrize("table", [1, 2])
+def test_join_nm_table_modes(kind, n, theta, table):
+    """The NM-join's shared-memory table -- bucketized CSR or the chained table of
+    (link in the top 16 bits of h, which the 2^16 partition digits fix) -- changes performance
+    only: COUNT and MATERIALIZE results equal the oracle's under both, including chains of
+    duplicated keys (Zipf, graph)."""
+    rk, rp, sk, sp = datagen.make_workload(kind, n, theta, seed=17)
+    on, oc, op = _oracle(rk, rp, sk, sp, pairs=True)
+    d = _dev(rk, rp, sk, sp)
+    cfg = gsh.make_config(pass_bits=(8, 8), nm_table=table)
+    r = gsh.join(*d, config=cfg)
+    assert (r.count, r.checksum) == (on, oc)
+    assert r.stats["nm_table"] == table
+    m = gsh.join(*d, mode="materialize", out_capacity=on, config=cfg)
+    assert (m.count, m.checksum, m.written) == (on, oc, on)
+    assert np.array_equal(_sorted_pairs(m.pairs), op)
