@@ -405,7 +405,9 @@ __device__ __forceinline__ void tile_issue(const ScatterArgs& a, int side, uint6
     }
 }
 
-template <int BLOCK, int IPT, int PASS>
+// TMAST: whole-sector bucket runs leave the staging buffer as TMA bulk stores (one per bucket
+// and tile, issued by the bucket's thread) instead of per-tuple stores.
+template <int BLOCK, int IPT, int PASS, bool TMAST>
 __global__ void __launch_bounds__(BLOCK) k_scatter(ScatterArgs a) {
     constexpr int TILE = BLOCK * IPT;
     extern __shared__ __align__(128) unsigned char smem_raw[];
@@ -545,6 +547,9 @@ __global__ void __launch_bounds__(BLOCK) k_scatter(ScatterArgs a) {
                     if (jj & 1) rk[jj >> 1] |= r << 16; else rk[jj >> 1] = r;
                 }
             }
+            // the previous tile's bulk stores must have read the staging buffer before any thread
+            // writes it again (after the barrier below)
+            if (TMAST && tid < nb) bulk_wait_read0();
             __syncthreads();
             if (last) un = S.claim;
             if (full) issue_next();
@@ -554,12 +559,18 @@ __global__ void __launch_bounds__(BLOCK) k_scatter(ScatterArgs a) {
             const uint32_t tc = (tid < nb) ? S.tcnt[tid] : 0u;
             const uint32_t cin = (tid < nb) ? S.carry[tid] : 0u;
             uint32_t all;
-            const uint32_t lstart = block_excl_scan_u32<BLOCK>(tc + cin, &all, S.scan_tmp);
+            // TMAST: one spare slot per bucket so the run starts at the parity of its output index
+            // (16-byte alignment of both ends of the bulk store)
+            uint32_t lstart = block_excl_scan_u32<BLOCK>(tc + cin + ((TMAST && tid < nb) ? 1u : 0u), &all, S.scan_tmp);
+            uint32_t my_w0 = 0, my_ew = 0;
             if (tid < nb) {
                 const uint32_t nxt = S.run[tid] + tc;
                 const uint32_t w0 = S.wpos[tid];
                 uint32_t ew = last ? nxt : (nxt & ~3u);
                 if (ew < w0) ew = w0;
+                if (TMAST) lstart += (lstart ^ w0) & 1u;
+                my_w0 = w0;
+                my_ew = ew;
                 S.local_start[tid] = lstart + cin;
                 S.gbase[tid] = w0 - lstart;
                 S.endw[tid] = ew;
@@ -603,18 +614,33 @@ __global__ void __launch_bounds__(BLOCK) k_scatter(ScatterArgs a) {
                 }
                 fence_proxy_async_smem();  // reads of the input tile precede the next TMA writes
             }
+            if (TMAST) fence_proxy_async_smem();  // staging writes precede the bulk stores' reads
             __syncthreads();
             if (!full) issue_next();
             // the < 4-tuple tail of each bucket moves to its carry slot; whole sectors go out
             if (tid < nb)
                 for (uint32_t k = 0; k < S.carry[tid]; ++k) S.cbuf[tid][k] = stage[S.tailpos[tid] + k];
             uint2* out = a.out[ui.side];
+            if (TMAST) {
+                // bucket tid's run [w0, ew) sits at stage[lstart ...]: an odd first index and an
+                // odd last one go out as single stores, the even-aligned middle as one bulk store
+                if (tid < nb && my_ew > my_w0) {
+                    const uint32_t hs = my_w0 & 1u;
+                    if (hs) st_stream_u2(out + my_w0, stage[lstart], wpol);
+                    const uint32_t a0 = my_w0 + hs;
+                    const uint32_t n2 = (my_ew - a0) & ~1u;
+                    if (n2) bulk_s2g_hint(out + a0, stage + lstart + hs, n2 * 8, wpol);
+                    if (a0 + n2 < my_ew) st_stream_u2(out + (my_ew - 1), stage[lstart + (my_ew - 1 - my_w0)], wpol);
+                    bulk_commit();
+                }
+            } else {
 #pragma unroll 4
-            for (uint32_t i = tid; i < all; i += BLOCK) {
-                const uint2 e = stage[i];
-                const uint32_t d = (e.x >> dshift) & dmask;
-                const uint32_t g = S.gbase[d] + i;
-                if (g < S.endw[d]) st_stream_u2(out + g, e, wpol);
+                for (uint32_t i = tid; i < all; i += BLOCK) {
+                    const uint2 e = stage[i];
+                    const uint32_t d = (e.x >> dshift) & dmask;
+                    const uint32_t g = S.gbase[d] + i;
+                    if (g < S.endw[d]) st_stream_u2(out + g, e, wpol);
+                }
             }
             __syncthreads();
         }
@@ -622,30 +648,33 @@ __global__ void __launch_bounds__(BLOCK) k_scatter(ScatterArgs a) {
         issued = true;  // the next unit's first tile (if any, and non-empty) is in flight
         if (u < total && unit_info(a, u, units0, p1).len == 0) issued = false;
     }
+    if (TMAST && tid < nb) bulk_wait0();  // shared memory must outlive the bulk stores' reads
 }
 
 size_t scatter_smem_bytes(int tile) {
     // input tile (+4 slack) and staging = tile + up to 3 carried tuples per bucket
-    return ((sizeof(ScatterSmem) + 127) & ~size_t(127)) + (size_t(tile) + 4) * 8 + (size_t(tile) + 3 * 256 + 4) * 8;
+    return ((sizeof(ScatterSmem) + 127) & ~size_t(127)) + (size_t(tile) + 4) * 8 + (size_t(tile) + 4 * 256 + 4) * 8;
 }
 
-template <int BLOCK, int IPT, int PASS>
+template <int BLOCK, int IPT, int PASS, bool TMAST>
 int launch_scatter_pass(const Plan& p, const ScatterArgs& a, cudaStream_t s) {
     const size_t smem = scatter_smem_bytes(BLOCK * IPT);
     static bool attr_set = false;
     if (!attr_set) {
-        cudaFuncSetAttribute(k_scatter<BLOCK, IPT, PASS>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        cudaFuncSetAttribute(k_scatter<BLOCK, IPT, PASS, TMAST>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             (int)smem);
         attr_set = true;
     }
     int occ = 0;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_scatter<BLOCK, IPT, PASS>, BLOCK, smem);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_scatter<BLOCK, IPT, PASS, TMAST>, BLOCK, smem);
     if (occ < 1) occ = 1;
-    k_scatter<BLOCK, IPT, PASS><<<(unsigned)(p.num_sms * occ), BLOCK, smem, s>>>(a);
+    k_scatter<BLOCK, IPT, PASS, TMAST><<<(unsigned)(p.num_sms * occ), BLOCK, smem, s>>>(a);
     return 1;
 }
-template <int BLOCK, int IPT>
+template <int BLOCK, int IPT, bool TMAST>
 int launch_scatter_cfg(const Plan& p, const ScatterArgs& a, cudaStream_t s) {
-    return a.pass == 1 ? launch_scatter_pass<BLOCK, IPT, 1>(p, a, s) : launch_scatter_pass<BLOCK, IPT, 2>(p, a, s);
+    return a.pass == 1 ? launch_scatter_pass<BLOCK, IPT, 1, TMAST>(p, a, s)
+                       : launch_scatter_pass<BLOCK, IPT, 2, TMAST>(p, a, s);
 }
 
 int launch_scatter(const Plan& p, int pass, const uint32_t* const keys[2], const uint32_t* const pays[2],
@@ -675,11 +704,11 @@ int launch_scatter(const Plan& p, int pass, const uint32_t* const keys[2], const
         const char* e = getenv("GSH_SCATTER_CFG");  // experiments only
         cfg = e ? atoi(e) : 0;
     }
+    // (TMA bulk stores per bucket run, cfg 1, measured slower on cfg2: 1.12 / 1.24 ms vs
+    // 1.06 / 1.17 ms for the per-tuple whole-sector stores -- barrier-bound, ALU 49 % vs 28 %)
     switch (cfg) {
-        case 1: return launch_scatter_cfg<384, 8>(p, a, s);
-        case 2: return launch_scatter_cfg<256, 12>(p, a, s);
-        case 3: return launch_scatter_cfg<256, 16>(p, a, s);
-        default: return launch_scatter_cfg<kScatterBlock, kScatterIpt>(p, a, s);
+        case 1: return launch_scatter_cfg<kScatterBlock, kScatterIpt, true>(p, a, s);
+        default: return launch_scatter_cfg<kScatterBlock, kScatterIpt, false>(p, a, s);
     }
 }
 

@@ -237,7 +237,7 @@ def test_repeatable_bit_exact():
     assert (a.count, a.checksum) == (b.count, b.checksum)
 
 
-@pytest.mark.parametrize("kind,n,theta", [("pkfk", 1 << 20, 0.0), ("uniform", (1 << 22) + 5, 0.0),
+@pytest.mark.parametrize("kind,n,theta", [("pkfk", 1 << 19, 0.0), ("uniform", (1 << 20) + 5, 0.0),
                                           ("zipf", 1 << 18, 0.5), ("zipf", 1 << 17, 1.0), ("graph", 1 << 17, 0.909)])
 @pytest.mark.parametrize("table", [1, 2])
 def test_join_nm_table_modes(kind, n, theta, table):
