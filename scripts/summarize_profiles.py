@@ -71,7 +71,7 @@ for i, key in ((0, "ms_pass1"), (1, "ms_pass2")):
     v = sum(x.get("dram__bytes_read.sum", 0) + x.get("dram__bytes_write.sum", 0) for x in xs) / max(len(xs), 1)
     if v:
         traffic[key] = v
-for kname, key in (("k_nmjoin", "ms_nmjoin"), ("k_hist2d", "ms_hist")):
+for kname, key in (("k_nmjoin_ring", "ms_nmjoin"), ("k_hist2d", "ms_hist")):
     xs = [x for x in ours if short(x["name"]) == kname]
     v = sum(x.get("dram__bytes_read.sum", 0) + x.get("dram__bytes_write.sum", 0) for x in xs) / max(len(xs), 1)
     if v:
@@ -129,7 +129,7 @@ if os.path.exists(rep):
         if k == "k_scatter":
             traffic["ms_pass1" if nscat % 2 == 0 else "ms_pass2"] = b
             nscat += 1
-        elif k == "k_nmjoin":
+        elif k == "k_nmjoin_ring":
             traffic["ms_nmjoin"] = b
         elif k == "k_hist2d":
             traffic["ms_hist"] = b
