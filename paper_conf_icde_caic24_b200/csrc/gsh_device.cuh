@@ -235,6 +235,31 @@ __device__ __forceinline__ void block_flush_u64x2(uint64_t a, uint64_t b, unsign
     }
 }
 
+// Block-wide exclusive scan where only the first NW warps hold non-zero values, with ONE
+// barrier: warp scans, the NW warp totals through shared memory, every thread sums the totals of
+// the warps before it (broadcast loads).  The caller must separate reuses of `smem` by a barrier.
+template <int NW>
+__device__ __forceinline__ uint32_t block_excl_scan_1bar(uint32_t v, uint32_t* total, uint32_t* smem /*NW*/) {
+    const uint32_t lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    uint32_t x = v;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t y = __shfl_up_sync(kFull, x, o);
+        if (lane >= (uint32_t)o) x += y;
+    }
+    if (lane == 31 && w < (uint32_t)NW) smem[w] = x;
+    __syncthreads();
+    uint32_t base = 0, tot = 0;
+#pragma unroll
+    for (int i = 0; i < NW; ++i) {
+        const uint32_t t = smem[i];
+        base += ((uint32_t)i < w) ? t : 0u;
+        tot += t;
+    }
+    *total = tot;
+    return base + x - v;
+}
+
 // Block-wide exclusive scan of one u32 per thread; returns exclusive prefix, *total = sum.
 template <int BLOCK>
 __device__ __forceinline__ uint32_t block_excl_scan_u32(uint32_t v, uint32_t* total, uint32_t* smem /*BLOCK/32+1*/) {

@@ -561,7 +561,7 @@ __global__ void __launch_bounds__(BLOCK) k_scatter(ScatterArgs a) {
             uint32_t all;
             // TMAST: one spare slot per bucket so the run starts at the parity of its output index
             // (16-byte alignment of both ends of the bulk store)
-            uint32_t lstart = block_excl_scan_u32<BLOCK>(tc + cin + ((TMAST && tid < nb) ? 1u : 0u), &all, S.scan_tmp);
+            uint32_t lstart = block_excl_scan_1bar<256 / 32>(tc + cin + ((TMAST && tid < nb) ? 1u : 0u), &all, S.scan_tmp);
             uint32_t my_w0 = 0, my_ew = 0;
             if (tid < nb) {
                 const uint32_t nxt = S.run[tid] + tc;
