@@ -53,6 +53,8 @@ def parse():
     ap.add_argument("--workload", default="cfg2", choices=sorted(WORKLOADS))
     ap.add_argument("--seed", type=int, default=0x6A5)
     ap.add_argument("--mode", default="count", choices=["count", "materialize"])
+    ap.add_argument("--detect", default="exact", choices=["exact", "sampled"],
+                    help="skew detection: exact counts (default) or the paper's 1%% sample + top-3 (L107, L112)")
     ap.add_argument("--out-cap", type=int, default=1 << 30, help="MATERIALIZE output capacity (pairs)")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -219,7 +221,10 @@ def main():
         dist.init_process_group("nccl", device_id=dev)
     rk, rp, sk, sp = make_data(kind, n, theta, args.seed, dev, rank)
     torch.cuda.synchronize()
-    cfg = gsh.make_config(timing=True, **json.loads(os.environ.get("GSH_BENCH_CFG", "{}")))  # experiments only
+    extra = json.loads(os.environ.get("GSH_BENCH_CFG", "{}"))  # experiments only
+    if args.detect == "sampled":
+        extra["detect_mode"] = 1
+    cfg = gsh.make_config(timing=True, **extra)
     if world > 1:
         from paper_conf_icde_caic24_b200 import sharded
 
@@ -330,7 +335,7 @@ def main():
             "steps": args.steps, "warmup": max(3, args.warmup), "ms_per_step": ms / args.steps,
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32",
             "data": "synthetic (datagen, seeded)",
-            "config": {"workload": desc, "n_r": n * world, "n_s": n * world, "mode": args.mode,
+            "config": {"workload": desc, "n_r": n * world, "n_s": n * world, "mode": args.mode, "detect": args.detect,
                        "parallelism": f"hash-sharded x{world}" if world > 1 else "single GPU",
                        "l2": "inputs 2 GiB per GPU > 126 MB L2: no flush needed", "seed": args.seed},
             "output_tuples_per_s": out_per_s, "count": r.count, "checksum": f"{r.checksum:#018x}",

@@ -99,6 +99,14 @@ typedef struct {
                                   digits cover the top 16 bits of fmix32(key), else bucketized
                                   CSR;  1 = always CSR;  2 = chained wherever possible.  The
                                   result never depends on it. */
+    int32_t detect_mode;       /* skewed-key detection in large partitions (L107, L112):
+                                  0 = exact counts of every key, skewed iff max(cnt_R, cnt_S) >= T_h
+                                  (default, R3/R4);  1 = the paper's sampling: every
+                                  sample_stride-th tuple of R_p ++ S_p goes into a linear-probing
+                                  table, the top_k most frequent sampled keys are skewed.  The
+                                  result never depends on it. */
+    uint32_t sample_stride;    /* detect_mode 1: 1 tuple in sample_stride is sampled.  0 = 100 (1 %) */
+    uint32_t top_k;            /* detect_mode 1: skewed keys per large partition.  0 = 3 (L112) */
 } gsh_config;
 
 /* Per-call result (host struct). */

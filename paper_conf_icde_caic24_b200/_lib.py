@@ -43,6 +43,9 @@ class GshConfig(ctypes.Structure):
         ("timing", i32),
         ("large_threshold", u32),
         ("nm_table", i32),
+        ("detect_mode", i32),
+        ("sample_stride", u32),
+        ("top_k", u32),
     ]
 
 

@@ -129,6 +129,11 @@ bool plan_build(Plan& p, uint64_t nR, uint64_t nS, const gsh_config* cfg_in, voi
     p.timing = cfg.timing;
     if (cfg.nm_table < 0 || cfg.nm_table > 2) return false;
     p.nm_table = cfg.nm_table;
+    if (cfg.detect_mode < 0 || cfg.detect_mode > 1) return false;
+    p.detect_mode = cfg.detect_mode;
+    p.sample_stride = cfg.sample_stride ? cfg.sample_stride : 100;
+    p.top_k = cfg.top_k ? cfg.top_k : 3;
+    if (p.top_k > 32) return false;
     if (p.force_normal && p.force_heavy) return false;
     p.hist_grid = num_sms;  // one 1024-thread CTA (128 KB of counters) per SM
     uint64_t t = next_pow2_u64(2 * (nR + nS));
@@ -226,6 +231,17 @@ gsh_status check_launch(const char* where) {
 }
 
 // Runs hist + scan + pass 1 + pass 2.  Returns kernels launched, or -1 after setting g_err.
+// Skew detection over the large partitions (L107, L112): exact counts of every key (detect_mode
+// 0), or the paper's sample + top-k per partition followed by exact counts of the chosen keys
+// (detect_mode 1); then the threshold pass that builds H.
+int run_detect(const Plan& p, uint32_t n_large, uint32_t gcap, cudaStream_t s) {
+    int l = launch_detect_prefix(p, n_large, s);
+    if (p.detect_mode == 1) l += launch_sample_topk(p, n_large, gcap, s);
+    l += launch_detect(p, n_large, gcap, s);
+    l += launch_select(p, gcap, s);
+    return l;
+}
+
 int run_partition(const Plan& p, const gsh_relation* R, const gsh_relation* S, cudaStream_t s) {
     int l = 0;
     l += launch_hist(p, R->keys, S->keys, s);
@@ -316,9 +332,7 @@ gsh_status gsh_join(const gsh_relation* R, const gsh_relation* S, gsh_out_mode m
         uint64_t gcap = next_pow2_u64(2 * (hs.large_tuples[0] + hs.large_tuples[1]));
         if (gcap < 1024) gcap = 1024;
         if (gcap > p.gt_cap_alloc) gcap = p.gt_cap_alloc;
-        launches += launch_detect_prefix(p, n_large, s);
-        launches += launch_detect(p, n_large, (uint32_t)gcap, s);
-        launches += launch_select(p, (uint32_t)gcap, s);
+        launches += run_detect(p, n_large, (uint32_t)gcap, s);
         e4 = tm.mark();
         if ((st = check_launch("detect")) != GSH_OK) return st;
         ce = cudaMemcpyAsync(&hs, p.st, sizeof(DevState), cudaMemcpyDeviceToHost, s);
@@ -488,9 +502,7 @@ gsh_status gsh_detect(const gsh_relation* R, const gsh_relation* S, const gsh_co
         uint64_t gcap = next_pow2_u64(2 * (hs.large_tuples[0] + hs.large_tuples[1]));
         if (gcap < 1024) gcap = 1024;
         if (gcap > p.gt_cap_alloc) gcap = p.gt_cap_alloc;
-        launch_detect_prefix(p, hs.n_large, s);
-        launch_detect(p, hs.n_large, (uint32_t)gcap, s);
-        launch_select(p, (uint32_t)gcap, s);
+        run_detect(p, hs.n_large, (uint32_t)gcap, s);
         if ((st = check_launch("detect")) != GSH_OK) return st;
         ce = cudaMemcpyAsync(&hs, p.st, sizeof(DevState), cudaMemcpyDeviceToHost, s);
         if (ce == cudaSuccess) ce = cudaStreamSynchronize(s);

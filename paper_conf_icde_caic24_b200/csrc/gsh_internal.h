@@ -81,6 +81,8 @@ struct Plan {
     int force_normal = 0, force_heavy = 0, timing = 0;
     int nm_table = 0;               // config: 0 auto, 1 CSR, 2 chained where possible
     int nm_chain = 0;               // chosen for this call (nm_ring.cu)
+    int detect_mode = 0;            // 0 exact counts, 1 sampled top-k (L107, L112)
+    uint32_t sample_stride = 100, top_k = 3;
     int num_sms = 148;
     int hist_grid = 148;            // histogram CTAs (1 per SM)
     uint32_t ngroups[2] = {0, 0};   // pass-2 chunk groups per side
@@ -133,6 +135,7 @@ int launch_scatter(const Plan& p, int pass, const uint32_t* const keys[2], const
 int launch_classify(const Plan& p, cudaStream_t s);
 int launch_detect_prefix(const Plan& p, uint32_t n_large, cudaStream_t s);
 int launch_detect(const Plan& p, uint32_t n_large, uint32_t gt_cap, cudaStream_t s);
+int launch_sample_topk(const Plan& p, uint32_t n_large, uint32_t gt_cap, cudaStream_t s);
 int launch_select(const Plan& p, uint32_t gt_cap, cudaStream_t s);
 int launch_heavy_prefix(const Plan& p, uint32_t n_heavy, uint32_t n_large, cudaStream_t s);
 int launch_split(const Plan& p, uint32_t n_large, uint32_t gt_cap, cudaStream_t s);

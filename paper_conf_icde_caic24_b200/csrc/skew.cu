@@ -149,6 +149,8 @@ __device__ __forceinline__ uint32_t gt_find(const unsigned long long* keys, uint
 // ------------------------------------------------------------------- a6: detect --
 constexpr int kDetBlock = 256;
 
+// FIND: count only keys already in the table (detect_mode 1: the sampled top-k keys).
+template <bool FIND>
 __global__ void __launch_bounds__(kDetBlock) k_detect(LargeView v, unsigned long long* gt_key, uint32_t* gt_cnt,
                                                      uint32_t cap_alloc, uint32_t logcap, DevState* st,
                                                      unsigned int* claim) {
@@ -170,9 +172,9 @@ __global__ void __launch_bounds__(kDetBlock) k_detect(LargeView v, unsigned long
             const unsigned long long key = valid ? ((uint64_t(side) << 32) | h) : ((2ull << 32) | lane_id());
             const uint32_t peers = __match_any_sync(kFull, key);
             if (valid && (peers & lanemask_lt()) == 0) {
-                uint32_t slot = gt_insert(gt_key, h, logcap);
+                const uint32_t slot = FIND ? gt_find(gt_key, h, logcap) : gt_insert(gt_key, h, logcap);
                 if (slot == kNoHeavy) {
-                    st->detect_overflow = 1;
+                    if (!FIND) st->detect_overflow = 1;
                 } else {
                     atomicAdd(&gt_cnt[size_t(side) * cap_alloc + slot], (uint32_t)__popc(peers));
                 }
@@ -185,12 +187,106 @@ int launch_detect(const Plan& p, uint32_t n_large, uint32_t gt_cap, cudaStream_t
     if (n_large == 0) return 0;
     uint32_t logcap = 0;
     while ((1u << logcap) < gt_cap) ++logcap;
-    cudaMemsetAsync(p.gt_key, 0, size_t(gt_cap) * sizeof(unsigned long long), s);
+    if (p.detect_mode == 0) cudaMemsetAsync(p.gt_key, 0, size_t(gt_cap) * sizeof(unsigned long long), s);
     cudaMemsetAsync(p.gt_cnt, 0, size_t(gt_cap) * sizeof(uint32_t), s);
     cudaMemsetAsync(p.gt_cnt + p.gt_cap_alloc, 0, size_t(gt_cap) * sizeof(uint32_t), s);
     LargeView v{{p.bufB[0], p.bufB[1]}, p.start, p.cnt, p.large_list, p.det_prefix, p.F, n_large};
-    k_detect<<<p.num_sms * 8, kDetBlock, 0, s>>>(v, p.gt_key, p.gt_cnt, p.gt_cap_alloc, logcap, p.st,
-                                                 &p.st->claim[2]);
+    if (p.detect_mode == 1)
+        k_detect<true><<<p.num_sms * 8, kDetBlock, 0, s>>>(v, p.gt_key, p.gt_cnt, p.gt_cap_alloc, logcap, p.st,
+                                                           &p.st->claim[2]);
+    else
+        k_detect<false><<<p.num_sms * 8, kDetBlock, 0, s>>>(v, p.gt_key, p.gt_cnt, p.gt_cap_alloc, logcap, p.st,
+                                                            &p.st->claim[2]);
+    return 1;
+}
+
+// ------------------------------------------------- a6 (paper-literal): sample + top-k --
+// "For each large partition, GSH samples (e.g., 1%) tuples to detect skewed keys.  GSH uses a
+// linear probing based hash table to compute the frequencies of sampled keys.  After sampling,
+// GSH marks the top-k most frequent keys in each large partition as the skewed key." (L107,
+// L112).  One CTA per large partition: every sample_stride-th tuple of R_p ++ S_p (positions
+// 0, stride, 2 stride, ...) is counted in a shared-memory linear-probing table; k rounds of a
+// block arg-max over (count, h) pick the top-k, which are inserted into the global table whose
+// exact counts k_detect<true> then takes.  A key whose probe sequence finds no free slot within
+// kDetectMaxProbe is dropped (a nearly full table; a large partition's sample is dominated by
+// its few skewed keys, so its distinct sampled keys are few); the choice affects
+// performance only -- split and the NM-join stay exact for any set of skewed keys.
+constexpr uint32_t kSampleSlots = 2048;
+constexpr int kSampleBlock = 256;
+
+__global__ void __launch_bounds__(kSampleBlock) k_sample_topk(LargeView v, uint32_t stride, uint32_t top_k,
+                                                             unsigned long long* gt_key, uint32_t logcap,
+                                                             DevState* st) {
+    __shared__ unsigned long long s_key[kSampleSlots];   // (1 << 32 | h), 0 = empty
+    __shared__ uint32_t s_cnt[kSampleSlots];
+    __shared__ unsigned long long s_red[kSampleBlock / 32];
+    for (uint32_t li = blockIdx.x; li < v.n_large; li += gridDim.x) {
+        for (uint32_t i = threadIdx.x; i < kSampleSlots; i += kSampleBlock) {
+            s_key[i] = 0;
+            s_cnt[i] = 0;
+        }
+        __syncthreads();
+        const uint32_t p = v.large_list[li];
+        const uint32_t cr = v.cnt[p], cs = v.cnt[v.F + p];
+        const uint64_t ns = (uint64_t(cr) + cs + stride - 1) / stride;
+        for (uint64_t k = threadIdx.x; k < ns; k += kSampleBlock) {
+            const uint64_t e = k * stride;
+            const int side = e >= cr;
+            const uint64_t off = side ? e - cr : e;
+            const uint32_t h = v.part[side][v.start[size_t(side) * (v.F + 1) + p] + off].x;
+            const unsigned long long tag = (1ull << 32) | h;
+            uint32_t slot = (h * 0x9E3779B1u) >> (32 - 11);   // linear probing (kSampleSlots = 2^11)
+            for (int probe = 0; probe < kDetectMaxProbe; ++probe) {
+                const unsigned long long cur = s_key[slot];
+                if (cur == tag) break;
+                if (cur == 0) {
+                    const unsigned long long prev = atomicCAS(&s_key[slot], 0ull, tag);
+                    if (prev == 0 || prev == tag) break;
+                }
+                slot = (slot + 1) & (kSampleSlots - 1);
+            }
+            if (s_key[slot] == tag) atomicAdd(&s_cnt[slot], 1u);
+        }
+        __syncthreads();
+        // top-k: k rounds of a block arg-max of (count << 32 | h) over the unchosen slots
+        for (uint32_t r = 0; r < top_k; ++r) {
+            unsigned long long best = 0;
+            uint32_t bslot = 0;
+            for (uint32_t i = threadIdx.x; i < kSampleSlots; i += kSampleBlock) {
+                const unsigned long long w = s_cnt[i] ? ((unsigned long long)s_cnt[i] << 32) | uint32_t(s_key[i]) : 0ull;
+                if (w > best) { best = w; bslot = i; }
+            }
+#pragma unroll
+            for (int o = 16; o > 0; o >>= 1) {
+                const unsigned long long ob = __shfl_xor_sync(kFull, best, o);
+                const uint32_t os = __shfl_xor_sync(kFull, bslot, o);
+                if (ob > best) { best = ob; bslot = os; }
+            }
+            if ((threadIdx.x & 31) == 0) s_red[threadIdx.x >> 5] = best;
+            __syncthreads();
+            unsigned long long top = 0;
+#pragma unroll
+            for (int w = 0; w < kSampleBlock / 32; ++w) top = s_red[w] > top ? s_red[w] : top;
+            if (top == 0) break;   // fewer than k distinct sampled keys (uniform across the block)
+            // the owner of the winning slot retires it and publishes the key
+            if ((threadIdx.x & 31) == 0 && best == top) {
+                s_cnt[bslot] = 0;
+                if (gt_insert(gt_key, uint32_t(top), logcap) == kNoHeavy) st->detect_overflow = 1;
+            }
+            __syncthreads();
+        }
+        __syncthreads();
+    }
+}
+
+int launch_sample_topk(const Plan& p, uint32_t n_large, uint32_t gt_cap, cudaStream_t s) {
+    if (n_large == 0) return 0;
+    uint32_t logcap = 0;
+    while ((1u << logcap) < gt_cap) ++logcap;
+    cudaMemsetAsync(p.gt_key, 0, size_t(gt_cap) * sizeof(unsigned long long), s);
+    LargeView v{{p.bufB[0], p.bufB[1]}, p.start, p.cnt, p.large_list, p.det_prefix, p.F, n_large};
+    const unsigned grid = (unsigned)umin64(n_large, uint64_t(p.num_sms) * 8);
+    k_sample_topk<<<grid, kSampleBlock, 0, s>>>(v, p.sample_stride, p.top_k, p.gt_key, logcap, p.st);
     return 1;
 }
 
@@ -224,7 +320,9 @@ int launch_select(const Plan& p, uint32_t gt_cap, cudaStream_t s) {
     const uint32_t B = p.b1 + p.b2;
     const uint32_t pshift = B ? (32 - p.route_bits - B) : 0;
     unsigned grid = (unsigned)umin64((gt_cap + 255) / 256, uint64_t(p.num_sms) * 16);
-    k_select<<<grid, 256, 0, s>>>(p.gt_key, p.gt_cnt, p.gt_hid, gt_cap, p.gt_cap_alloc, p.Th, p.force_heavy, pshift,
+    // detect_mode 1: the table holds exactly the sampled top-k keys, all skewed
+    const uint32_t th = p.detect_mode == 1 ? 1u : p.Th;
+    k_select<<<grid, 256, 0, s>>>(p.gt_key, p.gt_cnt, p.gt_hid, gt_cap, p.gt_cap_alloc, th, p.force_heavy, pshift,
                                   p.F - 1, p.F, p.H, p.part_heavy, p.st);
     return 1;
 }

@@ -255,3 +255,52 @@ def test_join_nm_table_modes(kind, n, theta, table):
     m = gsh.join(*d, mode="materialize", out_capacity=on, config=cfg)
     assert (m.count, m.checksum, m.written) == (on, oc, on)
     assert np.array_equal(_sorted_pairs(m.pairs), op)
+
+
+@pytest.mark.parametrize("theta,n", [(1.0, 1 << 18), (1.5, 1 << 17), (0.75, 1 << 18)])
+def test_sampled_detection_properties(theta, n):
+    """Paper-literal detection: a 1 % sample of each
+    large partition in a linear-probing table, its top-3 keys skewed.  Pins: every chosen key
+    lies in a large partition, at most k per partition, its counts in H are the EXACT counts
+    (np.unique), and the input's most frequent key -- which dominates its partition's sample --
+    is chosen."""
+    rk, rp, sk, sp = datagen.zipf_pair(n, n, theta, seed=3)
+    h, cr, cs, st = gsh.detect(*_dev(rk, rp, sk, sp), config=gsh.make_config(detect_mode=1))
+    B = st["pass_bits"][0] + st["pass_bits"][1]
+    L = st["large_threshold"]
+    rkn, skn = _np(rk), _np(sk)
+    szr = np.bincount(oracle.radix_digits(rkn, 0, B), minlength=1 << B)
+    szs = np.bincount(oracle.radix_digits(skn, 0, B), minlength=1 << B)
+    large = ((szr > L) | (szs > L)) & (szr > 0) & (szs > 0)
+    hh = h.numpy().astype(np.uint32)
+    assert len(hh) > 0
+    parts = (hh.astype(np.int64) >> (32 - B)) if B else np.zeros(len(hh), np.int64)
+    assert large[parts].all()
+    assert np.bincount(parts).max() <= 3
+    for side_h, got in ((oracle.fmix32(rkn), cr.numpy()), (oracle.fmix32(skn), cs.numpy())):
+        u, c = np.unique(side_h, return_counts=True)
+        idx = np.searchsorted(u, hh)
+        exact = np.where((idx < len(u)) & (u[np.minimum(idx, len(u) - 1)] == hh), c[np.minimum(idx, len(u) - 1)], 0)
+        assert np.array_equal(got, exact)
+    u, c = np.unique(oracle.fmix32(rkn), return_counts=True)
+    assert u[c.argmax()] in set(hh.tolist())
+
+
+@pytest.mark.parametrize("kind,n,theta,nmat", [("zipf", 1 << 18, 1.0, 40_000), ("zipf", 1 << 17, 1.5, 20_000),
+                                               ("zipf", 1 << 18, 0.75, 1 << 16), ("graph", 1 << 17, 0.909, 1 << 16)])
+def test_join_sampled_detection_exact(kind, n, theta, nmat):
+    """Which keys are treated as skewed changes performance only: with the sampled top-k
+    detection (normal remainders larger than C take the chunked NM-join) the join equals the
+    oracle bit-exactly: COUNT at n, MATERIALIZE at nmat (output size ~ n^2 sum p_k^2)."""
+    rk, rp, sk, sp = datagen.make_workload(kind, n, theta, seed=23)
+    on, oc, _ = _oracle(rk, rp, sk, sp)
+    cfg = gsh.make_config(detect_mode=1)
+    r = gsh.join(*_dev(rk, rp, sk, sp), config=cfg)
+    assert (r.count, r.checksum) == (on, oc)
+    assert r.stats["n_heavy"] > 0
+    rk, rp, sk, sp = datagen.make_workload(kind, nmat, theta, seed=23)
+    on, oc, op = _oracle(rk, rp, sk, sp, pairs=True)
+    d = _dev(rk, rp, sk, sp)
+    m = gsh.join(*d, mode="materialize", out_capacity=on, config=cfg)
+    assert (m.count, m.checksum, m.written) == (on, oc, on)
+    assert np.array_equal(_sorted_pairs(m.pairs), op)
