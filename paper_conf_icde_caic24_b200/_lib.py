@@ -10,7 +10,8 @@ import ctypes
 import os
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "lib", "libgsh.so")
+# GSH_LIB: experiments only (A/B builds of the same sources)
+LIB_PATH = os.environ.get("GSH_LIB") or os.path.join(_HERE, "lib", "libgsh.so")
 HEADER_PATH = os.path.join(os.path.dirname(_HERE), "include", "gsh.h")
 
 u32 = ctypes.c_uint32

@@ -14,8 +14,11 @@ constexpr int kScatterIpt = 8;                  // tuples per thread per tile
 constexpr int kScatterTile = kScatterBlock * kScatterIpt;  // 4096 tuples per tile
 constexpr int kScatterChunk = 4 * kScatterTile;  // 16384 input tuples per pass-1 work unit
 constexpr uint32_t kSliceChunks = 32;             // pass-1 chunks per joint-histogram slice
-constexpr uint32_t kGroupSlices = 8;              // slices per pass-2 chunk group
-constexpr uint32_t kGroupChunks = kSliceChunks * kGroupSlices;  // 256 chunks = 4M tuples
+#ifndef GSH_GROUP_SLICES
+#define GSH_GROUP_SLICES 16
+#endif
+constexpr uint32_t kGroupSlices = GSH_GROUP_SLICES;  // slices per pass-2 chunk group
+constexpr uint32_t kGroupChunks = kSliceChunks * kGroupSlices;  // 512 chunks = 8M tuples
 constexpr int kMaxDigitBits = 8;                // radix bits per pass (256 buckets)
 constexpr int kMaxPartBits = 16;                // b1 + b2 <= 16 (65536 partitions)
 constexpr int kHistBlock = 1024;

@@ -360,10 +360,9 @@ __device__ __forceinline__ UnitInfo unit_info(const ScatterArgs& a, uint32_t u, 
     return ui;
 }
 
-// Which tile elements arrive by TMA bulk copy: [head, head + nbulk); element i lives at shared
-// index i + shift (keeps the bulk destination 16-byte aligned).  The rest (an unaligned first
-// AoS tuple, a tail that is not a multiple of 16 bytes, or everything when the SoA inputs are
-// not 16-byte aligned) is loaded by its owning thread with ordinary loads.
+// Which tile elements arrive by TMA bulk copy (pass 1, SoA): [head, head + nbulk); element i lives
+// at shared index i + shift.  The rest (a tail that is not a multiple of 16 bytes, or everything
+// when the SoA inputs are not 16-byte aligned) is loaded by its owning thread with ordinary loads.
 struct LoadPlan {
     uint32_t head, nbulk, shift;
 };
@@ -377,31 +376,66 @@ __device__ __forceinline__ LoadPlan load_plan(const ScatterArgs& a, int side, ui
         lp.head = al ? 0 : len;
         lp.nbulk = al ? (len & ~3u) : 0;
         lp.shift = 0;
-    } else {
-        const uintptr_t ip = reinterpret_cast<uintptr_t>(a.in[side] + begin);
-        lp.head = umin32((ip & 15u) ? 1u : 0u, len);
-        lp.nbulk = (len - lp.head) & ~1u;
-        lp.shift = lp.head ? 1u : 0u;
+    } else {  // pass 2 always copies the 16-byte-aligned superset (see tile_geo)
+        lp.head = 0;
+        lp.nbulk = len;
+        lp.shift = 0;
     }
     return lp;
 }
 
-// Thread 0: arm `bar` and issue the bulk copies of tile [begin, begin + len) (read once: evict-first).
-__device__ __forceinline__ void tile_issue(const ScatterArgs& a, int side, uint64_t begin, uint32_t len, bool p1,
-                                           uint32_t* kdst, uint32_t* pdst, uint2* adst, uint64_t* bar,
-                                           uint64_t pol) {
-    const LoadPlan lp = load_plan(a, side, begin, len, p1);
+// Tile q of a unit [begin, begin + len).  Pass 1: TILE-aligned tiles of the (chunk-aligned) unit.
+// Pass 2 (AoS, 8-byte tuples): the first tile is one tuple shorter when `begin` is odd, so every
+// tile's 16-byte-aligned superset [tb - off, tb + ql rounded up to even) holds at most TILE tuples
+// and arrives by ONE bulk copy; the superset's extra (neighbouring units') tuples are masked.  The
+// workspace keeps >= 1 tuple of slack after each side, so the round-up never leaves it.
+struct TileGeo {
+    uint64_t tb;
+    uint32_t ql, off;
+};
+
+template <int TILE>
+__device__ __forceinline__ uint32_t tile_count(bool p1, uint64_t begin, uint32_t len) {
+    return p1 ? (len + TILE - 1) / TILE : (len + uint32_t(begin & 1) + TILE - 1) / TILE;
+}
+
+template <int TILE>
+__device__ __forceinline__ TileGeo tile_geo(bool p1, uint64_t begin, uint32_t len, uint32_t q) {
+    TileGeo g;
     if (p1) {
+        g.tb = begin + uint64_t(q) * TILE;
+        g.ql = umin32(TILE, len - q * TILE);
+        g.off = 0;
+    } else {
+        const uint32_t lead = uint32_t(begin & 1);
+        if (q == 0) {
+            g.tb = begin;
+            g.ql = umin32(TILE - lead, len);
+            g.off = lead;
+        } else {
+            g.tb = begin - lead + uint64_t(q) * TILE;
+            g.ql = (uint32_t)umin64(TILE, begin + len - g.tb);
+            g.off = 0;
+        }
+    }
+    return g;
+}
+
+// Thread 0: arm `bar` and issue the bulk copies of tile g (read once: evict-first).
+__device__ __forceinline__ void tile_issue(const ScatterArgs& a, int side, const TileGeo& g, bool p1, uint32_t* kdst,
+                                           uint32_t* pdst, uint2* adst, uint64_t* bar, uint64_t pol) {
+    if (p1) {
+        const LoadPlan lp = load_plan(a, side, g.tb, g.ql, p1);
         const uint32_t bytes = lp.nbulk * 4;
         mbar_arrive_expect_tx(bar, 2 * bytes);
         if (bytes) {
-            bulk_g2s_hint(kdst, a.keys[side] + begin, bytes, bar, pol);
-            bulk_g2s_hint(pdst, a.pays[side] + begin, bytes, bar, pol);
+            bulk_g2s_hint(kdst, a.keys[side] + g.tb, bytes, bar, pol);
+            bulk_g2s_hint(pdst, a.pays[side] + g.tb, bytes, bar, pol);
         }
     } else {
-        const uint32_t bytes = lp.nbulk * 8;
+        const uint32_t bytes = ((g.ql + g.off + 1) & ~1u) * 8;
         mbar_arrive_expect_tx(bar, bytes);
-        if (bytes) bulk_g2s_hint(adst + lp.head + lp.shift, a.in[side] + begin + lp.head, bytes, bar, pol);
+        if (bytes) bulk_g2s_hint(adst, a.in[side] + (g.tb - g.off), bytes, bar, pol);
     }
 }
 
@@ -410,6 +444,7 @@ __device__ __forceinline__ void tile_issue(const ScatterArgs& a, int side, uint6
 template <int BLOCK, int IPT, int PASS, bool TMAST>
 __global__ void __launch_bounds__(BLOCK) k_scatter(ScatterArgs a) {
     constexpr int TILE = BLOCK * IPT;
+    static_assert(TILE < 0xffff, "ranks are packed as u16 with 0xffff = masked");
     extern __shared__ __align__(128) unsigned char smem_raw[];
     ScatterSmem& S = *reinterpret_cast<ScatterSmem*>(smem_raw);
     unsigned char* buf0 = smem_raw + ((sizeof(ScatterSmem) + 127) & ~size_t(127));
@@ -440,7 +475,7 @@ __global__ void __launch_bounds__(BLOCK) k_scatter(ScatterArgs a) {
     bool issued = false;   // first tile of unit u already in flight
     while (u < total) {
         const UnitInfo ui = unit_info(a, u, units0, p1);
-        const uint32_t ntile = (ui.len + TILE - 1) / TILE;
+        const uint32_t ntile = tile_count<TILE>(p1, ui.begin, ui.len);
         if (ntile == 0) {  // empty unit (pass 2: digit absent from the group)
             __syncthreads();
             if (tid == 0) S.claim = atomicAdd(a.unit_ctr, 1u);
@@ -449,7 +484,7 @@ __global__ void __launch_bounds__(BLOCK) k_scatter(ScatterArgs a) {
             continue;
         }
         if (tid == 0 && !issued)
-            tile_issue(a, ui.side, ui.begin, umin32(TILE, ui.len), p1, ok, op, o2, &S.mbar, rpol);
+            tile_issue(a, ui.side, tile_geo<TILE>(p1, ui.begin, ui.len, 0), p1, ok, op, o2, &S.mbar, rpol);
         if (tid < nb) {
             uint32_t r0;
             const uint32_t pidx = ((ui.d1 << bits) | tid) << lowbits;
@@ -462,11 +497,12 @@ __global__ void __launch_bounds__(BLOCK) k_scatter(ScatterArgs a) {
         // (the first sync of the tile loop orders run[] before its use)
         uint32_t un = total;
         for (uint32_t q = 0; q < ntile; ++q) {
-            const uint32_t qb = q * TILE;
-            const uint32_t ql = umin32(TILE, ui.len - qb);
-            const uint64_t tb = ui.begin + qb;
+            const TileGeo geo = tile_geo<TILE>(p1, ui.begin, ui.len, q);
+            const uint32_t ql = geo.ql;
+            const uint64_t tb = geo.tb;
             const LoadPlan lp = load_plan(a, ui.side, tb, ql, p1);
-            const bool full = (ql == TILE) && lp.head == 0 && lp.nbulk == TILE;
+            // pass 2 always takes the vector path (masked superset); pass 1 when the tile is whole
+            const bool full = !p1 || ((ql == TILE) && lp.head == 0 && lp.nbulk == TILE);
             const bool last = (q + 1 == ntile);
             if (tid == 0 && last) S.claim = atomicAdd(a.unit_ctr, 1u);
             // TMA-prefetch the next tile (of this unit, or the first of the next unit) into the
@@ -474,11 +510,13 @@ __global__ void __launch_bounds__(BLOCK) k_scatter(ScatterArgs a) {
             auto issue_next = [&]() {
                 if (tid == 0) {
                     if (!last) {
-                        tile_issue(a, ui.side, tb + TILE, umin32(TILE, ui.len - qb - TILE), p1, ok, op, o2, &S.mbar,
+                        tile_issue(a, ui.side, tile_geo<TILE>(p1, ui.begin, ui.len, q + 1), p1, ok, op, o2, &S.mbar,
                                    rpol);
                     } else if (un < total) {
                         const UnitInfo nx = unit_info(a, un, units0, p1);
-                        if (nx.len) tile_issue(a, nx.side, nx.begin, umin32(TILE, nx.len), p1, ok, op, o2, &S.mbar, rpol);
+                        if (nx.len)
+                            tile_issue(a, nx.side, tile_geo<TILE>(p1, nx.begin, nx.len, 0), p1, ok, op, o2, &S.mbar,
+                                       rpol);
                     }
                 }
             };
@@ -504,13 +542,15 @@ __global__ void __launch_bounds__(BLOCK) k_scatter(ScatterArgs a) {
                         rk[2 * v] = r0 | (r1 << 16);
                         rk[2 * v + 1] = r2 | (r3 << 16);
                     }
-                } else {     // uint4 = 2 AoS tuples; slot 2 * v + c
+                } else {     // uint4 = 2 AoS tuples: shared slots 2u, 2u + 1 = tile elements 2u - off, ...
 #pragma unroll
                     for (int v = 0; v < NV; ++v) {
+                        const uint32_t i0 = 2 * (v * BLOCK + tid) - geo.off;   // wraps for slot 0 when off = 1
                         const uint4 x = reinterpret_cast<const uint4*>(o2)[v * BLOCK + tid];
                         xa[v] = x;
-                        const uint32_t r0 = atomicAdd(&S.tcnt[(x.x >> dshift) & dmask], 1u);
-                        const uint32_t r1 = atomicAdd(&S.tcnt[(x.z >> dshift) & dmask], 1u);
+                        uint32_t r0 = 0xffffu, r1 = 0xffffu;   // 0xffff = not in this tile
+                        if (i0 < ql) r0 = atomicAdd(&S.tcnt[(x.x >> dshift) & dmask], 1u);
+                        if (i0 + 1 < ql) r1 = atomicAdd(&S.tcnt[(x.z >> dshift) & dmask], 1u);
                         rk[v] = r0 | (r1 << 16);
                     }
                 }
@@ -594,12 +634,13 @@ __global__ void __launch_bounds__(BLOCK) k_scatter(ScatterArgs a) {
                         stage[S.local_start[(h4.w >> dshift) & dmask] + (rk[2 * v + 1] >> 16)] =
                             make_uint2(h4.w, p4.w);
                     }
-                } else {
+                } else {   // ranks < TILE <= 0xffff, so 0xffff marks a masked slot
 #pragma unroll
                     for (int v = 0; v < NV; ++v) {
                         const uint4 x = xa[v];
-                        stage[S.local_start[(x.x >> dshift) & dmask] + (rk[v] & 0xffffu)] = make_uint2(x.x, x.y);
-                        stage[S.local_start[(x.z >> dshift) & dmask] + (rk[v] >> 16)] = make_uint2(x.z, x.w);
+                        const uint32_t r0 = rk[v] & 0xffffu, r1 = rk[v] >> 16;
+                        if (r0 != 0xffffu) stage[S.local_start[(x.x >> dshift) & dmask] + r0] = make_uint2(x.x, x.y);
+                        if (r1 != 0xffffu) stage[S.local_start[(x.z >> dshift) & dmask] + r1] = make_uint2(x.z, x.w);
                     }
                 }
             } else {
