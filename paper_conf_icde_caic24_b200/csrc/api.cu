@@ -146,13 +146,26 @@ bool plan_build(Plan& p, uint64_t nR, uint64_t nS, const gsh_config* cfg_in, voi
         uint64_t hm = (nR + nS) / (p.Th ? p.Th : 1) + 1;
         p.h_max = hm < p.gt_cap_alloc ? hm : p.gt_cap_alloc;
     }
-    for (int s = 0; s < 2; ++s) {
-        p.nch1[s] = (uint32_t)((p.n[s] + kScatterChunk - 1) / kScatterChunk);
-        p.ngroups[s] = (p.nch1[s] + kGroupChunks - 1) / kGroupChunks;
+    // pass-1 units (= histogram slices): whole 16K-key chunks, about one unit per scatter CTA
+    // (2 per SM) and at most kHistMaxUnitChunks chunks; pass-2 groups of ~kGroupTuples tuples
+    {
+        const uint64_t nch0 = (p.n[0] + kScatterChunk - 1) / kScatterChunk, nch1 = (p.n[1] + kScatterChunk - 1) / kScatterChunk;
+        uint64_t uc = (nch0 + nch1 + 2 * uint64_t(num_sms) - 1) / (2 * uint64_t(num_sms));
+        if (uc < 1) uc = 1;
+        if (uc > kHistMaxUnitChunks) uc = kHistMaxUnitChunks;
+        p.unit_chunks = (uint32_t)uc;
+        const uint64_t ul = uc * kScatterChunk;
+        uint64_t gu = (kGroupTuples + ul / 2) / ul;
+        p.group_units = (uint32_t)(gu < 1 ? 1 : gu);
+        const uint64_t nch[2] = {nch0, nch1};
+        for (int s = 0; s < 2; ++s) {
+            p.nu1[s] = (uint32_t)((nch[s] + uc - 1) / uc);
+            p.ngroups[s] = (p.nu1[s] + p.group_units - 1) / p.group_units;
+        }
     }
     uint64_t scan_max = p.F + 1 > p.h_max + 1 ? p.F + 1 : p.h_max + 1;
     for (int s = 0; s < 2; ++s)
-        if (uint64_t(p.nch1[s]) * 256 + 1 > scan_max) scan_max = uint64_t(p.nch1[s]) * 256 + 1;
+        if (uint64_t(p.nu1[s]) * 256 + 1 > scan_max) scan_max = uint64_t(p.nu1[s]) * 256 + 1;
     p.scan_scratch_elems = scan_max / 4096 + 2;
 
     Carver c{reinterpret_cast<unsigned char*>(ws)};
@@ -169,11 +182,10 @@ bool plan_build(Plan& p, uint64_t nR, uint64_t nS, const gsh_config* cfg_in, voi
     p.bufB[1] = b ? b + nRp : nullptr;
     p.heavy_pay[0] = hp;
     p.heavy_pay[1] = hp ? hp + nR : nullptr;
-    const size_t nslices = (p.nch1[0] + kSliceChunks - 1) / kSliceChunks + (p.nch1[1] + kSliceChunks - 1) / kSliceChunks;
-    p.hist_partial = c.take<uint32_t>((nslices + 1) * F);
+    p.hist_partial = c.take<uint32_t>((size_t(p.nu1[0]) + p.nu1[1] + 1) * F);
     p.off2 = c.take<uint32_t>((size_t(p.ngroups[0]) + p.ngroups[1] + 1) * F);
-    p.c1cnt = c.take<uint32_t>((size_t(p.nch1[0]) + p.nch1[1]) * 256 + 1);
-    p.off1 = c.take<uint64_t>((size_t(p.nch1[0]) + p.nch1[1]) * 256 + 2);
+    p.c1cnt = c.take<uint32_t>((size_t(p.nu1[0]) + p.nu1[1]) * 256 + 1);
+    p.off1 = c.take<uint64_t>((size_t(p.nu1[0]) + p.nu1[1]) * 256 + 2);
     p.cnt = c.take<uint32_t>(2 * F);
     p.start = c.take<uint64_t>(2 * (F + 1));
     p.gt_key = c.take<unsigned long long>(p.gt_cap_alloc);

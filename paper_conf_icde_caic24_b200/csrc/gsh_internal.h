@@ -12,13 +12,9 @@ namespace gsh {
 constexpr int kScatterBlock = 512;              // threads per partition-scatter CTA
 constexpr int kScatterIpt = 8;                  // tuples per thread per tile
 constexpr int kScatterTile = kScatterBlock * kScatterIpt;  // 4096 tuples per tile
-constexpr int kScatterChunk = 4 * kScatterTile;  // 16384 input tuples per pass-1 work unit
-constexpr uint32_t kSliceChunks = 32;             // pass-1 chunks per joint-histogram slice
-#ifndef GSH_GROUP_SLICES
-#define GSH_GROUP_SLICES 16
-#endif
-constexpr uint32_t kGroupSlices = GSH_GROUP_SLICES;  // slices per pass-2 chunk group
-constexpr uint32_t kGroupChunks = kSliceChunks * kGroupSlices;  // 512 chunks = 8M tuples
+constexpr int kScatterChunk = 4 * kScatterTile;  // 16384 keys: the histogram's load granule
+constexpr uint32_t kHistMaxUnitChunks = 64;      // a pass-1 unit (= histogram slice) is <= 64 chunks = 2^20 tuples
+constexpr uint32_t kGroupTuples = 1u << 23;       // target tuples per pass-2 unit group (8M)
 constexpr int kMaxDigitBits = 8;                // radix bits per pass (256 buckets)
 constexpr int kMaxPartBits = 16;                // b1 + b2 <= 16 (65536 partitions)
 constexpr int kHistBlock = 1024;
@@ -88,7 +84,9 @@ struct Plan {
     uint32_t sample_stride = 100, top_k = 3;
     int num_sms = 148;
     int hist_grid = 148;            // histogram CTAs (1 per SM)
-    uint32_t ngroups[2] = {0, 0};   // pass-2 chunk groups per side
+    uint32_t ngroups[2] = {0, 0};   // pass-2 unit groups per side
+    uint32_t unit_chunks = 1;       // chunks per pass-1 unit (= histogram slice)
+    uint32_t group_units = 1;       // pass-1 units per pass-2 group
     uint32_t gt_cap_alloc = 0;      // detection table slots allocated
     uint64_t h_max = 0;             // skewed-key list capacity
     uint64_t scan_scratch_elems = 0;
@@ -97,10 +95,10 @@ struct Plan {
     uint2* bufA[2] = {nullptr, nullptr};      // pass-1 output, later normal remainders
     uint2* bufB[2] = {nullptr, nullptr};      // final partitions
     uint32_t* heavy_pay[2] = {nullptr, nullptr};  // skewed-key payload arrays
-    uint32_t* hist_partial = nullptr;         // [slices side0 + side1][F] joint counts per slice
-    uint32_t nch1[2] = {0, 0};                // pass-1 chunks per side
-    uint32_t* c1cnt = nullptr;                // [nch1[0] + nch1[1]][256] pass-1 digit counts per chunk
-    uint64_t* off1 = nullptr;                 // per side [256 * nch1 + 1] chunk/bucket output offsets
+    uint32_t* hist_partial = nullptr;         // [nu1[0] + nu1[1]][F] joint counts per pass-1 unit
+    uint32_t nu1[2] = {0, 0};                 // pass-1 units per side
+    uint32_t* c1cnt = nullptr;                // per side [256][nu1] pass-1 digit counts per unit
+    uint64_t* off1 = nullptr;                 // per side [256 * nu1 + 1] unit/bucket output offsets
     uint32_t* cnt = nullptr;                  // [2][F]
     uint64_t* start = nullptr;                // [2][F + 1]
     uint32_t* off2 = nullptr;                 // per side [ngroups][F] pass-2 unit offsets

@@ -36,39 +36,37 @@ int launch_hash(const uint32_t* keys, uint32_t* out, uint64_t n, cudaStream_t s)
 }
 
 // ------------------------------------------------------------------- a1: histogram --
-// One read of the keys yields the (d1, d2) histogram of BOTH partition passes.
+// One read of the keys yields the (d1, d2) histogram of BOTH partition passes, per pass-1 work
+// unit (a "slice" of unit_chunks chunks: the pass-1 scatter's unit IS the histogram slice, so
+// the pass-1 digit counts of a unit are the joint counts summed over d2 -- one shared atomic
+// per key).
 // F <= 2^15: u32 counters in shared memory, atomicAdd(.., 1) = hardware-aggregated
 // ATOMS.POPC.INC (skewed digits cost no more than spread ones; __match_any_sync costs ~64
 // cycles -- scripts/microbench_warp_ops.cu).
 // F > 2^15 (up to 2^16 bins): packed u16 counters, two bins per 32-bit word, so ONE CTA holds
-// all bins in 128 KB and every key is hashed once.  A slice (kSliceChunks chunks, <= 2^19
-// tuples) can wrap a u16 only if one pass-1 digit receives >= 2^16 of its keys (a joint bin
-// never holds more than its digit).  The exact per-chunk digit counts come with the same pass,
-// so a slice is counted with plain no-return atomics first; only a slice in which some digit
-// reached 2^16 (heavy skew) is recounted in exact mode, where wraps are accounted for from the
-// atomics' return values (all updates of a word are serialised, each returns the old word):
+// all bins in 128 KB and every key is hashed once.  A u16 can wrap (a bin reaching 2^16 keys in
+// one slice, heavy skew only), so wraps are accounted for from the atomics' return values (all
+// updates of a word are serialised, each returns the old word):
 //   * the lane whose increment takes a half from 0xffff to 0 sees old half == 0xffff;
 //   * a low-half wrap carries +1 into the high half -- recorded as a -1 correction of the high
 //     bin, and if that carry itself wrapped the high half (old high == 0xffff) as a high wrap.
 // true(low) = low + 65536 * wraps(low); true(high) = high + 65536 * wraps(high) - carries.
-// The (bin, delta) events of a slice (at most ~3 * 2^19 / 2^16) are applied at its flush.
-constexpr uint32_t kHistMaxEvents = 64;
+// The (bin, delta) events of a slice are applied at its flush: a slice holds <= kHistMaxUnitChunks
+// * 2^14 = 2^20 keys, so at most 16 wraps of 3 events each.
+constexpr uint32_t kHistMaxEvents = 128;
 static_assert(kScatterChunk == 16 * kHistBlock, "a full chunk is 4 uint4 per histogram thread");
-template <bool V>
-struct BoolTag {
-    static constexpr bool value = V;
-};
+static_assert(3 * ((uint64_t(kHistMaxUnitChunks) * kScatterChunk) >> 16) <= kHistMaxEvents, "wrap events of a slice");
 
 template <bool FAST16>
 __global__ void __launch_bounds__(kHistBlock, 1)
 k_hist2d(const uint32_t* __restrict__ k0, uint64_t n0, const uint32_t* __restrict__ k1, uint64_t n1,
          uint32_t shift, uint32_t nbits, uint32_t b2, uint32_t* __restrict__ partial, uint32_t* __restrict__ c1cnt,
-         uint32_t nch0, uint32_t nch1) {
+         uint32_t nu0, uint32_t nu1, uint32_t unit_chunks) {
     extern __shared__ uint32_t cnt[];
-    __shared__ uint32_t c1[2][256];
+    __shared__ uint32_t c1s[256];
     __shared__ uint32_t ev_bin[kHistMaxEvents];
     __shared__ int32_t ev_delta[kHistMaxEvents];
-    __shared__ uint32_t n_ev, s_redo;
+    __shared__ uint32_t n_ev;
     const uint32_t F = 1u << nbits;
     const uint32_t mask = F - 1;
     const bool packed = F > (1u << 15);
@@ -76,7 +74,7 @@ k_hist2d(const uint32_t* __restrict__ k0, uint64_t n0, const uint32_t* __restric
     const bool top16 = shift >= 16;
     const uint32_t nwords = packed ? F / 2 : F;
     const uint32_t d1n = (F >> b2) ? (F >> b2) : 1;
-    const uint32_t ns0 = (nch0 + kSliceChunks - 1) / kSliceChunks, ns1 = (nch1 + kSliceChunks - 1) / kSliceChunks;
+    const uint32_t per_d = packed ? ((1u << b2) >> 1) : (1u << b2);   // counter words per pass-1 digit
     auto event = [&](uint32_t bin, int32_t d) {
         const uint32_t e = atomicAdd(&n_ev, 1u);
         if (e < kHistMaxEvents) {
@@ -87,7 +85,7 @@ k_hist2d(const uint32_t* __restrict__ k0, uint64_t n0, const uint32_t* __restric
     auto count_exact = [&](uint32_t bin) {
         const uint32_t s16 = (bin & 1u) << 4;
         const uint32_t old = atomicAdd(&cnt[bin >> 1], 1u << s16);
-        if (((old >> s16) & 0xffffu) == 0xffffu) {  // a u16 wrapped
+        if (__builtin_expect(((old >> s16) & 0xffffu) == 0xffffu, 0)) {  // a u16 wrapped
             event(bin, 65536);
             if (s16 == 0) {
                 event(bin | 1u, -1);
@@ -95,128 +93,103 @@ k_hist2d(const uint32_t* __restrict__ k0, uint64_t n0, const uint32_t* __restric
             }
         }
     };
-    uint32_t* c1b = c1[0];
-    // EXACT: recount pass of a heavy slice (wrap accounting, no digit counts)
-    auto count_key = [&](uint32_t key, auto ex) {
-        constexpr bool EXACT = decltype(ex)::value;
+    auto count_key = [&](uint32_t key) {
         if (FAST16) {
-            const uint32_t h = hash32_top(key);
-            if (EXACT) {
-                count_exact(h >> 16);
-            } else {
-                atomicAdd(&cnt[h >> 17], 1u << ((h >> 12) & 16u));
-                atomicAdd(&c1b[h >> 24], 1u);
-            }
+            count_exact(hash32_top(key) >> 16);
         } else {
             const uint32_t bin = ((top16 ? hash32_top(key) : hash32(key)) >> shift) & mask;
-            if (EXACT) {
-                count_exact(bin);
-            } else {
-                if (packed) atomicAdd(&cnt[bin >> 1], 1u << ((bin & 1u) << 4)); else atomicAdd(&cnt[bin], 1u);
-                atomicAdd(&c1b[bin >> b2], 1u);
-            }
+            if (packed) count_exact(bin); else atomicAdd(&cnt[bin], 1u);
         }
     };
     for (uint32_t w = threadIdx.x; w < nwords; w += blockDim.x) cnt[w] = 0;
-    if (threadIdx.x < 512) c1[threadIdx.x >> 8][threadIdx.x & 255] = 0;
-    if (threadIdx.x == 0) n_ev = s_redo = 0;
+    if (threadIdx.x < 256) c1s[threadIdx.x] = 0;
+    if (threadIdx.x == 0) n_ev = 0;
     __syncthreads();
-    for (uint32_t it = blockIdx.x; it < ns0 + ns1; it += gridDim.x) {
-        const int side = it >= ns0;
-        const uint32_t sl = it - (side ? ns0 : 0);
+    for (uint32_t it = blockIdx.x; it < nu0 + nu1; it += gridDim.x) {
+        const int side = it >= nu0;
+        const uint32_t sl = it - (side ? nu0 : 0);
+        const uint32_t nu = side ? nu1 : nu0;
         const uint32_t* keys = side ? k1 : k0;
         const uint64_t n = side ? n1 : n0;
-        const uint32_t nch = side ? nch1 : nch0;
-        uint32_t* c1out = c1cnt + (side ? size_t(nch0) * 256 : 0);
+        const uint32_t nch = (uint32_t)((n + kScatterChunk - 1) / kScatterChunk);
+        uint32_t* c1out = c1cnt + (side ? size_t(nu0) * 256 : 0);
         const bool vec = ((reinterpret_cast<uintptr_t>(keys) & 15u) == 0);
-        const uint32_t c0 = sl * kSliceChunks, cend = umin32((sl + 1) * kSliceChunks, nch);
-        uint32_t dtot = 0;  // thread d < d1n: keys of digit d in this slice
+        const uint32_t c0 = sl * unit_chunks, cend = umin32(c0 + unit_chunks, nch);
         // Full chunks are loaded one chunk ahead (16 keys per thread in registers), so the
-        // loads of chunk c+1 are in flight while chunk c is counted and its pass-1 digit counts
-        // flushed; the two c1 buffers alternate so one barrier per chunk suffices.
-        auto run_slice = [&](auto ex) {
-            constexpr bool EXACT = decltype(ex)::value;
-            uint4 v[4];
-            auto load_chunk = [&](uint32_t c) {
-                const uint4* kv = reinterpret_cast<const uint4*>(keys + uint64_t(c) * kScatterChunk);
+        // loads of chunk c+1 are in flight while chunk c is counted.
+        uint4 v[4];
+        auto load_chunk = [&](uint32_t c) {
+            const uint4* kv = reinterpret_cast<const uint4*>(keys + uint64_t(c) * kScatterChunk);
 #pragma unroll
-                for (int u = 0; u < 4; ++u) v[u] = ld_stream_u4(kv + threadIdx.x + u * kHistBlock);
-            };
-            auto chunk_full = [&](uint32_t c) { return vec && uint64_t(c + 1) * kScatterChunk <= n; };
-            if (c0 < cend && chunk_full(c0)) load_chunk(c0);
-            for (uint32_t c = c0; c < cend; ++c) {
-                const uint64_t cb = uint64_t(c) * kScatterChunk;
-                const uint64_t ce = umin64(cb + kScatterChunk, n);
-                c1b = c1[c & 1];
-                if (chunk_full(c)) {
-                    uint4 cur[4];
-#pragma unroll
-                    for (int u = 0; u < 4; ++u) cur[u] = v[u];
-                    if (c + 1 < cend && chunk_full(c + 1)) load_chunk(c + 1);
-#pragma unroll
-                    for (int u = 0; u < 4; ++u) {
-                        const uint32_t kk[4] = {cur[u].x, cur[u].y, cur[u].z, cur[u].w};
-#pragma unroll
-                        for (int q = 0; q < 4; ++q) count_key(kk[q], ex);
-                    }
-                } else {  // the ragged last chunk, or keys not 16-byte aligned
-                    uint64_t done = cb;
-                    if (vec) {
-                        const uint4* kv = reinterpret_cast<const uint4*>(keys + cb);
-                        const uint64_t nv = (ce - cb) / 4;
-                        for (uint64_t i = threadIdx.x; i < nv; i += blockDim.x) {
-                            const uint4 w = ld_stream_u4(kv + i);
-                            const uint32_t kk[4] = {w.x, w.y, w.z, w.w};
-#pragma unroll
-                            for (int q = 0; q < 4; ++q) count_key(kk[q], ex);
-                        }
-                        done = cb + nv * 4;
-                    }
-                    for (uint64_t j = done + threadIdx.x; j < ce; j += blockDim.x) count_key(keys[j], ex);
-                }
-                if (!EXACT) {
-                    __syncthreads();
-                    if (threadIdx.x < d1n) {
-                        const uint32_t x = c1b[threadIdx.x];
-                        c1out[size_t(threadIdx.x) * nch + c] = x;
-                        c1b[threadIdx.x] = 0;
-                        dtot += x;
-                    }
-                }
-            }
+            for (int u = 0; u < 4; ++u) v[u] = ld_stream_u4(kv + threadIdx.x + u * kHistBlock);
         };
-        run_slice(BoolTag<false>{});
-        if (packed) {
-            if (threadIdx.x < d1n && dtot >= 65536u) s_redo = 1;
-            __syncthreads();
-            if (s_redo) {  // some u16 may have wrapped: recount the slice exactly (rare, skew only)
-                for (uint32_t w = threadIdx.x; w < nwords; w += blockDim.x) cnt[w] = 0;
-                __syncthreads();
-                run_slice(BoolTag<true>{});
+        auto chunk_full = [&](uint32_t c) { return vec && uint64_t(c + 1) * kScatterChunk <= n; };
+        if (c0 < cend && chunk_full(c0)) load_chunk(c0);
+        for (uint32_t c = c0; c < cend; ++c) {
+            const uint64_t cb = uint64_t(c) * kScatterChunk;
+            const uint64_t ce = umin64(cb + kScatterChunk, n);
+            if (chunk_full(c)) {
+                uint4 cur[4];
+#pragma unroll
+                for (int u = 0; u < 4; ++u) cur[u] = v[u];
+                if (c + 1 < cend && chunk_full(c + 1)) load_chunk(c + 1);
+#pragma unroll
+                for (int u = 0; u < 4; ++u) {
+                    const uint32_t kk[4] = {cur[u].x, cur[u].y, cur[u].z, cur[u].w};
+#pragma unroll
+                    for (int q = 0; q < 4; ++q) count_key(kk[q]);
+                }
+            } else {  // the ragged last chunk, or keys not 16-byte aligned
+                uint64_t done = cb;
+                if (vec) {
+                    const uint4* kv = reinterpret_cast<const uint4*>(keys + cb);
+                    const uint64_t nv = (ce - cb) / 4;
+                    for (uint64_t i = threadIdx.x; i < nv; i += blockDim.x) {
+                        const uint4 w = ld_stream_u4(kv + i);
+                        const uint32_t kk[4] = {w.x, w.y, w.z, w.w};
+#pragma unroll
+                        for (int q = 0; q < 4; ++q) count_key(kk[q]);
+                    }
+                    done = cb + nv * 4;
+                }
+                for (uint64_t j = done + threadIdx.x; j < ce; j += blockDim.x) count_key(keys[j]);
             }
         }
         __syncthreads();
-        // flush this slice's joint counts and reset
-        uint32_t* row = partial + (size_t(side ? ns0 : 0) + sl) * F;
-        if (packed) {
-            for (uint32_t w = threadIdx.x; w < nwords; w += blockDim.x) {
-                const uint32_t v = cnt[w];
-                reinterpret_cast<uint2*>(row)[w] = make_uint2(v & 0xffffu, v >> 16);
-                cnt[w] = 0;
+        // flush this slice's joint counts (and their per-d1 sums) and reset
+        uint32_t* row = partial + (size_t(side ? nu0 : 0) + sl) * F;
+        for (uint32_t w = threadIdx.x; w < nwords; w += blockDim.x) {
+            const uint32_t x = cnt[w];
+            uint32_t val;
+            if (packed) {
+                reinterpret_cast<uint2*>(row)[w] = make_uint2(x & 0xffffu, x >> 16);
+                val = (x & 0xffffu) + (x >> 16);
+            } else {
+                row[w] = x;
+                val = x;
             }
-            __syncthreads();
-            if (threadIdx.x == 0) {  // wrap corrections (sequential so repeated bins add up)
-                for (uint32_t e = 0; e < umin32(n_ev, kHistMaxEvents); ++e) row[ev_bin[e]] += ev_delta[e];
-                n_ev = 0;
-                s_redo = 0;
-            }
-        } else {
-            for (uint32_t w = threadIdx.x; w < nwords; w += blockDim.x) {
-                row[w] = cnt[w];
-                cnt[w] = 0;
+            cnt[w] = 0;
+            const uint32_t d = (packed ? 2 * w : w) >> b2;
+            if (per_d >= 32) {   // the warp's 32 words share one digit (whole warps: nwords % 32 == 0)
+                const uint32_t sum = __reduce_add_sync(kFull, val);
+                if ((threadIdx.x & 31) == 0 && sum) atomicAdd(&c1s[d], sum);
+            } else if (val) {
+                atomicAdd(&c1s[d], val);
             }
         }
         __syncthreads();
+        if (threadIdx.x == 0) {  // wrap corrections (sequential so repeated bins add up)
+            for (uint32_t e = 0; e < umin32(n_ev, kHistMaxEvents); ++e) {
+                row[ev_bin[e]] += ev_delta[e];
+                c1s[ev_bin[e] >> b2] += ev_delta[e];
+            }
+            n_ev = 0;
+        }
+        __syncthreads();
+        if (threadIdx.x < d1n) {
+            c1out[size_t(threadIdx.x) * nu + sl] = c1s[threadIdx.x];
+            c1s[threadIdx.x] = 0;
+        }
     }
 }
 
@@ -237,10 +210,12 @@ int launch_hist(const Plan& p, const uint32_t* k0, const uint32_t* k1, cudaStrea
     // DSMEM atomics, 3.6 ms, or DSMEM loads, 1.0 ms.)
     if (fast16)
         k_hist2d<true><<<p.hist_grid, kHistBlock, smem, s>>>(k0, p.n[0], k1, p.n[1], shift, nbits, p.b2,
-                                                             p.hist_partial, p.c1cnt, p.nch1[0], p.nch1[1]);
+                                                             p.hist_partial, p.c1cnt, p.nu1[0], p.nu1[1],
+                                                             p.unit_chunks);
     else
         k_hist2d<false><<<p.hist_grid, kHistBlock, smem, s>>>(k0, p.n[0], k1, p.n[1], shift, nbits, p.b2,
-                                                              p.hist_partial, p.c1cnt, p.nch1[0], p.nch1[1]);
+                                                              p.hist_partial, p.c1cnt, p.nu1[0], p.nu1[1],
+                                                              p.unit_chunks);
     return 1;
 }
 
@@ -249,7 +224,7 @@ int launch_hist(const Plan& p, const uint32_t* k0, const uint32_t* k1, cudaStrea
 // offsets relative to the partition start) and cnt[side][p] = |R_p| / |S_p|.
 __global__ void k_hist_reduce(const uint32_t* __restrict__ partial, uint32_t* __restrict__ cnt,
                               uint32_t* __restrict__ off2, uint32_t F, uint32_t ns0, uint32_t ns1, uint32_t ng0,
-                              uint32_t ng1) {
+                              uint32_t ng1, uint32_t group_units) {
     for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < 2 * F; i += gridDim.x * blockDim.x) {
         const uint32_t side = i / F, bin = i % F;
         const uint32_t ns = side ? ns1 : ns0, ng = side ? ng1 : ng0;
@@ -258,7 +233,7 @@ __global__ void k_hist_reduce(const uint32_t* __restrict__ partial, uint32_t* __
         uint32_t run = 0;
         for (uint32_t g = 0; g < ng; ++g) {
             o2[size_t(g) * F] = run;
-            const uint32_t s0 = g * kGroupSlices, s1 = umin32(s0 + kGroupSlices, ns);
+            const uint32_t s0 = g * group_units, s1 = umin32(s0 + group_units, ns);
             for (uint32_t s = s0; s < s1; ++s) run += base[size_t(s) * F];
         }
         cnt[i] = run;
@@ -270,26 +245,26 @@ struct CountAt {
     __device__ uint64_t operator()(uint64_t i) const { return c[i]; }
 };
 
-// Pass-1 chunk counts in (digit, chunk) order: the exclusive scan in that order IS the output
-// offset of chunk c's bucket-d run (start of bucket d + runs of d in earlier chunks).
+// Pass-1 unit counts in (digit, unit) order: the exclusive scan in that order IS the output
+// offset of unit u's bucket-d run (start of bucket d + runs of d in earlier units).
 struct ChunkDigit {
-    const uint32_t* c1;   // [256][nch] digit-major
+    const uint32_t* c1;   // [256][nu1] digit-major
     __device__ uint64_t operator()(uint64_t i) const { return c1[i]; }
 };
 
 int launch_hist_reduce_scan(const Plan& p, cudaStream_t s) {
     const uint32_t F = p.F;
-    const uint32_t ns0 = (p.nch1[0] + kSliceChunks - 1) / kSliceChunks, ns1 = (p.nch1[1] + kSliceChunks - 1) / kSliceChunks;
     unsigned grid = (2 * F + 255) / 256;
-    k_hist_reduce<<<grid, 256, 0, s>>>(p.hist_partial, p.cnt, p.off2, F, ns0, ns1, p.ngroups[0], p.ngroups[1]);
+    k_hist_reduce<<<grid, 256, 0, s>>>(p.hist_partial, p.cnt, p.off2, F, p.nu1[0], p.nu1[1], p.ngroups[0],
+                                       p.ngroups[1], p.group_units);
     int l = 1;
     for (int side = 0; side < 2; ++side)
         l += launch_scan(CountAt{p.cnt + size_t(side) * F}, F, p.start + size_t(side) * (F + 1), p.scan_scratch, s);
     uint64_t off = 0;
     for (int side = 0; side < 2; ++side) {
-        const uint64_t m = uint64_t(p.nch1[side]) * 256;
+        const uint64_t m = uint64_t(p.nu1[side]) * 256;
         if (m)
-            l += launch_scan(ChunkDigit{p.c1cnt + (side ? size_t(p.nch1[0]) * 256 : 0)}, m, p.off1 + off,
+            l += launch_scan(ChunkDigit{p.c1cnt + (side ? size_t(p.nu1[0]) * 256 : 0)}, m, p.off1 + off,
                              p.scan_scratch, s);
         off += m + 1;
     }
@@ -310,10 +285,11 @@ struct ScatterArgs {
     const uint2* in[2];        // pass 2 input (AoS pass-1 output)
     uint2* out[2];
     const uint64_t* start[2];  // final partition starts [F + 1] per side
-    const uint64_t* off1[2];   // [256 * nch1 + 1] per side: start of chunk c's run of digit d at d*nch1 + c
+    const uint64_t* off1[2];   // [256 * nu1 + 1] per side: start of unit u's run of digit d at d*nu1 + u
     const uint32_t* off2[2];   // [ngroups][F] per side: tuples of partition p in earlier chunk groups
     uint64_t n[2];
-    uint32_t nch1[2], ngroups[2];
+    uint32_t nu1[2], ngroups[2];     // pass-1 units (= histogram slices), pass-2 unit groups per side
+    uint32_t unit_len, group_units;  // tuples per pass-1 unit, pass-1 units per pass-2 group
     uint32_t pass, b1, b2, route_bits;
     unsigned int* unit_ctr;
 };
@@ -343,17 +319,17 @@ __device__ __forceinline__ UnitInfo unit_info(const ScatterArgs& a, uint32_t u, 
     UnitInfo ui;
     ui.side = (u >= units0) ? 1 : 0;
     const uint32_t lu = u - (ui.side ? units0 : 0);
-    const uint32_t nch = a.nch1[ui.side];
+    const uint32_t nch = a.nu1[ui.side];
     if (p1) {
         ui.d1 = 0;
         ui.grp = lu;
-        ui.begin = uint64_t(lu) * kScatterChunk;
-        ui.len = (uint32_t)umin64(kScatterChunk, a.n[ui.side] - ui.begin);
+        ui.begin = uint64_t(lu) * a.unit_len;
+        ui.len = (uint32_t)umin64(a.unit_len, a.n[ui.side] - ui.begin);
     } else {
         const uint32_t ng = a.ngroups[ui.side];
         ui.d1 = lu / ng;
         ui.grp = lu - ui.d1 * ng;
-        const uint32_t c0 = ui.grp * kGroupChunks, c1 = umin32(c0 + kGroupChunks, nch);
+        const uint32_t c0 = ui.grp * a.group_units, c1 = umin32(c0 + a.group_units, nch);
         ui.begin = a.off1[ui.side][size_t(ui.d1) * nch + c0];
         ui.len = (uint32_t)(a.off1[ui.side][size_t(ui.d1) * nch + c1] - ui.begin);
     }
@@ -460,8 +436,8 @@ __global__ void __launch_bounds__(BLOCK) k_scatter(ScatterArgs a) {
     const uint32_t dmask = nb - 1;
     const uint32_t dshift = (32 - a.route_bits - a.b1 - (p1 ? 0 : a.b2)) & 31;
     const uint32_t lowbits = p1 ? a.b2 : 0;
-    const uint32_t units0 = p1 ? a.nch1[0] : (1u << a.b1) * a.ngroups[0];
-    const uint32_t total = units0 + (p1 ? a.nch1[1] : (1u << a.b1) * a.ngroups[1]);
+    const uint32_t units0 = p1 ? a.nu1[0] : (1u << a.b1) * a.ngroups[0];
+    const uint32_t total = units0 + (p1 ? a.nu1[1] : (1u << a.b1) * a.ngroups[1]);
     const uint64_t rpol = policy_evict_first(), wpol = policy_evict_first();
 
     if (tid < 256) S.tcnt[tid] = 0;
@@ -488,7 +464,7 @@ __global__ void __launch_bounds__(BLOCK) k_scatter(ScatterArgs a) {
         if (tid < nb) {
             uint32_t r0;
             const uint32_t pidx = ((ui.d1 << bits) | tid) << lowbits;
-            if (p1) r0 = (uint32_t)a.off1[ui.side][size_t(tid) * a.nch1[ui.side] + ui.grp];
+            if (p1) r0 = (uint32_t)a.off1[ui.side][size_t(tid) * a.nu1[ui.side] + ui.grp];
             else r0 = (uint32_t)a.start[ui.side][pidx] + a.off2[ui.side][size_t(ui.grp) * (size_t(1) << (a.b1 + a.b2)) + pidx];
             S.run[tid] = r0;
             S.wpos[tid] = r0;
@@ -729,12 +705,14 @@ int launch_scatter(const Plan& p, int pass, const uint32_t* const keys[2], const
         a.out[side] = (pass == 1) ? p.bufA[side] : p.bufB[side];
         a.start[side] = p.start + size_t(side) * (p.F + 1);
         a.off1[side] = p.off1 + o1;
-        o1 += uint64_t(p.nch1[side]) * 256 + 1;
+        o1 += uint64_t(p.nu1[side]) * 256 + 1;
         a.off2[side] = p.off2 + (side ? size_t(p.ngroups[0]) * p.F : 0);
         a.n[side] = p.n[side];
-        a.nch1[side] = p.nch1[side];
+        a.nu1[side] = p.nu1[side];
         a.ngroups[side] = p.ngroups[side];
     }
+    a.unit_len = p.unit_chunks * kScatterChunk;
+    a.group_units = p.group_units;
     a.pass = pass;
     a.b1 = p.b1;
     a.b2 = p.b2;
