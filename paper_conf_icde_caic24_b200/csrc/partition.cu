@@ -299,8 +299,8 @@ struct ScatterSmem {
     uint32_t local_start[256];          // bucket start inside the staged tile
     uint32_t run[256];                  // next output index of bucket b for this unit
     uint32_t wpos[256];                 // first index of bucket b not yet written to memory
-    uint32_t gbase[256];                // output index of stage position 0 of bucket b (mod 2^32)
-    uint32_t endw[256];                 // write-out limit of bucket b for the current tile
+    uint2 gw[256];                      // bucket b: (output index of stage position 0 (mod 2^32),
+                                        //            write-out limit for the current tile)
     uint32_t tailpos[256];              // stage position of bucket b's carried tail
     uint2 cbuf[256][4];                 // carry: < 4 tuples (one 32 B sector) per bucket
     uint32_t carry[256];                // tuples in cbuf[b]
@@ -588,8 +588,7 @@ __global__ void __launch_bounds__(BLOCK) k_scatter(ScatterArgs a) {
                 my_w0 = w0;
                 my_ew = ew;
                 S.local_start[tid] = lstart + cin;
-                S.gbase[tid] = w0 - lstart;
-                S.endw[tid] = ew;
+                S.gw[tid] = make_uint2(w0 - lstart, ew);
                 S.tailpos[tid] = lstart + (ew - w0);
                 for (uint32_t k = 0; k < cin; ++k) stage[lstart + k] = S.cbuf[tid][k];
                 S.wpos[tid] = ew;
@@ -654,12 +653,14 @@ __global__ void __launch_bounds__(BLOCK) k_scatter(ScatterArgs a) {
 #pragma unroll 4
                 for (uint32_t i = tid; i < all; i += BLOCK) {
                     const uint2 e = stage[i];
-                    const uint32_t d = (e.x >> dshift) & dmask;
-                    const uint32_t g = S.gbase[d] + i;
-                    if (g < S.endw[d]) st_stream_u2(out + g, e, wpol);
+                    const uint2 ge = S.gw[(e.x >> dshift) & dmask];
+                    const uint32_t g = ge.x + i;
+                    if (g < ge.y) st_stream_u2(out + g, e, wpol);
                 }
             }
-            __syncthreads();
+            // No barrier here: the next tile's ranking touches only the input buffer and tcnt
+            // (reset in phase B), and everything this write-out reads (stage, gw, carry,
+            // tailpos) is rewritten only after the next tile's first barrier.
         }
         u = un;
         issued = true;  // the next unit's first tile (if any, and non-empty) is in flight
