@@ -167,6 +167,11 @@ bool plan_build(Plan& p, uint64_t nR, uint64_t nS, const gsh_config* cfg_in, voi
     for (int s = 0; s < 2; ++s)
         if (uint64_t(p.nu1[s]) * 256 + 1 > scan_max) scan_max = uint64_t(p.nu1[s]) * 256 + 1;
     p.scan_scratch_elems = scan_max / 4096 + 2;
+    {   // the histogram's four scans share one launch (launch_scan_u32_multi)
+        const uint64_t m4 = (2 * (uint64_t(p.F) + 4095) + (uint64_t(p.nu1[0]) * 256 + 4095) +
+                             (uint64_t(p.nu1[1]) * 256 + 4095)) / 4096 + 8;
+        if (m4 > p.scan_scratch_elems) p.scan_scratch_elems = m4;
+    }
 
     Carver c{reinterpret_cast<unsigned char*>(ws)};
     const size_t F = p.F;

@@ -83,9 +83,13 @@ k_hist2d(const uint32_t* __restrict__ k0, uint64_t n0, const uint32_t* __restric
         }
     };
     auto count_exact = [&](uint32_t bin) {
-        const uint32_t s16 = (bin & 1u) << 4;
-        const uint32_t old = atomicAdd(&cnt[bin >> 1], 1u << s16);
-        if (__builtin_expect(((old >> s16) & 0xffffu) == 0xffffu, 0)) {  // a u16 wrapped
+        // inc = 1 << (16 * (bin & 1)) and m = its half's mask, without variable shifts (the
+        // histogram is ALU-bound): a wrap is old's half == 0xffff, i.e. (~old & m) == 0
+        const uint32_t inc = umax32((bin & 1u) << 16, 1u);
+        const uint32_t m = inc * 0xffffu;
+        const uint32_t old = atomicAdd(&cnt[bin >> 1], inc);
+        if (__builtin_expect((~old & m) == 0, 0)) {  // a u16 wrapped
+            const uint32_t s16 = (bin & 1u) << 4;
             event(bin, 65536);
             if (s16 == 0) {
                 event(bin | 1u, -1);
@@ -257,18 +261,22 @@ int launch_hist_reduce_scan(const Plan& p, cudaStream_t s) {
     unsigned grid = (2 * F + 255) / 256;
     k_hist_reduce<<<grid, 256, 0, s>>>(p.hist_partial, p.cnt, p.off2, F, p.nu1[0], p.nu1[1], p.ngroups[0],
                                        p.ngroups[1], p.group_units);
-    int l = 1;
-    for (int side = 0; side < 2; ++side)
-        l += launch_scan(CountAt{p.cnt + size_t(side) * F}, F, p.start + size_t(side) * (F + 1), p.scan_scratch, s);
+    // four independent scans in one launch triple: partition starts per side, pass-1
+    // (digit, unit) offsets per side
+    ScanSegs g{};
+    g.k = 4;
     uint64_t off = 0;
     for (int side = 0; side < 2; ++side) {
+        g.in[side] = p.cnt + size_t(side) * F;
+        g.out[side] = p.start + size_t(side) * (F + 1);
+        g.n[side] = F;
         const uint64_t m = uint64_t(p.nu1[side]) * 256;
-        if (m)
-            l += launch_scan(ChunkDigit{p.c1cnt + (side ? size_t(p.nu1[0]) * 256 : 0)}, m, p.off1 + off,
-                             p.scan_scratch, s);
+        g.in[2 + side] = p.c1cnt + (side ? size_t(p.nu1[0]) * 256 : 0);
+        g.out[2 + side] = p.off1 + off;
+        g.n[2 + side] = m;
         off += m + 1;
     }
-    return l;
+    return 1 + launch_scan_u32_multi(g, p.scan_scratch, s);
 }
 
 // ------------------------------------------------------------- a3/a4: tile scatter --
