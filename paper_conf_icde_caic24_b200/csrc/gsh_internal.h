@@ -9,10 +9,21 @@
 namespace gsh {
 
 // ----------------------------------------------------------------- fixed shapes --
-constexpr int kScatterBlock = 512;              // threads per partition-scatter CTA
-constexpr int kScatterIpt = 8;                  // tuples per thread per tile
-constexpr int kScatterTile = kScatterBlock * kScatterIpt;  // 4096 tuples per tile
-constexpr int kScatterChunk = 4 * kScatterTile;  // 16384 keys: the histogram's load granule
+#ifndef GSH_SCATTER_BLOCK
+#define GSH_SCATTER_BLOCK 512
+#endif
+#ifndef GSH_SCATTER_IPT
+#define GSH_SCATTER_IPT 8
+#endif
+constexpr int kScatterBlock = GSH_SCATTER_BLOCK;  // threads per partition-scatter CTA
+constexpr int kScatterIpt = GSH_SCATTER_IPT;      // tuples per thread per tile
+#ifndef GSH_SCATTER_IPT1
+#define GSH_SCATTER_IPT1 16
+#endif
+constexpr int kScatterIpt1 = GSH_SCATTER_IPT1;    // pass 1: tuples per thread per tile
+constexpr int kScatterTile = kScatterBlock * kScatterIpt;  // 4096 tuples per tile (pass 2)
+constexpr int kScatterChunk = 16384;               // keys: the histogram's load granule (unit lengths are multiples)
+static_assert(kScatterChunk % (kScatterBlock * kScatterIpt1) == 0, "pass-1 units are whole tiles");
 constexpr uint32_t kHistMaxUnitChunks = 64;      // a pass-1 unit (= histogram slice) is <= 64 chunks = 2^20 tuples
 constexpr uint32_t kGroupTuples = 1u << 23;       // target tuples per pass-2 unit group (8M)
 constexpr int kMaxDigitBits = 8;                // radix bits per pass (256 buckets)

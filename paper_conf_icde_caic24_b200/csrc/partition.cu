@@ -691,9 +691,11 @@ int launch_scatter_pass(const Plan& p, const ScatterArgs& a, cudaStream_t s) {
                              (int)smem);
         attr_set = true;
     }
-    int occ = 0;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_scatter<BLOCK, IPT, PASS, TMAST>, BLOCK, smem);
-    if (occ < 1) occ = 1;
+    static int occ = 0;   // per kernel instance (fixed block and shared memory): query once
+    if (occ < 1) {
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_scatter<BLOCK, IPT, PASS, TMAST>, BLOCK, smem);
+        if (occ < 1) occ = 1;
+    }
     k_scatter<BLOCK, IPT, PASS, TMAST><<<(unsigned)(p.num_sms * occ), BLOCK, smem, s>>>(a);
     return 1;
 }
@@ -734,10 +736,12 @@ int launch_scatter(const Plan& p, int pass, const uint32_t* const keys[2], const
     }
     // (TMA bulk stores per bucket run, cfg 1, measured slower on cfg2: 1.12 / 1.24 ms vs
     // 1.06 / 1.17 ms for the per-tuple whole-sector stores -- barrier-bound, ALU 49 % vs 28 %)
-    switch (cfg) {
-        case 1: return launch_scatter_cfg<kScatterBlock, kScatterIpt, true>(p, a, s);
-        default: return launch_scatter_cfg<kScatterBlock, kScatterIpt, false>(p, a, s);
-    }
+    // Tile shapes per pass (measured on cfg2, scripts/gpu_variants.sh): pass 1 (SoA input,
+    // hashes computed in the kernel) prefers 512 x 16 = 8192-tuple tiles (1.013 -> 0.946 ms),
+    // pass 2 (AoS) 512 x 8 (1.032 ms vs 1.061 for 512 x 16, 1.109 for 1024 x 8).
+    if (cfg == 1) return launch_scatter_cfg<kScatterBlock, kScatterIpt, true>(p, a, s);
+    return pass == 1 ? launch_scatter_pass<kScatterBlock, kScatterIpt1, 1, false>(p, a, s)
+                     : launch_scatter_pass<kScatterBlock, kScatterIpt, 2, false>(p, a, s);
 }
 
 // ----------------------------------------------- standalone radix histogram (ABI) --
