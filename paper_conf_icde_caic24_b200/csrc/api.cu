@@ -217,27 +217,34 @@ bool plan_build(Plan& p, uint64_t nR, uint64_t nS, const gsh_config* cfg_in, voi
 
 namespace {
 
+// Phase timing (gsh_config.timing): events come from a per-thread pool created once, so a timed
+// call adds only cudaEventRecord / cudaEventElapsedTime on the host (a call is synchronous, so
+// the pool is free again when the next call on this thread starts).
 struct Timer {
     bool on;
     cudaStream_t s;
-    std::vector<cudaEvent_t> ev;
+    int used = 0;
+    static std::vector<cudaEvent_t>& pool() {
+        static thread_local std::vector<cudaEvent_t> p;
+        return p;
+    }
     explicit Timer(bool enable, cudaStream_t st) : on(enable), s(st) {}
     int mark() {
         if (!on) return -1;
-        cudaEvent_t e;
-        cudaEventCreate(&e);
-        cudaEventRecord(e, s);
-        ev.push_back(e);
-        return (int)ev.size() - 1;
+        auto& p = pool();
+        if (used == (int)p.size()) {
+            cudaEvent_t e;
+            if (cudaEventCreate(&e) != cudaSuccess) return -1;
+            p.push_back(e);
+        }
+        cudaEventRecord(p[used], s);
+        return used++;
     }
     float ms(int a, int b) {
         if (!on || a < 0 || b < 0) return 0.f;
         float t = 0.f;
-        cudaEventElapsedTime(&t, ev[a], ev[b]);
+        cudaEventElapsedTime(&t, pool()[a], pool()[b]);
         return t;
-    }
-    ~Timer() {
-        for (auto e : ev) cudaEventDestroy(e);
     }
 };
 
