@@ -19,7 +19,6 @@ import os
 import statistics
 import subprocess
 import sys
-import threading
 import time
 
 ROOT = os.path.dirname(os.path.abspath(__file__))
@@ -69,68 +68,84 @@ def hbm_peak():
         return FALLBACK_HBM_GBS, "fallback (B200_PROFILING.md)"
 
 
+_SAMPLER_SRC = r"""
+import json, sys, time
+import pynvml
+pynvml.nvmlInit()
+h = pynvml.nvmlDeviceGetHandleByIndex(int(sys.argv[1]))
+bits = {"hw_slowdown": 0x8, "sw_thermal_slowdown": 0x20, "hw_thermal_slowdown": 0x40, "sw_power_cap": 0x4}
+print(json.dumps({"max": pynvml.nvmlDeviceGetMaxClockInfo(h, pynvml.NVML_CLOCK_SM)}), flush=True)
+rows = []
+import select
+while True:
+    r, _, _ = select.select([sys.stdin], [], [], 0.02)
+    if r:
+        break
+    try:
+        sm = pynvml.nvmlDeviceGetClockInfo(h, pynvml.NVML_CLOCK_SM)
+        e = pynvml.nvmlDeviceGetCurrentClocksEventReasons(h)
+        rows.append((sm, [k for k, b in bits.items() if e & b]))
+    except Exception:
+        pass
+print(json.dumps({"rows": rows}), flush=True)
+"""
+
+
 class ClockSampler:
-    """SM clocks + throttle reasons sampled every 20 ms during the timed region (NVML; falls back
-    to `nvidia-smi -lms 100`)."""
+    """SM clocks + throttle reasons sampled every 20 ms during the timed region, by NVML in a
+    separate process (a sampler thread here would contend for the GIL with the launch loop and
+    open gaps between steps); falls back to `nvidia-smi -lms 100`."""
 
     def __init__(self, index: int):
         self.index = index
         self.rows = []
-        self.stop = threading.Event()
         self.proc = None
+        self.max_mhz = None
+        self.mode = None
 
     def __enter__(self):
         try:
-            import pynvml
-            pynvml.nvmlInit()
-            h = pynvml.nvmlDeviceGetHandleByIndex(self.index)
-            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(h, pynvml.NVML_CLOCK_SM)
-            bits = {"hw_slowdown": 0x8, "sw_thermal_slowdown": 0x20, "hw_thermal_slowdown": 0x40, "sw_power_cap": 0x4}
-
-            def poll():
-                while not self.stop.is_set():
-                    try:
-                        sm = pynvml.nvmlDeviceGetClockInfo(h, pynvml.NVML_CLOCK_SM)
-                        r = pynvml.nvmlDeviceGetCurrentClocksEventReasons(h)
-                        self.rows.append((sm, [k for k, b in bits.items() if r & b]))
-                    except Exception:
-                        pass
-                    time.sleep(0.02)
-            self.t = threading.Thread(target=poll, daemon=True)
-            self.t.start()
+            import pynvml  # noqa: F401  (the sampler process needs it)
+            self.proc = subprocess.Popen([sys.executable, "-c", _SAMPLER_SRC, str(self.index)], stdin=subprocess.PIPE,
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.max_mhz = json.loads(self.proc.stdout.readline())["max"]   # sampler is running
             self.mode = "nvml"
         except Exception:
+            self.proc = None
             self.mode = "smi"
-            self.max_mhz = None
             q = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
                  "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
             try:
                 self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={q}",
                                               "--format=csv,noheader,nounits", "-lms", "100"],
                                              stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
-                self.t = threading.Thread(target=self._read, daemon=True)
-                self.t.start()
             except Exception:
                 self.proc = None
         return self
 
-    def _read(self):
-        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        for line in self.proc.stdout:
-            p = [x.strip() for x in line.split(",")]
-            if len(p) == 6 and p[0].replace(".", "").isdigit():
-                self.max_mhz = float(p[1])
-                self.rows.append((float(p[0]), [names[i] for i in range(4) if p[2 + i].lower() == "active"]))
-
     def __exit__(self, *a):
-        self.stop.set()
-        if self.proc:
-            time.sleep(0.15)
-            self.proc.terminate()
-            try:
-                self.proc.wait(timeout=2)
-            except Exception:
-                self.proc.kill()
+        if not self.proc:
+            return
+        try:
+            if self.mode == "nvml":
+                out, _ = self.proc.communicate(input="stop\n", timeout=10)
+                for line in out.splitlines():
+                    if line.startswith("{"):
+                        d = json.loads(line)
+                        if "rows" in d:
+                            self.rows = [(float(r[0]), list(r[1])) for r in d["rows"]]
+            else:
+                time.sleep(0.15)
+                self.proc.terminate()
+                out, _ = self.proc.communicate(timeout=5)
+                names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+                for line in out.splitlines():
+                    p = [x.strip() for x in line.split(",")]
+                    if len(p) == 6 and p[0].replace(".", "").isdigit():
+                        self.max_mhz = float(p[1])
+                        self.rows.append((float(p[0]), [names[i] for i in range(4) if p[2 + i].lower() == "active"]))
+        except Exception:
+            self.proc.kill()
 
     def summary(self):
         if not self.rows:
@@ -224,6 +239,8 @@ def main():
     extra = json.loads(os.environ.get("GSH_BENCH_CFG", "{}"))  # experiments only
     if args.detect == "sampled":
         extra["detect_mode"] = 1
+    # per-phase CUDA events stay on inside the timed region (the roofline's kernel time is
+    # measured live there); they cost ~30 us of host time per call, included in the step time
     cfg = gsh.make_config(timing=True, **extra)
     if world > 1:
         from paper_conf_icde_caic24_b200 import sharded
