@@ -13,17 +13,25 @@ namespace gsh {
 #define GSH_SCATTER_BLOCK 512
 #endif
 #ifndef GSH_SCATTER_IPT
-#define GSH_SCATTER_IPT 8
+#define GSH_SCATTER_IPT 12
 #endif
 constexpr int kScatterBlock = GSH_SCATTER_BLOCK;  // threads per partition-scatter CTA
 constexpr int kScatterIpt = GSH_SCATTER_IPT;      // tuples per thread per tile
 #ifndef GSH_SCATTER_IPT1
-#define GSH_SCATTER_IPT1 16
+#define GSH_SCATTER_IPT1 20
 #endif
 constexpr int kScatterIpt1 = GSH_SCATTER_IPT1;    // pass 1: tuples per thread per tile
-constexpr int kScatterTile = kScatterBlock * kScatterIpt;  // 4096 tuples per tile (pass 2)
+#ifndef GSH_SCATTER_BLOCK2
+#define GSH_SCATTER_BLOCK2 448
+#endif
+constexpr int kScatterBlock2 = GSH_SCATTER_BLOCK2;  // pass 2: threads per CTA (tuples per thread: kScatterIpt)
+constexpr int kScatterTile = kScatterBlock * kScatterIpt;  // TMA-store experiment tile
 constexpr int kScatterChunk = 16384;               // keys: the histogram's load granule (unit lengths are multiples)
-static_assert(kScatterChunk % (kScatterBlock * kScatterIpt1) == 0, "pass-1 units are whole tiles");
+#ifndef GSH_SCATTER_BLOCK1
+#define GSH_SCATTER_BLOCK1 256
+#endif
+constexpr int kScatterBlock1 = GSH_SCATTER_BLOCK1;  // pass 1: threads per CTA
+static_assert(kScatterIpt1 % 4 == 0 && kScatterIpt % 2 == 0, "vector tile loads: uint4 = 4 keys / 2 tuples");
 constexpr uint32_t kHistMaxUnitChunks = 64;      // a pass-1 unit (= histogram slice) is <= 64 chunks = 2^20 tuples
 constexpr uint32_t kGroupTuples = 1u << 23;       // target tuples per pass-2 unit group (8M)
 constexpr int kMaxDigitBits = 8;                // radix bits per pass (256 buckets)

@@ -736,12 +736,14 @@ int launch_scatter(const Plan& p, int pass, const uint32_t* const keys[2], const
     }
     // (TMA bulk stores per bucket run, cfg 1, measured slower on cfg2: 1.12 / 1.24 ms vs
     // 1.06 / 1.17 ms for the per-tuple whole-sector stores -- barrier-bound, ALU 49 % vs 28 %)
-    // Tile shapes per pass (measured on cfg2, scripts/gpu_variants.sh): pass 1 (SoA input,
-    // hashes computed in the kernel) prefers 512 x 16 = 8192-tuple tiles (1.013 -> 0.946 ms),
-    // pass 2 (AoS) 512 x 8 (1.032 ms vs 1.061 for 512 x 16, 1.109 for 1024 x 8).
+    // Tile shapes per pass (measured on cfg2, scripts/gpu_variants.sh): the largest tiles that
+    // still let two CTAs share an SM's 227 KB win -- pass 1 (SoA, hashes in-kernel) 256 x 20 =
+    // 5120 tuples (0.927 ms; 512 x 8: 1.013, 512 x 16 at one CTA/SM: 0.944), pass 2 (AoS)
+    // 448 x 12 = 5376 tuples (0.976 ms; 512 x 8: 1.032, 384 x 12: 1.011, 512 x 12: 1.187).
+    // Tiles need not divide a unit: a unit's ragged last tile takes the scalar path.
     if (cfg == 1) return launch_scatter_cfg<kScatterBlock, kScatterIpt, true>(p, a, s);
-    return pass == 1 ? launch_scatter_pass<kScatterBlock, kScatterIpt1, 1, false>(p, a, s)
-                     : launch_scatter_pass<kScatterBlock, kScatterIpt, 2, false>(p, a, s);
+    return pass == 1 ? launch_scatter_pass<kScatterBlock1, kScatterIpt1, 1, false>(p, a, s)
+                     : launch_scatter_pass<kScatterBlock2, kScatterIpt, 2, false>(p, a, s);
 }
 
 // ----------------------------------------------- standalone radix histogram (ABI) --
