@@ -51,6 +51,31 @@ def test_cfg2_count_checksum_fullsize(cfg2):
     assert r.stats["n_large"] == 0  # uniform keys never trigger detection
 
 
+def test_pkfk_2e30_count_checksum():
+    """8x the bench size (|R| = |S| = 2^30): partitions average 16K tuples per side, beyond the
+    streamed NM kernel's staging limit, so the NM-join runs on the general (R-chunk, S-slice)
+    path; count = n_S and the closed-form checksum (oracle pair_hash over the generator's row
+    map, computed in chunks on the CPU) must still hold exactly."""
+    n = 1 << 30
+    if torch.cuda.get_device_properties(0).total_memory < (96 << 30):
+        pytest.skip("needs a GPU with >= 96 GB")
+    rk, rp, sk, sp = datagen.pkfk_pair(n, n, seed=0x6A5, device="cuda")
+    torch.cuda.synchronize()
+    r = gsh.join(rk, rp, sk, sp)
+    del rk, rp, sk, sp
+    torch.cuda.empty_cache()
+    assert r.count == n
+    expect = 0
+    step = 1 << 24
+    base = datagen.gen._stream_base(0x6A5, 1)
+    for b in range(0, n, step):
+        idx = torch.arange(b, b + step, dtype=torch.int64) + base
+        rows = (datagen.gen._srl(datagen.gen.splitmix64(idx), 1) % n).numpy().astype(np.uint32)
+        expect += int(np.sum(oracle.pair_hash(rows, np.arange(b, b + step, dtype=np.uint32)), dtype=np.uint64))
+    assert r.checksum == expect & ((1 << 64) - 1)
+    assert r.stats["n_large"] == 0
+
+
 def test_cfg2_materialize_fullsize(cfg2):
     rk, rp, sk, sp = cfg2
     r = gsh.join(rk, rp, sk, sp, mode="materialize", out_capacity=N2 + 16)
