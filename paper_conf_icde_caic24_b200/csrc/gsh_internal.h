@@ -52,8 +52,12 @@ constexpr uint32_t kRingBytes = (kRingGroups == 1 ? 192u : 160u) * 1024u;
 // being joined or queued behind one that is, so the producer only ever waits for progress);
 // half the ring keeps at least two in flight.
 constexpr uint32_t kRingItemMax = kRingBytes / 2;
-__host__ __device__ __forceinline__ bool ring_eligible(uint32_t rl, uint32_t sl) {
-    return rl > 0 && sl > 0 && rl <= kRingMaxR && (uint64_t(rl) + sl) * 8 + 32 <= kRingItemMax;
+// The chained table (links are 16-bit byte offsets) stages R sides up to kRingMaxRChain tuples;
+// the CSR table (packed-u16 bucket words) up to kRingMaxR.
+constexpr uint32_t kRingMaxRChain = 8190;
+__host__ __device__ __forceinline__ bool ring_eligible(uint32_t rl, uint32_t sl, bool chain) {
+    return rl > 0 && sl > 0 && rl <= (chain ? kRingMaxRChain : kRingMaxR) &&
+           (uint64_t(rl) + sl) * 8 + 32 <= kRingItemMax;
 }
 constexpr int kSkewBlock = 256;                 // skewed-key join CTA
 constexpr int kSkewSpt = 4;                     // S payloads per thread (registers)

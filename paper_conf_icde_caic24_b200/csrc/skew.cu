@@ -465,10 +465,11 @@ __global__ void k_nm_setup(const uint2* bufB0, const uint2* bufB1, const uint2* 
 struct NmItems {
     const NmPart* nm;
     uint32_t C;
+    int chain;   // the streamed kernel's table (its R-side limit differs)
     __device__ uint64_t operator()(uint64_t p) const {
         const NmPart d = nm[p];
         if (d.rlen == 0 || d.slen == 0) return 0;
-        if (ring_eligible(d.rlen, d.slen)) return 0;  // streamed kernel (nm_ring.cu)
+        if (ring_eligible(d.rlen, d.slen, chain != 0)) return 0;  // streamed kernel (nm_ring.cu)
         return uint64_t((d.rlen + C - 1) / C) * ((d.slen + kNmSlice - 1) / kNmSlice);
     }
 };
@@ -478,7 +479,7 @@ int launch_nm_setup(const Plan& p, uint32_t n_large, cudaStream_t s) {
     unsigned grid = (p.F + 255) / 256;
     k_nm_setup<<<grid, 256, 0, s>>>(p.bufB[0], p.bufB[1], p.bufA[0], p.bufA[1], p.start, p.cnt, p.large_idx,
                                     p.part_heavy, p.nrm_off, p.F, p.nm);
-    return 1 + launch_scan(NmItems{p.nm, p.C}, p.F, p.nm_prefix, p.scan_scratch, s);
+    return 1 + launch_scan(NmItems{p.nm, p.C, p.nm_chain}, p.F, p.nm_prefix, p.scan_scratch, s);
 }
 
 }  // namespace gsh

@@ -51,12 +51,14 @@ def test_cfg2_count_checksum_fullsize(cfg2):
     assert r.stats["n_large"] == 0  # uniform keys never trigger detection
 
 
-def test_pkfk_2e30_count_checksum():
-    """8x the bench size (|R| = |S| = 2^30): partitions average 16K tuples per side, beyond the
-    streamed NM kernel's staging limit, so the NM-join runs on the general (R-chunk, S-slice)
-    path; count = n_S and the closed-form checksum (oracle pair_hash over the generator's row
-    map, computed in chunks on the CPU) must still hold exactly."""
-    n = 1 << 30
+@pytest.mark.parametrize("logn", [28, 30])
+def test_pkfk_large_count_checksum(logn):
+    """2x and 8x the bench size.  |R| = |S| = 2^28: partitions average 4096 tuples per side, so
+    about half of them exceed the CSR staging limit and stream through the chained table's
+    larger one (kRingMaxRChain); 2^30: 16K per side, beyond any staging limit, so the NM-join
+    runs on the general (R-chunk, S-slice) path.  count = n_S and the closed-form checksum
+    (oracle pair_hash over the generator's row map, computed in chunks on the CPU) must hold."""
+    n = 1 << logn
     if torch.cuda.get_device_properties(0).total_memory < (96 << 30):
         pytest.skip("needs a GPU with >= 96 GB")
     rk, rp, sk, sp = datagen.pkfk_pair(n, n, seed=0x6A5, device="cuda")
