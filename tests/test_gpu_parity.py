@@ -84,18 +84,30 @@ def _keys_in_bins(bins, hi, nbits):
 @pytest.mark.parametrize("route_bits", [0, 1])
 def test_partition_histogram_u16_wraps(route_bits):
     """2^16 partitions use packed u16 counters per histogram slice: digits that
-    receive >= 2^16 keys of one 2^19-tuple slice wrap, both halves of one counter word wrap, and a
-    low-half carry can wrap the high half -- offsets must still equal the oracle's exact scan."""
+    receive >= 2^16 keys of one slice wrap, both halves of one counter word wrap, and a low-half
+    carry can wrap the high half -- offsets must still equal the oracle's exact scan.  Slices are
+    the pass-1 units (~one per scatter CTA, whole 16K-key chunks): at n = 2^24 + 2^21 per side
+    a slice holds 8 chunks = 2^17 keys, so 2^17 copies of one digit wrap its u16 twice."""
     pass_bits, B = (8, 8), 16
     ka, kb, kc = _keys_in_bins([0x1234, 0x1235, 0x7777], route_bits, B)   # ka, kb share a counter word
-    n = (1 << 20) + 77
+    n = (1 << 24) + (1 << 21) + 77
     g = np.random.default_rng(5)
     keys = g.integers(0, 1 << 32, n, dtype=np.uint64).astype(np.uint32)
-    pos = g.permutation(n)
-    keys[pos[:300_000]] = ka          # > 4 wraps of the even bin
-    keys[pos[300_000:560_000]] = kb   # ~4 wraps of the odd bin, interleaved with the carries
+    keys[: 1 << 18] = ka                                   # two whole slices of one (even) digit
+    keys[(1 << 18):(1 << 18) + (1 << 17):2] = ka           # a slice split evenly between the two
+    keys[(1 << 18) + 1:(1 << 18) + (1 << 17):2] = kb       # halves of one word: both wrap, with carries
+    pos = g.permutation(np.arange((1 << 19), n))
+    keys[pos[:300_000]] = ka
+    keys[pos[300_000:560_000]] = kb
     keys[pos[560_000:626_000]] = kc
-    keys[: 1 << 17] = ka              # the first slice almost all one digit
+    # precondition: with the library's unit sizing (api.cu plan_build) some slice holds >= 2^16
+    # keys of one digit, so the wrap accounting really runs
+    sms = torch.cuda.get_device_properties(0).multi_processor_count
+    nch = -(-n // 16384)
+    uc = min(64, max(1, -(-(2 * nch) // (2 * sms))))
+    dig = (oracle.fmix32(keys) << np.uint32(route_bits)) >> np.uint32(32 - B)
+    per_slice = [np.bincount(dig[u:u + uc * 16384], minlength=1 << B).max() for u in range(0, n, uc * 16384)]
+    assert max(per_slice) >= 1 << 16
     rk = torch.from_numpy(keys.view(np.int32).copy())
     rp = torch.arange(n, dtype=torch.int32)
     sk, sp = rk.flip(0).contiguous(), rp.clone()
