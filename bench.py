@@ -306,13 +306,15 @@ def main():
     except Exception:
         pass
     if dom == "ms_skewjoin":
-        # ALU roofline of the dense skewed-key tiles: 8 IMAD-pipe ops per pair (SASS), the IMAD
-        # pipe retires 64 lanes/clk/SM -> 8 pairs/clk/SM x 148 SMs x max SM clock
+        # ALU roofline of the dense skewed-key tiles: the inner loop's SASS issues
+        # 7.5 ALU-pipe ops per pair (LOP3 3.25, SHF 2.25, IADD3 2; the IMADs go to the FMA pipe),
+        # and the ALU pipe retires 64 lanes/clk/SM -> 64 / 7.5 = 8.53 pairs/clk/SM x 148 SMs x
+        # max SM clock (ncu on cfg1: ALU pipe 72.8 % busy = this kernel's frac)
         mhz = clocks.get("sm_max_mhz") or 1965.0
-        alu_peak = 8 * 148 * mhz * 1e6 / 1e9
+        alu_peak = (64 / 7.5) * 148 * mhz * 1e6 / 1e9
         achieved = st.get("skew_pairs", 0) / (phases[dom] / 1e3) / 1e9 if phases.get(dom) else None
         roofline = {"bound": "alu", "kernel": kernels[dom], "achieved": achieved, "peak": alu_peak,
-                    "peak_source": "derived: 8 pairs/clk/SM (IMAD pipe) x 148 SMs x max SM clock",
+                    "peak_source": "derived: 64 ALU lanes/clk/SM / 7.5 ALU ops per pair x 148 SMs x max SM clock",
                     "unit": "Gpairs/s", "frac": (achieved / alu_peak) if achieved else None, "traffic": traffic,
                     "algorithmic_pairs_per_launch": st.get("skew_pairs", 0)}
     else:
