@@ -306,17 +306,15 @@ def main():
     except Exception:
         pass
     if dom == "ms_skewjoin":
-        # Integer-pipe roofline of the dense skewed-key tiles, from the inner loop's
-        # SASS per pair: ALU pipe 7.0 ops (LOP3 3.25, SHF 2.25, IADD3 1.5), FMA pipe 9.25 issue
-        # slots (IMAD 3.25 + IMAD.IADD 2 + IMAD.WIDE 2 x 2 slots); both pipes retire 64 lanes/clk/SM
-        # for these integer ops (IMAD and IMAD.WIDE are not full rate: moving adds and shifts onto
-        # them made the phase slower) -> min(64/7.0, 64/9.25) = 6.92 pairs/clk/SM
-        # x 148 SMs x max SM clock
+        # ALU roofline of the dense skewed-key tiles: the inner loop's SASS issues
+        # 7.0 ALU-pipe ops per pair (LOP3 3.25, SHF 2.25, IADD3 1.5; the IMADs go to the FMA pipe,
+        # which ncu shows at ~1/3 of its issue rate), and the ALU pipe retires 64 lanes/clk/SM ->
+        # 64 / 7.0 = 9.14 pairs/clk/SM x 148 SMs x max SM clock
         mhz = clocks.get("sm_max_mhz") or 1965.0
-        alu_peak = min(64 / 7.0, 64 / 9.25) * 148 * mhz * 1e6 / 1e9
+        alu_peak = (64 / 7.0) * 148 * mhz * 1e6 / 1e9
         achieved = st.get("skew_pairs", 0) / (phases[dom] / 1e3) / 1e9 if phases.get(dom) else None
         roofline = {"bound": "alu", "kernel": kernels[dom], "achieved": achieved, "peak": alu_peak,
-                    "peak_source": "derived: 64 lanes/clk/SM / 9.25 FMA-pipe slots per pair (binding; ALU 7.0) x 148 SMs x max SM clock",
+                    "peak_source": "derived: 64 ALU lanes/clk/SM / 7.0 ALU ops per pair x 148 SMs x max SM clock",
                     "unit": "Gpairs/s", "frac": (achieved / alu_peak) if achieved else None, "traffic": traffic,
                     "algorithmic_pairs_per_launch": st.get("skew_pairs", 0)}
     else:
