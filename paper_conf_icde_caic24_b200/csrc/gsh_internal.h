@@ -42,12 +42,21 @@ constexpr uint32_t kMaxCapacity = 8192;         // largest NM build table (tuple
 constexpr uint32_t kNmSlice = 8192;             // S tuples probed per NM work item
 // Streamed NM-join (nm_ring.cu): one producer warp + kRingGroups consumer groups of
 // kRingGroupWarps warps; partition pairs staged by TMA in a shared-memory byte ring.
-constexpr int kRingGroups = 2;
-constexpr int kRingGroupWarps = 15;
+#ifndef GSH_RING_GROUPS
+#define GSH_RING_GROUPS 2
+#endif
+#ifndef GSH_RING_GROUP_WARPS
+#define GSH_RING_GROUP_WARPS 15
+#endif
+#ifndef GSH_RING_KB
+#define GSH_RING_KB (kRingGroups == 1 ? 192u : 160u)
+#endif
+constexpr int kRingGroups = GSH_RING_GROUPS;
+constexpr int kRingGroupWarps = GSH_RING_GROUP_WARPS;
 constexpr int kRingThreads = 32 + kRingGroups * kRingGroupWarps * 32;
 constexpr uint32_t kRingMaxR = 4096;            // largest staged R side = most CSR buckets
 constexpr uint32_t kRingSeBytes = kRingGroups * 2 * kRingMaxR * 4;  // bucket (start, end) tables
-constexpr uint32_t kRingBytes = (kRingGroups == 1 ? 192u : 160u) * 1024u;
+constexpr uint32_t kRingBytes = GSH_RING_KB * 1024u;
 // An item (R_p and S_p spans, 16-byte aligned) must fit the empty ring (every resident item is
 // being joined or queued behind one that is, so the producer only ever waits for progress);
 // half the ring keeps at least two in flight.
