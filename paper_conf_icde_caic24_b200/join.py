@@ -8,7 +8,6 @@ no CPU path: calling with CPU tensors raises.
 from __future__ import annotations
 
 import ctypes
-from dataclasses import dataclass, field
 
 import torch
 
@@ -39,14 +38,26 @@ def make_config(capacity: int = 0, pass_bits=None, heavy_threshold: int = 0, rou
     return cfg
 
 
-@dataclass
 class JoinResult:
-    count: int
-    checksum: int
-    written: int = 0
-    overflow: bool = False
-    pairs: torch.Tensor | None = None   # (written, 2) int32 view of (payload_R, payload_S)
-    stats: dict = field(default_factory=dict)
+    """count, checksum (mod 2^64), written, overflow, pairs ((written, 2) int32 view of
+    (payload_R, payload_S) or None) and stats (every gsh_result field, built on first access)."""
+
+    __slots__ = ("count", "checksum", "written", "overflow", "pairs", "_stats", "_raw")
+
+    def __init__(self, count: int, checksum: int, written: int = 0, overflow: bool = False,
+                 pairs: torch.Tensor | None = None, stats: dict | None = None, raw=None):
+        self.count, self.checksum, self.written, self.overflow, self.pairs = count, checksum, written, overflow, pairs
+        self._stats, self._raw = stats, raw
+
+    @property
+    def stats(self) -> dict:
+        if self._stats is None:
+            self._stats = self._raw.as_dict() if self._raw is not None else {}
+        return self._stats
+
+    def __repr__(self) -> str:
+        return (f"JoinResult(count={self.count}, checksum={self.checksum:#x}, written={self.written}, "
+                f"overflow={self.overflow})")
 
 
 def _check_dev(t: torch.Tensor, name: str) -> torch.Tensor:
@@ -130,20 +141,22 @@ def join(r_keys: torch.Tensor, r_payloads: torch.Tensor, s_keys: torch.Tensor, s
         if not out.is_contiguous():
             raise ValueError("out must be contiguous")
         outp = GshOutput(out.data_ptr() if out.numel() else None, out.shape[0])
-    nb = workspace_bytes(R.n, S.n, config)
-    ws = workspace if workspace is not None else _default_ws.get(nb, dev)
-    if ws.numel() < nb:
-        raise ValueError(f"workspace too small ({ws.numel()} < {nb} bytes)")
+    if workspace is not None:   # gsh_join itself rejects a too-small workspace (GSH_ERR_INVALID)
+        ws = workspace
+    else:
+        ws = _default_ws.get(workspace_bytes(R.n, S.n, config), dev)
     res = GshResult()
-    with torch.cuda.device(dev):
-        st = lib.gsh_join(ctypes.byref(R), ctypes.byref(S), _lib.GSH_OUT_MATERIALIZE if mat else _lib.GSH_OUT_COUNT,
-                          ctypes.byref(outp) if outp is not None else None, ws.data_ptr(), ws.numel(),
-                          ctypes.byref(config) if config is not None else None, _stream_handle(stream),
-                          ctypes.byref(res))
+    args = (ctypes.byref(R), ctypes.byref(S), _lib.GSH_OUT_MATERIALIZE if mat else _lib.GSH_OUT_COUNT,
+            ctypes.byref(outp) if outp is not None else None, ws.data_ptr(), ws.numel(),
+            ctypes.byref(config) if config is not None else None, _stream_handle(stream), ctypes.byref(res))
+    if dev.index == torch.cuda.current_device():
+        st = lib.gsh_join(*args)
+    else:
+        with torch.cuda.device(dev):
+            st = lib.gsh_join(*args)
     check(st, "gsh_join")
-    d = res.as_dict()
     return JoinResult(count=int(res.count), checksum=int(res.checksum), written=int(res.written),
-                      overflow=bool(res.overflow), pairs=(out[: res.written] if mat else None), stats=d)
+                      overflow=bool(res.overflow), pairs=(out[: res.written] if mat else None), raw=res)
 
 
 def join_host(r_keys, r_payloads, s_keys, s_payloads, mode: str = "count", out=None, out_capacity=None,
@@ -182,7 +195,7 @@ def join_host(r_keys, r_payloads, s_keys, s_payloads, mode: str = "count", out=N
                                ctypes.byref(res))
     check(st, "gsh_join_host")
     return JoinResult(count=int(res.count), checksum=int(res.checksum), written=int(res.written),
-                      overflow=bool(res.overflow), pairs=(out[: res.written] if mat else None), stats=res.as_dict())
+                      overflow=bool(res.overflow), pairs=(out[: res.written] if mat else None), raw=res)
 
 
 # ------------------------------------------------------------------ step entry points
