@@ -114,3 +114,40 @@ def test_zipf_2e24_closed_form_and_invariance(theta):
     assert (r2.count, r2.checksum) == (r.count, r.checksum)
     r3 = gsh.join(rk, rp, sk, sp, config=gsh.make_config(large_threshold=1, heavy_threshold=2))
     assert (r3.count, r3.checksum) == (r.count, r.checksum)
+
+
+@pytest.mark.parametrize("theta", [0.25, 0.5])
+def test_cfg3_materialize_fullsize(theta):
+    """cfg3 at its full size (|R| = |S| = 2^27, both sides Zipf theta, N = n) in MATERIALIZE mode
+    (SURVEY §8(c) P3): count equals the closed form from exact key histograms, written == count,
+    every written pair is a real match (payload = row id), no pair repeats, and the oracle's
+    checksum over the written pairs equals the returned one -- together the pair multiset is M."""
+    n = N2
+    rk, rp, sk, sp = datagen.zipf_pair(n, n, theta, seed=0x6A5, device="cuda")
+    expect = _closed_form(rk, sk)
+    r = gsh.join(rk, rp, sk, sp, mode="materialize", out_capacity=expect + 16)
+    assert (r.count, r.written, r.overflow) == (expect, expect, False)
+    p = r.pairs.long() & 0xFFFFFFFF
+    a, b = p[:, 0], p[:, 1]
+    assert bool((rk[a] == sk[b]).all())
+    assert torch.unique((a << 32) | b).numel() == expect
+    del p, a, b
+    pc = r.pairs.cpu().numpy().view(np.uint32)
+    chk = 0
+    for s in range(0, expect, 1 << 24):
+        chk += int(np.sum(oracle.pair_hash(pc[s:s + (1 << 24), 0], pc[s:s + (1 << 24), 1]), dtype=np.uint64))
+    assert chk & ((1 << 64) - 1) == r.checksum
+    if theta == 0.5:
+        assert r.stats["n_heavy"] > 0    # the skewed-key phase wrote part of the pairs
+
+
+def test_cfg3_theta075_count_fullsize():
+    """cfg3 at theta = 0.75, full size (2.6e11 pairs: COUNT only): count equals the closed form, and
+    the checksum is identical when every pair goes through the NM-join instead (no detection)."""
+    n = N2
+    rk, rp, sk, sp = datagen.zipf_pair(n, n, 0.75, seed=0x6A5, device="cuda")
+    r = gsh.join(rk, rp, sk, sp)
+    assert r.count == _closed_form(rk, sk)
+    assert r.stats["n_heavy"] > 0 and r.stats["n_large"] > 0
+    r2 = gsh.join(rk, rp, sk, sp, config=gsh.make_config(force_all_normal=True))
+    assert (r2.count, r2.checksum) == (r.count, r.checksum)
