@@ -32,6 +32,8 @@ constexpr int kScatterChunk = 16384;               // keys: the histogram's load
 #endif
 constexpr int kScatterBlock1 = GSH_SCATTER_BLOCK1;  // pass 1: threads per CTA
 static_assert(kScatterIpt1 % 4 == 0 && kScatterIpt % 2 == 0, "vector tile loads: uint4 = 4 keys / 2 tuples");
+static_assert(kScatterBlock1 >= 256 && kScatterBlock2 >= 256 && kScatterBlock >= 256,
+              "scatter CTAs keep one thread per bucket (2^kMaxDigitBits = 256)");
 constexpr uint32_t kHistMaxUnitChunks = 64;      // a pass-1 unit (= histogram slice) is <= 64 chunks = 2^20 tuples
 constexpr uint32_t kGroupTuples = 1u << 23;       // target tuples per pass-2 unit group (8M)
 constexpr int kMaxDigitBits = 8;                // radix bits per pass (256 buckets)
