@@ -30,5 +30,18 @@ for w in order + sorted(set(rows) - set(order)):
     out.append(f"| {d['config']['workload']} | {d['value']:.3g} | {d['output_tuples_per_s']:.3g} | {d['ms_per_step']:.3f} | "
                f"{p['ms_hist']:.3f} | {p['ms_pass1']:.3f} | {p['ms_pass2']:.3f} | {p['ms_detect']:.3f} | {p['ms_split']:.3f} | "
                f"{p['ms_nmjoin']:.3f} | {p['ms_skewjoin']:.3f} | {s['n_heavy']} | {s['n_large']} |")
+mat = sorted(glob.glob(os.path.join(ROOT, "gpurun_out", "sweepmat_*.json")))
+if mat:
+    out += ["", "MATERIALIZE (`--mode materialize --out-cap 2^30`: pairs written to an 8 GiB device buffer; the NM-join"
+                " counts each item's matches, reserves one output range, then emits)", "",
+            "| workload | input tuples/s | output tuples/s | ms/step | NM | skew | written | overflow |", "|---|---|---|---|---|---|---|---|"]
+    for f in mat:
+        try:
+            d = json.load(open(f))
+        except Exception:
+            continue
+        p, s_ = d["phases_ms"], d["stats"]
+        out.append(f"| {d['config']['workload']} | {d['value']:.3g} | {d['output_tuples_per_s']:.3g} | {d['ms_per_step']:.3f} | "
+                   f"{p['ms_nmjoin']:.3f} | {p['ms_skewjoin']:.3f} | {s_['written']} | {s_['overflow']} |")
 open(os.path.join(ROOT, "profiles", f"{tag}_sweep.md"), "w").write("\n".join(out) + "\n")
 print("\n".join(out))
