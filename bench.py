@@ -232,6 +232,8 @@ def main():
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     kind, n, theta, desc = WORKLOADS[args.workload]
+    if args.mode == "materialize":
+        desc = desc.replace("COUNT", "MATERIALIZE")
     dist = None
     if world > 1:
         import torch.distributed as dist

@@ -41,7 +41,7 @@ if mat:
         except Exception:
             continue
         p, s_ = d["phases_ms"], d["stats"]
-        out.append(f"| {d['config']['workload']} | {d['value']:.3g} | {d['output_tuples_per_s']:.3g} | {d['ms_per_step']:.3f} | "
+        out.append(f"| {d['config']['workload'].replace('COUNT', 'MATERIALIZE')} | {d['value']:.3g} | {d['output_tuples_per_s']:.3g} | {d['ms_per_step']:.3f} | "
                    f"{p['ms_nmjoin']:.3f} | {p['ms_skewjoin']:.3f} | {s_['written']} | {s_['overflow']} |")
 open(os.path.join(ROOT, "profiles", f"{tag}_sweep.md"), "w").write("\n".join(out) + "\n")
 print("\n".join(out))
