@@ -234,11 +234,25 @@ __global__ void k_hist_reduce(const uint32_t* __restrict__ partial, uint32_t* __
         const uint32_t ns = side ? ns1 : ns0, ng = side ? ng1 : ng0;
         const uint32_t* base = partial + size_t(side ? ns0 : 0) * F + bin;
         uint32_t* o2 = off2 + size_t(side ? ng0 : 0) * F + bin;
-        uint32_t run = 0;
-        for (uint32_t g = 0; g < ng; ++g) {
-            o2[size_t(g) * F] = run;
-            const uint32_t s0 = g * group_units, s1 = umin32(s0 + group_units, ns);
-            for (uint32_t s = s0; s < s1; ++s) run += base[size_t(s) * F];
+        // slices in order, 8 loads in flight per thread; off2 of group g = the running sum when
+        // its first slice comes up
+        (void)ng;
+        uint32_t run = 0, g = 0, left = 0;
+        for (uint32_t s = 0; s < ns; s += 8) {
+            uint32_t v[8];
+#pragma unroll
+            for (int k = 0; k < 8; ++k) v[k] = (s + k < ns) ? base[size_t(s + k) * F] : 0u;
+#pragma unroll
+            for (int k = 0; k < 8; ++k) {
+                if (s + k < ns) {
+                    if (left == 0) {
+                        o2[size_t(g++) * F] = run;
+                        left = group_units;
+                    }
+                    --left;
+                    run += v[k];
+                }
+            }
         }
         cnt[i] = run;
     }
