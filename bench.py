@@ -297,8 +297,11 @@ def main():
     st = r.stats
     heavy_t = st.get("heavy_tuples_r", 0) + st.get("heavy_tuples_s", 0)
     # algorithmic bytes per launch: hist 4 B, each pass 16 B, NM 8 B per normal tuple
-    algo = {"ms_hist": 4 * n_tot, "ms_pass1": 16 * n_tot, "ms_pass2": 16 * n_tot, "ms_nmjoin": 8 * (n_tot - heavy_t)}
-    kernels = {"ms_pass1": "k_scatter (pass 1)", "ms_pass2": "k_scatter (pass 2)", "ms_nmjoin": "k_nmjoin_ring",
+    # (+ the pre-partition pass beyond 2^28 per side: 4 B count + 16 B split per tuple; with it the
+    # phase figures below are summed over the 2^prepass_bits sub-joins)
+    algo = {"ms_hist": 4 * n_tot, "ms_pass1": 16 * n_tot, "ms_pass2": 16 * n_tot, "ms_nmjoin": 8 * (n_tot - heavy_t),
+            "ms_prepass": 20 * n_tot}
+    kernels = {"ms_prepass": "k_split_count + k_split_scatter", "ms_pass1": "k_scatter (pass 1)", "ms_pass2": "k_scatter (pass 2)", "ms_nmjoin": "k_nmjoin_ring",
                "ms_hist": "k_hist2d", "ms_skewjoin": "k_skewjoin"}
     dom = max(list(algo) + ["ms_skewjoin"], key=lambda k: phases.get(k, 0.0))
     traffic = None

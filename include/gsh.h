@@ -107,6 +107,13 @@ typedef struct {
                                   result never depends on it. */
     uint32_t sample_stride;    /* detect_mode 1: 1 tuple in sample_stride is sampled.  0 = 100 (1 %) */
     uint32_t top_k;            /* detect_mode 1: skewed keys per large partition.  0 = 3 (L112) */
+    int32_t prepass_bits;      /* pre-partition pass: split R and S by this many
+                                  hash bits below route_bits and join each of the 2^bits
+                                  sub-problems separately, so partitions stay shared-memory
+                                  sized beyond the 2^16-partition limit of the two radix passes
+                                  (L106).  0 = auto (enough bits that each side's share is
+                                  <= 2^28 tuples; none up to 2^28);  -1 = off;  1..8 = forced.
+                                  The result never depends on it. */
 } gsh_config;
 
 /* Per-call result (host struct). */
@@ -130,13 +137,16 @@ typedef struct {
     uint32_t large_threshold;  /* L actually used */
     int32_t nm_table;          /* NM-join table used by the streamed kernel: 1 = CSR, 2 = chained */
     float ms_hist, ms_pass1, ms_pass2, ms_detect, ms_split, ms_nmjoin, ms_skewjoin, ms_total;
+    uint32_t prepass_bits;     /* pre-partition bits actually used (0 = none) */
+    float ms_prepass;          /* pre-partition pass (count + scatter), included in ms_total */
 } gsh_result;
 
 /* Fill *cfg with defaults (all auto, no hooks, timing off). */
 GSH_API void gsh_config_default(gsh_config *cfg);
 
 /* Bytes of device workspace gsh_join needs for these sizes (independent of the data).
- * Roughly 20 B per input tuple plus O(fanout) tables; see DESIGN.md §5. */
+ * Roughly 20 B per input tuple plus O(fanout) tables, + 16 B per tuple when the pre-partition
+ * pass runs (gsh_config.prepass_bits); see DESIGN.md §5. */
 GSH_API size_t gsh_workspace_bytes(uint64_t n_r, uint64_t n_s, const gsh_config *cfg);
 
 /*

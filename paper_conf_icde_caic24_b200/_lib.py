@@ -47,6 +47,7 @@ class GshConfig(ctypes.Structure):
         ("detect_mode", i32),
         ("sample_stride", u32),
         ("top_k", u32),
+        ("prepass_bits", i32),
     ]
 
 
@@ -78,6 +79,8 @@ class GshResult(ctypes.Structure):
         ("ms_nmjoin", ctypes.c_float),
         ("ms_skewjoin", ctypes.c_float),
         ("ms_total", ctypes.c_float),
+        ("prepass_bits", u32),
+        ("ms_prepass", ctypes.c_float),
     ]
 
     def as_dict(self) -> dict:

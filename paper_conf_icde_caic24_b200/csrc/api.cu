@@ -223,12 +223,17 @@ namespace {
 struct Timer {
     bool on;
     cudaStream_t s;
-    int used = 0;
+    int used, saved;
     static std::vector<cudaEvent_t>& pool() {
         static thread_local std::vector<cudaEvent_t> p;
         return p;
     }
-    explicit Timer(bool enable, cudaStream_t st) : on(enable), s(st) {}
+    static int& top() {   // first free pool slot; nested timers (pre-pass sub-joins) stack above
+        static thread_local int t = 0;
+        return t;
+    }
+    explicit Timer(bool enable, cudaStream_t st) : on(enable), s(st), used(top()), saved(top()) {}
+    ~Timer() { top() = saved; }
     int mark() {
         if (!on) return -1;
         auto& p = pool();
@@ -238,6 +243,7 @@ struct Timer {
             p.push_back(e);
         }
         cudaEventRecord(p[used], s);
+        top() = used + 1;
         return used++;
     }
     float ms(int a, int b) {
@@ -299,14 +305,82 @@ void gsh_config_default(gsh_config* cfg) {
     cfg->pass_bits[1] = -1;
 }
 
-size_t gsh_workspace_bytes(uint64_t n_r, uint64_t n_s, const gsh_config* cfg) {
+static size_t direct_workspace_bytes(uint64_t n_r, uint64_t n_s, const gsh_config* cfg) {
     Plan p;
     if (!plan_build(p, n_r, n_s, cfg, nullptr, device_sms())) return 0;
     return p.bytes;
 }
 
-gsh_status gsh_join(const gsh_relation* R, const gsh_relation* S, gsh_out_mode mode, const gsh_output* out,
-                    void* workspace, size_t workspace_bytes, const gsh_config* cfg, void* stream, gsh_result* res) {
+// Pre-partition pass bits (gsh_config.prepass_bits): auto = enough hash bits that each side's
+// sub-problem is <= 2^28 tuples (the two radix passes then keep partitions within the NM ring).
+// Returns -1 on a bad value.
+static int prepass_bits_for(uint64_t n_r, uint64_t n_s, const gsh_config* cfg) {
+    const int32_t want = cfg ? cfg->prepass_bits : 0;
+    const uint32_t rb = cfg ? cfg->route_bits : 0;
+    if (want < -1 || want > 8) return -1;
+    int r = 0;
+    if (want > 0) {
+        r = want;
+    } else if (want == 0) {
+        const uint64_t nmax = n_r > n_s ? n_r : n_s;
+        while (r < 8 && (nmax >> r) > (1ull << 28)) ++r;
+    }
+    if (r > 0 && rb + (uint32_t)r > 16) return want > 0 ? -1 : 0;
+    return r;
+}
+
+// Sub-problem config: the pre-partition bits are consumed like routing bits; no further pre-pass.
+static gsh_config sub_config(const gsh_config* cfg, int r) {
+    gsh_config c;
+    gsh_config_default(&c);
+    if (cfg) c = *cfg;
+    c.route_bits += (uint32_t)r;
+    c.prepass_bits = -1;
+    return c;
+}
+
+constexpr uint64_t kPrepassAlign = 64;   // tuples (256 B of u32)
+
+struct Prepass {
+    size_t sub_ws;        // workspace of one sub-problem's join (sized for the whole input)
+    uint32_t* rk; uint32_t* rp; uint32_t* sk; uint32_t* sp;
+    uint64_t* counts;     // [2][256]
+    uint64_t* offs;       // [2][256]
+    uint64_t* cur;        // [2][256]
+    size_t bytes;
+};
+
+static Prepass prepass_layout(uint64_t n_r, uint64_t n_s, const gsh_config* sub, unsigned char* base) {
+    Prepass q{};
+    q.sub_ws = direct_workspace_bytes(n_r, n_s, sub);
+    if (!q.sub_ws) return q;
+    size_t off = align256(q.sub_ws);
+    auto take = [&](size_t bytes) { unsigned char* p = base ? base + off : nullptr; off += align256(bytes); return p; };
+    // each sub-problem starts 256-byte aligned (kPrepassAlign tuples): the radix passes' vector
+    // and TMA bulk loads then see aligned inputs
+    q.rk = reinterpret_cast<uint32_t*>(take((n_r + 256 * kPrepassAlign) * 4));
+    q.rp = reinterpret_cast<uint32_t*>(take((n_r + 256 * kPrepassAlign) * 4));
+    q.sk = reinterpret_cast<uint32_t*>(take((n_s + 256 * kPrepassAlign) * 4));
+    q.sp = reinterpret_cast<uint32_t*>(take((n_s + 256 * kPrepassAlign) * 4));
+    q.counts = reinterpret_cast<uint64_t*>(take(2 * 256 * 8));
+    q.offs = reinterpret_cast<uint64_t*>(take(2 * 256 * 8));
+    q.cur = reinterpret_cast<uint64_t*>(take(2 * 256 * 8));
+    q.bytes = off;
+    return q;
+}
+
+size_t gsh_workspace_bytes(uint64_t n_r, uint64_t n_s, const gsh_config* cfg) {
+    const int r = prepass_bits_for(n_r, n_s, cfg);
+    if (r < 0) return 0;
+    if (r == 0) return direct_workspace_bytes(n_r, n_s, cfg);
+    const gsh_config sub = sub_config(cfg, r);
+    const Prepass q = prepass_layout(n_r, n_s, &sub, nullptr);
+    return q.sub_ws ? q.bytes : 0;
+}
+
+static gsh_status join_direct(const gsh_relation* R, const gsh_relation* S, gsh_out_mode mode, const gsh_output* out,
+                              void* workspace, size_t workspace_bytes, const gsh_config* cfg, void* stream,
+                              gsh_result* res) {
     if (!res) return fail(GSH_ERR_INVALID, "res is NULL");
     std::memset(res, 0, sizeof(*res));
     if (mode != GSH_OUT_COUNT && mode != GSH_OUT_MATERIALIZE) return fail(GSH_ERR_INVALID, "bad mode");
@@ -406,6 +480,116 @@ gsh_status gsh_join(const gsh_relation* R, const gsh_relation* S, gsh_out_mode m
         res->ms_skewjoin = tm.ms(e6, e7);
         res->ms_total = tm.ms(e0, e7);
     }
+    return GSH_OK;
+}
+
+// gsh_join: the direct path, or (beyond 2^28 tuples per side, or when forced) the pre-partition
+// pass -- split R and S by `r` hash bits below route_bits (route.cu k_split_*), then join each
+// of the 2^r sub-problems with the direct path.  Matches never cross sub-problems (equal keys,
+// equal h); count / checksum add mod 2^64, MATERIALIZE pairs are appended.
+gsh_status gsh_join(const gsh_relation* R, const gsh_relation* S, gsh_out_mode mode, const gsh_output* out,
+                    void* workspace, size_t workspace_bytes, const gsh_config* cfg, void* stream, gsh_result* res) {
+    if (!res) return fail(GSH_ERR_INVALID, "res is NULL");
+    std::memset(res, 0, sizeof(*res));
+    if (!validate_rel(R) || !validate_rel(S)) return fail(GSH_ERR_INVALID, "invalid relation (NULL or n >= 2^32)");
+    const int r = prepass_bits_for(R->n, S->n, cfg);
+    if (r < 0) return fail(GSH_ERR_INVALID, "invalid gsh_config (prepass_bits)");
+    if (r == 0 || R->n == 0 || S->n == 0)
+        return join_direct(R, S, mode, out, workspace, workspace_bytes, cfg, stream, res);
+    if (mode != GSH_OUT_COUNT && mode != GSH_OUT_MATERIALIZE) return fail(GSH_ERR_INVALID, "bad mode");
+    const bool mat = (mode == GSH_OUT_MATERIALIZE);
+    if (mat && (!out || (!out->pairs && out->capacity > 0)))
+        return fail(GSH_ERR_INVALID, "MATERIALIZE needs an output buffer");
+    const gsh_config sub = sub_config(cfg, r);
+    if (!workspace || (reinterpret_cast<uintptr_t>(workspace) & 255u))
+        return fail(GSH_ERR_INVALID, "workspace NULL or not 256-byte aligned");
+    const Prepass q = prepass_layout(R->n, S->n, &sub, reinterpret_cast<unsigned char*>(workspace));
+    if (!q.sub_ws) return fail(GSH_ERR_INVALID, "invalid gsh_config");
+    if (workspace_bytes < q.bytes) return fail(GSH_ERR_INVALID, "workspace too small");
+    cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+    const bool timing = cfg && cfg->timing;
+    Timer tm(timing, s);
+    const uint32_t G = 1u << r, skip = sub.route_bits - (uint32_t)r;
+    const int e0 = tm.mark();
+    cudaError_t ce = cudaMemsetAsync(q.counts, 0, 3 * align256(2 * 256 * 8), s);
+    if (ce != cudaSuccess) return cuda_fail(ce, "prepass memset");
+    int launches = 0;
+    launches += launch_split_count(R->keys, R->n, skip, (uint32_t)r, q.counts, s);
+    launches += launch_split_count(S->keys, S->n, skip, (uint32_t)r, q.counts + 256, s);
+    gsh_status st = check_launch("prepass count");
+    if (st != GSH_OK) return st;
+    uint64_t hc[512], ho[512];
+    ce = cudaMemcpyAsync(hc, q.counts, sizeof(hc), cudaMemcpyDeviceToHost, s);
+    if (ce == cudaSuccess) ce = cudaStreamSynchronize(s);
+    if (ce != cudaSuccess) return cuda_fail(ce, "prepass counts");
+    for (int side = 0; side < 2; ++side) {
+        uint64_t acc = 0, tot = 0;
+        for (uint32_t g = 0; g < 256; ++g) {
+            ho[side * 256 + g] = acc;
+            const uint64_t c = g < G ? hc[side * 256 + g] : 0;
+            acc = (acc + c + kPrepassAlign - 1) & ~(kPrepassAlign - 1);
+            tot += c;
+        }
+        if (tot != (side ? S->n : R->n)) return fail(GSH_ERR_INTERNAL, "prepass count mismatch");
+    }
+    ce = cudaMemcpyAsync(q.offs, ho, sizeof(ho), cudaMemcpyHostToDevice, s);
+    if (ce != cudaSuccess) return cuda_fail(ce, "prepass offsets");
+    launches += launch_split_scatter(R->keys, R->payloads, R->n, skip, (uint32_t)r, q.offs, q.cur, q.rk, q.rp, s);
+    launches += launch_split_scatter(S->keys, S->payloads, S->n, skip, (uint32_t)r, q.offs + 256, q.cur + 256,
+                                     q.sk, q.sp, s);
+    const int e1 = tm.mark();
+    if ((st = check_launch("prepass scatter")) != GSH_OK) return st;
+    const uint64_t cap = mat ? out->capacity : 0;
+    uint64_t written = 0;
+    gsh_result acc;
+    std::memset(&acc, 0, sizeof(acc));
+    for (uint32_t g = 0; g < G; ++g) {
+        const gsh_relation sR{q.rk + ho[g], q.rp + ho[g], hc[g]};
+        const gsh_relation sS{q.sk + ho[256 + g], q.sp + ho[256 + g], hc[256 + g]};
+        gsh_output so{mat && out->pairs ? out->pairs + 2 * written : nullptr, cap - written};
+        gsh_result sr;
+        st = join_direct(&sR, &sS, mode, mat ? &so : nullptr, workspace, q.sub_ws, &sub, stream, &sr);
+        if (st != GSH_OK) return st;
+        written += sr.written;
+        acc.count += sr.count;
+        acc.checksum += sr.checksum;
+        acc.normal_count += sr.normal_count;
+        acc.normal_checksum += sr.normal_checksum;
+        acc.heavy_tuples_r += sr.heavy_tuples_r;
+        acc.heavy_tuples_s += sr.heavy_tuples_s;
+        acc.skew_pairs += sr.skew_pairs;
+        acc.n_heavy += sr.n_heavy;
+        acc.n_large += sr.n_large;
+        acc.detect_overflow |= sr.detect_overflow;
+        acc.launches += sr.launches;
+        if (sR.n && sS.n) {   // parameters of a non-empty sub-problem
+            acc.pass_bits[0] = sr.pass_bits[0];
+            acc.pass_bits[1] = sr.pass_bits[1];
+            acc.capacity = sr.capacity;
+            acc.heavy_threshold = sr.heavy_threshold;
+            acc.large_threshold = sr.large_threshold;
+            acc.nm_table = sr.nm_table;
+        }
+        acc.ms_hist += sr.ms_hist;
+        acc.ms_pass1 += sr.ms_pass1;
+        acc.ms_pass2 += sr.ms_pass2;
+        acc.ms_detect += sr.ms_detect;
+        acc.ms_split += sr.ms_split;
+        acc.ms_nmjoin += sr.ms_nmjoin;
+        acc.ms_skewjoin += sr.ms_skewjoin;
+    }
+    const int e2 = tm.mark();
+    acc.written = mat ? written : 0;
+    acc.overflow = mat ? (acc.count > cap ? 1u : 0u) : 0u;
+    acc.launches += (uint32_t)launches;
+    acc.prepass_bits = (uint32_t)r;
+    if (timing) {
+        ce = cudaStreamSynchronize(s);
+        if (ce != cudaSuccess) return cuda_fail(ce, "prepass timing");
+        acc.ms_prepass = tm.ms(e0, e1);
+        acc.ms_total = tm.ms(e0, e2);
+    }
+    *res = acc;
     return GSH_OK;
 }
 

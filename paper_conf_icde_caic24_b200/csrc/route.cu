@@ -107,4 +107,175 @@ int launch_count_keys(const uint32_t* keys, uint64_t n, const uint32_t* q, uint6
     return 1;
 }
 
+// ---------------------------------------------------------------------------------------------
+// Split pass (DESIGN.md §5 "split pass"): beyond 2^28 tuples per side the two radix passes
+// (<= 2^16 partitions) leave partitions larger than the NM ring stages, so gsh_join first splits
+// both relations by `rb` hash bits below the `skip` bits already consumed (multi-GPU routing) and
+// joins each of the 2^rb sub-problems separately.  Equal keys have equal h, so every match lies
+// inside one sub-problem (partitioning by the hash of the key).  SoA in, SoA out.
+// Bucket peers are found with rb + 1 ballots (no __match_any_sync); one shared-memory atomic per
+// (warp, bucket) and one global cursor atomic per (tile, bucket).
+
+__device__ __forceinline__ uint32_t split_dest(uint32_t k, uint32_t skip, uint32_t rb) {
+    return (hash32(k) << skip) >> (32 - rb);
+}
+
+// lanes of this warp holding the same bucket d (valid lanes only)
+__device__ __forceinline__ uint32_t split_peers(bool v, uint32_t d, uint32_t rb) {
+    uint32_t peers = __ballot_sync(kFull, v);
+    for (uint32_t b = 0; b < rb; ++b) {
+        const bool bit = (d >> b) & 1u;
+        const uint32_t m = __ballot_sync(kFull, bit);
+        peers &= bit ? m : ~m;
+    }
+    return peers;
+}
+
+constexpr int kSplitBlock = 512;
+constexpr int kSplitIpt = 16;
+constexpr uint64_t kSplitTile = uint64_t(kSplitBlock) * kSplitIpt;
+
+// 8 independent key loads per thread in flight (one per 512-key stride of a 4096-key tile), so the
+// pass streams at HBM rate rather than at one load per thread's latency.
+__global__ void __launch_bounds__(kSplitBlock) k_split_count(const uint32_t* __restrict__ keys, uint64_t n,
+                                                            uint32_t skip, uint32_t rb, unsigned long long* counts) {
+    constexpr int kIpt = 8;
+    constexpr uint64_t kTile = uint64_t(kSplitBlock) * kIpt;
+    __shared__ uint32_t c[256];
+    const uint32_t G = 1u << rb;
+    for (uint32_t i = threadIdx.x; i < G; i += blockDim.x) c[i] = 0;
+    __syncthreads();
+    const uint64_t ntiles = (n + kTile - 1) / kTile;
+    for (uint64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
+        uint32_t k[kIpt];
+#pragma unroll
+        for (int j = 0; j < kIpt; ++j) {
+            const uint64_t i = t * kTile + uint64_t(j) * kSplitBlock + threadIdx.x;
+            k[j] = i < n ? __ldcs(keys + i) : 0u;
+        }
+#pragma unroll
+        for (int j = 0; j < kIpt; ++j) {
+            const bool v = t * kTile + uint64_t(j) * kSplitBlock + threadIdx.x < n;
+            const uint32_t d = v ? split_dest(k[j], skip, rb) : 0u;
+            const uint32_t peers = split_peers(v, d, rb);
+            if (v && (peers & lanemask_lt()) == 0) atomicAdd(&c[d], (uint32_t)__popc(peers));
+        }
+    }
+    __syncthreads();
+    for (uint32_t i = threadIdx.x; i < G; i += blockDim.x)
+        if (c[i]) atomicAdd(&counts[i], (unsigned long long)c[i]);
+}
+
+// One 8192-tuple tile per iteration: rank every tuple within its bucket (ballot peers + one shared
+// atomic per (warp, bucket)), reserve each bucket's run with one global atomic, permute the tile
+// into shared memory grouped by bucket, then write it out with consecutive threads on consecutive
+// addresses of a run (coalesced; only run ends touch partial sectors).
+constexpr size_t kSplitSmem = kSplitTile * (4 + 4 + 1);
+
+__global__ void __launch_bounds__(kSplitBlock, 2) k_split_scatter(const uint32_t* __restrict__ keys,
+                                                              const uint32_t* __restrict__ pays, uint64_t n,
+                                                              uint32_t skip, uint32_t rb,
+                                                              const uint64_t* __restrict__ off,
+                                                              unsigned long long* cur, uint32_t* __restrict__ ok,
+                                                              uint32_t* __restrict__ op) {
+    extern __shared__ uint4 split_dyn[];
+    uint32_t* s_k = reinterpret_cast<uint32_t*>(split_dyn);
+    uint32_t* s_p = s_k + kSplitTile;
+    uint8_t* s_d = reinterpret_cast<uint8_t*>(s_p + kSplitTile);
+    __shared__ uint32_t cnt[256], pre[256];
+    __shared__ unsigned long long base[256];
+    const uint32_t G = 1u << rb;
+    const uint64_t ntiles = (n + kSplitTile - 1) / kSplitTile;
+    for (uint64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
+        for (uint32_t i = threadIdx.x; i < G; i += blockDim.x) cnt[i] = 0;
+        __syncthreads();
+        const uint64_t t0 = t * kSplitTile;
+        uint32_t k[kSplitIpt], p[kSplitIpt], dr[kSplitIpt];  // dr = bucket << 16 | rank in tile
+#pragma unroll
+        for (int j = 0; j < kSplitIpt; ++j) {
+            const uint64_t idx = t0 + uint64_t(j) * kSplitBlock + threadIdx.x;
+            const bool v = idx < n;
+            k[j] = v ? keys[idx] : 0u;
+            p[j] = v ? pays[idx] : 0u;
+        }
+#pragma unroll
+        for (int j = 0; j < kSplitIpt; ++j) {
+            const bool v = t0 + uint64_t(j) * kSplitBlock + threadIdx.x < n;
+            const uint32_t d = v ? split_dest(k[j], skip, rb) : 0u;
+            const uint32_t peers = split_peers(v, d, rb);
+            const uint32_t leader = peers ? __ffs(peers) - 1 : 0;
+            uint32_t b = 0;
+            if (v && lane_id() == leader) b = atomicAdd(&cnt[d], (uint32_t)__popc(peers));
+            b = __shfl_sync(kFull, b, leader);  // every lane calls; invalid lanes discard it
+            dr[j] = v ? (d << 16 | (b + __popc(peers & lanemask_lt()))) : 0xffffffffu;
+        }
+        __syncthreads();
+        for (uint32_t i = threadIdx.x; i < G; i += blockDim.x)
+            base[i] = cnt[i] ? off[i] + atomicAdd(&cur[i], (unsigned long long)cnt[i]) : 0ull;
+        if (threadIdx.x < 32) {   // exclusive scan of the tile's bucket counts (8 buckets per lane)
+            uint32_t c[8], s = 0;
+#pragma unroll
+            for (int q = 0; q < 8; ++q) {
+                const uint32_t i = threadIdx.x * 8 + q;
+                c[q] = i < G ? cnt[i] : 0u;
+                s += c[q];
+            }
+            uint32_t incl = s;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const uint32_t y = __shfl_up_sync(kFull, incl, o);
+                if (threadIdx.x >= (uint32_t)o) incl += y;
+            }
+            uint32_t e = incl - s;
+#pragma unroll
+            for (int q = 0; q < 8; ++q) {
+                const uint32_t i = threadIdx.x * 8 + q;
+                if (i < G) pre[i] = e;
+                e += c[q];
+            }
+        }
+        __syncthreads();
+#pragma unroll
+        for (int j = 0; j < kSplitIpt; ++j) {
+            if (dr[j] != 0xffffffffu) {
+                const uint32_t d = dr[j] >> 16, q = pre[d] + (dr[j] & 0xffffu);
+                s_k[q] = k[j];
+                s_p[q] = p[j];
+                s_d[q] = (uint8_t)d;
+            }
+        }
+        __syncthreads();
+        const uint32_t tn = (uint32_t)umin64(kSplitTile, n - t0);
+        for (uint32_t i = threadIdx.x; i < tn; i += kSplitBlock) {
+            const uint32_t d = s_d[i];
+            const uint64_t pos = base[d] + (i - pre[d]);
+            ok[pos] = s_k[i];
+            op[pos] = s_p[i];
+        }
+        __syncthreads();  // cnt / base / pre / staging reused by the next tile
+    }
+}
+
+int launch_split_count(const uint32_t* keys, uint64_t n, uint32_t skip, uint32_t rb, uint64_t* counts,
+                       cudaStream_t s) {
+    if (n == 0) return 0;
+    unsigned grid = (unsigned)umin64((n + kSplitBlock * 8 - 1) / (kSplitBlock * 8), 148 * 4);
+    k_split_count<<<grid, kSplitBlock, 0, s>>>(keys, n, skip, rb, reinterpret_cast<unsigned long long*>(counts));
+    return 1;
+}
+
+int launch_split_scatter(const uint32_t* keys, const uint32_t* pays, uint64_t n, uint32_t skip, uint32_t rb,
+                         const uint64_t* off, uint64_t* cur, uint32_t* ok, uint32_t* op, cudaStream_t s) {
+    if (n == 0) return 0;
+    unsigned grid = (unsigned)umin64((n + kSplitTile - 1) / kSplitTile, 148 * 4);
+    static bool attr = false;   // > 48 KB of dynamic shared memory needs the opt-in once
+    if (!attr) {
+        cudaFuncSetAttribute(k_split_scatter, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSplitSmem);
+        attr = true;
+    }
+    k_split_scatter<<<grid, kSplitBlock, kSplitSmem, s>>>(keys, pays, n, skip, rb, off,
+                                                 reinterpret_cast<unsigned long long*>(cur), ok, op);
+    return 1;
+}
+
 }  // namespace gsh

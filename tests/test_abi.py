@@ -74,6 +74,22 @@ def test_workspace_sizing_is_monotone_and_rejects_bad_config():
         gsh.workspace_bytes(100, 100, gsh.make_config(pass_bits=(9, 1)))
     with pytest.raises(ValueError):
         gsh.workspace_bytes(100, 100, gsh.make_config(force_all_heavy=True, force_all_normal=True))
+    with pytest.raises(ValueError):
+        gsh.workspace_bytes(100, 100, gsh.make_config(prepass_bits=9))
+    with pytest.raises(ValueError):   # pre-pass bits stack on the routing bits (<= 16 in total)
+        gsh.workspace_bytes(100, 100, gsh.make_config(prepass_bits=2, route_bits=15))
+
+
+def test_prepass_workspace_adds_split_copies():
+    """The pre-partition pass (gsh_config.prepass_bits) needs the sub-problem workspace plus SoA
+    copies of both sides (16 B per tuple); auto mode adds it only beyond 2^28 tuples per side."""
+    n = 1 << 20
+    plain = gsh.workspace_bytes(n, n, gsh.make_config(prepass_bits=-1))
+    assert gsh.workspace_bytes(n, n) == plain
+    forced = gsh.workspace_bytes(n, n, gsh.make_config(prepass_bits=2))
+    assert forced >= plain + 16 * n
+    big = 1 << 29
+    assert gsh.workspace_bytes(big, big) >= gsh.workspace_bytes(big, big, gsh.make_config(prepass_bits=-1)) + 16 * big
 
 
 def test_argument_errors_before_any_launch():

@@ -55,8 +55,8 @@ def test_cfg2_count_checksum_fullsize(cfg2):
 def test_pkfk_large_count_checksum(logn):
     """2x and 8x the bench size.  |R| = |S| = 2^28: partitions average 4096 tuples per side, so
     about half of them exceed the CSR staging limit and stream through the chained table's
-    larger one (kRingMaxRChain); 2^30: 16K per side, beyond any staging limit, so the NM-join
-    runs on the general (R-chunk, S-slice) path.  count = n_S and the closed-form checksum
+    larger one (kRingMaxRChain); 2^30: the pre-partition pass splits both sides by 2 hash bits
+    into four 2^28 sub-problems (gsh_config.prepass_bits auto).  count = n_S and the closed-form checksum
     (oracle pair_hash over the generator's row map, computed in chunks on the CPU) must hold."""
     n = 1 << logn
     if torch.cuda.get_device_properties(0).total_memory < (96 << 30):
@@ -76,6 +76,7 @@ def test_pkfk_large_count_checksum(logn):
         expect += int(np.sum(oracle.pair_hash(rows, np.arange(b, b + step, dtype=np.uint32)), dtype=np.uint64))
     assert r.checksum == expect & ((1 << 64) - 1)
     assert r.stats["n_large"] == 0
+    assert r.stats["prepass_bits"] == (2 if logn == 30 else 0)
 
 
 def test_cfg2_materialize_fullsize(cfg2):

@@ -198,6 +198,35 @@ def test_join_invariant_under_config(cfg):
     assert (r.count, r.checksum) == (on, oc)
 
 
+@pytest.mark.parametrize("bits", [1, 3, 8])
+@pytest.mark.parametrize("kind,n,theta", [("pkfk", (1 << 18) + 7, 0.0), ("zipf", 1 << 17, 1.0),
+                                          ("graph", 1 << 16, 0.909), ("uniform", 1000, 0.0)])
+def test_join_prepass_exact(kind, n, theta, bits):
+    """Pre-partition pass (gsh_config.prepass_bits; auto beyond 2^28 tuples per side): splitting R
+    and S by hash bits and joining the sub-problems changes performance only -- COUNT and
+    MATERIALIZE equal the oracle's, pairs as a multiset, also with routing bits above it."""
+    rk, rp, sk, sp = datagen.make_workload(kind, n, theta, seed=29)
+    on, oc, op = _oracle(rk, rp, sk, sp, pairs=True)
+    d = _dev(rk, rp, sk, sp)
+    r = gsh.join(*d, config=gsh.make_config(prepass_bits=bits, timing=True))
+    assert (r.count, r.checksum) == (on, oc)
+    assert r.stats["prepass_bits"] == bits and r.stats["ms_prepass"] > 0
+    m = gsh.join(*d, mode="materialize", out_capacity=on + 3, config=gsh.make_config(prepass_bits=bits, route_bits=2))
+    assert (m.count, m.checksum, m.written, m.overflow) == (on, oc, on, False)
+    assert np.array_equal(_sorted_pairs(m.pairs), op)
+
+
+def test_join_prepass_overflow_subset():
+    rk, rp, sk, sp = datagen.zipf_pair(30_000, 30_000, 1.0, seed=8)
+    on, oc, _ = _oracle(rk, rp, sk, sp)
+    cap = on // 3
+    r = gsh.join(*_dev(rk, rp, sk, sp), mode="materialize", out_capacity=cap, config=gsh.make_config(prepass_bits=2))
+    assert (r.count, r.checksum, r.written, r.overflow) == (on, oc, cap, True)
+    got = _sorted_pairs(r.pairs)
+    assert np.all(_np(rk)[got[:, 0]] == _np(sk)[got[:, 1]])
+    assert np.unique(got, axis=0).shape[0] == got.shape[0]
+
+
 def test_join_edge_cases():
     # all keys equal (one giant skewed key), extremes of the key range, no matches, empty sides
     z = torch.zeros
