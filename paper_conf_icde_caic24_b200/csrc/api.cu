@@ -347,6 +347,9 @@ struct Prepass {
     uint64_t* counts;     // [2][256]
     uint64_t* offs;       // [2][256]
     uint64_t* cur;        // [2][256]
+    uint32_t* tile_cnt[2];   // rb <= 3: per-(bucket, tile) counts, bucket-major
+    uint64_t* tpfx[2];       // their exclusive prefix
+    uint64_t* scratch;       // scan scratch
     size_t bytes;
 };
 
@@ -365,6 +368,12 @@ static Prepass prepass_layout(uint64_t n_r, uint64_t n_s, const gsh_config* sub,
     q.counts = reinterpret_cast<uint64_t*>(take(2 * 256 * 8));
     q.offs = reinterpret_cast<uint64_t*>(take(2 * 256 * 8));
     q.cur = reinterpret_cast<uint64_t*>(take(2 * 256 * 8));
+    const uint64_t nt[2] = {8 * split_tiles(n_r), 8 * split_tiles(n_s)};
+    for (int side = 0; side < 2; ++side) {
+        q.tile_cnt[side] = reinterpret_cast<uint32_t*>(take(nt[side] * 4));
+        q.tpfx[side] = reinterpret_cast<uint64_t*>(take((nt[side] + 1) * 8));
+    }
+    q.scratch = reinterpret_cast<uint64_t*>(take(((nt[0] > nt[1] ? nt[0] : nt[1]) / 4096 + 8) * 8));
     q.bytes = off;
     return q;
 }
@@ -514,8 +523,16 @@ gsh_status gsh_join(const gsh_relation* R, const gsh_relation* S, gsh_out_mode m
     cudaError_t ce = cudaMemsetAsync(q.counts, 0, 3 * align256(2 * 256 * 8), s);
     if (ce != cudaSuccess) return cuda_fail(ce, "prepass memset");
     int launches = 0;
-    launches += launch_split_count(R->keys, R->n, skip, (uint32_t)r, q.counts, s);
-    launches += launch_split_count(S->keys, S->n, skip, (uint32_t)r, q.counts + 256, s);
+    const bool tiled = r <= 3;   // atomic-free register-ranked kernels (G <= 8)
+    if (tiled) {
+        launches += launch_split_count_tiles(R->keys, R->n, skip, (uint32_t)r, q.tile_cnt[0], q.counts, s);
+        launches += launch_split_count_tiles(S->keys, S->n, skip, (uint32_t)r, q.tile_cnt[1], q.counts + 256, s);
+        launches += launch_split_tile_scan(q.tile_cnt[0], R->n, (uint32_t)r, q.tpfx[0], q.scratch, s);
+        launches += launch_split_tile_scan(q.tile_cnt[1], S->n, (uint32_t)r, q.tpfx[1], q.scratch, s);
+    } else {
+        launches += launch_split_count(R->keys, R->n, skip, (uint32_t)r, q.counts, s);
+        launches += launch_split_count(S->keys, S->n, skip, (uint32_t)r, q.counts + 256, s);
+    }
     gsh_status st = check_launch("prepass count");
     if (st != GSH_OK) return st;
     uint64_t hc[512], ho[512];
@@ -534,9 +551,16 @@ gsh_status gsh_join(const gsh_relation* R, const gsh_relation* S, gsh_out_mode m
     }
     ce = cudaMemcpyAsync(q.offs, ho, sizeof(ho), cudaMemcpyHostToDevice, s);
     if (ce != cudaSuccess) return cuda_fail(ce, "prepass offsets");
-    launches += launch_split_scatter(R->keys, R->payloads, R->n, skip, (uint32_t)r, q.offs, q.cur, q.rk, q.rp, s);
-    launches += launch_split_scatter(S->keys, S->payloads, S->n, skip, (uint32_t)r, q.offs + 256, q.cur + 256,
-                                     q.sk, q.sp, s);
+    if (tiled) {
+        launches += launch_split_scatter_tiles(R->keys, R->payloads, R->n, skip, (uint32_t)r, q.offs, q.tpfx[0],
+                                               q.rk, q.rp, s);
+        launches += launch_split_scatter_tiles(S->keys, S->payloads, S->n, skip, (uint32_t)r, q.offs + 256,
+                                               q.tpfx[1], q.sk, q.sp, s);
+    } else {
+        launches += launch_split_scatter(R->keys, R->payloads, R->n, skip, (uint32_t)r, q.offs, q.cur, q.rk, q.rp, s);
+        launches += launch_split_scatter(S->keys, S->payloads, S->n, skip, (uint32_t)r, q.offs + 256, q.cur + 256,
+                                         q.sk, q.sp, s);
+    }
     const int e1 = tm.mark();
     if ((st = check_launch("prepass scatter")) != GSH_OK) return st;
     const uint64_t cap = mat ? out->capacity : 0;

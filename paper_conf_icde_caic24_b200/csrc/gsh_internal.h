@@ -190,6 +190,14 @@ int launch_split_count(const uint32_t* keys, uint64_t n, uint32_t skip, uint32_t
                        cudaStream_t s);
 int launch_split_scatter(const uint32_t* keys, const uint32_t* pays, uint64_t n, uint32_t skip, uint32_t rb,
                          const uint64_t* off, uint64_t* cur, uint32_t* ok, uint32_t* op, cudaStream_t s);
+uint64_t split_tiles(uint64_t n);
+int launch_split_count_tiles(const uint32_t* keys, uint64_t n, uint32_t skip, uint32_t rb, uint32_t* tile_cnt,
+                             uint64_t* counts, cudaStream_t s);
+int launch_split_tile_scan(const uint32_t* tile_cnt, uint64_t n, uint32_t rb, uint64_t* tpfx, uint64_t* scratch,
+                           cudaStream_t s);
+int launch_split_scatter_tiles(const uint32_t* keys, const uint32_t* pays, uint64_t n, uint32_t skip, uint32_t rb,
+                               const uint64_t* off, const uint64_t* tpfx, uint32_t* ok, uint32_t* op,
+                               cudaStream_t s);
 int launch_count_keys(const uint32_t* keys, uint64_t n, const uint32_t* q, uint64_t m, uint64_t* counts,
                       cudaStream_t s);
 int launch_radix_hist(const uint32_t* keys, uint64_t n, uint32_t hi_bits, uint32_t nbits, uint64_t* hist,

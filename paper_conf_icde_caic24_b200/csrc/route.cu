@@ -256,6 +256,211 @@ __global__ void __launch_bounds__(kSplitBlock, 2) k_split_scatter(const uint32_t
     }
 }
 
+// ---- rb <= 3 (G <= 8; auto mode up to 2^31 tuples per side): no atomics.  Every lane of a warp
+// computes the warp's G bucket masks from rb + 1 ballots, so per-(warp, bucket) counts and ranks
+// stay in warp-uniform registers.  The count kernel writes per-(bucket, tile) counts, one scan
+// (bucket-major) gives every tile its write offset in each bucket, and the scatter needs neither
+// a shared nor a global atomic.
+template <int RB>
+__device__ __forceinline__ void split_masks(bool v, uint32_t d, uint32_t (&eq)[1 << RB]) {
+    const uint32_t m = __ballot_sync(kFull, v);
+    uint32_t mb[RB];
+#pragma unroll
+    for (int b = 0; b < RB; ++b) mb[b] = __ballot_sync(kFull, (d >> b) & 1u);
+#pragma unroll
+    for (int g = 0; g < (1 << RB); ++g) {
+        uint32_t e = m;
+#pragma unroll
+        for (int b = 0; b < RB; ++b) e &= ((g >> b) & 1) ? mb[b] : ~mb[b];
+        eq[g] = e;
+    }
+}
+
+constexpr int kSplitWarps = kSplitBlock / 32;
+
+template <int RB>
+__global__ void __launch_bounds__(kSplitBlock, 2) k_split_count_tiles(const uint32_t* __restrict__ keys, uint64_t n,
+                                                                  uint32_t skip, uint32_t* __restrict__ tile_cnt,
+                                                                  unsigned long long* counts) {
+    constexpr int G = 1 << RB;
+    __shared__ uint32_t s_wc[kSplitWarps][G];
+    const uint64_t ntiles = (n + kSplitTile - 1) / kSplitTile;
+    const uint32_t warp = threadIdx.x >> 5;
+    // the next tile's keys are loaded while this tile's counts are reduced (k[] is free by then)
+    uint32_t k[kSplitIpt];
+    auto load = [&](uint64_t tt) {
+#pragma unroll
+        for (int j = 0; j < kSplitIpt; ++j) {
+            const uint64_t i = tt * kSplitTile + uint64_t(j) * kSplitBlock + threadIdx.x;
+            k[j] = (tt < ntiles && i < n) ? __ldcs(keys + i) : 0u;
+        }
+    };
+    load(blockIdx.x);
+    for (uint64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
+        const uint64_t t0 = t * kSplitTile;
+        uint32_t wc[G];
+#pragma unroll
+        for (int g = 0; g < G; ++g) wc[g] = 0;
+#pragma unroll
+        for (int j = 0; j < kSplitIpt; ++j) {
+            const bool v = t0 + uint64_t(j) * kSplitBlock + threadIdx.x < n;
+            uint32_t eq[G];
+            split_masks<RB>(v, v ? split_dest(k[j], skip, RB) : 0u, eq);
+#pragma unroll
+            for (int g = 0; g < G; ++g) wc[g] += __popc(eq[g]);
+        }
+        load(t + gridDim.x);
+        if (lane_id() == 0) {
+#pragma unroll
+            for (int g = 0; g < G; ++g) s_wc[warp][g] = wc[g];
+        }
+        __syncthreads();
+        if (threadIdx.x < G) {
+            uint32_t c = 0;
+            for (int w = 0; w < kSplitWarps; ++w) c += s_wc[w][threadIdx.x];
+            tile_cnt[uint64_t(threadIdx.x) * ntiles + t] = c;
+            if (c) atomicAdd(&counts[threadIdx.x], (unsigned long long)c);
+        }
+        __syncthreads();
+    }
+}
+
+template <int RB>
+__global__ void __launch_bounds__(kSplitBlock, 2) k_split_scatter_tiles(
+    const uint32_t* __restrict__ keys, const uint32_t* __restrict__ pays, uint64_t n, uint32_t skip,
+    const uint64_t* __restrict__ off, const uint64_t* __restrict__ tpfx, uint32_t* __restrict__ ok,
+    uint32_t* __restrict__ op) {
+    constexpr int G = 1 << RB;
+    extern __shared__ uint4 split_dyn[];
+    uint32_t* s_k = reinterpret_cast<uint32_t*>(split_dyn);
+    uint32_t* s_p = s_k + kSplitTile;
+    uint8_t* s_d = reinterpret_cast<uint8_t*>(s_p + kSplitTile);
+    __shared__ uint32_t s_wc[kSplitWarps][G];   // per-warp counts, then per-warp bases within the tile
+    __shared__ uint32_t pre[G];
+    __shared__ unsigned long long base[G];
+    const uint64_t ntiles = (n + kSplitTile - 1) / kSplitTile;
+    const uint32_t warp = threadIdx.x >> 5;
+    // the next tile is loaded into k[] / p[] before this tile's write-out (they are free once the
+    // tile sits permuted in shared memory), so its load latency overlaps the stores
+    uint32_t k[kSplitIpt], p[kSplitIpt], dr[kSplitIpt];  // dr = bucket << 16 | rank in the warp
+    auto load = [&](uint64_t tt) {
+#pragma unroll
+        for (int j = 0; j < kSplitIpt; ++j) {
+            const uint64_t idx = tt * kSplitTile + uint64_t(j) * kSplitBlock + threadIdx.x;
+            const bool v = tt < ntiles && idx < n;
+            k[j] = v ? __ldcs(keys + idx) : 0u;
+            p[j] = v ? __ldcs(pays + idx) : 0u;
+        }
+    };
+    load(blockIdx.x);
+    for (uint64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
+        const uint64_t t0 = t * kSplitTile;
+        uint32_t wc[G];
+#pragma unroll
+        for (int g = 0; g < G; ++g) wc[g] = 0;
+#pragma unroll
+        for (int j = 0; j < kSplitIpt; ++j) {
+            const bool v = t0 + uint64_t(j) * kSplitBlock + threadIdx.x < n;
+            const uint32_t d = v ? split_dest(k[j], skip, RB) : 0u;
+            uint32_t eq[G];
+            split_masks<RB>(v, d, eq);
+            uint32_t r = 0;
+#pragma unroll
+            for (int g = 0; g < G; ++g) {
+                if ((uint32_t)g == d) r = wc[g] + __popc(eq[g] & lanemask_lt());
+                wc[g] += __popc(eq[g]);
+            }
+            dr[j] = v ? (d << 16 | r) : 0xffffffffu;
+        }
+        if (lane_id() == 0) {
+#pragma unroll
+            for (int g = 0; g < G; ++g) s_wc[warp][g] = wc[g];
+        }
+        __syncthreads();
+        if (threadIdx.x < G) {
+            const uint32_t g = threadIdx.x;
+            uint32_t before = 0;   // tuples of the tile in buckets < g
+            for (uint32_t h = 0; h < g; ++h)
+                for (int w = 0; w < kSplitWarps; ++w) before += s_wc[w][h];
+            pre[g] = before;
+            uint32_t acc = 0;
+            for (int w = 0; w < kSplitWarps; ++w) {
+                const uint32_t c = s_wc[w][g];
+                s_wc[w][g] = acc;
+                acc += c;
+            }
+            base[g] = off[g] + (tpfx[uint64_t(g) * ntiles + t] - tpfx[uint64_t(g) * ntiles]);
+        }
+        __syncthreads();
+#pragma unroll
+        for (int j = 0; j < kSplitIpt; ++j) {
+            if (dr[j] != 0xffffffffu) {
+                const uint32_t d = dr[j] >> 16, q = pre[d] + s_wc[warp][d] + (dr[j] & 0xffffu);
+                s_k[q] = k[j];
+                s_p[q] = p[j];
+                s_d[q] = (uint8_t)d;
+            }
+        }
+        __syncthreads();
+        load(t + gridDim.x);
+        const uint32_t tn = (uint32_t)umin64(kSplitTile, n - t0);
+        for (uint32_t i = threadIdx.x; i < tn; i += kSplitBlock) {
+            const uint32_t d = s_d[i];
+            const uint64_t pos = base[d] + (i - pre[d]);
+            ok[pos] = s_k[i];
+            op[pos] = s_p[i];
+        }
+        __syncthreads();
+    }
+}
+
+struct TileCount {
+    const uint32_t* c;
+    __device__ uint64_t operator()(uint64_t i) const { return c[i]; }
+};
+
+uint64_t split_tiles(uint64_t n) { return (n + kSplitTile - 1) / kSplitTile; }
+
+// rb in 1..3: per-(bucket, tile) counts into tile_cnt[G * ntiles], bucket totals added to counts[G]
+int launch_split_count_tiles(const uint32_t* keys, uint64_t n, uint32_t skip, uint32_t rb, uint32_t* tile_cnt,
+                             uint64_t* counts, cudaStream_t s) {
+    if (n == 0) return 0;
+    const unsigned grid = (unsigned)umin64(split_tiles(n), 148 * 4);
+    auto* c = reinterpret_cast<unsigned long long*>(counts);
+    if (rb == 1) k_split_count_tiles<1><<<grid, kSplitBlock, 0, s>>>(keys, n, skip, tile_cnt, c);
+    else if (rb == 2) k_split_count_tiles<2><<<grid, kSplitBlock, 0, s>>>(keys, n, skip, tile_cnt, c);
+    else k_split_count_tiles<3><<<grid, kSplitBlock, 0, s>>>(keys, n, skip, tile_cnt, c);
+    return 1;
+}
+
+// exclusive bucket-major prefix of tile_cnt (G * ntiles + 1 values) into tpfx
+int launch_split_tile_scan(const uint32_t* tile_cnt, uint64_t n, uint32_t rb, uint64_t* tpfx, uint64_t* scratch,
+                           cudaStream_t s) {
+    if (n == 0) return 0;
+    return launch_scan(TileCount{tile_cnt}, (uint64_t(1) << rb) * split_tiles(n), tpfx, scratch, s);
+}
+
+int launch_split_scatter_tiles(const uint32_t* keys, const uint32_t* pays, uint64_t n, uint32_t skip, uint32_t rb,
+                               const uint64_t* off, const uint64_t* tpfx, uint32_t* ok, uint32_t* op,
+                               cudaStream_t s) {
+    if (n == 0) return 0;
+    static bool attr = false;
+    if (!attr) {
+        cudaFuncSetAttribute(k_split_scatter_tiles<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSplitSmem);
+        cudaFuncSetAttribute(k_split_scatter_tiles<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSplitSmem);
+        cudaFuncSetAttribute(k_split_scatter_tiles<3>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSplitSmem);
+        attr = true;
+    }
+    const unsigned grid = (unsigned)umin64(split_tiles(n), 148 * 2);
+    if (rb == 1)
+        k_split_scatter_tiles<1><<<grid, kSplitBlock, kSplitSmem, s>>>(keys, pays, n, skip, off, tpfx, ok, op);
+    else if (rb == 2)
+        k_split_scatter_tiles<2><<<grid, kSplitBlock, kSplitSmem, s>>>(keys, pays, n, skip, off, tpfx, ok, op);
+    else
+        k_split_scatter_tiles<3><<<grid, kSplitBlock, kSplitSmem, s>>>(keys, pays, n, skip, off, tpfx, ok, op);
+    return 1;
+}
+
 int launch_split_count(const uint32_t* keys, uint64_t n, uint32_t skip, uint32_t rb, uint64_t* counts,
                        cudaStream_t s) {
     if (n == 0) return 0;
