@@ -276,12 +276,39 @@ __device__ __forceinline__ void split_masks(bool v, uint32_t d, uint32_t (&eq)[1
     }
 }
 
+// Element of slot j (0..kSplitIpt) of this thread within tile t0: scalar layout = one element per
+// 512-stride; VEC layout = 4 consecutive elements per uint4 (slots 4v..4v+3 of vector v).  Any
+// bijection onto the tile is correct: counts are per tile, ranks are computed where they are used.
+template <bool VEC>
+__device__ __forceinline__ uint64_t split_elem(uint64_t t0, int j) {
+    return VEC ? t0 + (uint64_t((j >> 2) * kSplitBlock + threadIdx.x) << 2) + (j & 3)
+               : t0 + uint64_t(j) * kSplitBlock + threadIdx.x;
+}
+
+template <bool VEC>
+__device__ __forceinline__ void split_load(const uint32_t* __restrict__ src, uint64_t t0, uint64_t n,
+                                           uint32_t (&x)[kSplitIpt]) {
+    if (VEC && t0 + kSplitTile <= n) {
+#pragma unroll
+        for (int v = 0; v < kSplitIpt / 4; ++v) {
+            const uint4 w = __ldcs(reinterpret_cast<const uint4*>(src + split_elem<true>(t0, 4 * v)));
+            x[4 * v] = w.x; x[4 * v + 1] = w.y; x[4 * v + 2] = w.z; x[4 * v + 3] = w.w;
+        }
+    } else {
+#pragma unroll
+        for (int j = 0; j < kSplitIpt; ++j) {
+            const uint64_t i = split_elem<VEC>(t0, j);
+            x[j] = i < n ? __ldcs(src + i) : 0u;
+        }
+    }
+}
+
 constexpr int kSplitWarps = kSplitBlock / 32;
 
-template <int RB>
+template <int RB, bool VEC>
 __global__ void __launch_bounds__(kSplitBlock, 2) k_split_count_tiles(const uint32_t* __restrict__ keys, uint64_t n,
-                                                                  uint32_t skip, uint32_t* __restrict__ tile_cnt,
-                                                                  unsigned long long* counts) {
+                                                                     uint32_t skip, uint32_t* __restrict__ tile_cnt,
+                                                                     unsigned long long* counts) {
     constexpr int G = 1 << RB;
     __shared__ uint32_t s_wc[kSplitWarps][G];
     const uint64_t ntiles = (n + kSplitTile - 1) / kSplitTile;
@@ -289,11 +316,7 @@ __global__ void __launch_bounds__(kSplitBlock, 2) k_split_count_tiles(const uint
     // the next tile's keys are loaded while this tile's counts are reduced (k[] is free by then)
     uint32_t k[kSplitIpt];
     auto load = [&](uint64_t tt) {
-#pragma unroll
-        for (int j = 0; j < kSplitIpt; ++j) {
-            const uint64_t i = tt * kSplitTile + uint64_t(j) * kSplitBlock + threadIdx.x;
-            k[j] = (tt < ntiles && i < n) ? __ldcs(keys + i) : 0u;
-        }
+        if (tt < ntiles) split_load<VEC>(keys, tt * kSplitTile, n, k);
     };
     load(blockIdx.x);
     for (uint64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
@@ -303,7 +326,7 @@ __global__ void __launch_bounds__(kSplitBlock, 2) k_split_count_tiles(const uint
         for (int g = 0; g < G; ++g) wc[g] = 0;
 #pragma unroll
         for (int j = 0; j < kSplitIpt; ++j) {
-            const bool v = t0 + uint64_t(j) * kSplitBlock + threadIdx.x < n;
+            const bool v = split_elem<VEC>(t0, j) < n;
             uint32_t eq[G];
             split_masks<RB>(v, v ? split_dest(k[j], skip, RB) : 0u, eq);
 #pragma unroll
@@ -325,7 +348,7 @@ __global__ void __launch_bounds__(kSplitBlock, 2) k_split_count_tiles(const uint
     }
 }
 
-template <int RB>
+template <int RB, bool VEC>
 __global__ void __launch_bounds__(kSplitBlock, 2) k_split_scatter_tiles(
     const uint32_t* __restrict__ keys, const uint32_t* __restrict__ pays, uint64_t n, uint32_t skip,
     const uint64_t* __restrict__ off, const uint64_t* __restrict__ tpfx, uint32_t* __restrict__ ok,
@@ -344,14 +367,12 @@ __global__ void __launch_bounds__(kSplitBlock, 2) k_split_scatter_tiles(
     // tile sits permuted in shared memory), so its load latency overlaps the stores
     uint32_t k[kSplitIpt], p[kSplitIpt], dr[kSplitIpt];  // dr = bucket << 16 | rank in the warp
     auto load = [&](uint64_t tt) {
-#pragma unroll
-        for (int j = 0; j < kSplitIpt; ++j) {
-            const uint64_t idx = tt * kSplitTile + uint64_t(j) * kSplitBlock + threadIdx.x;
-            const bool v = tt < ntiles && idx < n;
-            k[j] = v ? __ldcs(keys + idx) : 0u;
-            p[j] = v ? __ldcs(pays + idx) : 0u;
+        if (tt < ntiles) {
+            split_load<VEC>(keys, tt * kSplitTile, n, k);
+            split_load<VEC>(pays, tt * kSplitTile, n, p);
         }
     };
+    const uint32_t lt = lanemask_lt();
     load(blockIdx.x);
     for (uint64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
         const uint64_t t0 = t * kSplitTile;
@@ -360,17 +381,19 @@ __global__ void __launch_bounds__(kSplitBlock, 2) k_split_scatter_tiles(
         for (int g = 0; g < G; ++g) wc[g] = 0;
 #pragma unroll
         for (int j = 0; j < kSplitIpt; ++j) {
-            const bool v = t0 + uint64_t(j) * kSplitBlock + threadIdx.x < n;
+            const bool v = split_elem<VEC>(t0, j) < n;
             const uint32_t d = v ? split_dest(k[j], skip, RB) : 0u;
             uint32_t eq[G];
             split_masks<RB>(v, d, eq);
-            uint32_t r = 0;
+            uint32_t mine = 0, r0 = 0;
 #pragma unroll
             for (int g = 0; g < G; ++g) {
-                if ((uint32_t)g == d) r = wc[g] + __popc(eq[g] & lanemask_lt());
+                const bool is = (uint32_t)g == d;
+                mine = is ? eq[g] : mine;
+                r0 = is ? wc[g] : r0;
                 wc[g] += __popc(eq[g]);
             }
-            dr[j] = v ? (d << 16 | r) : 0xffffffffu;
+            dr[j] = v ? (d << 16 | (r0 + __popc(mine & lt))) : 0xffffffffu;
         }
         if (lane_id() == 0) {
 #pragma unroll
@@ -422,14 +445,22 @@ struct TileCount {
 uint64_t split_tiles(uint64_t n) { return (n + kSplitTile - 1) / kSplitTile; }
 
 // rb in 1..3: per-(bucket, tile) counts into tile_cnt[G * ntiles], bucket totals added to counts[G]
+template <bool VEC>
+void split_count_tiles_rb(const uint32_t* keys, uint64_t n, uint32_t skip, uint32_t rb, uint32_t* tile_cnt,
+                          unsigned long long* c, unsigned grid, cudaStream_t s) {
+    if (rb == 1) k_split_count_tiles<1, VEC><<<grid, kSplitBlock, 0, s>>>(keys, n, skip, tile_cnt, c);
+    else if (rb == 2) k_split_count_tiles<2, VEC><<<grid, kSplitBlock, 0, s>>>(keys, n, skip, tile_cnt, c);
+    else k_split_count_tiles<3, VEC><<<grid, kSplitBlock, 0, s>>>(keys, n, skip, tile_cnt, c);
+}
+
+// rb in 1..3: per-(bucket, tile) counts into tile_cnt[G * ntiles], bucket totals added to counts[G]
 int launch_split_count_tiles(const uint32_t* keys, uint64_t n, uint32_t skip, uint32_t rb, uint32_t* tile_cnt,
                              uint64_t* counts, cudaStream_t s) {
     if (n == 0) return 0;
     const unsigned grid = (unsigned)umin64(split_tiles(n), 148 * 4);
     auto* c = reinterpret_cast<unsigned long long*>(counts);
-    if (rb == 1) k_split_count_tiles<1><<<grid, kSplitBlock, 0, s>>>(keys, n, skip, tile_cnt, c);
-    else if (rb == 2) k_split_count_tiles<2><<<grid, kSplitBlock, 0, s>>>(keys, n, skip, tile_cnt, c);
-    else k_split_count_tiles<3><<<grid, kSplitBlock, 0, s>>>(keys, n, skip, tile_cnt, c);
+    if ((reinterpret_cast<uintptr_t>(keys) & 15u) == 0) split_count_tiles_rb<true>(keys, n, skip, rb, tile_cnt, c, grid, s);
+    else split_count_tiles_rb<false>(keys, n, skip, rb, tile_cnt, c, grid, s);
     return 1;
 }
 
@@ -440,24 +471,33 @@ int launch_split_tile_scan(const uint32_t* tile_cnt, uint64_t n, uint32_t rb, ui
     return launch_scan(TileCount{tile_cnt}, (uint64_t(1) << rb) * split_tiles(n), tpfx, scratch, s);
 }
 
+template <int RB, bool VEC>
+void split_scatter_tiles_one(const uint32_t* keys, const uint32_t* pays, uint64_t n, uint32_t skip,
+                             const uint64_t* off, const uint64_t* tpfx, uint32_t* ok, uint32_t* op, cudaStream_t s) {
+    static bool attr = false;   // > 48 KB of dynamic shared memory needs the opt-in once
+    if (!attr) {
+        cudaFuncSetAttribute(k_split_scatter_tiles<RB, VEC>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             (int)kSplitSmem);
+        attr = true;
+    }
+    const unsigned grid = (unsigned)umin64(split_tiles(n), 148 * 2);
+    k_split_scatter_tiles<RB, VEC><<<grid, kSplitBlock, kSplitSmem, s>>>(keys, pays, n, skip, off, tpfx, ok, op);
+}
+
 int launch_split_scatter_tiles(const uint32_t* keys, const uint32_t* pays, uint64_t n, uint32_t skip, uint32_t rb,
                                const uint64_t* off, const uint64_t* tpfx, uint32_t* ok, uint32_t* op,
                                cudaStream_t s) {
     if (n == 0) return 0;
-    static bool attr = false;
-    if (!attr) {
-        cudaFuncSetAttribute(k_split_scatter_tiles<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSplitSmem);
-        cudaFuncSetAttribute(k_split_scatter_tiles<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSplitSmem);
-        cudaFuncSetAttribute(k_split_scatter_tiles<3>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSplitSmem);
-        attr = true;
+    const bool vec = ((reinterpret_cast<uintptr_t>(keys) | reinterpret_cast<uintptr_t>(pays)) & 15u) == 0;
+    if (vec) {
+        if (rb == 1) split_scatter_tiles_one<1, true>(keys, pays, n, skip, off, tpfx, ok, op, s);
+        else if (rb == 2) split_scatter_tiles_one<2, true>(keys, pays, n, skip, off, tpfx, ok, op, s);
+        else split_scatter_tiles_one<3, true>(keys, pays, n, skip, off, tpfx, ok, op, s);
+    } else {
+        if (rb == 1) split_scatter_tiles_one<1, false>(keys, pays, n, skip, off, tpfx, ok, op, s);
+        else if (rb == 2) split_scatter_tiles_one<2, false>(keys, pays, n, skip, off, tpfx, ok, op, s);
+        else split_scatter_tiles_one<3, false>(keys, pays, n, skip, off, tpfx, ok, op, s);
     }
-    const unsigned grid = (unsigned)umin64(split_tiles(n), 148 * 2);
-    if (rb == 1)
-        k_split_scatter_tiles<1><<<grid, kSplitBlock, kSplitSmem, s>>>(keys, pays, n, skip, off, tpfx, ok, op);
-    else if (rb == 2)
-        k_split_scatter_tiles<2><<<grid, kSplitBlock, kSplitSmem, s>>>(keys, pays, n, skip, off, tpfx, ok, op);
-    else
-        k_split_scatter_tiles<3><<<grid, kSplitBlock, kSplitSmem, s>>>(keys, pays, n, skip, off, tpfx, ok, op);
     return 1;
 }
 
