@@ -161,6 +161,9 @@ GSH_API size_t gsh_workspace_bytes(uint64_t n_r, uint64_t n_s, const gsh_config 
  *   cfg        : NULL = defaults.
  *   stream     : cudaStream_t as void*.
  *   res        : host result, filled after the stream is synchronised.
+ * Beyond 2^28 tuples per side (or with cfg->prepass_bits > 0) both relations are first split
+ * by hash bits into 2^prepass_bits sub-problems (split copies in the workspace), which are
+ * joined one after another on `stream`; count / checksum / written cover all of them.
  * Returns GSH_ERR_INVALID for NULL pointers with n > 0, MATERIALIZE without output,
  * a too-small or misaligned workspace, n >= 2^32, or bad config values.
  */
