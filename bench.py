@@ -41,6 +41,7 @@ WORKLOADS = {
     "zipf15s": ("zipf", 1 << 22, 1.5, "cfg3-shaped (scaled): |R|=|S|=2^22 Zipf theta=1.5 both sides, COUNT"),
     "graph": ("graph", 1 << 26, 0.909, "cfg4-shaped (scaled): 2^26-edge power-law graph self-join (dst, src), COUNT"),
     "pkfk28": ("pkfk", 1 << 28, 0.0, "scale point: |R|=|S|=2^28 uniform 1:1 PK-FK (cfg5's per-GPU share at G=8), COUNT"),
+    "pkfk29": ("pkfk", 1 << 29, 0.0, "scale point: |R|=|S|=2^29 uniform 1:1 PK-FK (4x cfg2; 2^30 input tuples), COUNT"),
     "pkfk30": ("pkfk", 1 << 30, 0.0, "scale point: |R|=|S|=2^30 uniform 1:1 PK-FK (8x cfg2; 2^31 input tuples), COUNT"),
 }
 
