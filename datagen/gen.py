@@ -150,6 +150,16 @@ def pkfk_pair(n_r: int, n_s: int, seed: int = 0, device="cpu"):
     return _to_i32(rk64), _payloads(n_r, device), _to_i32(sk64), _payloads(n_s, device)
 
 
+def pkfk_zipf_pair(n_r: int, n_s: int, theta: float, seed: int = 0, device="cpu"):
+    """Skewed-FK PK-FK: R = n_r distinct keys (row r holds key map(r)); each S row references R row
+    rank ~ Zipf(theta) over the n_r rows (the interval array of PAPER.md L139), so R is unique and
+    S is skewed: count == n_s exactly, cnt_R = 1 for every key."""
+    T = torch.from_numpy(zipf_thresholds(max(n_r, 1), theta)).to(device)
+    rk = _to_i32(rank_to_key(torch.arange(n_r, dtype=torch.int64, device=device), seed))
+    sk = zipf_keys(n_s, T, seed, seed, 1, device) if n_r else torch.zeros(0, dtype=torch.int32, device=device)
+    return rk, _payloads(n_r, device), sk, _payloads(sk.numel(), device)
+
+
 def graph_pair(n_edges: int, n_vertices: int, theta: float = 1.0 / (2.1 - 1.0), seed: int = 0,
                device="cpu"):
     """Power-law graph edge self-join (SURVEY reading #18; PAPER.md L13 motivation).
@@ -163,7 +173,7 @@ def graph_pair(n_edges: int, n_vertices: int, theta: float = 1.0 / (2.1 - 1.0), 
 
 
 def make_workload(kind: str, n: int, theta: float = 0.0, seed: int = 0, device="cpu", n_s: int | None = None):
-    """Convenience dispatcher used by tests / bench: kind in {zipf, uniform, pkfk, graph}."""
+    """Convenience dispatcher used by tests / bench: kind in {zipf, uniform, pkfk, pkfk_zipf, graph}."""
     n_s = n if n_s is None else n_s
     if kind == "zipf":
         return zipf_pair(n, n_s, theta, None, seed, device)
@@ -171,6 +181,8 @@ def make_workload(kind: str, n: int, theta: float = 0.0, seed: int = 0, device="
         return uniform_pair(n, n_s, seed, device)
     if kind == "pkfk":
         return pkfk_pair(n, n_s, seed, device)
+    if kind == "pkfk_zipf":
+        return pkfk_zipf_pair(n, n_s, theta, seed, device)
     if kind == "graph":
         v = max(1, n // 16)
         return graph_pair(n, v, theta if theta else 1.0 / 1.1, seed, device)

@@ -218,40 +218,109 @@ GSH_API gsh_status gsh_detect(const gsh_relation *R, const gsh_relation *S, cons
                       uint32_t *h_keys, uint32_t *h_cnt_r, uint32_t *h_cnt_s, uint64_t cap,
                       uint64_t *h_n, gsh_result *res);
 
-/* -------------------------------------------------------------- multi-GPU routing --
- * Hash sharding over G = 2^route_bits ranks: a normal tuple goes to rank
- * top_route_bits(fmix32(key)); a tuple whose key is in the agreed skewed set goes to the
- * extra "heavy" bucket G (S stays local, R is all-gathered by the driver).             */
+/* ------------------------------------------------------ multi-GPU hash sharding --
+ * SURVEY.md §8(e), a north-star addition: the paper runs on one A100 (§V-A).
+ * One process (or logical rank) per GPU; rank g holds any shard of R and S.  The driver
+ * (paper_conf_icde_caic24_b200/sharded.py) calls these per-rank steps between collectives
+ * (torch.distributed over NCCL, or an in-process exchange for the one-GPU test harness):
+ *   1. gsh_shard_plan: the single-GPU rule's parameters for the GLOBAL sizes;
+ *   2. gsh_shard_histogram -> all_reduce(sum) -> global partition sizes;
+ *   3. gsh_shard_candidates: keys of globally large partitions (L107) whose LOCAL count
+ *      max(cnt_R, cnt_S) reaches tau = ceil(T_h / G) (pigeonhole: a key whose global count
+ *      reaches T_h reaches tau on some rank) -> all_gather;
+ *   4. gsh_shard_agree: union of the gathered candidates + this rank's exact counts of each
+ *      -> all_reduce(sum);  5. gsh_shard_select: skewed iff max(cnt_R, cnt_S) >= T_h (L112) --
+ *      the single-GPU rule applied to the whole input, identical list on every rank;
+ *   6. gsh_heavy_set_build + gsh_route_count / gsh_route_scatter: a normal tuple goes to rank
+ *      top_route_bits(h), a tuple of a skewed key to the "heavy" destination G (S_k stays
+ *      local, R_k is all-gathered), so no GPU receives a skewed key's full S.
+ * Keys are identified by h = fmix32(key) throughout (a bijection, so h equality is key equality).
+ */
+typedef struct {
+    uint32_t world;            /* G, a power of two <= 256 */
+    uint32_t route_bits;       /* log2 G */
+    uint32_t part_bits;        /* B: partition bits of the skew rule (top B bits of h) */
+    uint32_t large_threshold;  /* L: a partition is large iff |R_p| > L or |S_p| > L (both > 0) */
+    uint32_t heavy_threshold;  /* T_h: skewed iff max(cnt_R, cnt_S) >= T_h (global counts) */
+    uint32_t cand_threshold;   /* tau = ceil(T_h / G): local candidate threshold */
+    int32_t force_all_normal;  /* gsh_config hook: no partition is large, no skewed key */
+} gsh_shard_params;
 
-/* d_counts[0..G] (device u64, caller zeroes): tuples per destination, index G = heavy.
- * d_heavy_keys: device array of n_heavy keys (raw keys, not hashes) sorted ascending. */
+/* Parameters for global sizes n_r_global, n_s_global over `world` ranks; B, L and T_h are what
+ * gsh_join would use on one GPU holding the whole input (cfg as for gsh_join; NULL = defaults).
+ * Host-only (no CUDA call).  GSH_ERR_INVALID for a bad world or config. */
+GSH_API gsh_status gsh_shard_plan(uint64_t n_r_global, uint64_t n_s_global, uint32_t world,
+                                  const gsh_config *cfg, gsh_shard_params *out);
+
+/* d_hist (device u64[2 << part_bits], overwritten): d_hist[d] = #{R tuples with top part_bits
+ * of h == d}, d_hist[2^part_bits + d] the same for S (the L106 "count" of the local shard). */
+GSH_API gsh_status gsh_shard_histogram(const gsh_relation *R, const gsh_relation *S,
+                                       const gsh_shard_params *p, uint64_t *d_hist, void *stream);
+
+/* Device workspace of gsh_shard_candidates for a local shard of n_r + n_s tuples (holds the
+ * local count table reused by gsh_shard_agree; keep it alive between the two calls). */
+GSH_API size_t gsh_shard_workspace_bytes(uint64_t n_r, uint64_t n_s);
+
+/* Local skew candidates.  d_hist_global: device u64[2 << part_bits], the all-reduced histogram.
+ * Counts every key of a globally large partition exactly (both sides) into a table in
+ * `workspace`, then writes the h of every key with local max(cnt_R, cnt_S) >= cand_threshold
+ * to d_cand (device u32[cap], unspecified order); *h_n = how many (host).  *h_overflow (host,
+ * may be NULL) = 1 iff the count table filled: keys were dropped from the candidates, which
+ * keeps the join exact (an unflagged skewed key is simply routed as a normal key) but loses
+ * its skew handling.  GSH_ERR_INVALID if *h_n > cap (nothing beyond cap is written). */
+GSH_API gsh_status gsh_shard_candidates(const gsh_relation *R, const gsh_relation *S,
+                                        const gsh_shard_params *p, const uint64_t *d_hist_global,
+                                        void *workspace, size_t workspace_bytes, void *stream,
+                                        uint32_t *d_cand, uint64_t cap, uint64_t *h_n,
+                                        uint32_t *h_overflow);
+
+/* Device workspace of gsh_shard_agree for a gathered buffer of n_gathered slots (world x
+ * stride); also enough for gsh_shard_select on m <= n_gathered union keys. */
+GSH_API size_t gsh_shard_agree_workspace_bytes(uint64_t n_gathered);
+
+/* Union of the all-gathered candidates.  d_gathered: device u32[world * stride], rank g's
+ * h_sizes[g] (host u64[world]) candidates at [g * stride, g * stride + h_sizes[g]).  Writes
+ * the distinct values to d_union (device u32[cap]) in order of FIRST occurrence in the
+ * gathered buffer -- the same order on every rank, since every rank holds the same buffer --
+ * and this rank's exact counts of each to d_counts (device u64[2 * cap], interleaved
+ * cnt_R, cnt_S), looked up in the table cand_ws (the workspace of this rank's
+ * gsh_shard_candidates call).  *h_n = number of distinct values (host).  world * stride < 2^32. */
+GSH_API gsh_status gsh_shard_agree(const void *cand_ws, size_t cand_ws_bytes,
+                                   const uint32_t *d_gathered, uint32_t world, uint64_t stride,
+                                   const uint64_t *h_sizes, void *workspace, size_t workspace_bytes,
+                                   void *stream, uint32_t *d_union, uint64_t *d_counts, uint64_t cap,
+                                   uint64_t *h_n);
+
+/* Skewed keys (L112 reading): d_heavy[i] (device u32[cap]) = the union keys with global
+ * max(cnt_R, cnt_S) >= heavy_threshold, in union order (stable compaction: identical on every
+ * rank).  d_counts: device u64[2 * m], the all-reduced interleaved counts.  *h_n (host). */
+GSH_API gsh_status gsh_shard_select(const uint32_t *d_union, const uint64_t *d_counts, uint64_t m,
+                                    const gsh_shard_params *p, void *workspace,
+                                    size_t workspace_bytes, void *stream, uint32_t *d_heavy,
+                                    uint64_t cap, uint64_t *h_n);
+
+/* Bytes of the open-addressing set of n_heavy skewed keys (0 for an empty set). */
+GSH_API size_t gsh_heavy_set_bytes(uint64_t n_heavy);
+
+/* Build the set of the n skewed keys d_heavy (device u32 h values) in d_set (device,
+ * 256-byte aligned, >= gsh_heavy_set_bytes(n) bytes).  Synchronises `stream`. */
+GSH_API gsh_status gsh_heavy_set_build(const uint32_t *d_heavy, uint64_t n, void *d_set,
+                                       size_t set_bytes, void *stream);
+
+/* Tuples per destination: d_counts[0..G] (device u64[G + 1], overwritten), G = 2^route_bits;
+ * destination d < G = top route_bits of h (normal key), d = G = skewed key (member of the
+ * set d_set / set_bytes from gsh_heavy_set_build; NULL / 0 = no skewed keys).  route_bits <= 8. */
 GSH_API gsh_status gsh_route_count(const uint32_t *d_keys, uint64_t n, uint32_t route_bits,
-                           const uint32_t *d_heavy_keys, uint64_t n_heavy,
-                           uint64_t *d_counts, void *stream);
+                                   const void *d_set, size_t set_bytes, uint64_t *d_counts,
+                                   void *stream);
 
-/* Scatter tuples into destination-grouped SoA send buffers.  d_offsets[0..G]: device u64
- * exclusive scan of gsh_route_count's counts.  d_cursor: device u64[G+1] scratch the
- * caller zeroes.  Order inside a destination group is unspecified. */
+/* Scatter every tuple to its destination (as gsh_route_count).  d_dst: device u64[2 (G + 1)],
+ * d_dst[2d] / d_dst[2d + 1] = device addresses of destination d's key / payload arrays, each
+ * with room for its count; d_cursor: device u64[G + 1] scratch (overwritten).  The order of
+ * tuples inside a destination is unspecified. */
 GSH_API gsh_status gsh_route_scatter(const uint32_t *d_keys, const uint32_t *d_payloads, uint64_t n,
-                             uint32_t route_bits, const uint32_t *d_heavy_keys, uint64_t n_heavy,
-                             const uint64_t *d_offsets, uint64_t *d_cursor,
-                             uint32_t *d_out_keys, uint32_t *d_out_payloads, void *stream);
-
-/* Exact local counts of query keys: d_counts[q] += #{i : d_keys[i] == d_query[q]} for a
- * device array d_query of m keys sorted ascending (d_counts device u64[m], caller zeroes). */
-GSH_API gsh_status gsh_count_keys(const uint32_t *d_keys, uint64_t n, const uint32_t *d_query,
-                          uint64_t m, uint64_t *d_counts, void *stream);
-
-/* Candidate skewed keys of a shard: keys whose partition (top part_bits of fmix32 below
- * hi_bits) is flagged in d_large (device u8[2^part_bits]) and whose local count on either
- * side is >= threshold.  Writes raw keys to d_cand (device, cap entries), count to *h_n. */
-GSH_API gsh_status gsh_local_candidates(const gsh_relation *R, const gsh_relation *S, uint32_t hi_bits,
-                                uint32_t part_bits, const uint8_t *d_large, uint32_t threshold,
-                                void *workspace, size_t workspace_bytes, void *stream,
-                                uint32_t *d_cand, uint64_t cap, uint64_t *h_n);
-
-/* Workspace for gsh_local_candidates. */
-GSH_API size_t gsh_candidates_workspace_bytes(uint64_t n_r, uint64_t n_s);
+                                     uint32_t route_bits, const void *d_set, size_t set_bytes,
+                                     const uint64_t *d_dst, uint64_t *d_cursor, void *stream);
 
 /* ------------------------------------------------------------------- diagnostics -- */
 GSH_API const char *gsh_status_string(gsh_status s);

@@ -175,7 +175,9 @@ def heavy_rule(rk, sk, part_bits: int, large_threshold: int, threshold: int, rou
     readings of DESIGN.md §3 (exact counts replace the 1 % sample, north star):
 
       partition p = top `part_bits` bits of h below `route_bits` (final partitions);
-      large(p)  <=>  |R_p| > L  or  |S_p| > L,  L = large_threshold   (L107 threshold)
+      large(p)  <=>  (|R_p| > L  or  |S_p| > L)  and  |R_p| > 0  and  |S_p| > 0
+                     L = large_threshold   (L107 threshold; R5: a partition with an
+                     empty side produces no result tuple, so it is never treated as large)
       heavy(k)  <=>  k lies in a large partition and
                      max(cnt_R(k), cnt_S(k)) >= threshold            (L112 'top-k')
 
@@ -189,7 +191,7 @@ def heavy_rule(rk, sk, part_bits: int, large_threshold: int, threshold: int, rou
     nparts = 1 << part_bits
     szr = np.bincount(pr, minlength=nparts)
     szs = np.bincount(ps, minlength=nparts)
-    large = (szr > large_threshold) | (szs > large_threshold)
+    large = ((szr > large_threshold) | (szs > large_threshold)) & (szr > 0) & (szs > 0)
     ur, cr = np.unique(hr[large[pr]], return_counts=True)
     us, cs = np.unique(hs[large[ps]], return_counts=True)
     allk = np.union1d(ur, us).astype(np.uint32)

@@ -93,6 +93,18 @@ class GshResult(ctypes.Structure):
         return d
 
 
+class GshShardParams(ctypes.Structure):
+    _fields_ = [
+        ("world", u32),
+        ("route_bits", u32),
+        ("part_bits", u32),
+        ("large_threshold", u32),
+        ("heavy_threshold", u32),
+        ("cand_threshold", u32),
+        ("force_all_normal", i32),
+    ]
+
+
 # (name, restype, argtypes) for every entry point declared in include/gsh.h
 _PROTOS = [
     ("gsh_config_default", None, [ctypes.POINTER(GshConfig)]),
@@ -111,12 +123,22 @@ _PROTOS = [
     ("gsh_detect", ctypes.c_int, [ctypes.POINTER(GshRelation), ctypes.POINTER(GshRelation),
                                   ctypes.POINTER(GshConfig), vp, ctypes.c_size_t, vp, p32, p32, p32, u64, p64,
                                   ctypes.POINTER(GshResult)]),
-    ("gsh_route_count", ctypes.c_int, [vp, u64, u32, vp, u64, vp, vp]),
-    ("gsh_route_scatter", ctypes.c_int, [vp, vp, u64, u32, vp, u64, vp, vp, vp, vp, vp]),
-    ("gsh_count_keys", ctypes.c_int, [vp, u64, vp, u64, vp, vp]),
-    ("gsh_local_candidates", ctypes.c_int, [ctypes.POINTER(GshRelation), ctypes.POINTER(GshRelation), u32, u32, vp,
-                                            u32, vp, ctypes.c_size_t, vp, vp, u64, p64]),
-    ("gsh_candidates_workspace_bytes", ctypes.c_size_t, [u64, u64]),
+    ("gsh_shard_plan", ctypes.c_int, [u64, u64, u32, ctypes.POINTER(GshConfig), ctypes.POINTER(GshShardParams)]),
+    ("gsh_shard_histogram", ctypes.c_int, [ctypes.POINTER(GshRelation), ctypes.POINTER(GshRelation),
+                                           ctypes.POINTER(GshShardParams), vp, vp]),
+    ("gsh_shard_workspace_bytes", ctypes.c_size_t, [u64, u64]),
+    ("gsh_shard_candidates", ctypes.c_int, [ctypes.POINTER(GshRelation), ctypes.POINTER(GshRelation),
+                                            ctypes.POINTER(GshShardParams), vp, vp, ctypes.c_size_t, vp, vp, u64,
+                                            p64, p32]),
+    ("gsh_shard_agree_workspace_bytes", ctypes.c_size_t, [u64]),
+    ("gsh_shard_agree", ctypes.c_int, [vp, ctypes.c_size_t, vp, u32, u64, p64, vp, ctypes.c_size_t, vp, vp, vp, u64,
+                                       p64]),
+    ("gsh_shard_select", ctypes.c_int, [vp, vp, u64, ctypes.POINTER(GshShardParams), vp, ctypes.c_size_t, vp, vp, u64,
+                                        p64]),
+    ("gsh_heavy_set_bytes", ctypes.c_size_t, [u64]),
+    ("gsh_heavy_set_build", ctypes.c_int, [vp, u64, vp, ctypes.c_size_t, vp]),
+    ("gsh_route_count", ctypes.c_int, [vp, u64, u32, vp, ctypes.c_size_t, vp, vp]),
+    ("gsh_route_scatter", ctypes.c_int, [vp, vp, u64, u32, vp, ctypes.c_size_t, vp, vp, vp]),
     ("gsh_status_string", ctypes.c_char_p, [ctypes.c_int]),
     ("gsh_last_error", ctypes.c_char_p, []),
     ("gsh_version", ctypes.c_int, []),

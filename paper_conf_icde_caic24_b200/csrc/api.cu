@@ -17,11 +17,6 @@
 namespace gsh {
 // defined in join.cu
 uint32_t nm_table_slots(uint32_t rl);
-// defined in skew.cu
-size_t cand_table_slots(uint64_t nR, uint64_t nS);
-int launch_candidates(const uint32_t* kr, uint64_t nR, const uint32_t* ks, uint64_t nS, uint32_t hi_bits,
-                      uint32_t part_bits, const uint8_t* large, uint32_t threshold, void* ws, uint32_t* out,
-                      uint64_t outcap, unsigned long long* d_nout, cudaStream_t s);
 }  // namespace gsh
 
 using namespace gsh;
@@ -143,7 +138,10 @@ bool plan_build(Plan& p, uint64_t nR, uint64_t nS, const gsh_config* cfg_in, voi
     if (p.force_heavy)
         p.h_max = p.gt_cap_alloc;
     else {
+        // exact rule: a skewed key holds >= T_h tuples on one side; sampled rule (detect_mode 1):
+        // up to top_k keys per large partition, whatever their counts
         uint64_t hm = (nR + nS) / (p.Th ? p.Th : 1) + 1;
+        if (p.detect_mode == 1 && uint64_t(p.F) * p.top_k > hm) hm = uint64_t(p.F) * p.top_k;
         p.h_max = hm < p.gt_cap_alloc ? hm : p.gt_cap_alloc;
     }
     // pass-1 units (= histogram slices): whole 16K-key chunks, about one unit per scatter CTA
@@ -210,6 +208,25 @@ bool plan_build(Plan& p, uint64_t nR, uint64_t nS, const gsh_config* cfg_in, voi
     p.nm_prefix = c.take<uint64_t>(F + 1);
     p.scan_scratch = c.take<uint64_t>(p.scan_scratch_elems);
     p.bytes = c.off;
+    return true;
+}
+
+// Error helpers for the other C-ABI translation units (shard.cu): same thread-local message.
+gsh_status api_fail(gsh_status st, const char* msg) { return fail(st, msg); }
+gsh_status api_cuda(const char* where) {
+    const cudaError_t e = cudaGetLastError();
+    return e == cudaSuccess ? GSH_OK : cuda_fail(e, where);
+}
+
+// The single-GPU rule's parameters for global sizes (multi-GPU skew agreement, gsh_shard_plan):
+// partition bits B = b1 + b2, large-partition threshold L and skewed-key threshold T_h, exactly as
+// plan_build derives them for one GPU holding the whole input.
+bool shard_plan_params(uint64_t nR, uint64_t nS, const gsh_config* cfg, uint32_t* B, uint32_t* L, uint32_t* Th) {
+    Plan p;
+    if (!plan_build(p, nR, nS, cfg, nullptr, 148)) return false;
+    *B = p.b1 + p.b2;
+    *L = p.L;
+    *Th = p.Th;
     return true;
 }
 
@@ -431,6 +448,8 @@ static gsh_status join_direct(const gsh_relation* R, const gsh_relation* S, gsh_
     cudaError_t ce = cudaMemcpyAsync(&hs, p.st, sizeof(DevState), cudaMemcpyDeviceToHost, s);
     if (ce == cudaSuccess) ce = cudaStreamSynchronize(s);
     if (ce != cudaSuccess) return cuda_fail(ce, "classify sync");
+    if (hs.route_mismatch)
+        return fail(GSH_ERR_INVALID, "gsh_config.route_bits: the tuples do not all share the top route_bits of h");
     const uint32_t n_large = hs.n_large;
     uint32_t n_heavy = 0;
     p.nm_slots = nm_table_slots(hs.max_rlen < p.C ? (hs.max_rlen ? hs.max_rlen : 1) : p.C);
@@ -446,7 +465,7 @@ static gsh_status join_direct(const gsh_relation* R, const gsh_relation* S, gsh_
         if (ce == cudaSuccess) ce = cudaStreamSynchronize(s);
         if (ce != cudaSuccess) return cuda_fail(ce, "detect sync");
         n_heavy = hs.n_heavy;
-        if (n_heavy > p.h_max) return fail(GSH_ERR_INTERNAL, "skewed-key list overflow");
+        if (hs.heavy_overflow || n_heavy > p.h_max) return fail(GSH_ERR_INTERNAL, "skewed-key list overflow");
         launches += launch_heavy_prefix(p, n_heavy, n_large, s);
         launches += launch_split(p, n_large, (uint32_t)gcap, s);
         e5 = tm.mark();
@@ -739,6 +758,7 @@ gsh_status gsh_detect(const gsh_relation* R, const gsh_relation* S, const gsh_co
         ce = cudaMemcpyAsync(&hs, p.st, sizeof(DevState), cudaMemcpyDeviceToHost, s);
         if (ce == cudaSuccess) ce = cudaStreamSynchronize(s);
         if (ce != cudaSuccess) return cuda_fail(ce, "detect sync");
+        if (hs.heavy_overflow || hs.n_heavy > p.h_max) return fail(GSH_ERR_INTERNAL, "skewed-key list overflow");
     }
     if (res) {
         res->n_large = hs.n_large;
@@ -766,63 +786,6 @@ gsh_status gsh_detect(const gsh_relation* R, const gsh_relation* S, const gsh_co
             h_cnt_s[i] = hk[i].cnt_s;
         }
     }
-    return GSH_OK;
-}
-
-gsh_status gsh_route_count(const uint32_t* d_keys, uint64_t n, uint32_t route_bits, const uint32_t* d_heavy_keys,
-                           uint64_t n_heavy, uint64_t* d_counts, void* stream) {
-    if (route_bits > 8) return fail(GSH_ERR_INVALID, "route_bits > 8");
-    if ((n && !d_keys) || !d_counts || (n_heavy && !d_heavy_keys)) return fail(GSH_ERR_INVALID, "NULL pointer");
-    launch_route_count(d_keys, n, route_bits, d_heavy_keys, n_heavy, d_counts, reinterpret_cast<cudaStream_t>(stream));
-    return check_launch("route_count");
-}
-
-gsh_status gsh_route_scatter(const uint32_t* d_keys, const uint32_t* d_payloads, uint64_t n, uint32_t route_bits,
-                             const uint32_t* d_heavy_keys, uint64_t n_heavy, const uint64_t* d_offsets,
-                             uint64_t* d_cursor, uint32_t* d_out_keys, uint32_t* d_out_payloads, void* stream) {
-    if (route_bits > 8) return fail(GSH_ERR_INVALID, "route_bits > 8");
-    if (n && (!d_keys || !d_payloads || !d_offsets || !d_cursor || !d_out_keys || !d_out_payloads))
-        return fail(GSH_ERR_INVALID, "NULL pointer");
-    if (n_heavy && !d_heavy_keys) return fail(GSH_ERR_INVALID, "NULL heavy keys");
-    launch_route_scatter(d_keys, d_payloads, n, route_bits, d_heavy_keys, n_heavy, d_offsets, d_cursor, d_out_keys,
-                         d_out_payloads, reinterpret_cast<cudaStream_t>(stream));
-    return check_launch("route_scatter");
-}
-
-gsh_status gsh_count_keys(const uint32_t* d_keys, uint64_t n, const uint32_t* d_query, uint64_t m, uint64_t* d_counts,
-                          void* stream) {
-    if ((n && !d_keys) || (m && (!d_query || !d_counts))) return fail(GSH_ERR_INVALID, "NULL pointer");
-    launch_count_keys(d_keys, n, d_query, m, d_counts, reinterpret_cast<cudaStream_t>(stream));
-    return check_launch("count_keys");
-}
-
-size_t gsh_candidates_workspace_bytes(uint64_t n_r, uint64_t n_s) {
-    return align256(cand_table_slots(n_r, n_s) * 16 + 16) + 256;
-}
-
-gsh_status gsh_local_candidates(const gsh_relation* R, const gsh_relation* S, uint32_t hi_bits, uint32_t part_bits,
-                                const uint8_t* d_large, uint32_t threshold, void* workspace, size_t workspace_bytes,
-                                void* stream, uint32_t* d_cand, uint64_t cap, uint64_t* h_n) {
-    if (!validate_rel(R) || !validate_rel(S)) return fail(GSH_ERR_INVALID, "invalid relation");
-    if (part_bits > 16 || hi_bits + part_bits > 32 || !d_large || !h_n || (cap && !d_cand))
-        return fail(GSH_ERR_INVALID, "bad argument");
-    const size_t need = gsh_candidates_workspace_bytes(R->n, S->n);
-    if (!workspace || workspace_bytes < need || (reinterpret_cast<uintptr_t>(workspace) & 255u))
-        return fail(GSH_ERR_INVALID, "workspace NULL, misaligned or too small");
-    cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
-    unsigned long long* d_nout =
-        reinterpret_cast<unsigned long long*>(reinterpret_cast<unsigned char*>(workspace) + need - 256);
-    cudaMemsetAsync(d_nout, 0, 8, s);
-    launch_candidates(R->keys, R->n, S->keys, S->n, hi_bits, part_bits, d_large, threshold ? threshold : 1, workspace,
-                      d_cand, cap, d_nout, s);
-    gsh_status st = check_launch("candidates");
-    if (st != GSH_OK) return st;
-    unsigned long long nout = 0;
-    cudaError_t ce = cudaMemcpyAsync(&nout, d_nout, 8, cudaMemcpyDeviceToHost, s);
-    if (ce == cudaSuccess) ce = cudaStreamSynchronize(s);
-    if (ce != cudaSuccess) return cuda_fail(ce, "candidates sync");
-    *h_n = nout;
-    if (nout > cap) return fail(GSH_ERR_INVALID, "candidate capacity too small");
     return GSH_OK;
 }
 

@@ -2,6 +2,7 @@
 #pragma once
 #include <cstddef>
 #include <cstdint>
+#include <mutex>
 #include <cuda_runtime.h>
 
 #include "../../include/gsh.h"
@@ -90,7 +91,22 @@ struct DevState {
     unsigned long long skew_claim;                 // tile claim counter
     unsigned int n_large, n_heavy, detect_overflow, max_rlen;  // max_rlen: largest |R_p| with |S_p| > 0
     unsigned int claim[8];                         // per-kernel work claim counters
+    unsigned int route_mismatch;                   // route_bits > 0: tuples differ in the top route bits
+    unsigned int heavy_overflow;                   // more skewed keys than the list H holds
 };
+
+// Per-(call site, device) one-time setup (kernel attributes): concurrent host threads wait until
+// it has run; a process driving several devices runs it once on each.
+constexpr int kMaxDevices = 64;
+template <class Fn>
+inline void once_per_device(std::once_flag (&flags)[kMaxDevices], Fn&& fn) {
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= kMaxDevices) {
+        fn();
+        return;
+    }
+    std::call_once(flags[dev], fn);
+}
 
 // Skewed-key side list entry H[k].
 struct HeavyKey {

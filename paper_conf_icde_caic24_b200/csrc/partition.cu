@@ -57,11 +57,15 @@ constexpr uint32_t kHistMaxEvents = 128;
 static_assert(kScatterChunk == 16 * kHistBlock, "a full chunk is 4 uint4 per histogram thread");
 static_assert(3 * ((uint64_t(kHistMaxUnitChunks) * kScatterChunk) >> 16) <= kHistMaxEvents, "wrap events of a slice");
 
-template <bool FAST16>
+// CHECK (route_bits > 0): also verify the caller's gsh_config.route_bits assertion -- every tuple
+// shares the top route_bits of h -- by OR-ing t and ~t over all keys (t = those bits): they are all
+// equal iff (OR t) & (OR ~t) has no bit set.  The NM-join's chained table relies on it.
+template <bool FAST16, bool CHECK>
 __global__ void __launch_bounds__(kHistBlock, 1)
 k_hist2d(const uint32_t* __restrict__ k0, uint64_t n0, const uint32_t* __restrict__ k1, uint64_t n1,
          uint32_t shift, uint32_t nbits, uint32_t b2, uint32_t* __restrict__ partial, uint32_t* __restrict__ c1cnt,
-         uint32_t nu0, uint32_t nu1, uint32_t unit_chunks) {
+         uint32_t nu0, uint32_t nu1, uint32_t unit_chunks, uint32_t rshift, DevState* st) {
+    uint32_t r_or = 0, r_nor = 0;
     extern __shared__ uint32_t cnt[];
     __shared__ uint32_t c1s[256];
     __shared__ uint32_t ev_bin[kHistMaxEvents];
@@ -101,7 +105,13 @@ k_hist2d(const uint32_t* __restrict__ k0, uint64_t n0, const uint32_t* __restric
         if (FAST16) {
             count_exact(hash32_top(key) >> 16);
         } else {
-            const uint32_t bin = ((top16 ? hash32_top(key) : hash32(key)) >> shift) & mask;
+            const uint32_t hk = top16 ? hash32_top(key) : hash32(key);
+            if (CHECK) {
+                const uint32_t t = hk >> rshift;
+                r_or |= t;
+                r_nor |= ~t;
+            }
+            const uint32_t bin = (hk >> shift) & mask;
             if (packed) count_exact(bin); else atomicAdd(&cnt[bin], 1u);
         }
     };
@@ -195,6 +205,11 @@ k_hist2d(const uint32_t* __restrict__ k0, uint64_t n0, const uint32_t* __restric
             c1s[threadIdx.x] = 0;
         }
     }
+    if (CHECK) {
+        r_or = __reduce_or_sync(kFull, r_or);
+        r_nor = __reduce_or_sync(kFull, r_nor);
+        if ((threadIdx.x & 31) == 0 && (r_or & r_nor & ((1u << (32 - rshift)) - 1))) atomicOr(&st->route_mismatch, 1u);
+    }
 }
 
 int launch_hist(const Plan& p, const uint32_t* k0, const uint32_t* k1, cudaStream_t s) {
@@ -202,24 +217,29 @@ int launch_hist(const Plan& p, const uint32_t* k0, const uint32_t* k1, cudaStrea
     const uint32_t shift = nbits ? (32 - p.route_bits - nbits) : 0;
     const uint32_t F = 1u << nbits;
     const size_t smem = size_t(F > (1u << 15) ? F / 2 : F) * 4;
-    static bool attr_set = false;
-    if (!attr_set) {
-        cudaFuncSetAttribute(k_hist2d<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, 128 * 1024);
-        cudaFuncSetAttribute(k_hist2d<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, 128 * 1024);
-        attr_set = true;
-    }
+    static std::once_flag attr_once[kMaxDevices];
+    once_per_device(attr_once, [] {
+        cudaFuncSetAttribute(k_hist2d<false, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, 128 * 1024);
+        cudaFuncSetAttribute(k_hist2d<false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, 128 * 1024);
+        cudaFuncSetAttribute(k_hist2d<true, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, 128 * 1024);
+    });
     const bool fast16 = nbits == 16 && p.route_bits == 0 && p.b2 == 8;
+    const uint32_t rshift = 32 - p.route_bits;
     // (Rejected, kept in history: CTA pairs each counting one half of 2^16 u32 bins -- every key
     // hashed twice, ALU-bound at 0.76 ms for 2^28 keys; a cluster pair exchanging bins through
     // DSMEM atomics, 3.6 ms, or DSMEM loads, 1.0 ms.)
     if (fast16)
-        k_hist2d<true><<<p.hist_grid, kHistBlock, smem, s>>>(k0, p.n[0], k1, p.n[1], shift, nbits, p.b2,
-                                                             p.hist_partial, p.c1cnt, p.nu1[0], p.nu1[1],
-                                                             p.unit_chunks);
+        k_hist2d<true, false><<<p.hist_grid, kHistBlock, smem, s>>>(k0, p.n[0], k1, p.n[1], shift, nbits, p.b2,
+                                                                    p.hist_partial, p.c1cnt, p.nu1[0], p.nu1[1],
+                                                                    p.unit_chunks, rshift, p.st);
+    else if (p.route_bits)
+        k_hist2d<false, true><<<p.hist_grid, kHistBlock, smem, s>>>(k0, p.n[0], k1, p.n[1], shift, nbits, p.b2,
+                                                                    p.hist_partial, p.c1cnt, p.nu1[0], p.nu1[1],
+                                                                    p.unit_chunks, rshift, p.st);
     else
-        k_hist2d<false><<<p.hist_grid, kHistBlock, smem, s>>>(k0, p.n[0], k1, p.n[1], shift, nbits, p.b2,
-                                                              p.hist_partial, p.c1cnt, p.nu1[0], p.nu1[1],
-                                                              p.unit_chunks);
+        k_hist2d<false, false><<<p.hist_grid, kHistBlock, smem, s>>>(k0, p.n[0], k1, p.n[1], shift, nbits, p.b2,
+                                                                     p.hist_partial, p.c1cnt, p.nu1[0], p.nu1[1],
+                                                                     p.unit_chunks, rshift, p.st);
     return 1;
 }
 
@@ -699,16 +719,19 @@ size_t scatter_smem_bytes(int tile) {
 template <int BLOCK, int IPT, int PASS, bool TMAST>
 int launch_scatter_pass(const Plan& p, const ScatterArgs& a, cudaStream_t s) {
     const size_t smem = scatter_smem_bytes(BLOCK * IPT);
-    static bool attr_set = false;
-    if (!attr_set) {
+    static std::once_flag attr_once[kMaxDevices];   // > 48 KB of dynamic shared memory: opt in once per device
+    once_per_device(attr_once, [&] {
         cudaFuncSetAttribute(k_scatter<BLOCK, IPT, PASS, TMAST>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                              (int)smem);
-        attr_set = true;
-    }
-    static int occ = 0;   // per kernel instance (fixed block and shared memory): query once
+    });
+    static int occ_dev[kMaxDevices] = {0};   // per kernel instance and device: query once
+    int dev = 0;
+    cudaGetDevice(&dev);
+    int& occ = occ_dev[dev >= 0 && dev < kMaxDevices ? dev : 0];
     if (occ < 1) {
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_scatter<BLOCK, IPT, PASS, TMAST>, BLOCK, smem);
-        if (occ < 1) occ = 1;
+        int o = 0;
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, k_scatter<BLOCK, IPT, PASS, TMAST>, BLOCK, smem);
+        occ = o < 1 ? 1 : o;
     }
     k_scatter<BLOCK, IPT, PASS, TMAST><<<(unsigned)(p.num_sms * occ), BLOCK, smem, s>>>(a);
     return 1;
@@ -794,11 +817,10 @@ int launch_radix_hist(const uint32_t* keys, uint64_t n, uint32_t hi_bits, uint32
     const uint32_t shift = nbits ? (32 - hi_bits - nbits) : 0;
     const int use_smem = nbits <= 14;
     size_t smem = use_smem ? size_t(F) * 4 : 0;
-    static bool attr_set = false;
-    if (!attr_set) {
+    static std::once_flag attr_once[kMaxDevices];   // > 48 KB of dynamic shared memory: opt in once per device
+    once_per_device(attr_once, [&] {
         cudaFuncSetAttribute(k_radix_hist, cudaFuncAttributeMaxDynamicSharedMemorySize, 64 * 1024);
-        attr_set = true;
-    }
+    });
     unsigned grid = (unsigned)umin64((n + 1023) / 1024, 148);
     k_radix_hist<<<grid, 1024, smem, s>>>(keys, n, shift, F - 1, reinterpret_cast<unsigned long long*>(hist),
                                           use_smem);

@@ -17,6 +17,7 @@
 #include "gsh_device.cuh"
 #include "gsh_internal.h"
 #include "gsh_scan.cuh"
+#include "gsh_table.cuh"
 
 namespace gsh {
 
@@ -110,40 +111,6 @@ __device__ __forceinline__ uint2 item_tuple(const LargeView& v, const ItemRange&
     side = e >= r.cr;
     uint64_t off = side ? (e - r.cr) : e;
     return v.part[side][v.start[size_t(side) * (v.F + 1) + r.p] + off];
-}
-
-__device__ __forceinline__ uint32_t gt_slot0(uint32_t h, uint32_t logcap) {
-    return (h * 0x9E3779B1u) >> (32 - logcap);
-}
-
-// Insert-or-find h; returns slot or kNoHeavy when the probe budget is exhausted.
-__device__ __forceinline__ uint32_t gt_insert(unsigned long long* keys, uint32_t h, uint32_t logcap) {
-    const unsigned long long tag = (1ull << 32) | h;
-    const uint32_t mask = (1u << logcap) - 1;
-    uint32_t slot = gt_slot0(h, logcap);
-    for (int probe = 0; probe < kDetectMaxProbe; ++probe) {
-        unsigned long long cur = keys[slot];
-        if (cur == tag) return slot;
-        if (cur == 0) {
-            unsigned long long prev = atomicCAS(&keys[slot], 0ull, tag);
-            if (prev == 0 || prev == tag) return slot;
-        }
-        slot = (slot + 1) & mask;
-    }
-    return kNoHeavy;
-}
-
-__device__ __forceinline__ uint32_t gt_find(const unsigned long long* keys, uint32_t h, uint32_t logcap) {
-    const unsigned long long tag = (1ull << 32) | h;
-    const uint32_t mask = (1u << logcap) - 1;
-    uint32_t slot = gt_slot0(h, logcap);
-    for (int probe = 0; probe < kDetectMaxProbe; ++probe) {
-        unsigned long long cur = keys[slot];
-        if (cur == tag) return slot;
-        if (cur == 0) return kNoHeavy;
-        slot = (slot + 1) & mask;
-    }
-    return kNoHeavy;
 }
 
 // ------------------------------------------------------------------- a6: detect --
@@ -294,7 +261,7 @@ int launch_sample_topk(const Plan& p, uint32_t n_large, uint32_t gt_cap, cudaStr
 __global__ void k_select(const unsigned long long* __restrict__ gt_key, const uint32_t* __restrict__ gt_cnt,
                          uint32_t* __restrict__ gt_hid, uint32_t cap, uint32_t cap_alloc, uint32_t Th,
                          int force_heavy, uint32_t pshift, uint32_t pmask, uint32_t F, HeavyKey* __restrict__ H,
-                         uint32_t* __restrict__ part_heavy, DevState* st) {
+                         uint64_t h_max, uint32_t* __restrict__ part_heavy, DevState* st) {
     for (uint32_t slot = blockIdx.x * blockDim.x + threadIdx.x; slot < cap; slot += gridDim.x * blockDim.x) {
         const unsigned long long kw = gt_key[slot];
         if (kw == 0) continue;
@@ -305,6 +272,11 @@ __global__ void k_select(const unsigned long long* __restrict__ gt_key, const ui
         if (heavy) {
             const uint32_t p = part_of(h, pshift, pmask);
             hid = atomicAdd(&st->n_heavy, 1u);
+            if (hid >= h_max) {   // the side list is full: the call fails (GSH_ERR_INTERNAL)
+                st->heavy_overflow = 1;
+                gt_hid[slot] = kNoHeavy;
+                continue;
+            }
             H[hid] = HeavyKey{h, cr, cs, p};
             if (cr) atomicAdd(&part_heavy[p], cr);
             if (cs) atomicAdd(&part_heavy[F + p], cs);
@@ -323,7 +295,7 @@ int launch_select(const Plan& p, uint32_t gt_cap, cudaStream_t s) {
     // detect_mode 1: the table holds exactly the sampled top-k keys, all skewed
     const uint32_t th = p.detect_mode == 1 ? 1u : p.Th;
     k_select<<<grid, 256, 0, s>>>(p.gt_key, p.gt_cnt, p.gt_hid, gt_cap, p.gt_cap_alloc, th, p.force_heavy, pshift,
-                                  p.F - 1, p.F, p.H, p.part_heavy, p.st);
+                                  p.F - 1, p.F, p.H, p.h_max, p.part_heavy, p.st);
     return 1;
 }
 
@@ -484,72 +456,3 @@ int launch_nm_setup(const Plan& p, uint32_t n_large, cudaStream_t s) {
 
 }  // namespace gsh
 
-namespace gsh {
-
-// ----------------------------------------------- multi-GPU: local skew candidates --
-// Exact local counts of every key whose partition is flagged large (globally agreed flags),
-// then keys with local max(cnt_R, cnt_S) >= threshold are emitted as candidates (by hash h).
-__global__ void k_cand_count(const uint32_t* __restrict__ keys, uint64_t n, int side, uint32_t pshift,
-                             uint32_t pmask, const uint8_t* __restrict__ large, unsigned long long* gt_key,
-                             uint32_t* gt_cnt, uint32_t cap, uint32_t logcap, unsigned int* overflow) {
-    for (uint64_t i = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; i - threadIdx.x < n;
-         i += uint64_t(gridDim.x) * blockDim.x) {
-        bool v = i < n;
-        uint32_t h = v ? hash32(keys[i]) : 0u;
-        v = v && large[part_of(h, pshift, pmask)];
-        const unsigned long long key = v ? h : ((1ull << 32) | lane_id());
-        const uint32_t peers = __match_any_sync(kFull, key);
-        if (v && (peers & lanemask_lt()) == 0) {
-            uint32_t slot = gt_insert(gt_key, h, logcap);
-            if (slot == kNoHeavy) *overflow = 1;
-            else atomicAdd(&gt_cnt[size_t(side) * cap + slot], (uint32_t)__popc(peers));
-        }
-    }
-}
-
-__global__ void k_cand_select(const unsigned long long* __restrict__ gt_key, const uint32_t* __restrict__ gt_cnt,
-                              uint32_t cap, uint32_t threshold, uint32_t* out, unsigned long long outcap,
-                              unsigned long long* nout) {
-    for (uint32_t slot = blockIdx.x * blockDim.x + threadIdx.x; slot < cap; slot += gridDim.x * blockDim.x) {
-        const unsigned long long kw = gt_key[slot];
-        if (kw == 0) continue;
-        if (max(gt_cnt[slot], gt_cnt[cap + slot]) >= threshold) {
-            unsigned long long i = atomicAdd(nout, 1ull);
-            if (i < outcap) out[i] = (uint32_t)kw;
-        }
-    }
-}
-
-size_t cand_table_slots(uint64_t nR, uint64_t nS) {
-    uint64_t t = 2 * (nR + nS);
-    uint64_t c = 1024;
-    while (c < t && c < (1ull << 26)) c <<= 1;
-    return (size_t)c;
-}
-
-int launch_candidates(const uint32_t* kr, uint64_t nR, const uint32_t* ks, uint64_t nS, uint32_t hi_bits,
-                      uint32_t part_bits, const uint8_t* large, uint32_t threshold, void* ws, uint32_t* out,
-                      uint64_t outcap, unsigned long long* d_nout, cudaStream_t s) {
-    const uint32_t cap = (uint32_t)cand_table_slots(nR, nS);
-    uint32_t logcap = 0;
-    while ((1u << logcap) < cap) ++logcap;
-    unsigned long long* gt_key = reinterpret_cast<unsigned long long*>(ws);
-    uint32_t* gt_cnt = reinterpret_cast<uint32_t*>(gt_key + cap);
-    unsigned int* overflow = gt_cnt + 2 * size_t(cap);
-    cudaMemsetAsync(ws, 0, size_t(cap) * 16 + 16, s);
-    const uint32_t pshift = part_bits ? (32 - hi_bits - part_bits) : 0;
-    const uint32_t pmask = (1u << part_bits) - 1;
-    int l = 0;
-    if (nR) {
-        k_cand_count<<<148 * 8, 512, 0, s>>>(kr, nR, 0, pshift, pmask, large, gt_key, gt_cnt, cap, logcap, overflow);
-        ++l;
-    }
-    if (nS) {
-        k_cand_count<<<148 * 8, 512, 0, s>>>(ks, nS, 1, pshift, pmask, large, gt_key, gt_cnt, cap, logcap, overflow);
-        ++l;
-    }
-    k_cand_select<<<148 * 4, 256, 0, s>>>(gt_key, gt_cnt, cap, threshold, out, outcap, d_nout);
-    return l + 1;
-}
-
-}  // namespace gsh

@@ -8,6 +8,7 @@ no CPU path: calling with CPU tensors raises.
 from __future__ import annotations
 
 import ctypes
+import threading
 
 import torch
 
@@ -80,27 +81,32 @@ def _rel(keys: torch.Tensor, pays: torch.Tensor, side: str) -> GshRelation:
                        keys.numel())
 
 
-def _stream_handle(stream) -> int | None:
+def _stream_handle(stream, device=None) -> int | None:
+    """cudaStream_t of `stream`; None = torch's current stream of `device` (per thread)."""
     if stream is None:
-        return torch.cuda.current_stream().cuda_stream
+        return torch.cuda.current_stream(device).cuda_stream
     if isinstance(stream, torch.cuda.Stream):
         return stream.cuda_stream
     return int(stream)
 
 
 class Workspace:
-    """Grow-only device scratch buffer (torch caching allocator), one per device."""
+    """Grow-only device scratch buffer (torch caching allocator), one per (device, thread): calls
+    from several host threads (e.g. logical ranks sharing a GPU) never share scratch."""
 
     def __init__(self):
-        self._buf: dict[int, torch.Tensor] = {}
+        self._tls = threading.local()
 
     def get(self, nbytes: int, device: torch.device) -> torch.Tensor:
         idx = device.index if device.index is not None else torch.cuda.current_device()
-        b = self._buf.get(idx)
+        bufs = getattr(self._tls, "bufs", None)
+        if bufs is None:
+            bufs = self._tls.bufs = {}
+        b = bufs.get(idx)
         if b is None or b.numel() < nbytes:
-            self._buf.pop(idx, None)
+            bufs.pop(idx, None)
             b = torch.empty(max(nbytes, 256), dtype=torch.uint8, device=torch.device("cuda", idx))
-            self._buf[idx] = b
+            bufs[idx] = b
         return b
 
 
@@ -149,7 +155,7 @@ def join(r_keys: torch.Tensor, r_payloads: torch.Tensor, s_keys: torch.Tensor, s
     res = GshResult()
     args = (ctypes.byref(R), ctypes.byref(S), _lib.GSH_OUT_MATERIALIZE if mat else _lib.GSH_OUT_COUNT,
             ctypes.byref(outp) if outp is not None else None, ws.data_ptr(), ws.numel(),
-            ctypes.byref(config) if config is not None else None, _stream_handle(stream), ctypes.byref(res))
+            ctypes.byref(config) if config is not None else None, _stream_handle(stream, dev), ctypes.byref(res))
     if dev.index == torch.cuda.current_device():
         st = lib.gsh_join(*args)
     else:
@@ -192,7 +198,7 @@ def join_host(r_keys, r_payloads, s_keys, s_payloads, mode: str = "count", out=N
     with torch.cuda.device(dev):
         st = lib.gsh_join_host(ctypes.byref(R), ctypes.byref(S), 1 if mat else 0,
                                ctypes.byref(outp) if outp is not None else None, ws.data_ptr(), ws.numel(),
-                               ctypes.byref(config) if config is not None else None, _stream_handle(stream),
+                               ctypes.byref(config) if config is not None else None, _stream_handle(stream, dev),
                                ctypes.byref(res))
     check(st, "gsh_join_host")
     return JoinResult(count=int(res.count), checksum=int(res.checksum), written=int(res.written),
@@ -207,7 +213,7 @@ def hash_keys(keys: torch.Tensor, stream=None) -> torch.Tensor:
     out = torch.empty_like(k, dtype=torch.int32)
     with torch.cuda.device(k.device):
         check(lib.gsh_hash_keys(k.data_ptr() if k.numel() else None, out.data_ptr() if k.numel() else None,
-                                k.numel(), _stream_handle(stream)), "gsh_hash_keys")
+                                k.numel(), _stream_handle(stream, k.device)), "gsh_hash_keys")
     return out
 
 
@@ -218,7 +224,7 @@ def radix_histogram(keys: torch.Tensor, hi_bits: int, nbits: int, stream=None) -
     hist = torch.zeros(1 << nbits, dtype=torch.int64, device=k.device)
     with torch.cuda.device(k.device):
         check(lib.gsh_radix_histogram(k.data_ptr() if k.numel() else None, k.numel(), hi_bits, nbits,
-                                      hist.data_ptr(), None, 0, _stream_handle(stream)), "gsh_radix_histogram")
+                                      hist.data_ptr(), None, 0, _stream_handle(stream, k.device)), "gsh_radix_histogram")
     return hist
 
 
@@ -240,7 +246,7 @@ def partition(r_keys, r_payloads, s_keys, s_payloads, config: GshConfig | None =
     bits = (ctypes.c_uint32 * 2)()
     with torch.cuda.device(dev):
         check(lib.gsh_partition(ctypes.byref(R), ctypes.byref(S), ctypes.byref(config) if config is not None else None,
-                                ws.data_ptr(), ws.numel(), _stream_handle(stream), part_r.data_ptr(),
+                                ws.data_ptr(), ws.numel(), _stream_handle(stream, dev), part_r.data_ptr(),
                                 part_s.data_ptr(), off_r.data_ptr(), off_s.data_ptr(), bits), "gsh_partition")
     F = 1 << (bits[0] + bits[1])
     return part_r[: R.n], part_s[: S.n], off_r[: F + 1], off_s[: F + 1], (int(bits[0]), int(bits[1]))
@@ -263,7 +269,7 @@ def detect(r_keys, r_payloads, s_keys, s_payloads, config: GshConfig | None = No
     res = GshResult()
     with torch.cuda.device(dev):
         check(lib.gsh_detect(ctypes.byref(R), ctypes.byref(S), ctypes.byref(config) if config is not None else None,
-                             ws.data_ptr(), ws.numel(), _stream_handle(stream), hk, cr, cs, cap, ctypes.byref(n),
+                             ws.data_ptr(), ws.numel(), _stream_handle(stream, dev), hk, cr, cs, cap, ctypes.byref(n),
                              ctypes.byref(res)), "gsh_detect")
     m = int(n.value)
     h = torch.tensor(list(hk[:m]), dtype=torch.int64)

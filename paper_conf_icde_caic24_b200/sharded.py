@@ -1,252 +1,477 @@
-"""Multi-GPU GSH: hash sharding over one node with torch.distributed (NCCL over NVLink/NVSwitch).
+"""Multi-GPU GSH: hash sharding over one node (a north-star addition --
+the paper runs on one A100).
 
-SURVEY.md §8(e) / row a11 (a north-star addition; the paper runs on one A100):
+One process per GPU (torch.distributed, NCCL over NVLink/NVSwitch), or G logical ranks sharing one
+GPU in one process (`LocalWorld`, the one-GPU test harness of SURVEY §4(i)).  Per rank:
 
-  1. positional shards: rank g holds rows of R and S (any split);
-  2. skew agreement: global partition histogram (all_reduce) -> globally large partitions
-     (the single-GPU rule of PAPER.md L107 on global sizes); each rank proposes the keys of
-     large partitions whose LOCAL count reaches ceil(T_h / G) (pigeonhole: any key with global
-     count >= T_h reaches it on some rank); all_gather + sorted union; exact local counts of the
-     union, all_reduce -> the global skewed set H = {k : max(cnt_R, cnt_S) >= T_h}, identical on
-     every rank and equal to the single-GPU rule on the whole input;
-  3. normal tuples: routed to rank top_log2(G)_bits(fmix32(key)) with all_to_all_single (split
-     sizes exchanged first);
-  4. skewed keys: S_k stays local, R_k is broadcast to every rank, so no GPU receives a skewed
-     key's full S (only |R_k| x |S_k,local| work per rank);
-  5. local GSH join of (received normal R + all skewed R) x (received normal S + local skewed S);
-  6. all_reduce(sum) of (count, checksum) mod 2^64 == the single-GPU result bit-exactly.
+  1. agreement (gsh_shard_*): global partition histogram (all_reduce) -> globally large
+     partitions (L107) -> local candidates with local max(cnt_R, cnt_S) >= ceil(T_h / G)
+     -> all_gather -> union in first-occurrence order + exact local counts -> all_reduce ->
+     skewed keys max(cnt_R, cnt_S) >= T_h (L112): the single-GPU rule on the whole input, the
+     same list on every rank;
+  2. routing (gsh_route_*): a normal tuple goes to rank top_log2(G)_bits(fmix32(key)); a tuple of
+     a skewed key stays on this rank (S) or is broadcast (R), so no GPU receives a skewed key's
+     full S.  The route kernel writes every tuple straight into its final buffer: this rank's own
+     normal tuples into the receive buffer, its skewed R tuples into the all-gathered R_H buffer,
+     the rest into the send buffer of the all-to-all;
+  3. exchange: all_to_all of the normal tuples, all-gather of the skewed R tuples;
+  4. two local GSH joins (gsh_join): the received normal shard (every tuple's top route bits of h
+     equal this rank's id, which gsh_config.route_bits asserts), and all ranks' R_H x local S_H
+     with route_bits = 0 (skewed keys carry arbitrary top bits);
+  5. all_reduce(sum) of (count, checksum) mod 2^64: the single-GPU result bit-exactly.
 
-Every data-path step is a libgsh.so kernel (route_count / route_scatter / count_keys /
-local_candidates / gsh_join); torch.distributed only moves bytes.  The `ops` hook exists so the
-host-side protocol can be exercised on CPU with gloo and a test double (tests/ only).
+Every data-path step is a libgsh.so kernel; PyTorch provides device memory, streams and the
+process group.  `ops` / `comm` are hooks so the host protocol runs on CPU with gloo and an oracle
+test double (tests/ only).
 """
 from __future__ import annotations
 
 import ctypes
-import math
+import threading
+import time
 
 import torch
 import torch.distributed as dist
 
 from . import _lib
-from .join import _check_dev, _rel, _stream_handle, join, make_config
-from ._lib import check, load
+from ._lib import GshShardParams, check, load
+from .join import JoinResult, _check_dev, _rel, _stream_handle, join, make_config
 
 M64 = (1 << 64) - 1
+NVLINK_GBS = 900.0   # NVLink 5 per GPU per direction (B200_PROFILING.md)
 
 
-def _cfg_params(n_global: int, config) -> tuple[int, int, int]:
-    """(B, L, T_h) exactly as plan_build() derives them (api.cu) for n = max side size:
-    radix bits, large-partition threshold, skewed-key threshold."""
-    if config is not None and config.pass_bits[0] >= 0 and config.pass_bits[1] >= 0:
-        B = int(config.pass_bits[0]) + int(config.pass_bits[1])
-    else:
-        B = 0
-        while B < 16 and (n_global >> B) > 2048:
-            B += 1
-    F = 1 << B
-    if config is not None and config.large_threshold:
-        L = int(config.large_threshold)
-    else:
-        mean = float(n_global) / float(F)
-        L = max(64, int(mean + 8.0 * math.sqrt(max(mean, 1.0))) + 1)
-    Th = int(config.heavy_threshold) if (config is not None and config.heavy_threshold) else 64
-    return B, L, Th
+# --------------------------------------------------------------------------- communicators
+class TorchComm:
+    """Collectives of the protocol over a torch.distributed process group (NCCL on GPUs, gloo on
+    CPU).  Integer tensors only; sizes travel as int64 tensors on the data's device."""
+
+    def __init__(self, group=None, device=None):
+        self.group = group
+        self.rank = dist.get_rank(group)
+        self.world = dist.get_world_size(group)
+        self.device = device
+
+    def _src(self, g: int) -> int:
+        return dist.get_global_rank(self.group, g) if self.group is not None else g
+
+    def all_reduce_(self, t: torch.Tensor) -> None:
+        dist.all_reduce(t, group=self.group)
+
+    def all_gather_sizes(self, n: int) -> list[int]:
+        t = torch.tensor([n], dtype=torch.int64, device=self.device)
+        out = [torch.zeros_like(t) for _ in range(self.world)]
+        dist.all_gather(out, t, group=self.group)
+        return [int(x.item()) for x in out]
+
+    def all_gather_pad(self, t: torch.Tensor, m: int) -> torch.Tensor:
+        """[world * m] buffer; rank g's tensor at [g * m, g * m + len)."""
+        out = torch.zeros(self.world * max(m, 1), dtype=t.dtype, device=t.device)
+        pad = torch.zeros(max(m, 1), dtype=t.dtype, device=t.device)
+        pad[: t.numel()] = t
+        dist.all_gather(list(out.view(self.world, -1).unbind(0)), pad, group=self.group)
+        return out
+
+    def all_to_all_v(self, out: torch.Tensor, inp: torch.Tensor, out_splits: list[int], in_splits: list[int]) -> None:
+        if sum(out_splits) == 0 and sum(in_splits) == 0 and self.world == 1:
+            return
+        dist.all_to_all_single(out, inp, out_splits, in_splits, group=self.group)
+
+    def all_gather_v_(self, buf: torch.Tensor, sizes: list[int]) -> None:
+        """In place: rank g's segment [sum(sizes[:g]), +sizes[g]) of `buf` is sent to every rank
+        (this rank's own segment must already be in place)."""
+        off = 0
+        for g, n in enumerate(sizes):
+            if n:
+                dist.broadcast(buf[off: off + n], src=self._src(g), group=self.group)
+            off += n
 
 
+class LocalWorld:
+    """G logical ranks in one process (one host thread each, any device), exchanging through
+    device copies: the one-GPU multi-rank harness.  Every collective is a
+    deposit / barrier / copy / barrier round; each rank synchronises its own stream before it
+    deposits, so peers read finished data."""
+
+    def __init__(self, world: int):
+        self.world = world
+        self.barrier = threading.Barrier(world)
+        self.slots: list = [None] * world
+
+    def comm(self, rank: int) -> "LocalComm":
+        return LocalComm(self, rank)
+
+
+class LocalComm:
+    def __init__(self, w: LocalWorld, rank: int):
+        self.w, self.rank, self.world = w, rank, w.world
+
+    def _round(self, obj, fn):
+        if torch.cuda.is_available():
+            torch.cuda.current_stream().synchronize()
+        self.w.slots[self.rank] = obj
+        self.w.barrier.wait()
+        try:
+            r = fn(list(self.w.slots))
+            if torch.cuda.is_available():
+                torch.cuda.current_stream().synchronize()
+        finally:
+            self.w.barrier.wait()
+        return r
+
+    def all_reduce_(self, t: torch.Tensor) -> None:
+        s = self._round(t, lambda xs: sum(x.clone() for x in xs))
+        t.copy_(s)
+
+    def all_gather_sizes(self, n: int) -> list[int]:
+        return self._round(int(n), lambda xs: list(xs))
+
+    def all_gather_pad(self, t: torch.Tensor, m: int) -> torch.Tensor:
+        out = torch.zeros(self.world * max(m, 1), dtype=t.dtype, device=t.device)
+
+        def fn(xs):
+            for g, x in enumerate(xs):
+                out[g * max(m, 1): g * max(m, 1) + x.numel()].copy_(x)
+        self._round(t, fn)
+        return out
+
+    def all_to_all_v(self, out, inp, out_splits, in_splits) -> None:
+        me = self.rank
+
+        def fn(xs):
+            o = 0
+            for g, (x, isp) in enumerate(xs):
+                n = isp[me]
+                assert n == out_splits[g]
+                if n:
+                    src = sum(isp[:me])
+                    out[o: o + n].copy_(x[src: src + n])
+                o += out_splits[g]
+        self._round((inp, list(in_splits)), fn)
+
+    def all_gather_v_(self, buf, sizes) -> None:
+        me = self.rank
+
+        def fn(xs):
+            off = 0
+            for g, x in enumerate(xs):
+                if g != me and sizes[g]:
+                    buf[off: off + sizes[g]].copy_(x[off: off + sizes[g]])
+                off += sizes[g]
+        self._round(buf, fn)
+
+
+# ------------------------------------------------------------------------------- CUDA ops
 class CudaOps:
-    """The production data path: every call is a libgsh.so kernel launch."""
+    """The production per-rank steps: every call is a libgsh.so entry point (include/gsh.h)."""
 
-    def radix_histogram(self, keys, hi_bits, nbits):
-        from .join import radix_histogram
-        return radix_histogram(keys, hi_bits, nbits)
+    def __init__(self, device: torch.device):
+        self.dev = device
+        self.events: list[tuple[str, torch.cuda.Event]] = []
+        self.launches = 0   # libgsh kernels launched by the protocol steps (the joins report their own)
 
-    def local_candidates(self, rk, rp, sk, sp, part_bits, large_u8, threshold):
+    # plumbing
+    def tensor(self, vals, dtype=torch.int64):
+        return torch.tensor(vals, dtype=dtype, device=self.dev)
+
+    def empty(self, n: int):
+        return torch.empty(max(int(n), 1), dtype=torch.int32, device=self.dev)[: int(n)]
+
+    def stream(self):
+        return _stream_handle(None, self.dev)
+
+    def mark(self, name: str) -> None:
+        e = torch.cuda.Event(enable_timing=True)
+        e.record(torch.cuda.current_stream(self.dev))
+        self.events.append((name, e))
+
+    def phase_ms(self) -> dict:
+        torch.cuda.current_stream(self.dev).synchronize()
+        return {f"ms_{n}": float(a.elapsed_time(b)) for (_, a), (n, b) in zip(self.events, self.events[1:])}
+
+    # steps
+    def histogram(self, rk, sk, P):
+        h = torch.empty(2 << P.part_bits, dtype=torch.int64, device=self.dev)
+        R, S = _rel(rk, rk, "R"), _rel(sk, sk, "S")
+        check(load().gsh_shard_histogram(ctypes.byref(R), ctypes.byref(S), ctypes.byref(P), h.data_ptr(),
+                                         self.stream()), "gsh_shard_histogram")
+        self.launches += (R.n > 0) + (S.n > 0)
+        return h
+
+    def candidates(self, state, rk, rp, sk, sp, P, hist):
         lib = load()
         R, S = _rel(rk, rp, "R"), _rel(sk, sp, "S")
-        nb = lib.gsh_candidates_workspace_bytes(R.n, S.n)
-        ws = torch.empty(int(nb), dtype=torch.uint8, device=rk.device)
-        cap = max(1, (R.n + S.n) // max(threshold, 1) + 1)
-        out = torch.empty(cap, dtype=torch.int32, device=rk.device)
+        nb = int(lib.gsh_shard_workspace_bytes(R.n, S.n))
+        state["cand_ws"] = ws = torch.empty(nb, dtype=torch.uint8, device=self.dev)
+        cap = max(1024, (R.n + S.n) // 64)
+        while True:
+            out = torch.empty(cap, dtype=torch.int32, device=self.dev)
+            n, ovf = ctypes.c_uint64(0), ctypes.c_uint32(0)
+            st = lib.gsh_shard_candidates(ctypes.byref(R), ctypes.byref(S), ctypes.byref(P), hist.data_ptr(),
+                                          ws.data_ptr(), ws.numel(), self.stream(), out.data_ptr(), cap,
+                                          ctypes.byref(n), ctypes.byref(ovf))
+            if st == _lib.GSH_ERR_INVALID and n.value > cap:
+                cap = int(n.value)
+                continue
+            check(st, "gsh_shard_candidates")
+            self.launches += 2 + (R.n > 0) + (S.n > 0)
+            return out[: n.value], bool(ovf.value)
+
+    def agree(self, state, gathered, sizes, stride):
+        lib = load()
+        G = len(sizes)
+        ws = torch.empty(int(lib.gsh_shard_agree_workspace_bytes(G * max(stride, 1))), dtype=torch.uint8,
+                         device=self.dev)
+        state["agree_ws"] = ws
+        cap = max(1, sum(sizes))
+        uni = torch.empty(cap, dtype=torch.int32, device=self.dev)
+        cnt = torch.zeros(2 * cap, dtype=torch.int64, device=self.dev)
+        hs = (ctypes.c_uint64 * G)(*sizes)
         n = ctypes.c_uint64(0)
-        check(lib.gsh_local_candidates(ctypes.byref(R), ctypes.byref(S), 0, part_bits, large_u8.data_ptr(), threshold,
-                                       ws.data_ptr(), ws.numel(), _stream_handle(None), out.data_ptr(), cap,
-                                       ctypes.byref(n)), "gsh_local_candidates")
-        return out[: n.value].to(torch.int64) & 0xFFFFFFFF
+        cw = state["cand_ws"]
+        check(lib.gsh_shard_agree(cw.data_ptr(), cw.numel(), gathered.data_ptr(), G, max(stride, 1), hs,
+                                  ws.data_ptr(), ws.numel(), self.stream(), uni.data_ptr(), cnt.data_ptr(), cap,
+                                  ctypes.byref(n)), "gsh_shard_agree")
+        m = int(n.value)
+        self.launches += 5 if sum(sizes) else 0
+        return uni[:m], cnt[: 2 * m]
 
-    def count_keys(self, keys, q_sorted_i32):
+    def select(self, state, uni, cnt, P):
         lib = load()
-        counts = torch.zeros(q_sorted_i32.numel(), dtype=torch.int64, device=keys.device)
-        if keys.numel() and q_sorted_i32.numel():
-            check(lib.gsh_count_keys(keys.data_ptr(), keys.numel(), q_sorted_i32.data_ptr(), q_sorted_i32.numel(),
-                                     counts.data_ptr(), _stream_handle(None)), "gsh_count_keys")
-        return counts
+        m = uni.numel()
+        heavy = torch.empty(max(m, 1), dtype=torch.int32, device=self.dev)
+        n = ctypes.c_uint64(0)
+        ws = state.get("agree_ws")
+        check(lib.gsh_shard_select(uni.data_ptr() if m else None, cnt.data_ptr() if m else None, m, ctypes.byref(P),
+                                   ws.data_ptr() if ws is not None else None, ws.numel() if ws is not None else 0,
+                                   self.stream(), heavy.data_ptr(), m, ctypes.byref(n)), "gsh_shard_select")
+        nh = int(n.value)
+        self.launches += (4 if m else 0) + (1 if nh else 0)
+        heavy = heavy[:nh]
+        sb = int(lib.gsh_heavy_set_bytes(nh))
+        state["set"] = hset = torch.empty(max(sb, 256), dtype=torch.uint8, device=self.dev)
+        state["set_bytes"] = sb
+        check(lib.gsh_heavy_set_build(heavy.data_ptr() if nh else None, nh, hset.data_ptr(), sb, self.stream()),
+              "gsh_heavy_set_build")
+        return heavy
 
-    def route(self, keys, pays, route_bits, heavy_sorted_i32):
-        lib = load()
-        G = 1 << route_bits
-        dev = keys.device
-        counts = torch.zeros(G + 1, dtype=torch.int64, device=dev)
-        hp = heavy_sorted_i32.data_ptr() if heavy_sorted_i32.numel() else None
-        check(lib.gsh_route_count(keys.data_ptr() if keys.numel() else None, keys.numel(), route_bits, hp,
-                                  heavy_sorted_i32.numel(), counts.data_ptr(), _stream_handle(None)), "route_count")
-        host_counts = counts.cpu().tolist()
-        offs = [0]
-        for c in host_counts:
-            offs.append(offs[-1] + c)
-        off_t = torch.tensor(offs, dtype=torch.int64, device=dev)
-        cur = torch.zeros(G + 1, dtype=torch.int64, device=dev)
-        ok = torch.empty(max(keys.numel(), 1), dtype=torch.int32, device=dev)
-        op = torch.empty(max(keys.numel(), 1), dtype=torch.int32, device=dev)
-        if keys.numel():
-            check(lib.gsh_route_scatter(keys.data_ptr(), pays.data_ptr(), keys.numel(), route_bits, hp,
-                                        heavy_sorted_i32.numel(), off_t.data_ptr(), cur.data_ptr(), ok.data_ptr(),
-                                        op.data_ptr(), _stream_handle(None)), "route_scatter")
-        return ok[: keys.numel()], op[: keys.numel()], host_counts
+    def route_count(self, state, keys, rb):
+        G1 = (1 << rb) + 1
+        c = torch.empty(G1, dtype=torch.int64, device=self.dev)
+        check(load().gsh_route_count(keys.data_ptr() if keys.numel() else None, keys.numel(), rb,
+                                     state["set"].data_ptr() if state["set_bytes"] else None, state["set_bytes"],
+                                     c.data_ptr(), self.stream()), "gsh_route_count")
+        self.launches += keys.numel() > 0
+        return [int(x) for x in c.cpu().tolist()]
 
-    def join(self, rk, rp, sk, sp, config):
-        r = join(rk, rp, sk, sp, config=config)
-        return r.count, r.checksum, r.stats
+    def route_scatter(self, state, keys, pays, rb, dst):
+        """dst[d] = (keys_tensor, pays_tensor, offset): destination d's run starts at offset."""
+        if keys.numel() == 0:
+            return
+        ptrs = []
+        for k, p, off in dst:
+            ptrs += [k.data_ptr() + 4 * off if k.numel() else 0, p.data_ptr() + 4 * off if p.numel() else 0]
+        d_dst = self.tensor([x - (1 << 64) if x >= (1 << 63) else x for x in ptrs])
+        cur = torch.empty(len(dst), dtype=torch.int64, device=self.dev)
+        check(load().gsh_route_scatter(keys.data_ptr(), pays.data_ptr(), keys.numel(), rb,
+                                       state["set"].data_ptr() if state["set_bytes"] else None, state["set_bytes"],
+                                       d_dst.data_ptr(), cur.data_ptr(), self.stream()), "gsh_route_scatter")
+        state.setdefault("keep", []).append(d_dst)
+        self.launches += 1
 
-
-def _to_i32_sorted(h64: torch.Tensor) -> torch.Tensor:
-    """u32 values held in int64, sorted ascending -> same bit patterns as int32 (kernels compare
-    as unsigned)."""
-    h = torch.sort(h64).values
-    return torch.where(h >= (1 << 31), h - (1 << 32), h).to(torch.int32)
-
-
-def _allgather_var(t: torch.Tensor, group) -> torch.Tensor:
-    """all_gather of a variable-length 1-D int64 tensor -> concatenation over ranks."""
-    G = dist.get_world_size(group)
-    n = torch.tensor([t.numel()], dtype=torch.int64, device=t.device)
-    sizes = [torch.zeros_like(n) for _ in range(G)]
-    dist.all_gather(sizes, n, group=group)
-    sizes = [int(s.item()) for s in sizes]
-    m = max(sizes) if sizes else 0
-    pad = torch.zeros(max(m, 1), dtype=t.dtype, device=t.device)
-    pad[: t.numel()] = t
-    bufs = [torch.empty_like(pad) for _ in range(G)]
-    dist.all_gather(bufs, pad, group=group)
-    return torch.cat([b[:s] for b, s in zip(bufs, sizes)])
+    def join(self, rk, rp, sk, sp, config, out=None):
+        mode = "materialize" if out is not None else "count"
+        r = join(rk, rp, sk, sp, mode=mode, out=out, config=config)
+        self.launches += r.stats.get("launches", 0)
+        return r.count, r.checksum, r.written, r.stats
 
 
-def agree_heavy(rk, rp, sk, sp, config=None, group=None, ops=None):
-    """Steps 1-2: the globally agreed skewed-key set (sorted hashes as int32) + global parameters."""
-    ops = ops or CudaOps()
-    dev = rk.device
-    n = torch.tensor([rk.numel(), sk.numel()], dtype=torch.int64, device=dev)
-    dist.all_reduce(n, group=group)
-    n_r, n_s = int(n[0]), int(n[1])
-    B, L, Th = _cfg_params(max(n_r, n_s), config)
-    hr = ops.radix_histogram(rk, 0, B)
-    hs = ops.radix_histogram(sk, 0, B)
-    h = torch.stack([hr, hs])
-    dist.all_reduce(h, group=group)
-    large = ((h[0] > L) | (h[1] > L)) & (h[0] > 0) & (h[1] > 0)
-    if config is not None and config.force_all_normal:
-        large[:] = False
-    G = dist.get_world_size(group)
-    empty = torch.zeros(0, dtype=torch.int32, device=dev)
-    if not bool(large.any()):
-        return empty, (B, L, Th, n_r, n_s)
-    tau = max(1, -(-Th // G))
-    cand = ops.local_candidates(rk, rp, sk, sp, B, large.to(torch.uint8), tau)
-    allc = _allgather_var(cand, group)
-    q = torch.unique(allc)  # sorted int64 u32 values
-    if q.numel() == 0:
-        return empty, (B, L, Th, n_r, n_s)
-    q32 = _to_i32_sorted(q)
-    cnt = torch.stack([ops.count_keys(rk, q32), ops.count_keys(sk, q32)])
-    dist.all_reduce(cnt, group=group)
-    heavy = q[torch.maximum(cnt[0], cnt[1]) >= Th]
-    return _to_i32_sorted(heavy), (B, L, Th, n_r, n_s)
+# ------------------------------------------------------------------------------- protocol
+def shard_plan(n_r: int, n_s: int, world: int, config=None) -> GshShardParams:
+    """gsh_shard_plan: the single-GPU rule's (B, L, T_h) for the global sizes + tau (host-only)."""
+    P = GshShardParams()
+    check(load().gsh_shard_plan(n_r, n_s, world, ctypes.byref(config) if config is not None else None,
+                                ctypes.byref(P)), "gsh_shard_plan")
+    return P
 
 
-def _exchange_normal(keys, pays, counts, G, group):
-    """all_to_all of the destination-grouped normal tuples (first G groups)."""
-    dev = keys.device
-    send = torch.tensor(counts[:G], dtype=torch.int64, device=dev)
-    recv = torch.empty_like(send)
-    dist.all_to_all_single(recv, send, group=group)
-    in_splits = [int(c) for c in counts[:G]]
-    out_splits = [int(c) for c in recv.cpu().tolist()]
-    tot_in = sum(in_splits)
-    tot_out = sum(out_splits)
-    ok = torch.empty(tot_out, dtype=torch.int32, device=dev)
-    op = torch.empty(tot_out, dtype=torch.int32, device=dev)
-    dist.all_to_all_single(ok, keys[:tot_in].contiguous(), out_splits, in_splits, group=group)
-    dist.all_to_all_single(op, pays[:tot_in].contiguous(), out_splits, in_splits, group=group)
-    return ok, op
+def _copy_cfg(c, **kw):
+    n = _lib.GshConfig()
+    if c is None:
+        n = make_config()
+    else:
+        ctypes.memmove(ctypes.byref(n), ctypes.byref(c), ctypes.sizeof(c))
+    for k, v in kw.items():
+        setattr(n, k, v)
+    return n
 
 
-def _broadcast_heavy_r(hk, hp, group):
-    """Every rank receives every rank's skewed R tuples (exact-size broadcasts, no padding)."""
-    G = dist.get_world_size(group)
-    dev = hk.device
-    n = torch.tensor([hk.numel()], dtype=torch.int64, device=dev)
-    sizes = [torch.zeros_like(n) for _ in range(G)]
-    dist.all_gather(sizes, n, group=group)
-    sizes = [int(s.item()) for s in sizes]
-    me = dist.get_rank(group)
-    tot = sum(sizes)
-    ok = torch.empty(tot, dtype=torch.int32, device=dev)
-    op = torch.empty(tot, dtype=torch.int32, device=dev)
-    off = 0
-    for g, s in enumerate(sizes):
-        if s:
-            if g == me:
-                ok[off: off + s].copy_(hk)
-                op[off: off + s].copy_(hp)
-            src = dist.get_global_rank(group, g) if group is not None else g
-            dist.broadcast(ok[off: off + s], src=src, group=group)
-            dist.broadcast(op[off: off + s], src=src, group=group)
-        off += s
-    return ok, op
+def _s64(x: int) -> int:
+    x &= M64
+    return x - (1 << 64) if x >= (1 << 63) else x
 
 
-def join_sharded(rk, rp, sk, sp, config=None, group=None, ops=None):
-    """Hash-sharded GSH join of this rank's shards; returns a JoinResult-like object whose
-    count/checksum are GLOBAL (identical on all ranks)."""
-    from .join import JoinResult
-    ops = ops or CudaOps()
-    if isinstance(ops, CudaOps):
+def agree_heavy(rk, rp, sk, sp, P, comm, ops, state):
+    """Step 1: the globally agreed skewed keys (int32 h values, identical list on every rank)."""
+    hist = ops.histogram(rk, sk, P)
+    comm.all_reduce_(hist)
+    cand, cand_ovf = ops.candidates(state, rk, rp, sk, sp, P, hist)
+    sizes = comm.all_gather_sizes(cand.numel())
+    stride = max(sizes) if sizes else 0
+    state["cand_overflow"] = cand_ovf
+    state["n_cand"] = sum(sizes)
+    if stride == 0:
+        return ops.select(state, cand[:0], ops.tensor([], dtype=torch.int64), P)
+    gathered = comm.all_gather_pad(cand, stride)
+    uni, cnt = ops.agree(state, gathered, sizes, stride)
+    comm.all_reduce_(cnt)
+    state["n_union"] = uni.numel()
+    return ops.select(state, uni, cnt, P)
+
+
+def join_sharded(rk, rp, sk, sp, config=None, group=None, ops=None, comm=None, mode: str = "count", out=None):
+    """Hash-sharded GSH join of this rank's shards (any positional split of R and S over the ranks).
+
+    Returns a JoinResult whose count / checksum are GLOBAL (identical on all ranks); in
+    "materialize" mode `out` ((capacity, 2) int32 CUDA tensor) receives this rank's pairs and
+    `written` counts them.  stats: per-phase ms, exchanged bytes and their NVLink fraction."""
+    if ops is None:
         rk, rp = _check_dev(rk, "r_keys"), _check_dev(rp, "r_payloads")
         sk, sp = _check_dev(sk, "s_keys"), _check_dev(sp, "s_payloads")
-    G = dist.get_world_size(group)
+        ops = CudaOps(rk.device)
+    if comm is None:
+        comm = TorchComm(group, rk.device)
+    G, me = comm.world, comm.rank
     if G & (G - 1):
         raise ValueError("world size must be a power of two (route bits)")
-    rb = G.bit_length() - 1
-    heavy, (B, L, Th, n_r, n_s) = agree_heavy(rk, rp, sk, sp, config, group, ops)
-    rks, rps, rc = ops.route(rk, rp, rb, heavy)
-    sks, sps, sc = ops.route(sk, sp, rb, heavy)
-    rk_n, rp_n = _exchange_normal(rks, rps, rc, G, group)
-    sk_n, sp_n = _exchange_normal(sks, sps, sc, G, group)
-    nr_h = rc[G]
-    ns_h = sc[G]
-    r_off = sum(rc[:G])
-    s_off = sum(sc[:G])
-    rk_h, rp_h = _broadcast_heavy_r(rks[r_off: r_off + nr_h], rps[r_off: r_off + nr_h], group)
-    # local inputs: normal received + skewed (R: all ranks', S: local)
-    lrk = torch.cat([rk_n, rk_h])
-    lrp = torch.cat([rp_n, rp_h])
-    lsk = torch.cat([sk_n, sks[s_off: s_off + ns_h]])
-    lsp = torch.cat([sp_n, sps[s_off: s_off + ns_h]])
-    lcfg = make_config() if config is None else _copy_cfg(config)
-    lcfg.route_bits = rb
-    cnt, chk, stats = ops.join(lrk, lrp, lsk, lsp, lcfg)
-    dev = rk.device
-    t = torch.tensor([cnt, chk - (1 << 64) if chk >= (1 << 63) else chk], dtype=torch.int64, device=dev)
-    dist.all_reduce(t, group=group)
-    gc = int(t[0]) & M64
-    gk = int(t[1]) & M64
-    stats = dict(stats)
-    stats.update({"n_heavy_global": int(heavy.numel()), "local_r": int(lrk.numel()), "local_s": int(lsk.numel()),
-                  "heavy_r_recv": int(rk_h.numel()), "route_bits": rb})
-    return JoinResult(count=gc, checksum=gk, stats=stats)
+    if mode not in ("count", "materialize"):
+        raise ValueError("mode must be 'count' or 'materialize'")
+    state: dict = {}
+    ops.mark("start")
+    n = ops.tensor([rk.numel(), sk.numel()])
+    comm.all_reduce_(n)
+    n_r, n_s = (int(x) for x in n.tolist())
+    P = shard_plan(n_r, n_s, G, config)
+    rb = int(P.route_bits)
+    heavy = agree_heavy(rk, rp, sk, sp, P, comm, ops, state)
+    ops.mark("agree")
+
+    # routing plan: destination counts, then every buffer laid out so the route kernel writes
+    # each tuple to its final place
+    rc = ops.route_count(state, rk, rb)
+    sc = ops.route_count(state, sk, rb)
+    send = ops.tensor([[rc[d], sc[d]] for d in range(G)]).reshape(-1)
+    recv = ops.tensor([0] * (2 * G))
+    comm.all_to_all_v(recv, send, [2] * G, [2] * G)
+    recv = recv.reshape(G, 2).tolist()
+    rh_sizes = comm.all_gather_sizes(rc[G])
+    rr = [int(recv[g][0]) if g != me else 0 for g in range(G)]   # from other ranks
+    rs = [int(recv[g][1]) if g != me else 0 for g in range(G)]
+    rsend = [rc[d] if d != me else 0 for d in range(G)]
+    ssend = [sc[d] if d != me else 0 for d in range(G)]
+    nr_other, ns_other = sum(rr), sum(rs)
+    Rn = (ops.empty(nr_other + rc[me]), ops.empty(nr_other + rc[me]))    # normal R: [others | own]
+    Sn = (ops.empty(ns_other + sc[me]), ops.empty(ns_other + sc[me]))
+    Rh = (ops.empty(sum(rh_sizes)), ops.empty(sum(rh_sizes)))            # skewed R of every rank
+    Sh = (ops.empty(sc[G]), ops.empty(sc[G]))                            # local skewed S
+    Rx = (ops.empty(sum(rsend)), ops.empty(sum(rsend)))                  # send buffers
+    Sx = (ops.empty(sum(ssend)), ops.empty(sum(ssend)))
+
+    def dst_list(own, own_off, x, xsend, heavy_buf, heavy_off):
+        d, off = [], 0
+        for g in range(G):
+            if g == me:
+                d.append((own[0], own[1], own_off))
+            else:
+                d.append((x[0], x[1], off))
+                off += xsend[g]
+        d.append((heavy_buf[0], heavy_buf[1], heavy_off))
+        return d
+
+    ops.route_scatter(state, rk, rp, rb, dst_list(Rn, nr_other, Rx, rsend, Rh, sum(rh_sizes[:me])))
+    ops.route_scatter(state, sk, sp, rb, dst_list(Sn, ns_other, Sx, ssend, Sh, 0))
+    ops.mark("route")
+    for i in range(2):
+        comm.all_to_all_v(Rn[i][:nr_other], Rx[i], rr, rsend)
+        comm.all_to_all_v(Sn[i][:ns_other], Sx[i], rs, ssend)
+    ops.mark("exchange")
+    for i in range(2):
+        comm.all_gather_v_(Rh[i], rh_sizes)
+    ops.mark("broadcast")
+
+    # local joins: the routed normal shard under route_bits = rb, the skewed keys under 0
+    cfg_n = _copy_cfg(config, route_bits=rb, timing=1)
+    cfg_h = _copy_cfg(config, route_bits=0, timing=1)
+    mat = mode == "materialize"
+    o1 = out if mat else None
+    c1, k1, w1, st1 = ops.join(Rn[0], Rn[1], Sn[0], Sn[1], cfg_n, o1)
+    ops.mark("join_normal")
+    o2 = out[w1:] if mat else None
+    if Rh[0].numel() and Sh[0].numel():
+        c2, k2, w2, st2 = ops.join(Rh[0], Rh[1], Sh[0], Sh[1], cfg_h, o2)
+    else:
+        c2, k2, w2, st2 = 0, 0, 0, {}
+    ops.mark("join_heavy")
+    t = ops.tensor([_s64(c1 + c2), _s64(k1 + k2)])
+    comm.all_reduce_(t)
+    gc, gk = (int(x) & M64 for x in t.tolist())
+    ops.mark("reduce")
+    phases = ops.phase_ms()
+    xbytes = 8 * (sum(rsend) + sum(ssend))
+    bbytes = 8 * (sum(rh_sizes) - rh_sizes[me])
+    stats = {
+        "world": G, "rank": me, "route_bits": rb, "part_bits": int(P.part_bits),
+        "large_threshold": int(P.large_threshold), "heavy_threshold": int(P.heavy_threshold),
+        "cand_threshold": int(P.cand_threshold), "n_heavy_global": int(heavy.numel()),
+        "n_candidates_gathered": state.get("n_cand", 0), "n_union": state.get("n_union", 0),
+        "candidate_table_overflow": bool(state.get("cand_overflow", False)),
+        "local_r": rk.numel(), "local_s": sk.numel(),
+        "normal_r": Rn[0].numel(), "normal_s": Sn[0].numel(), "heavy_r": Rh[0].numel(), "heavy_s": Sh[0].numel(),
+        "exchange_send_bytes": xbytes, "broadcast_recv_bytes": bbytes,
+        "count_normal": c1, "count_heavy": c2, "written": w1 + w2,
+        "join_normal": st1, "join_heavy": st2, "launches": getattr(ops, "launches", 0),
+    }
+    stats.update(phases)
+    for name, nbytes in (("exchange", xbytes), ("broadcast", bbytes)):
+        ms = phases.get(f"ms_{name}", 0.0)
+        gbs = nbytes / (ms * 1e6) if ms > 0 else None
+        stats[f"{name}_GBps"] = gbs
+        stats[f"{name}_nvlink_frac"] = gbs / NVLINK_GBS if gbs is not None else None
+    return JoinResult(count=gc, checksum=gk, written=w1 + w2, overflow=bool(st1.get("overflow", 0) or
+                                                                            st2.get("overflow", 0)),
+                      pairs=(out[: w1 + w2] if mat else None), stats=stats)
 
 
-def _copy_cfg(c):
-    n = _lib.GshConfig()
-    ctypes.memmove(ctypes.byref(n), ctypes.byref(c), ctypes.sizeof(c))
-    return n
+def run_local(world: int, shards, config=None, mode: str = "count", out_capacity: int = 0, device=None):
+    """Run join_sharded for `world` logical ranks on ONE device (threads + LocalWorld): the
+    one-GPU multi-rank harness.  shards[g] = (rk, rp, sk, sp) CUDA tensors of rank g.  Returns the
+    per-rank JoinResults (rank order)."""
+    lw = LocalWorld(world)
+    dev = torch.device(device) if device is not None else shards[0][0].device
+    res: list = [None] * world
+    err: list = []
+
+    def worker(g):
+        try:
+            with torch.cuda.device(dev):
+                s = torch.cuda.Stream(dev)
+                with torch.cuda.stream(s):
+                    out = (torch.empty((out_capacity, 2), dtype=torch.int32, device=dev)
+                           if mode == "materialize" else None)
+                    res[g] = join_sharded(*shards[g], config=config, comm=lw.comm(g), mode=mode, out=out)
+                s.synchronize()
+        except BaseException as e:  # surface the first failure, release the other ranks
+            err.append(e)
+            lw.barrier.abort()
+
+    th = [threading.Thread(target=worker, args=(g,)) for g in range(world)]
+    t0 = time.perf_counter()
+    for t in th:
+        t.start()
+    for t in th:
+        t.join()
+    if err:
+        raise err[0]
+    for r in res:
+        r.stats["wall_s"] = time.perf_counter() - t0
+    return res

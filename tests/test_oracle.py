@@ -329,10 +329,29 @@ def test_heavy_rule_bruteforce():
         expect = []
         for x in set(cntr) | set(cnts):
             p = part(x)
-            if szr.get(p, 0) > cap or szs.get(p, 0) > cap:
+            if (szr.get(p, 0) > cap or szs.get(p, 0) > cap) and szr.get(p, 0) > 0 and szs.get(p, 0) > 0:
                 if max(cntr.get(x, 0), cnts.get(x, 0)) >= thr:
                     h = int(oracle.fmix32(np.array([x], np.uint32))[0])
                     expect.append((h, cntr.get(x, 0), cnts.get(x, 0)))
         expect.sort()
         got = list(zip(hk.tolist(), cr.tolist(), cs.tolist()))
         assert got == expect
+
+
+def test_heavy_rule_empty_side_partition():
+    """DESIGN.md R5: a partition holding many R tuples but no S tuple is not large (it yields no
+    result tuple), so its keys are never skewed; the same key with one matching S tuple is."""
+    pb = 4
+    part = lambda a: (oracle.fmix32(np.asarray(a, np.uint32)) >> np.uint32(32 - pb)).astype(np.int64)  # noqa: E731
+    cand = np.arange(1, 5000, dtype=np.uint32)
+    pc = part(cand)
+    k_big = int(cand[0])
+    others = cand[pc != pc[0]][:200]          # S keys from other partitions only
+    rk = np.concatenate([np.full(500, k_big), others]).astype(np.uint32)
+    sk = others.copy()
+    hk, _, _ = oracle.heavy_rule(rk, sk, pb, 100, 50)
+    assert k_big not in set(oracle.fmix32(np.asarray(hk, np.uint32)).tolist()) and hk.size == 0
+    sk2 = np.concatenate([sk, [k_big]]).astype(np.uint32)   # one S tuple: the partition becomes large
+    hk2, cr2, cs2 = oracle.heavy_rule(rk, sk2, pb, 100, 50)
+    h_big = int(oracle.fmix32(np.array([k_big], np.uint32))[0])
+    assert hk2.tolist() == [h_big] and cr2.tolist() == [500] and cs2.tolist() == [1]
