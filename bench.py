@@ -32,7 +32,7 @@ import torch  # noqa: E402
 MEASURED_PEAKS = os.path.join(ROOT, "MEASURED_PEAKS.json")
 PROFILE_SUMMARY = os.path.join(ROOT, "profiles", "ncu_traffic.json")
 FALLBACK_HBM_GBS = 6650.0  # /opt/skills/guides/B200_PROFILING.md fallback
-DEVSTATE_BYTES = 152        # sizeof(gsh::DevState): D2H'd twice per step (classify + final)
+DEVSTATE_BYTES = 168        # sizeof(gsh::DevState): D2H'd twice per step (classify + final)
 
 WORKLOADS = {
     # name: (kind, n per side (per rank), theta, description)
@@ -40,6 +40,8 @@ WORKLOADS = {
     "cfg1": ("zipf", 1 << 20, 1.0, "cfg1: |R|=|S|=2^20 Zipf theta=1.0 both sides, COUNT"),
     "zipf05": ("zipf", 1 << 27, 0.5, "cfg3 point: |R|=|S|=2^27 Zipf theta=0.5 both sides, COUNT"),
     "zipf075": ("zipf", 1 << 27, 0.75, "cfg3 point: |R|=|S|=2^27 Zipf theta=0.75 both sides, COUNT"),
+    "zipf10": ("zipf", 1 << 27, 1.0, "cfg3 point: |R|=|S|=2^27 Zipf theta=1.0 both sides (use --input-side), COUNT"),
+    "zipf15": ("zipf", 1 << 27, 1.5, "cfg3 point: |R|=|S|=2^27 Zipf theta=1.5 both sides (use --input-side), COUNT"),
     "zipf10s": ("zipf", 1 << 24, 1.0, "cfg3-shaped (scaled): |R|=|S|=2^24 Zipf theta=1.0 both sides, COUNT"),
     "zipf15s": ("zipf", 1 << 22, 1.5, "cfg3-shaped (scaled): |R|=|S|=2^22 Zipf theta=1.5 both sides, COUNT"),
     "graph": ("graph", 1 << 26, 0.909, "cfg4-shaped (scaled): 2^26-edge power-law graph self-join (dst, src), COUNT"),
@@ -64,6 +66,9 @@ def parse():
     ap.add_argument("--out-cap", type=int, default=1 << 30, help="MATERIALIZE output capacity (pairs)")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-sweep", action="store_true", help="skip the theta_sweep sub-object (N=1 only)")
+    ap.add_argument("--input-side", action="store_true",
+                    help="time only the input side (partition, detect, split): gsh_config.input_side_only")
     ap.add_argument("--fake-ranks", type=int, default=0,
                     help="run the sharded step for G logical ranks on one GPU (code-path check, not a headline)")
     return ap.parse_args()
@@ -257,6 +262,68 @@ def run_reference(args, rank, world):
         "output_tuples_per_step": cnt}))
 
 
+def pass_fractions(ph, st, n_tot):
+    """HBM fraction of every input-side pass (algorithmic bytes) of one join."""
+    peak, _ = hbm_peak()
+    large = st.get("large_tuples", None)
+    out = {}
+    for k, b in (("ms_hist", 4 * n_tot), ("ms_pass1", 16 * n_tot), ("ms_pass2", 16 * n_tot)):
+        ms = ph.get(k) or 0.0
+        out[k.replace("ms_", "") + "_frac"] = (b / (ms * 1e6)) / peak if ms > 0 else None
+    if large:
+        for k, b in (("ms_detect", 8 * large), ("ms_split", 16 * large)):
+            ms = ph.get(k) or 0.0
+            out[k.replace("ms_", "") + "_frac"] = (b / (ms * 1e6)) / peak if ms > 0 else None
+    return out
+
+
+SWEEP = [  # (theta, n per side, input side only): BASELINE configs[2] points at full size
+    (0.5, 1 << 27, False), (0.75, 1 << 27, False), (1.0, 1 << 27, True), (1.5, 1 << 27, True)]
+DENSE = [(1.0, 1 << 24), (1.5, 1 << 22)]   # skewed-key phase at the largest sizes that finish in ~1-2 s
+
+
+def theta_sweep(gsh, dev, seed, steps=3):
+    """configs[2]: |R|=|S|=2^27 both-sides Zipf at theta in {0.5, 0.75, 1.0, 1.5}: per-phase ms and the
+    HBM fraction of every input-side pass (theta >= 1.0: input side only -- the output is 8e13 to
+    3e15 pairs), plus the skewed-key phase's pairs/s at the largest sizes that finish in seconds."""
+    import datagen
+    out = {"points": [], "dense": []}
+    for theta, n, inp in SWEEP:
+        rk, rp, sk, sp = datagen.make_workload("zipf", n, theta, seed=seed, device=dev)
+        cfg = gsh.make_config(timing=True, input_side_only=inp)
+        ws = torch.empty(gsh.workspace_bytes(n, n, cfg), dtype=torch.uint8, device=dev)
+        r = gsh.join(rk, rp, sk, sp, config=cfg, workspace=ws)
+        ph = {}
+        for _ in range(steps):
+            r = gsh.join(rk, rp, sk, sp, config=cfg, workspace=ws)
+            for k, v in r.stats.items():
+                if k.startswith("ms_"):
+                    ph[k] = ph.get(k, 0.0) + v / steps
+        st = dict(r.stats)
+        pt = {"theta": theta, "n_per_side": n, "input_side_only": inp, "phases_ms": ph,
+              "n_large": st["n_large"], "n_heavy": st["n_heavy"],
+              "heavy_tuples": st["heavy_tuples_r"] + st["heavy_tuples_s"], "skew_pairs": st["skew_pairs"]}
+        pt.update(pass_fractions(ph, st, 2 * n))
+        if not inp:
+            pt["count"] = r.count
+            pt["input_tuples_per_s"] = 2 * n / (ph["ms_total"] / 1e3)
+            pt["output_tuples_per_s"] = r.count / (ph["ms_total"] / 1e3)
+        out["points"].append(pt)
+        del rk, rp, sk, sp, ws
+    for theta, n in DENSE:
+        rk, rp, sk, sp = datagen.make_workload("zipf", n, theta, seed=seed, device=dev)
+        cfg = gsh.make_config(timing=True)
+        r = gsh.join(rk, rp, sk, sp, config=cfg)
+        st = r.stats
+        out["dense"].append({"theta": theta, "n_per_side": n, "count": r.count, "ms_total": st["ms_total"],
+                             "ms_skewjoin": st["ms_skewjoin"], "skew_pairs": st["skew_pairs"],
+                             "skew_pairs_per_s": st["skew_pairs"] / (st["ms_skewjoin"] / 1e3),
+                             "output_tuples_per_s": r.count / (st["ms_total"] / 1e3)})
+        del rk, rp, sk, sp
+    torch.cuda.empty_cache()
+    return out
+
+
 def flatten(r, world):
     """(phases_ms, launches, join stats) of one step's result: the single-GPU gsh_join stats, or for
     the sharded step its protocol phases plus the routed normal shard's per-kernel phases."""
@@ -352,6 +419,8 @@ def main():
         extra["detect_mode"] = 1
     # per-phase CUDA events stay on inside the timed region (the roofline's kernel time is
     # measured live there); they cost ~30 us of host time per call, included in the step time
+    if args.input_side:
+        extra["input_side_only"] = True
     cfg = gsh.make_config(timing=True, **extra)
     fake = args.fake_ranks if world == 1 else 0   # 1 = the sharded protocol with one rank
     if fake >= 1:
@@ -456,6 +525,13 @@ def main():
                "d2h_bytes_per_step": d2h, "steps": ke, "ms_per_step": ems / ke, "api": api}
         del hk
 
+    sweep = None
+    if world == 1 and not fake and not args.no_sweep and args.workload == "cfg2" and args.mode == "count":
+        del rk, rp, sk, sp, ws
+        torch.cuda.empty_cache()
+        sweep = theta_sweep(gsh, dev, args.seed)
+        rk, rp, sk, sp = make_data(kind, n, theta, args.seed, dev, rank)
+
     base = None
     if rank == 0 and world == 1 and not fake and not args.no_cpu_baseline:
         base = cpu_baseline(kind, n, theta, args.seed, rk, rp, sk, sp, r)
@@ -479,6 +555,9 @@ def main():
         }
         if multi:
             line["sharded"] = sharded_summary(phases, r.stats, fake or world)
+        if sweep is not None:
+            line["theta_sweep"] = sweep
+        line["pass_fractions"] = pass_fractions(phases, jst, n_tot)
         print(json.dumps(line))
     if dist:
         dist.destroy_process_group()

@@ -114,6 +114,10 @@ typedef struct {
                                   (L106).  0 = auto (enough bits that each side's share is
                                   <= 2^28 tuples; none up to 2^28);  -1 = off;  1..8 = forced.
                                   The result never depends on it. */
+    int32_t input_side_only;   /* measurement hook: run the input side (partition, classify,
+                                  detect, split) and stop before the NM-join and the skewed-key
+                                  join; count / checksum / written are then 0.  Used to time the
+                                  partition passes on inputs whose output takes minutes. */
 } gsh_config;
 
 /* Per-call result (host struct). */
@@ -139,6 +143,7 @@ typedef struct {
     float ms_hist, ms_pass1, ms_pass2, ms_detect, ms_split, ms_nmjoin, ms_skewjoin, ms_total;
     uint32_t prepass_bits;     /* pre-partition bits actually used (0 = none) */
     float ms_prepass;          /* pre-partition pass (count + scatter), included in ms_total */
+    uint64_t large_tuples;     /* R + S tuples in large partitions (read by detect and split) */
 } gsh_result;
 
 /* Fill *cfg with defaults (all auto, no hooks, timing off). */

@@ -48,6 +48,7 @@ class GshConfig(ctypes.Structure):
         ("sample_stride", u32),
         ("top_k", u32),
         ("prepass_bits", i32),
+        ("input_side_only", i32),
     ]
 
 
@@ -81,6 +82,7 @@ class GshResult(ctypes.Structure):
         ("ms_total", ctypes.c_float),
         ("prepass_bits", u32),
         ("ms_prepass", ctypes.c_float),
+        ("large_tuples", u64),
     ]
 
     def as_dict(self) -> dict:

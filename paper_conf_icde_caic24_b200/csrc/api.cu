@@ -120,6 +120,7 @@ bool plan_build(Plan& p, uint64_t nR, uint64_t nS, const gsh_config* cfg_in, voi
         p.L = (uint32_t)(l < 64 ? 64 : l);
     }
     p.force_normal = cfg.force_all_normal;
+    p.input_only = cfg.input_side_only;
     p.force_heavy = cfg.force_all_heavy;
     p.timing = cfg.timing;
     if (cfg.nm_table < 0 || cfg.nm_table > 2) return false;
@@ -145,21 +146,24 @@ bool plan_build(Plan& p, uint64_t nR, uint64_t nS, const gsh_config* cfg_in, voi
         p.h_max = hm < p.gt_cap_alloc ? hm : p.gt_cap_alloc;
     }
     // pass-1 units (= histogram slices): whole 16K-key chunks, about one unit per scatter CTA
-    // (2 per SM) and at most kHistMaxUnitChunks chunks; pass-2 groups of ~kGroupTuples tuples
+    // (2 per SM) and at most kHistMaxUnitChunks chunks.  Pass-2 units: ranges of consecutive
+    // slices of one pass-1 partition holding >= T tuples (planned on the device from the
+    // histogram, largest partitions first), so a skewed pass-1 partition spreads over many CTAs.
     {
         const uint64_t nch0 = (p.n[0] + kScatterChunk - 1) / kScatterChunk, nch1 = (p.n[1] + kScatterChunk - 1) / kScatterChunk;
         uint64_t uc = (nch0 + nch1 + 2 * uint64_t(num_sms) - 1) / (2 * uint64_t(num_sms));
         if (uc < 1) uc = 1;
         if (uc > kHistMaxUnitChunks) uc = kHistMaxUnitChunks;
         p.unit_chunks = (uint32_t)uc;
-        const uint64_t ul = uc * kScatterChunk;
-        uint64_t gu = (kGroupTuples + ul / 2) / ul;
-        p.group_units = (uint32_t)(gu < 1 ? 1 : gu);
         const uint64_t nch[2] = {nch0, nch1};
-        for (int s = 0; s < 2; ++s) {
-            p.nu1[s] = (uint32_t)((nch[s] + uc - 1) / uc);
-            p.ngroups[s] = (p.nu1[s] + p.group_units - 1) / p.group_units;
-        }
+        for (int s = 0; s < 2; ++s) p.nu1[s] = (uint32_t)((nch[s] + uc - 1) / uc);
+        if (p.nu1[0] > 4096 || p.nu1[1] > 4096) return false;   // k_hist_reduce stages <= 4096 slices
+        uint64_t T = kGroupTuples >> p.b1;
+        const uint64_t bal = (nR + nS) / (uint64_t(num_sms) * 8);   // >= 8 units per SM
+        if (bal < T) T = bal;
+        if (T < kPass2MinUnit) T = kPass2MinUnit;
+        p.u2_target = (uint32_t)T;
+        for (int s = 0; s < 2; ++s) p.u2_max[s] = (uint32_t)(p.n[s] / T + (1u << p.b1) + 1);
     }
     uint64_t scan_max = p.F + 1 > p.h_max + 1 ? p.F + 1 : p.h_max + 1;
     for (int s = 0; s < 2; ++s)
@@ -186,8 +190,10 @@ bool plan_build(Plan& p, uint64_t nR, uint64_t nS, const gsh_config* cfg_in, voi
     p.heavy_pay[0] = hp;
     p.heavy_pay[1] = hp ? hp + nR : nullptr;
     p.hist_partial = c.take<uint32_t>((size_t(p.nu1[0]) + p.nu1[1] + 1) * F);
-    p.off2 = c.take<uint32_t>((size_t(p.ngroups[0]) + p.ngroups[1] + 1) * F);
+    p.off2 = c.take<uint32_t>((size_t(p.u2_max[0]) + p.u2_max[1]) * (size_t(1) << p.b2));
+    p.u2_info = c.take<uint4>(size_t(p.u2_max[0]) + p.u2_max[1]);
     p.c1cnt = c.take<uint32_t>((size_t(p.nu1[0]) + p.nu1[1]) * 256 + 1);
+    p.slice_dom = c.take<uint32_t>(size_t(p.nu1[0]) + p.nu1[1] + 1);
     p.off1 = c.take<uint64_t>((size_t(p.nu1[0]) + p.nu1[1]) * 256 + 2);
     p.cnt = c.take<uint32_t>(2 * F);
     p.start = c.take<uint64_t>(2 * (F + 1));
@@ -198,6 +204,7 @@ bool plan_build(Plan& p, uint64_t nR, uint64_t nS, const gsh_config* cfg_in, voi
     p.large_idx = c.take<uint32_t>(F);
     p.part_heavy = c.take<uint32_t>(2 * F);
     p.det_prefix = c.take<uint64_t>(F + 1);
+    p.det_prefix2 = c.take<uint64_t>(F + 1);
     p.nrm_off = c.take<uint64_t>(2 * (F + 1));
     p.nrm_cur = c.take<uint32_t>(2 * F);
     p.H = c.take<HeavyKey>(p.h_max);
@@ -470,6 +477,28 @@ static gsh_status join_direct(const gsh_relation* R, const gsh_relation* S, gsh_
         launches += launch_split(p, n_large, (uint32_t)gcap, s);
         e5 = tm.mark();
     }
+    if (p.input_only) {   // measurement hook: stop after the input side
+        ce = cudaMemcpyAsync(&hs, p.st, sizeof(DevState), cudaMemcpyDeviceToHost, s);
+        if (ce == cudaSuccess) ce = cudaStreamSynchronize(s);
+        if (ce != cudaSuccess) return cuda_fail(ce, "input-side sync");
+        res->heavy_tuples_r = hs.heavy_tuples[0];
+        res->heavy_tuples_s = hs.heavy_tuples[1];
+        res->large_tuples = hs.large_tuples[0] + hs.large_tuples[1];
+        res->skew_pairs = hs.skew_pairs;
+        res->n_heavy = n_heavy;
+        res->n_large = n_large;
+        res->detect_overflow = hs.detect_overflow;
+        res->launches = (uint32_t)launches;
+        if (p.timing) {
+            res->ms_hist = tm.ms(e0, e1);
+            res->ms_pass1 = tm.ms(e1, e2);
+            res->ms_pass2 = tm.ms(e2, e3);
+            res->ms_detect = n_large ? tm.ms(e3, e4) : 0.f;
+            res->ms_split = n_large ? tm.ms(e4, e5) : 0.f;
+            res->ms_total = tm.ms(e0, e5);
+        }
+        return GSH_OK;
+    }
     // Chained NM table (L115) when the partition digits fix the top 16 bits of h (the chain link
     // then lives there) and, in auto mode, no partition is large (no duplicated keys that would
     // serialise a chain walk; the CSR table flattens those across the warp).
@@ -493,6 +522,7 @@ static gsh_status join_direct(const gsh_relation* R, const gsh_relation* S, gsh_
     res->overflow = mat ? (res->count > cap ? 1u : 0u) : 0u;  // items skip reserving once full
     res->heavy_tuples_r = hs.heavy_tuples[0];
     res->heavy_tuples_s = hs.heavy_tuples[1];
+    res->large_tuples = hs.large_tuples[0] + hs.large_tuples[1];
     res->skew_pairs = hs.skew_pairs;
     res->n_heavy = n_heavy;
     res->n_large = n_large;
@@ -601,6 +631,7 @@ gsh_status gsh_join(const gsh_relation* R, const gsh_relation* S, gsh_out_mode m
         acc.heavy_tuples_r += sr.heavy_tuples_r;
         acc.heavy_tuples_s += sr.heavy_tuples_s;
         acc.skew_pairs += sr.skew_pairs;
+        acc.large_tuples += sr.large_tuples;
         acc.n_heavy += sr.n_heavy;
         acc.n_large += sr.n_large;
         acc.detect_overflow |= sr.detect_overflow;

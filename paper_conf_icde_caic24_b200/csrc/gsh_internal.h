@@ -36,7 +36,8 @@ static_assert(kScatterIpt1 % 4 == 0 && kScatterIpt % 2 == 0, "vector tile loads:
 static_assert(kScatterBlock1 >= 256 && kScatterBlock2 >= 256 && kScatterBlock >= 256,
               "scatter CTAs keep one thread per bucket (2^kMaxDigitBits = 256)");
 constexpr uint32_t kHistMaxUnitChunks = 64;      // a pass-1 unit (= histogram slice) is <= 64 chunks = 2^20 tuples
-constexpr uint32_t kGroupTuples = 1u << 23;       // target tuples per pass-2 unit group (8M)
+constexpr uint32_t kGroupTuples = 1u << 23;       // pass-2 unit target = kGroupTuples >> b1 (32K at b1 = 8)
+constexpr uint32_t kPass2MinUnit = 4096;          // smallest pass-2 unit target (tuples)
 constexpr int kMaxDigitBits = 8;                // radix bits per pass (256 buckets)
 constexpr int kMaxPartBits = 16;                // b1 + b2 <= 16 (65536 partitions)
 constexpr int kHistBlock = 1024;
@@ -75,7 +76,7 @@ constexpr int kSkewBlock = 256;                 // skewed-key join CTA
 constexpr int kSkewSpt = 4;                     // S payloads per thread (registers)
 constexpr int kSkewTileS = kSkewBlock * kSkewSpt;  // 1024
 constexpr int kSkewTileR = 64;                  // R payloads per tile (shared memory)
-constexpr uint32_t kDetectChunk = 4096;         // tuples per detect / split work item
+constexpr uint32_t kDetectChunk = 2048;         // tuples per split (and sampled-detect) work item
 constexpr uint32_t kNoHeavy = 0xffffffffu;
 constexpr int kDetectMaxProbe = 64;   // a full table degrades to "normal", never to a long probe
 
@@ -92,6 +93,7 @@ struct DevState {
     unsigned int n_large, n_heavy, detect_overflow, max_rlen;  // max_rlen: largest |R_p| with |S_p| > 0
     unsigned int claim[8];                         // per-kernel work claim counters
     unsigned int route_mismatch;                   // route_bits > 0: tuples differ in the top route bits
+    unsigned int u2_front, u2_back;                // pass-2 units at the front / back of the list
     unsigned int heavy_overflow;                   // more skewed keys than the list H holds
 };
 
@@ -127,16 +129,17 @@ struct Plan {
     uint32_t C = 4096, Th = 64, L = 4096;  // NM capacity, skew-key threshold, large-partition threshold
     uint32_t nm_slots = 0;          // NM build-table slots (set after classification; 0 = from C)
     uint32_t F = 1;                 // 1 << (b1 + b2)
-    int force_normal = 0, force_heavy = 0, timing = 0;
+    int force_normal = 0, force_heavy = 0, timing = 0, input_only = 0;
     int nm_table = 0;               // config: 0 auto, 1 CSR, 2 chained where possible
     int nm_chain = 0;               // chosen for this call (nm_ring.cu)
     int detect_mode = 0;            // 0 exact counts, 1 sampled top-k (L107, L112)
     uint32_t sample_stride = 100, top_k = 3;
     int num_sms = 148;
     int hist_grid = 148;            // histogram CTAs (1 per SM)
-    uint32_t ngroups[2] = {0, 0};   // pass-2 unit groups per side
     uint32_t unit_chunks = 1;       // chunks per pass-1 unit (= histogram slice)
-    uint32_t group_units = 1;       // pass-1 units per pass-2 group
+    uint32_t u2_target = 0;         // pass-2 unit size target T (tuples): units = slice ranges of a
+                                    // pass-1 partition holding >= T tuples (the last one: any)
+    uint32_t u2_max[2] = {0, 0};    // bound on pass-2 units per side: n / T + 2^b1 + 1
     uint32_t gt_cap_alloc = 0;      // detection table slots allocated
     uint64_t h_max = 0;             // skewed-key list capacity
     uint64_t scan_scratch_elems = 0;
@@ -148,10 +151,14 @@ struct Plan {
     uint32_t* hist_partial = nullptr;         // [nu1[0] + nu1[1]][F] joint counts per pass-1 unit
     uint32_t nu1[2] = {0, 0};                 // pass-1 units per side
     uint32_t* c1cnt = nullptr;                // per side [256][nu1] pass-1 digit counts per unit
+    uint32_t* slice_dom = nullptr;            // [nu1[0] + nu1[1]] dominant pass-1 digit per unit or ~0
     uint64_t* off1 = nullptr;                 // per side [256 * nu1 + 1] unit/bucket output offsets
     uint32_t* cnt = nullptr;                  // [2][F]
     uint64_t* start = nullptr;                // [2][F + 1]
-    uint32_t* off2 = nullptr;                 // per side [ngroups][F] pass-2 unit offsets
+    uint32_t* off2 = nullptr;                 // [u2_max[0] + u2_max[1]][2^b2] pass-2 unit offsets in
+                                              // their final partitions (relative to its start)
+    uint4* u2_info = nullptr;                 // [u2_max[0] + u2_max[1]] pass-2 units: (side << 8 | d1,
+                                              // first slice, end slice, -); large rows' units at the front
     DevState* st = nullptr;
     unsigned long long* gt_key = nullptr;     // [gt_cap_alloc]  (1 << 32 | h), 0 = empty
     uint32_t* gt_cnt = nullptr;               // [2][gt_cap_alloc]
@@ -159,7 +166,8 @@ struct Plan {
     uint32_t* large_list = nullptr;           // [F]
     uint32_t* large_idx = nullptr;            // [F] partition -> large index or kNoHeavy
     uint32_t* part_heavy = nullptr;           // [2][F]  skewed tuples per partition
-    uint64_t* det_prefix = nullptr;           // [F + 1] detect/split items per large partition
+    uint64_t* det_prefix = nullptr;           // [F + 1] split (and sampled-detect) items per large partition
+    uint64_t* det_prefix2 = nullptr;          // [F + 1] exact-detect items per large partition
     uint64_t* nrm_off = nullptr;              // [2][F + 1] normal remainder offsets (large idx)
     HeavyKey* H = nullptr;                    // [h_max]
     uint64_t* h_off = nullptr;                // [2][h_max + 1]

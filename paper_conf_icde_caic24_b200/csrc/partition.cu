@@ -15,6 +15,8 @@
 #include <cstdio>
 #include <cstdlib>
 
+#include <type_traits>
+
 #include "gsh_device.cuh"
 #include "gsh_internal.h"
 #include "gsh_scan.cuh"
@@ -64,8 +66,10 @@ template <bool FAST16, bool CHECK>
 __global__ void __launch_bounds__(kHistBlock, 1)
 k_hist2d(const uint32_t* __restrict__ k0, uint64_t n0, const uint32_t* __restrict__ k1, uint64_t n1,
          uint32_t shift, uint32_t nbits, uint32_t b2, uint32_t* __restrict__ partial, uint32_t* __restrict__ c1cnt,
-         uint32_t nu0, uint32_t nu1, uint32_t unit_chunks, uint32_t rshift, DevState* st) {
+         uint32_t nu0, uint32_t nu1, uint32_t unit_chunks, uint32_t rshift, DevState* st,
+         uint32_t* __restrict__ slice_dom) {
     uint32_t r_or = 0, r_nor = 0;
+    __shared__ uint32_t s_dom;
     extern __shared__ uint32_t cnt[];
     __shared__ uint32_t c1s[256];
     __shared__ uint32_t ev_bin[kHistMaxEvents];
@@ -200,10 +204,20 @@ k_hist2d(const uint32_t* __restrict__ k0, uint64_t n0, const uint32_t* __restric
             n_ev = 0;
         }
         __syncthreads();
+        // the slice's dominant pass-1 digit (>= 1/8 of it: skewed data), for the pass-1 scatter
+        const uint64_t slen = umin64(n, uint64_t(cend) * kScatterChunk) - uint64_t(c0) * kScatterChunk;
+        if (threadIdx.x == 0) s_dom = 0;
+        __syncthreads();
         if (threadIdx.x < d1n) {
-            c1out[size_t(threadIdx.x) * nu + sl] = c1s[threadIdx.x];
+            const uint32_t c = c1s[threadIdx.x];
+            c1out[size_t(threadIdx.x) * nu + sl] = c;
             c1s[threadIdx.x] = 0;
+            const uint32_t w = __reduce_max_sync(__activemask(),
+                                                 (uint32_t)umin64(slen ? uint64_t(c) * 256 / slen : 0, 256) << 8 | threadIdx.x);
+            if ((threadIdx.x & 31) == 0) atomicMax(&s_dom, w);
         }
+        __syncthreads();
+        if (threadIdx.x == 0) slice_dom[(side ? nu0 : 0) + sl] = (s_dom >> 8) >= 32 ? (s_dom & 255u) : 0xffffffffu;
     }
     if (CHECK) {
         r_or = __reduce_or_sync(kFull, r_or);
@@ -231,51 +245,121 @@ int launch_hist(const Plan& p, const uint32_t* k0, const uint32_t* k1, cudaStrea
     if (fast16)
         k_hist2d<true, false><<<p.hist_grid, kHistBlock, smem, s>>>(k0, p.n[0], k1, p.n[1], shift, nbits, p.b2,
                                                                     p.hist_partial, p.c1cnt, p.nu1[0], p.nu1[1],
-                                                                    p.unit_chunks, rshift, p.st);
+                                                                    p.unit_chunks, rshift, p.st, p.slice_dom);
     else if (p.route_bits)
         k_hist2d<false, true><<<p.hist_grid, kHistBlock, smem, s>>>(k0, p.n[0], k1, p.n[1], shift, nbits, p.b2,
                                                                     p.hist_partial, p.c1cnt, p.nu1[0], p.nu1[1],
-                                                                    p.unit_chunks, rshift, p.st);
+                                                                    p.unit_chunks, rshift, p.st, p.slice_dom);
     else
         k_hist2d<false, false><<<p.hist_grid, kHistBlock, smem, s>>>(k0, p.n[0], k1, p.n[1], shift, nbits, p.b2,
                                                                      p.hist_partial, p.c1cnt, p.nu1[0], p.nu1[1],
-                                                                     p.unit_chunks, rshift, p.st);
+                                                                     p.unit_chunks, rshift, p.st, p.slice_dom);
     return 1;
 }
 
-// --------------------------------------------------- a2: reduce partials + prefix scans --
-// Per (side, partition p): off2[side][g][p] = tuples of p in chunk groups before g (pass-2 unit
-// offsets relative to the partition start) and cnt[side][p] = |R_p| / |S_p|.
-__global__ void k_hist_reduce(const uint32_t* __restrict__ partial, uint32_t* __restrict__ cnt,
-                              uint32_t* __restrict__ off2, uint32_t F, uint32_t ns0, uint32_t ns1, uint32_t ng0,
-                              uint32_t ng1, uint32_t group_units) {
-    for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < 2 * F; i += gridDim.x * blockDim.x) {
-        const uint32_t side = i / F, bin = i % F;
-        const uint32_t ns = side ? ns1 : ns0, ng = side ? ng1 : ng0;
-        const uint32_t* base = partial + size_t(side ? ns0 : 0) * F + bin;
-        uint32_t* o2 = off2 + size_t(side ? ng0 : 0) * F + bin;
-        // slices in order, 8 loads in flight per thread; off2 of group g = the running sum when
-        // its first slice comes up
-        (void)ng;
-        uint32_t run = 0, g = 0, left = 0;
-        for (uint32_t s = 0; s < ns; s += 8) {
-            uint32_t v[8];
+// --------------------------------------------- a2: reduce partials + pass-2 unit plan --
+// One CTA per pass-1 partition row (side, d1); thread b handles final partition p = (d1, b).
+//
+// Pass-2 units: a unit is a range of consecutive histogram slices [c0, c1) of ONE pass-1
+// partition: the runs those slices wrote into partition d1 in pass 1, contiguous there.  Slice s
+// belongs to unit floor(P_incl(s) / T) (P_incl = tuples of d1 in slices <= s), so units hold about
+// T tuples and a slice whose run alone exceeds T is a unit of its own: a skewed pass-1 partition
+// (38 % of a side at theta = 1.5) spreads over many CTAs instead of one.  Units of large rows
+// (>= 4x the mean row) are allocated from the front of the unit list, the rest from the back, so
+// the dynamic claim order runs the biggest units first (longest-processing-time-first).
+//
+// Then per thread: cnt[side][p] = |R_p| / |S_p|, and off2[u][b] = tuples of p in the slices before
+// unit u's first one (u's write offset in partition p, relative to the partition start).
+constexpr int kSlicesPerThread = 16;
+constexpr uint32_t kMaxSlices = 256 * kSlicesPerThread;   // >= 2^32 tuples / (64 chunks of 16K)
+
+__global__ void __launch_bounds__(256) k_hist_reduce(const uint32_t* __restrict__ partial,
+                                                     const uint32_t* __restrict__ c1cnt, uint32_t* __restrict__ cnt,
+                                                     uint32_t* __restrict__ off2, uint4* __restrict__ uinfo,
+                                                     uint32_t F, uint32_t b1, uint32_t b2, uint32_t ns0, uint32_t ns1,
+                                                     uint32_t T, uint32_t big, uint32_t ucap, DevState* st) {
+    __shared__ uint32_t starts[kMaxSlices + 1];
+    __shared__ uint32_t scan_tmp[256 / 32 + 1];
+    __shared__ uint32_t s_base, s_units;
+    const uint32_t side = blockIdx.x >> b1, d1 = blockIdx.x & ((1u << b1) - 1);
+    const uint32_t ns = side ? ns1 : ns0;
+    const uint32_t* row = c1cnt + (side ? size_t(ns0) * 256 : 0) + size_t(d1) * ns;
+    // (1) unit starts of this row: thread t owns slices [16t, 16t + 16) (ns <= kMaxSlices)
+    constexpr int K = kSlicesPerThread;
+    uint32_t v[K], loc = 0;
 #pragma unroll
-            for (int k = 0; k < 8; ++k) v[k] = (s + k < ns) ? base[size_t(s + k) * F] : 0u;
+    for (int k = 0; k < K; ++k) {
+        const uint32_t sl = K * threadIdx.x + k;
+        v[k] = sl < ns ? row[sl] : 0u;
+        loc += v[k];
+    }
+    uint32_t rtot = 0;
+    uint32_t pex = block_excl_scan_u32<256>(loc, &rtot, scan_tmp);   // tuples before my first slice
+    uint32_t flag = 0, nflag = 0;   // flag bit k: slice K t + k starts a unit
+#pragma unroll
+    for (int k = 0; k < K; ++k) {
+        const uint32_t sl = K * threadIdx.x + k;
+        const uint32_t pin = pex + v[k];
+        // start: slice 0 of a non-empty row, or the unit id floor(P_incl / T) advances past a
+        // non-empty prefix (leading empty slices stay in unit 0)
+        const bool f = (sl < ns) && ((sl == 0 && rtot > 0) || (pex > 0 && pin / T > pex / T));
+        flag |= uint32_t(f) << k;
+        nflag += f;
+        pex = pin;
+    }
+    __syncthreads();   // scan_tmp reuse
+    uint32_t units = 0;
+    uint32_t j = block_excl_scan_u32<256>(nflag, &units, scan_tmp);
+#pragma unroll
+    for (int k = 0; k < K; ++k)
+        if ((flag >> k) & 1u) starts[j++] = K * threadIdx.x + k;
+    if (threadIdx.x == 0) {
+        starts[units] = ns;
+        uint32_t base = 0;
+        if (units) {
+            if (rtot >= big) base = atomicAdd(&st->u2_front, units);
+            else base = ucap - atomicAdd(&st->u2_back, units) - units;
+        }
+        s_base = base;
+        s_units = units;
+    }
+    __syncthreads();
+    const uint32_t ub = s_base, uc = s_units;
+    for (uint32_t q = threadIdx.x; q < uc; q += blockDim.x)
+        uinfo[ub + q] = make_uint4(side << 8 | d1, starts[q], starts[q + 1], 0xffffffffu);
+    // (2) per final partition p = (d1, b): running sum over slices, recorded at unit starts
+    const uint32_t b = threadIdx.x;
+    uint32_t run = 0;
+    if (b < (1u << b2)) {
+        const uint32_t bin = (d1 << b2) | b;
+        const uint32_t* base = partial + size_t(side ? ns0 : 0) * F + bin;
+        uint32_t jj = 0, next = uc ? starts[0] : 0xffffffffu;
+        for (uint32_t s = 0; s < ns; s += 8) {   // 8 loads in flight per thread
+            uint32_t x[8];
+#pragma unroll
+            for (int k = 0; k < 8; ++k) x[k] = (s + k < ns) ? base[size_t(s + k) * F] : 0u;
 #pragma unroll
             for (int k = 0; k < 8; ++k) {
-                if (s + k < ns) {
-                    if (left == 0) {
-                        o2[size_t(g++) * F] = run;
-                        left = group_units;
-                    }
-                    --left;
-                    run += v[k];
+                if (s + k == next) {
+                    off2[(size_t(ub + jj) << b2) + b] = run;
+                    ++jj;
+                    next = jj < uc ? starts[jj] : 0xffffffffu;
                 }
+                run += x[k];
             }
         }
-        cnt[i] = run;
+        cnt[size_t(side) * F + bin] = run;
     }
+    // (3) the row's dominant final partition (>= 1/8 of the row: skewed data) for every unit of
+    // the row: the pass-2 scatter ranks its tuples with ballots instead of shared atomics
+    const uint32_t w = __reduce_max_sync(kFull, (uint32_t)umin64(rtot ? uint64_t(run) * 256 / rtot : 0, 256) << 8 | b);
+    __syncthreads();   // scan_tmp is free
+    if ((threadIdx.x & 31) == 0) scan_tmp[threadIdx.x >> 5] = w;
+    __syncthreads();
+    uint32_t best = 0;
+    for (int i = 0; i < 8; ++i) best = umax32(best, scan_tmp[i]);
+    const uint32_t dom = (best >> 8) >= 32 ? (best & 255u) : 0xffffffffu;
+    for (uint32_t q = threadIdx.x; q < uc; q += blockDim.x) uinfo[ub + q].w = dom;
 }
 
 struct CountAt {
@@ -292,9 +376,10 @@ struct ChunkDigit {
 
 int launch_hist_reduce_scan(const Plan& p, cudaStream_t s) {
     const uint32_t F = p.F;
-    unsigned grid = (2 * F + 255) / 256;
-    k_hist_reduce<<<grid, 256, 0, s>>>(p.hist_partial, p.cnt, p.off2, F, p.nu1[0], p.nu1[1], p.ngroups[0],
-                                       p.ngroups[1], p.group_units);
+    const uint64_t mean_row = (p.n[0] + p.n[1]) / (2ull << p.b1);
+    const uint32_t big = (uint32_t)umin64(4 * mean_row + 1, 0xffffffffull);
+    k_hist_reduce<<<2u << p.b1, 256, 0, s>>>(p.hist_partial, p.c1cnt, p.cnt, p.off2, p.u2_info, F, p.b1, p.b2,
+                                             p.nu1[0], p.nu1[1], p.u2_target, big, p.u2_max[0] + p.u2_max[1], p.st);
     // four independent scans in one launch triple: partition starts per side, pass-1
     // (digit, unit) offsets per side
     ScanSegs g{};
@@ -328,10 +413,14 @@ struct ScatterArgs {
     uint2* out[2];
     const uint64_t* start[2];  // final partition starts [F + 1] per side
     const uint64_t* off1[2];   // [256 * nu1 + 1] per side: start of unit u's run of digit d at d*nu1 + u
-    const uint32_t* off2[2];   // [ngroups][F] per side: tuples of partition p in earlier chunk groups
+    const uint32_t* off2;      // [pass-2 unit][2^b2]: unit's write offset in each of its partitions
+    const uint4* u2_info;      // pass-2 units (side << 8 | d1, first slice, end slice, dominant bucket)
+    const uint32_t* p1_dom;    // pass-1 units: dominant pass-1 digit of the slice, or 0xffffffff
+    const unsigned int* u2_fb;      // (front, back) unit counts (device, from k_hist_reduce)
+    uint32_t u2_cap;           // unit list capacity: front units at [0, f), back units at [cap - b, cap)
     uint64_t n[2];
-    uint32_t nu1[2], ngroups[2];     // pass-1 units (= histogram slices), pass-2 unit groups per side
-    uint32_t unit_len, group_units;  // tuples per pass-1 unit, pass-1 units per pass-2 group
+    uint32_t nu1[2];           // pass-1 units (= histogram slices) per side
+    uint32_t unit_len;         // tuples per pass-1 unit
     uint32_t pass, b1, b2, route_bits;
     unsigned int* unit_ctr;
 };
@@ -348,16 +437,22 @@ struct ScatterSmem {
     uint32_t carry[256];                // tuples in cbuf[b]
     uint32_t scan_tmp[33];
     uint32_t claim;
+    uint32_t wdom[32];                  // per warp: tuples of the dominant bucket in this tile
+    uint32_t wdoff[32];                 // their exclusive prefix over warps
     uint64_t mbar;                      // TMA completion of the tile buffer
 };
 
 struct UnitInfo {
     int side;
     uint32_t d1, grp, len;
+    uint32_t dom;   // dominant bucket of the unit (skewed data) or 0xffffffff
     uint64_t begin;
 };
 
-__device__ __forceinline__ UnitInfo unit_info(const ScatterArgs& a, uint32_t u, uint32_t units0, bool p1) {
+// Pass 1: unit u = histogram slice (side 1 from units0 on).  Pass 2: claim index u maps to the
+// unit list's front part [0, units0) or, shifted by back_off, its back part.
+__device__ __forceinline__ UnitInfo unit_info(const ScatterArgs& a, uint32_t u, uint32_t units0, uint32_t back_off,
+                                              bool p1) {
     UnitInfo ui;
     ui.side = (u >= units0) ? 1 : 0;
     const uint32_t lu = u - (ui.side ? units0 : 0);
@@ -367,13 +462,17 @@ __device__ __forceinline__ UnitInfo unit_info(const ScatterArgs& a, uint32_t u, 
         ui.grp = lu;
         ui.begin = uint64_t(lu) * a.unit_len;
         ui.len = (uint32_t)umin64(a.unit_len, a.n[ui.side] - ui.begin);
+        ui.dom = a.p1_dom[u];
     } else {
-        const uint32_t ng = a.ngroups[ui.side];
-        ui.d1 = lu / ng;
-        ui.grp = lu - ui.d1 * ng;
-        const uint32_t c0 = ui.grp * a.group_units, c1 = umin32(c0 + a.group_units, nch);
-        ui.begin = a.off1[ui.side][size_t(ui.d1) * nch + c0];
-        ui.len = (uint32_t)(a.off1[ui.side][size_t(ui.d1) * nch + c1] - ui.begin);
+        const uint32_t li = u < units0 ? u : u + back_off;
+        const uint4 inf = a.u2_info[li];
+        ui.side = (int)(inf.x >> 8);
+        ui.d1 = inf.x & 255u;
+        ui.grp = li;
+        const uint32_t nc = a.nu1[ui.side];
+        ui.begin = a.off1[ui.side][size_t(ui.d1) * nc + inf.y];
+        ui.len = (uint32_t)(a.off1[ui.side][size_t(ui.d1) * nc + inf.z] - ui.begin);
+        ui.dom = inf.w;
     }
     return ui;
 }
@@ -460,9 +559,9 @@ __device__ __forceinline__ void tile_issue(const ScatterArgs& a, int side, const
 // TMAST: whole-sector bucket runs leave the staging buffer as TMA bulk stores (one per bucket
 // and tile, issued by the bucket's thread) instead of per-tuple stores.
 template <int BLOCK, int IPT, int PASS, bool TMAST>
-__global__ void __launch_bounds__(BLOCK) k_scatter(ScatterArgs a) {
+__global__ void __launch_bounds__(BLOCK, 2) k_scatter(ScatterArgs a) {
     constexpr int TILE = BLOCK * IPT;
-    static_assert(TILE < 0xffff, "ranks are packed as u16 with 0xffff = masked");
+    static_assert(TILE < 0x7fff, "ranks are packed as u16: bit 15 = dominant bucket, 0xffff = masked");
     extern __shared__ __align__(128) unsigned char smem_raw[];
     ScatterSmem& S = *reinterpret_cast<ScatterSmem*>(smem_raw);
     unsigned char* buf0 = smem_raw + ((sizeof(ScatterSmem) + 127) & ~size_t(127));
@@ -478,8 +577,9 @@ __global__ void __launch_bounds__(BLOCK) k_scatter(ScatterArgs a) {
     const uint32_t dmask = nb - 1;
     const uint32_t dshift = (32 - a.route_bits - a.b1 - (p1 ? 0 : a.b2)) & 31;
     const uint32_t lowbits = p1 ? a.b2 : 0;
-    const uint32_t units0 = p1 ? a.nu1[0] : (1u << a.b1) * a.ngroups[0];
-    const uint32_t total = units0 + (p1 ? a.nu1[1] : (1u << a.b1) * a.ngroups[1]);
+    const uint32_t units0 = p1 ? a.nu1[0] : a.u2_fb[0];
+    const uint32_t total = p1 ? a.nu1[0] + a.nu1[1] : a.u2_fb[0] + a.u2_fb[1];
+    const uint32_t back_off = p1 ? 0u : a.u2_cap - total;
     const uint64_t rpol = policy_evict_first(), wpol = policy_evict_first();
 
     if (tid < 256) S.tcnt[tid] = 0;
@@ -492,7 +592,7 @@ __global__ void __launch_bounds__(BLOCK) k_scatter(ScatterArgs a) {
     uint32_t par = 0;
     bool issued = false;   // first tile of unit u already in flight
     while (u < total) {
-        const UnitInfo ui = unit_info(a, u, units0, p1);
+        const UnitInfo ui = unit_info(a, u, units0, back_off, p1);
         const uint32_t ntile = tile_count<TILE>(p1, ui.begin, ui.len);
         if (ntile == 0) {  // empty unit (pass 2: digit absent from the group)
             __syncthreads();
@@ -507,11 +607,17 @@ __global__ void __launch_bounds__(BLOCK) k_scatter(ScatterArgs a) {
             uint32_t r0;
             const uint32_t pidx = ((ui.d1 << bits) | tid) << lowbits;
             if (p1) r0 = (uint32_t)a.off1[ui.side][size_t(tid) * a.nu1[ui.side] + ui.grp];
-            else r0 = (uint32_t)a.start[ui.side][pidx] + a.off2[ui.side][size_t(ui.grp) * (size_t(1) << (a.b1 + a.b2)) + pidx];
+            else r0 = (uint32_t)a.start[ui.side][pidx] + a.off2[(size_t(ui.grp) << a.b2) + tid];
             S.run[tid] = r0;
             S.wpos[tid] = r0;
             S.carry[tid] = 0;
         }
+        // Dominant bucket (skewed data: one key's bucket holds >= 1/8 of the slice / pass-1
+        // partition, from the histogram pass): its tuples are ranked with warp ballots and per-warp
+        // register counters instead of shared-memory atomics, which serialise when most lanes of
+        // every warp hit the same counter.
+        const uint32_t dom = ui.dom;
+        const bool dom_on = dom != 0xffffffffu;
         // (the first sync of the tile loop orders run[] before its use)
         uint32_t un = total;
         for (uint32_t q = 0; q < ntile; ++q) {
@@ -531,7 +637,7 @@ __global__ void __launch_bounds__(BLOCK) k_scatter(ScatterArgs a) {
                         tile_issue(a, ui.side, tile_geo<TILE>(p1, ui.begin, ui.len, q + 1), p1, ok, op, o2, &S.mbar,
                                    rpol);
                     } else if (un < total) {
-                        const UnitInfo nx = unit_info(a, un, units0, p1);
+                        const UnitInfo nx = unit_info(a, un, units0, back_off, p1);
                         if (nx.len)
                             tile_issue(a, nx.side, tile_geo<TILE>(p1, nx.begin, nx.len, 0), p1, ok, op, o2, &S.mbar,
                                        rpol);
@@ -540,12 +646,29 @@ __global__ void __launch_bounds__(BLOCK) k_scatter(ScatterArgs a) {
             };
             mbar_wait(&S.mbar, par);
             par ^= 1;
-            uint32_t rk[IPT / 2];  // ranks, packed 2 x u16
+            uint32_t rk[IPT / 2];  // ranks, packed 2 x u16 (bit 15: dominant-bucket rank; 0xffff: masked)
+            uint32_t wrun = 0;     // this warp's dominant-bucket tuples so far in this tile
+            // rank of one tuple of bucket b: dominant bucket by ballot, others by shared atomics
             // full tile: the input stays in registers from the ranking to the staging step, so
             // the input buffer is free (and the next tile's TMA issued) after the first barrier
             constexpr int NV = p1 ? IPT / 4 : IPT / 2;
             uint4 xa[NV], xb[p1 ? NV : 1];
-            if (full) {  // whole tile arrived by TMA: vector shared loads, no bounds checks
+            // (two instantiations of the full-tile ranking: DOM = the unit has a dominant bucket)
+            auto rank_tile = [&](auto dom_tag) {
+                constexpr bool DOM = decltype(dom_tag)::value;
+                auto rank_of = [&](bool valid, uint32_t b) -> uint32_t {
+                    if constexpr (DOM) {
+                        const bool isd = valid && b == dom;
+                        const uint32_t m = __ballot_sync(kFull, isd);
+                        uint32_t r = 0xffffu;
+                        if (isd) r = 0x8000u | (wrun + __popc(m & lanemask_lt()));
+                        else if (valid) r = atomicAdd(&S.tcnt[b], 1u);
+                        wrun += __popc(m);
+                        return r;
+                    } else {
+                        return valid ? atomicAdd(&S.tcnt[b], 1u) : 0xffffu;
+                    }
+                };
                 if (p1) {    // uint4 = 4 keys; slot 4 * v + c of element 4 * (v * BLOCK + tid) + c
 #pragma unroll
                     for (int v = 0; v < NV; ++v) {
@@ -553,10 +676,10 @@ __global__ void __launch_bounds__(BLOCK) k_scatter(ScatterArgs a) {
                         xb[v] = reinterpret_cast<const uint4*>(op)[v * BLOCK + tid];
                         x.x = hash32(x.x); x.y = hash32(x.y); x.z = hash32(x.z); x.w = hash32(x.w);
                         xa[v] = x;
-                        const uint32_t r0 = atomicAdd(&S.tcnt[(x.x >> dshift) & dmask], 1u);
-                        const uint32_t r1 = atomicAdd(&S.tcnt[(x.y >> dshift) & dmask], 1u);
-                        const uint32_t r2 = atomicAdd(&S.tcnt[(x.z >> dshift) & dmask], 1u);
-                        const uint32_t r3 = atomicAdd(&S.tcnt[(x.w >> dshift) & dmask], 1u);
+                        const uint32_t r0 = rank_of(true, (x.x >> dshift) & dmask);
+                        const uint32_t r1 = rank_of(true, (x.y >> dshift) & dmask);
+                        const uint32_t r2 = rank_of(true, (x.z >> dshift) & dmask);
+                        const uint32_t r3 = rank_of(true, (x.w >> dshift) & dmask);
                         rk[2 * v] = r0 | (r1 << 16);
                         rk[2 * v + 1] = r2 | (r3 << 16);
                     }
@@ -566,12 +689,16 @@ __global__ void __launch_bounds__(BLOCK) k_scatter(ScatterArgs a) {
                         const uint32_t i0 = 2 * (v * BLOCK + tid) - geo.off;   // wraps for slot 0 when off = 1
                         const uint4 x = reinterpret_cast<const uint4*>(o2)[v * BLOCK + tid];
                         xa[v] = x;
-                        uint32_t r0 = 0xffffu, r1 = 0xffffu;   // 0xffff = not in this tile
-                        if (i0 < ql) r0 = atomicAdd(&S.tcnt[(x.x >> dshift) & dmask], 1u);
-                        if (i0 + 1 < ql) r1 = atomicAdd(&S.tcnt[(x.z >> dshift) & dmask], 1u);
+                        // 0xffff = not in this tile
+                        const uint32_t r0 = rank_of(i0 < ql, (x.x >> dshift) & dmask);
+                        const uint32_t r1 = rank_of(i0 + 1 < ql, (x.z >> dshift) & dmask);
                         rk[v] = r0 | (r1 << 16);
                     }
                 }
+            };
+            if (full) {  // whole tile arrived by TMA: vector shared loads, no bounds checks
+                if (dom_on) rank_tile(std::true_type{});
+                else rank_tile(std::false_type{});
                 fence_proxy_async_smem();  // reads of the input tile precede the next TMA writes
             } else {
 #pragma unroll
@@ -605,6 +732,7 @@ __global__ void __launch_bounds__(BLOCK) k_scatter(ScatterArgs a) {
                     if (jj & 1) rk[jj >> 1] |= r << 16; else rk[jj >> 1] = r;
                 }
             }
+            if ((tid & 31) == 0) S.wdom[tid >> 5] = wrun;
             // the previous tile's bulk stores must have read the staging buffer before any thread
             // writes it again (after the barrier below)
             if (TMAST && tid < nb) bulk_wait_read0();
@@ -614,7 +742,22 @@ __global__ void __launch_bounds__(BLOCK) k_scatter(ScatterArgs a) {
             // Write combining: bucket b's staged run = [carry from the previous tile | this tile's
             // tuples]; only whole 32-byte sectors are written, the < 4-tuple remainder carries
             // over (the unit's last tile flushes everything).  u32 offsets (n < 2^32).
-            const uint32_t tc = (tid < nb) ? S.tcnt[tid] : 0u;
+            uint32_t tc = (tid < nb) ? S.tcnt[tid] : 0u;
+            if (dom_on) {
+                constexpr uint32_t NW = BLOCK / 32;
+                if (tid == dom)
+                    for (uint32_t w = 0; w < NW; ++w) tc += S.wdom[w];
+                if (tid < 32) {   // exclusive prefix of the warps' dominant counts
+                    const uint32_t c = tid < NW ? S.wdom[tid] : 0u;
+                    uint32_t x = c;
+#pragma unroll
+                    for (int o = 1; o < 32; o <<= 1) {
+                        const uint32_t y = __shfl_up_sync(kFull, x, o);
+                        if (tid >= (uint32_t)o) x += y;
+                    }
+                    if (tid < NW) S.wdoff[tid] = x - c;
+                }
+            }
             const uint32_t cin = (tid < nb) ? S.carry[tid] : 0u;
             uint32_t all;
             // TMAST: one spare slot per bucket so the run starts at the parity of its output index
@@ -640,24 +783,27 @@ __global__ void __launch_bounds__(BLOCK) k_scatter(ScatterArgs a) {
             }
             __syncthreads();
             if (full) {
+                // staging position of a tuple of bucket b with rank r (bit 15: dominant bucket)
+                const uint32_t dbase = dom_on ? S.local_start[dom & 255u] + S.wdoff[tid >> 5] : 0u;
+                auto spos = [&](uint32_t b, uint32_t r) {
+                    return (r & 0x8000u) ? dbase + (r & 0x7fffu) : S.local_start[b] + r;
+                };
                 if (p1) {
 #pragma unroll
                     for (int v = 0; v < NV; ++v) {
                         const uint4 h4 = xa[v], p4 = xb[v];
-                        stage[S.local_start[(h4.x >> dshift) & dmask] + (rk[2 * v] & 0xffffu)] = make_uint2(h4.x, p4.x);
-                        stage[S.local_start[(h4.y >> dshift) & dmask] + (rk[2 * v] >> 16)] = make_uint2(h4.y, p4.y);
-                        stage[S.local_start[(h4.z >> dshift) & dmask] + (rk[2 * v + 1] & 0xffffu)] =
-                            make_uint2(h4.z, p4.z);
-                        stage[S.local_start[(h4.w >> dshift) & dmask] + (rk[2 * v + 1] >> 16)] =
-                            make_uint2(h4.w, p4.w);
+                        stage[spos((h4.x >> dshift) & dmask, rk[2 * v] & 0xffffu)] = make_uint2(h4.x, p4.x);
+                        stage[spos((h4.y >> dshift) & dmask, rk[2 * v] >> 16)] = make_uint2(h4.y, p4.y);
+                        stage[spos((h4.z >> dshift) & dmask, rk[2 * v + 1] & 0xffffu)] = make_uint2(h4.z, p4.z);
+                        stage[spos((h4.w >> dshift) & dmask, rk[2 * v + 1] >> 16)] = make_uint2(h4.w, p4.w);
                     }
-                } else {   // ranks < TILE <= 0xffff, so 0xffff marks a masked slot
+                } else {   // ranks < TILE <= 0x7fff, so 0xffff marks a masked slot
 #pragma unroll
                     for (int v = 0; v < NV; ++v) {
                         const uint4 x = xa[v];
                         const uint32_t r0 = rk[v] & 0xffffu, r1 = rk[v] >> 16;
-                        if (r0 != 0xffffu) stage[S.local_start[(x.x >> dshift) & dmask] + r0] = make_uint2(x.x, x.y);
-                        if (r1 != 0xffffu) stage[S.local_start[(x.z >> dshift) & dmask] + r1] = make_uint2(x.z, x.w);
+                        if (r0 != 0xffffu) stage[spos((x.x >> dshift) & dmask, r0)] = make_uint2(x.x, x.y);
+                        if (r1 != 0xffffu) stage[spos((x.z >> dshift) & dmask, r1)] = make_uint2(x.z, x.w);
                     }
                 }
             } else {
@@ -706,7 +852,7 @@ __global__ void __launch_bounds__(BLOCK) k_scatter(ScatterArgs a) {
         }
         u = un;
         issued = true;  // the next unit's first tile (if any, and non-empty) is in flight
-        if (u < total && unit_info(a, u, units0, p1).len == 0) issued = false;
+        if (u < total && unit_info(a, u, units0, back_off, p1).len == 0) issued = false;
     }
     if (TMAST && tid < nb) bulk_wait0();  // shared memory must outlive the bulk stores' reads
 }
@@ -754,13 +900,15 @@ int launch_scatter(const Plan& p, int pass, const uint32_t* const keys[2], const
         a.start[side] = p.start + size_t(side) * (p.F + 1);
         a.off1[side] = p.off1 + o1;
         o1 += uint64_t(p.nu1[side]) * 256 + 1;
-        a.off2[side] = p.off2 + (side ? size_t(p.ngroups[0]) * p.F : 0);
         a.n[side] = p.n[side];
         a.nu1[side] = p.nu1[side];
-        a.ngroups[side] = p.ngroups[side];
     }
+    a.off2 = p.off2;
+    a.u2_info = p.u2_info;
+    a.u2_fb = &p.st->u2_front;
+    a.p1_dom = p.slice_dom;
+    a.u2_cap = p.u2_max[0] + p.u2_max[1];
     a.unit_len = p.unit_chunks * kScatterChunk;
-    a.group_units = p.group_units;
     a.pass = pass;
     a.b1 = p.b1;
     a.b2 = p.b2;

@@ -53,20 +53,26 @@ int launch_classify(const Plan& p, cudaStream_t s) {
     return 1;
 }
 
-// Items of detect / split: ceil((|R_p| + |S_p|) / kDetectChunk) per large partition.
+// Work items of detect / split: ceil((|R_p| + |S_p|) / chunk) per large partition, never spanning
+// two partitions.  Detect uses kDetectItem-tuple items (one shared-memory count table flush per
+// item), split kDetectChunk-tuple items (every tuple held in registers across its two phases).
+constexpr uint32_t kDetectItem = 16384;
+
 struct DetectItems {
     const uint32_t* cnt;
     const uint32_t* large_list;
-    uint32_t F;
+    uint32_t F, chunk;
     __device__ uint64_t operator()(uint64_t i) const {
         uint32_t p = large_list[i];
         uint64_t t = uint64_t(cnt[p]) + cnt[F + p];
-        return (t + kDetectChunk - 1) / kDetectChunk;
+        return (t + chunk - 1) / chunk;
     }
 };
 
 int launch_detect_prefix(const Plan& p, uint32_t n_large, cudaStream_t s) {
-    return launch_scan(DetectItems{p.cnt, p.large_list, p.F}, n_large, p.det_prefix, p.scan_scratch, s);
+    return launch_scan(DetectItems{p.cnt, p.large_list, p.F, kDetectChunk}, n_large, p.det_prefix, p.scan_scratch,
+                       s) +
+           launch_scan(DetectItems{p.cnt, p.large_list, p.F, kDetectItem}, n_large, p.det_prefix2, p.scan_scratch, s);
 }
 
 // Locate item `it` among large partitions: returns large index li and chunk c.
@@ -86,7 +92,7 @@ struct LargeView {
     const uint32_t* cnt;      // [2][F]
     const uint32_t* large_list;
     const uint64_t* det_prefix;
-    uint32_t F, n_large;
+    uint32_t F, n_large, chunk;
 };
 
 // The element range of one item: tuples [e0, e1) of the concatenation R_p ++ S_p.
@@ -102,8 +108,8 @@ __device__ __forceinline__ ItemRange item_range(const LargeView& v, uint64_t it)
     r.cr = v.cnt[r.p];
     r.cs = v.cnt[v.F + r.p];
     uint64_t c = it - v.det_prefix[r.li];
-    r.e0 = c * kDetectChunk;
-    r.e1 = umin64(r.e0 + kDetectChunk, uint64_t(r.cr) + r.cs);
+    r.e0 = c * v.chunk;
+    r.e1 = umin64(r.e0 + v.chunk, uint64_t(r.cr) + r.cs);
     return r;
 }
 
@@ -150,6 +156,145 @@ __global__ void __launch_bounds__(kDetBlock) k_detect(LargeView v, unsigned long
     }
 }
 
+// Exact detection (detect_mode 0): per-item shared-memory count tables.  A CTA claims
+// an item (<= kDetectItem tuples of ONE large partition), counts every key of it in a shared-memory
+// linear-probing table keyed by h (0 marks an empty slot; the key with h = 0 has its own counters),
+// then merges each distinct key ONCE into the global table -- a skewed key costs one global atomic
+// per item instead of one per warp.  Every key lives in exactly one partition, so when the whole
+// partition is this one item its counts are exact and only keys reaching T_h are merged (the rest
+// are normal, and "not in the table" means normal to split and select); keys of partitions spanning
+// several items are all merged.  A key that finds no shared slot within kDetSmemProbe goes to the
+// global table directly (exact either way).
+constexpr uint32_t kDetSmemSlots = 6144;   // 72 KB: three CTAs per SM
+constexpr int kDetSmemProbe = 32;
+constexpr size_t kDetSmemBytes = size_t(kDetSmemSlots) * 12;
+
+__global__ void __launch_bounds__(kDetBlock, 3) k_detect_smem(LargeView v, unsigned long long* gt_key, uint32_t* gt_cnt,
+                                                          uint32_t cap_alloc, uint32_t logcap, uint32_t Th,
+                                                          int force_heavy, DevState* st, unsigned int* claim) {
+    extern __shared__ uint32_t det_dyn[];
+    uint32_t* s_key = det_dyn;                  // h, 0 = empty
+    uint32_t* s_cr = det_dyn + kDetSmemSlots;
+    uint32_t* s_cs = s_cr + kDetSmemSlots;
+    __shared__ uint32_t s_zero[2];              // counts of the key with h = 0
+    __shared__ unsigned int s_it;
+    for (uint32_t i = threadIdx.x; i < kDetSmemSlots; i += kDetBlock) {
+        s_key[i] = 0;
+        s_cr[i] = 0;
+        s_cs[i] = 0;
+    }
+    if (threadIdx.x < 2) s_zero[threadIdx.x] = 0;
+    const uint64_t total = v.det_prefix[v.n_large];
+    auto merge = [&](uint32_t h, uint32_t cr, uint32_t cs) {
+        const uint32_t g = gt_insert(gt_key, h, logcap);
+        if (g == kNoHeavy) {
+            st->detect_overflow = 1;
+        } else {
+            if (cr) atomicAdd(&gt_cnt[g], cr);
+            if (cs) atomicAdd(&gt_cnt[size_t(cap_alloc) + g], cs);
+        }
+    };
+    // count k_r R and k_s S occurrences of h (K1: one occurrence of one side, which compiles to
+    // ATOMS.POPC.INC: the lanes of a warp on one counter cost one instruction)
+    auto count = [&](uint32_t h, uint32_t kr, uint32_t ks, bool K1) {
+        if (h == 0) {
+            if (kr) atomicAdd(&s_zero[0], kr);
+            if (ks) atomicAdd(&s_zero[1], ks);
+            return;
+        }
+        uint32_t slot = __umulhi(h * 0x9E3779B1u, kDetSmemSlots);
+        for (int probe = 0; probe < kDetSmemProbe; ++probe) {
+            const uint32_t cur = s_key[slot];
+            bool hit = cur == h;
+            if (!hit && cur == 0) {
+                const uint32_t prev = atomicCAS(&s_key[slot], 0u, h);
+                hit = prev == 0 || prev == h;
+            }
+            if (hit) {
+                if (K1) {
+                    atomicAdd(ks ? &s_cs[slot] : &s_cr[slot], 1u);
+                } else {
+                    if (kr) atomicAdd(&s_cr[slot], kr);
+                    if (ks) atomicAdd(&s_cs[slot], ks);
+                }
+                return;
+            }
+            slot = slot + 1 == kDetSmemSlots ? 0 : slot + 1;
+        }
+        merge(h, kr, ks);   // shared table crowded: count globally
+    };
+    const uint32_t lane = lane_id();
+    for (;;) {
+        if (threadIdx.x == 0) s_it = atomicAdd(claim, 1u);
+        __syncthreads();
+        const uint64_t it = s_it;
+        if (it >= total) break;
+        const ItemRange r = item_range(v, it);
+        const uint2* pr = v.part[0] + v.start[r.p];
+        const uint2* ps = v.part[1] + v.start[size_t(v.F) + 1 + r.p];
+        // the whole partition in this item: local counts are exact, merge only possible skewed keys
+        const bool whole = r.e0 == 0 && r.e1 == uint64_t(r.cr) + r.cs;
+        const uint32_t keep = (whole && !force_heavy) ? Th : 1u;
+        // Warp reference key: lanes holding the warp's current reference key are counted in
+        // registers (one ballot per side), so a skewed key's tuples cost no shared atomics; the
+        // reference moves to another lane's key when it matched fewer than 8 lanes.
+        uint32_t ref = 0, pend_r = 0, pend_s = 0;
+        bool has_ref = false;
+        constexpr int U = 8;   // independent loads in flight per thread; the next batch loads while
+                               // this one is counted
+        uint32_t hn[U];
+        auto load = [&](uint64_t base) {
+#pragma unroll
+            for (int u = 0; u < U; ++u) {
+                const uint64_t e = base + uint64_t(u) * kDetBlock + threadIdx.x;
+                hn[u] = e < r.e1 ? (e < r.cr ? pr[e].x : ps[e - r.cr].x) : 0u;
+            }
+        };
+        load(r.e0);
+        for (uint64_t base = r.e0; base < r.e1; base += uint64_t(U) * kDetBlock) {
+            uint32_t h[U];
+#pragma unroll
+            for (int u = 0; u < U; ++u) h[u] = hn[u];
+            if (base + uint64_t(U) * kDetBlock < r.e1) load(base + uint64_t(U) * kDetBlock);
+#pragma unroll
+            for (int u = 0; u < U; ++u) {
+                const uint64_t e = base + uint64_t(u) * kDetBlock + threadIdx.x;
+                const bool valid = e < r.e1, side = e >= r.cr;
+                const bool isref = has_ref && valid && h[u] == ref;
+                const uint32_t m1 = __ballot_sync(kFull, isref && side), ma = __ballot_sync(kFull, isref);
+                pend_s += __popc(m1);
+                pend_r += __popc(ma & ~m1);
+                const bool other = valid && !isref;
+                if (other) count(h[u], side ? 0u : 1u, side ? 1u : 0u, true);
+                const uint32_t mo = __ballot_sync(kFull, other);
+                if (__popc(ma) < 8 && mo) {
+                    if (lane == 0 && (pend_r | pend_s)) count(ref, pend_r, pend_s, false);
+                    pend_r = pend_s = 0;
+                    ref = __shfl_sync(kFull, h[u], __ffs(mo) - 1);
+                    has_ref = true;
+                }
+            }
+        }
+        if (lane == 0 && (pend_r | pend_s)) count(ref, pend_r, pend_s, false);
+        __syncthreads();
+        for (uint32_t i = threadIdx.x; i < kDetSmemSlots; i += kDetBlock) {   // merge + clear
+            const uint32_t k = s_key[i];
+            if (k) {
+                const uint32_t cr = s_cr[i], cs = s_cs[i];
+                if (max(cr, cs) >= keep) merge(k, cr, cs);
+                s_key[i] = 0;
+                s_cr[i] = 0;
+                s_cs[i] = 0;
+            }
+        }
+        if (threadIdx.x == 0 && (s_zero[0] | s_zero[1])) {
+            if (max(s_zero[0], s_zero[1]) >= keep) merge(0u, s_zero[0], s_zero[1]);
+            s_zero[0] = s_zero[1] = 0;
+        }
+        __syncthreads();
+    }
+}
+
 int launch_detect(const Plan& p, uint32_t n_large, uint32_t gt_cap, cudaStream_t s) {
     if (n_large == 0) return 0;
     uint32_t logcap = 0;
@@ -157,13 +302,21 @@ int launch_detect(const Plan& p, uint32_t n_large, uint32_t gt_cap, cudaStream_t
     if (p.detect_mode == 0) cudaMemsetAsync(p.gt_key, 0, size_t(gt_cap) * sizeof(unsigned long long), s);
     cudaMemsetAsync(p.gt_cnt, 0, size_t(gt_cap) * sizeof(uint32_t), s);
     cudaMemsetAsync(p.gt_cnt + p.gt_cap_alloc, 0, size_t(gt_cap) * sizeof(uint32_t), s);
-    LargeView v{{p.bufB[0], p.bufB[1]}, p.start, p.cnt, p.large_list, p.det_prefix, p.F, n_large};
+    LargeView v{{p.bufB[0], p.bufB[1]}, p.start, p.cnt, p.large_list, p.det_prefix, p.F, n_large, kDetectChunk};
     if (p.detect_mode == 1)
         k_detect<true><<<p.num_sms * 8, kDetBlock, 0, s>>>(v, p.gt_key, p.gt_cnt, p.gt_cap_alloc, logcap, p.st,
                                                            &p.st->claim[2]);
-    else
-        k_detect<false><<<p.num_sms * 8, kDetBlock, 0, s>>>(v, p.gt_key, p.gt_cnt, p.gt_cap_alloc, logcap, p.st,
-                                                            &p.st->claim[2]);
+    else {
+        static std::once_flag attr_once[kMaxDevices];
+        once_per_device(attr_once, [] {
+            cudaFuncSetAttribute(k_detect_smem, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kDetSmemBytes);
+        });
+        LargeView v2 = v;
+        v2.det_prefix = p.det_prefix2;
+        v2.chunk = kDetectItem;
+        k_detect_smem<<<p.num_sms * 3, kDetBlock, kDetSmemBytes, s>>>(v2, p.gt_key, p.gt_cnt, p.gt_cap_alloc, logcap,
+                                                                      p.Th, p.force_heavy, p.st, &p.st->claim[2]);
+    }
     return 1;
 }
 
@@ -251,7 +404,7 @@ int launch_sample_topk(const Plan& p, uint32_t n_large, uint32_t gt_cap, cudaStr
     uint32_t logcap = 0;
     while ((1u << logcap) < gt_cap) ++logcap;
     cudaMemsetAsync(p.gt_key, 0, size_t(gt_cap) * sizeof(unsigned long long), s);
-    LargeView v{{p.bufB[0], p.bufB[1]}, p.start, p.cnt, p.large_list, p.det_prefix, p.F, n_large};
+    LargeView v{{p.bufB[0], p.bufB[1]}, p.start, p.cnt, p.large_list, p.det_prefix, p.F, n_large, kDetectChunk};
     const unsigned grid = (unsigned)umin64(n_large, uint64_t(p.num_sms) * 8);
     k_sample_topk<<<grid, kSampleBlock, 0, s>>>(v, p.sample_stride, p.top_k, p.gt_key, logcap, p.st);
     return 1;
@@ -340,64 +493,164 @@ int launch_heavy_prefix(const Plan& p, uint32_t n_heavy, uint32_t n_large, cudaS
 }
 
 // -------------------------------------------------------------------- a7: split --
-__global__ void __launch_bounds__(kDetBlock) k_split(LargeView v, const unsigned long long* gt_key,
-                                                    const uint32_t* gt_hid, uint32_t logcap,
-                                                    const uint64_t* h_off, uint64_t h_stride, uint32_t* h_cur,
-                                                    uint32_t h_max, uint32_t* heavy_pay_r, uint32_t* heavy_pay_s,
-                                                    const uint64_t* nrm_off, uint32_t* nrm_cur, uint2* out_r,
-                                                    uint2* out_s, unsigned int* claim) {
+// "checks each R tuple against the skewed keys.  If the tuple is skewed, it is appended to an
+// array allocated for the associated skewed key ... Otherwise ... appends the tuple to a normal
+// partition" (L114); same for S.  A CTA claims an item (<= kDetectChunk tuples of ONE large
+// partition, 16 per thread, held in registers) and splits it in two phases: (1) every tuple gets
+// its skewed-key id (global table lookup) and a rank inside the item -- per (side, key) for skewed
+// tuples through a shared-memory table, per side for normal ones -- from shared-memory atomics
+// (ATOMS.POPC.INC: lanes of a warp on one counter get consecutive ranks in one instruction);
+// (2) one global atomic per distinct (side, key) and per side reserves the item's runs, and the
+// tuples are written at base + rank (consecutive for runs of one key: coalesced).
+constexpr uint32_t kSplitHidSlots = 2 * kDetectChunk;   // an item's distinct (side, key) always fit
+constexpr int kSplitIpt = kDetectChunk / kDetBlock;
+constexpr size_t kSplitSmemBytes = size_t(kSplitHidSlots) * 8;
+static_assert(kSplitIpt * kDetBlock == kDetectChunk, "split item = 8 tuples per thread");
+static_assert(kSplitHidSlots == 4096, "slot hash below takes 12 bits");
+
+__global__ void __launch_bounds__(kDetBlock, 4) k_split(LargeView v, const unsigned long long* __restrict__ gt_key,
+                                                    const uint32_t* __restrict__ gt_hid, uint32_t logcap,
+                                                    const uint64_t* __restrict__ h_off, uint64_t h_stride,
+                                                    uint32_t* h_cur, uint32_t h_max, uint32_t* heavy_pay_r,
+                                                    uint32_t* heavy_pay_s, const uint64_t* __restrict__ nrm_off,
+                                                    uint32_t* nrm_cur, uint2* out_r, uint2* out_s,
+                                                    unsigned int* claim) {
+    extern __shared__ uint32_t split_dyn[];
+    uint32_t* s_key = split_dyn;                    // (hid << 1 | side) + 1, 0 = empty
+    uint32_t* s_cnt = split_dyn + kSplitHidSlots;   // count, then the item's run base
+    __shared__ uint32_t s_nrm[2], s_nbase[2];
     __shared__ unsigned int s_it;
+    for (uint32_t i = threadIdx.x; i < kSplitHidSlots; i += kDetBlock) {
+        s_key[i] = 0;
+        s_cnt[i] = 0;
+    }
+    if (threadIdx.x < 2) s_nrm[threadIdx.x] = 0;
     const uint64_t total = v.det_prefix[v.n_large];
-    const uint32_t lane = lane_id();
-    const uint32_t ltm = lanemask_lt();
     for (;;) {
         if (threadIdx.x == 0) s_it = atomicAdd(claim, 1u);
         __syncthreads();
         const uint64_t it = s_it;
-        __syncthreads();
         if (it >= total) break;
         const ItemRange r = item_range(v, it);
-        for (uint64_t base = r.e0; base < r.e1; base += kDetBlock) {
-            const uint64_t e = base + threadIdx.x;
-            const bool valid = e < r.e1;
-            int side = 0;
-            uint2 t = make_uint2(0, 0);
-            if (valid) t = item_tuple(v, r, e, side);
-            // one table lookup per distinct key in the warp
-            const unsigned long long key = valid ? ((uint64_t(side) << 32) | t.x) : ((2ull << 32) | lane);
-            const uint32_t peers = __match_any_sync(kFull, key);
-            const uint32_t leader = __ffs(peers) - 1;
-            uint32_t hid = kNoHeavy;
-            if (valid && lane == leader) {
-                uint32_t slot = gt_find(gt_key, t.x, logcap);
-                hid = (slot == kNoHeavy) ? kNoHeavy : gt_hid[slot];
-            }
-            hid = __shfl_sync(kFull, hid, leader);
-            // heavy: append payload to its key array (warp-aggregated cursor per (side, key))
-            const bool heavy = valid && hid != kNoHeavy;
-            uint32_t pos = 0;
-            if (heavy && lane == leader) pos = atomicAdd(&h_cur[size_t(side) * h_max + hid], (uint32_t)__popc(peers));
-            pos = __shfl_sync(kFull, pos, leader) + __popc(peers & ltm);
-            if (heavy) {
-                uint32_t* dst = side ? heavy_pay_s : heavy_pay_r;
-                dst[h_off[size_t(side) * h_stride + hid] + pos] = t.y;
-            }
-            // normal: compact into the normal remainder of this large partition
-            const bool normal = valid && hid == kNoHeavy;
+        const uint2* pr = v.part[0] + v.start[r.p];
+        const uint2* ps = v.part[1] + v.start[size_t(v.F) + 1 + r.p];
+        uint2 t[kSplitIpt];
+        // rk: skewed = shared slot << 16 | rank; normal = 1 << 31 | side << 16 | rank; none = ~0
+        uint32_t rk[kSplitIpt];
 #pragma unroll
-            for (int sd = 0; sd < 2; ++sd) {
-                const uint32_t m = __ballot_sync(kFull, normal && side == sd);
-                if (m == 0) continue;
-                const uint32_t lead = __ffs(m) - 1;
-                uint32_t b = 0;
-                if (lane == lead) b = atomicAdd(&nrm_cur[size_t(sd) * v.F + r.li], (uint32_t)__popc(m));
-                b = __shfl_sync(kFull, b, lead);
-                if (normal && side == sd) {
-                    uint2* dst = sd ? out_s : out_r;
-                    dst[nrm_off[size_t(sd) * (v.F + 1) + r.li] + b + __popc(m & ltm)] = t;
-                }
+        for (int j = 0; j < kSplitIpt; ++j) {
+            const uint64_t e = r.e0 + uint64_t(j) * kDetBlock + threadIdx.x;
+            t[j] = e < r.e1 ? (e < r.cr ? pr[e] : ps[e - r.cr]) : make_uint2(0, 0);
+        }
+        // skewed-key ids: the first probe of every tuple is issued before any is resolved (the
+        // table holds only possible skewed keys, so most first probes find an empty slot)
+        uint32_t probe0 = 0;   // 2 bits per tuple: 0 = first slot empty (normal), 1 = found there, 2 = probe on
+        {
+            unsigned long long w0[kSplitIpt];
+#pragma unroll
+            for (int j = 0; j < kSplitIpt; ++j) w0[j] = gt_key[gt_slot0(t[j].x, logcap)];
+#pragma unroll
+            for (int j = 0; j < kSplitIpt; ++j) {
+                const uint32_t st2 = w0[j] == ((1ull << 32) | t[j].x) ? 1u : (w0[j] == 0 ? 0u : 2u);
+                probe0 |= st2 << (2 * j);
             }
         }
+        // Ranks: normal tuples by one shared atomic per (warp, side); skewed tuples of the warp's
+        // reference key by one shared atomic per warp (lanes ranked by ballot prefix); other skewed
+        // tuples one shared atomic each, the reference moving to one of their keys whenever it
+        // matched fewer than 8 lanes (skewed items are dominated by one key).
+        uint32_t ref = 0, ref_slot = 0;   // warp-uniform; key 0 = none
+        const uint32_t lane = lane_id(), ltm = lanemask_lt();
+#pragma unroll
+        for (int j = 0; j < kSplitIpt; ++j) {
+            const uint64_t e = r.e0 + uint64_t(j) * kDetBlock + threadIdx.x;
+            const bool valid = e < r.e1;
+            const uint32_t side = e >= r.cr;
+            const uint32_t st2 = (probe0 >> (2 * j)) & 3u;
+            uint32_t g = kNoHeavy;
+            if (valid && st2) g = st2 == 1 ? gt_slot0(t[j].x, logcap) : gt_find(gt_key, t[j].x, logcap);
+            const uint32_t id = g == kNoHeavy ? kNoHeavy : gt_hid[g];
+            const bool heavy = valid && id != kNoHeavy;
+            const uint32_t key = heavy ? ((id << 1 | side) + 1) : 0u;
+            uint32_t rr = 0xffffffffu;
+#pragma unroll
+            for (uint32_t sd = 0; sd < 2; ++sd) {
+                const uint32_t m = __ballot_sync(kFull, valid && !heavy && side == sd);
+                if (m) {
+                    const uint32_t lead = __ffs(m) - 1;
+                    uint32_t b = 0;
+                    if (lane == lead) b = atomicAdd(&s_nrm[sd], (uint32_t)__popc(m));
+                    b = __shfl_sync(kFull, b, lead);
+                    if ((m >> lane) & 1u) rr = 1u << 31 | sd << 16 | (b + __popc(m & ltm));
+                }
+            }
+            const uint32_t mr = __ballot_sync(kFull, heavy && key == ref);
+            if (mr) {
+                const uint32_t lead = __ffs(mr) - 1;
+                uint32_t b = 0;
+                if (lane == lead) b = atomicAdd(&s_cnt[ref_slot], (uint32_t)__popc(mr));
+                b = __shfl_sync(kFull, b, lead);
+                if ((mr >> lane) & 1u) rr = ref_slot << 16 | (b + __popc(mr & ltm));
+            }
+            const bool other = heavy && key != ref;
+            if (other) {
+                uint32_t slot = (key * 0x9E3779B1u) >> (32 - 12);   // kSplitHidSlots = 2^12
+                for (;;) {   // an item has <= kDetectChunk distinct keys: a free slot always exists
+                    const uint32_t cur = s_key[slot];
+                    if (cur == key) break;
+                    if (cur == 0) {
+                        const uint32_t prev = atomicCAS(&s_key[slot], 0u, key);
+                        if (prev == 0 || prev == key) break;
+                    }
+                    slot = (slot + 1) & (kSplitHidSlots - 1);
+                }
+                rr = slot << 16 | atomicAdd(&s_cnt[slot], 1u);
+            }
+            const uint32_t mo = __ballot_sync(kFull, other);
+            if (__popc(mr) < 8 && mo) {
+                const uint32_t lead = __ffs(mo) - 1;
+                ref = __shfl_sync(kFull, key, lead);
+                ref_slot = __shfl_sync(kFull, rr >> 16, lead);
+            }
+            rk[j] = rr;
+        }
+        __syncthreads();
+        // reserve this item's runs: one global atomic per distinct (side, key) and per side
+        for (uint32_t i = threadIdx.x; i < kSplitHidSlots; i += kDetBlock) {
+            const uint32_t key = s_key[i];
+            if (key) {
+                const uint32_t id = (key - 1) >> 1, side = (key - 1) & 1u;
+                s_cnt[i] = atomicAdd(&h_cur[size_t(side) * h_max + id], s_cnt[i]);
+            }
+        }
+        if (threadIdx.x < 2 && s_nrm[threadIdx.x])
+            s_nbase[threadIdx.x] = atomicAdd(&nrm_cur[size_t(threadIdx.x) * v.F + r.li], s_nrm[threadIdx.x]);
+        __syncthreads();
+#pragma unroll
+        for (int j = 0; j < kSplitIpt; ++j) {
+            if (rk[j] == 0xffffffffu) continue;
+            const uint32_t rank = rk[j] & 0xffffu;
+            if (rk[j] >> 31) {
+                const uint32_t side = (rk[j] >> 16) & 1u;
+                uint2* dst = side ? out_s : out_r;
+                dst[nrm_off[size_t(side) * (v.F + 1) + r.li] + s_nbase[side] + rank] = t[j];
+            } else {
+                const uint32_t slot = rk[j] >> 16;
+                const uint32_t key = s_key[slot] - 1;
+                uint32_t* dst = (key & 1u) ? heavy_pay_s : heavy_pay_r;
+                dst[h_off[size_t(key & 1u) * h_stride + (key >> 1)] + s_cnt[slot] + rank] = t[j].y;
+            }
+        }
+        __syncthreads();
+        // clear the slots this item used (each thread its own tuples' slots; repeats are harmless)
+#pragma unroll
+        for (int j = 0; j < kSplitIpt; ++j) {
+            if ((rk[j] >> 31) == 0) {
+                s_key[rk[j] >> 16] = 0;
+                s_cnt[rk[j] >> 16] = 0;
+            }
+        }
+        if (threadIdx.x < 2) s_nrm[threadIdx.x] = 0;
     }
 }
 
@@ -405,10 +658,15 @@ int launch_split(const Plan& p, uint32_t n_large, uint32_t gt_cap, cudaStream_t 
     if (n_large == 0) return 0;
     uint32_t logcap = 0;
     while ((1u << logcap) < gt_cap) ++logcap;
-    LargeView v{{p.bufB[0], p.bufB[1]}, p.start, p.cnt, p.large_list, p.det_prefix, p.F, n_large};
-    k_split<<<p.num_sms * 8, kDetBlock, 0, s>>>(v, p.gt_key, p.gt_hid, logcap, p.h_off, p.h_max + 1, p.h_cur,
-                                                (uint32_t)p.h_max, p.heavy_pay[0], p.heavy_pay[1], p.nrm_off,
-                                                p.nrm_cur, p.bufA[0], p.bufA[1], &p.st->claim[3]);
+    static std::once_flag attr_once[kMaxDevices];
+    once_per_device(attr_once, [] {
+        cudaFuncSetAttribute(k_split, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSplitSmemBytes);
+    });
+    LargeView v{{p.bufB[0], p.bufB[1]}, p.start, p.cnt, p.large_list, p.det_prefix, p.F, n_large, kDetectChunk};
+    k_split<<<p.num_sms * 4, kDetBlock, kSplitSmemBytes, s>>>(v, p.gt_key, p.gt_hid, logcap, p.h_off, p.h_max + 1,
+                                                             p.h_cur, (uint32_t)p.h_max, p.heavy_pay[0],
+                                                             p.heavy_pay[1], p.nrm_off, p.nrm_cur, p.bufA[0],
+                                                             p.bufA[1], &p.st->claim[3]);
     return 1;
 }
 

@@ -19,7 +19,7 @@ from ._lib import GshConfig, GshOutput, GshRelation, GshResult, check, load
 def make_config(capacity: int = 0, pass_bits=None, heavy_threshold: int = 0, route_bits: int = 0,
                 force_all_normal: bool = False, force_all_heavy: bool = False, timing: bool = False,
                 large_threshold: int = 0, nm_table: int = 0, detect_mode: int = 0, sample_stride: int = 0,
-                top_k: int = 0, prepass_bits: int = 0) -> GshConfig:
+                top_k: int = 0, prepass_bits: int = 0, input_side_only: bool = False) -> GshConfig:
     """Build a gsh_config (see include/gsh.h for each field's meaning)."""
     cfg = _lib.default_config()
     cfg.capacity = int(capacity)
@@ -37,6 +37,7 @@ def make_config(capacity: int = 0, pass_bits=None, heavy_threshold: int = 0, rou
     cfg.sample_stride = int(sample_stride)
     cfg.top_k = int(top_k)
     cfg.prepass_bits = int(prepass_bits)
+    cfg.input_side_only = int(bool(input_side_only))
     return cfg
 
 

@@ -211,9 +211,19 @@ def test_join_prepass_exact(kind, n, theta, bits):
     r = gsh.join(*d, config=gsh.make_config(prepass_bits=bits, timing=True))
     assert (r.count, r.checksum) == (on, oc)
     assert r.stats["prepass_bits"] == bits and r.stats["ms_prepass"] > 0
-    m = gsh.join(*d, mode="materialize", out_capacity=on + 3, config=gsh.make_config(prepass_bits=bits, route_bits=2))
+    m = gsh.join(*d, mode="materialize", out_capacity=on + 3, config=gsh.make_config(prepass_bits=bits))
     assert (m.count, m.checksum, m.written, m.overflow) == (on, oc, on, False)
     assert np.array_equal(_sorted_pairs(m.pairs), op)
+    # below routing bits: a shard whose tuples all share the top 2 bits of h (route_bits asserts it)
+    u = lambda t: t.numpy().view(np.uint32)  # noqa: E731
+    kr = (oracle.fmix32(u(rk)) >> 30) == 2
+    ks = (oracle.fmix32(u(sk)) >> 30) == 2
+    sh = [t[torch.from_numpy(m_)] for t, m_ in ((rk, kr), (rp, kr), (sk, ks), (sp, ks))]
+    on2, oc2, op2 = _oracle(*sh, pairs=True)
+    m2 = gsh.join(*_dev(*sh), mode="materialize", out_capacity=on2 + 3,
+                  config=gsh.make_config(prepass_bits=bits, route_bits=2))
+    assert (m2.count, m2.checksum, m2.written, m2.overflow) == (on2, oc2, on2, False)
+    assert np.array_equal(_sorted_pairs(m2.pairs), op2)
 
 
 @pytest.mark.parametrize("bits", [2, 3])
