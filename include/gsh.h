@@ -114,6 +114,9 @@ typedef struct {
                                   (L106).  0 = auto (enough bits that each side's share is
                                   <= 2^28 tuples; none up to 2^28);  -1 = off;  1..8 = forced.
                                   The result never depends on it. */
+    int32_t heavy_detail;      /* test hook: the skewed-key join also sums
+                                  each skewed key's checksum share C_k into the workspace, read
+                                  back with gsh_heavy_detail.  Not with the pre-partition pass. */
     int32_t input_side_only;   /* measurement hook: run the input side (partition, classify,
                                   detect, split) and stop before the NM-join and the skewed-key
                                   join; count / checksum / written are then 0.  Used to time the
@@ -190,6 +193,19 @@ GSH_API size_t gsh_host_workspace_bytes(uint64_t n_r, uint64_t n_s, gsh_out_mode
 GSH_API gsh_status gsh_join_host(const gsh_relation *R, const gsh_relation *S, gsh_out_mode mode,
                          const gsh_output *out, void *workspace, size_t workspace_bytes,
                          const gsh_config *cfg, void *stream, gsh_result *res);
+
+/* Decomposition of the last gsh_join on this workspace (cfg->heavy_detail = 1, COUNT or
+ * MATERIALIZE, no pre-partition pass): for every skewed key k (unspecified
+ * order) h_keys[k] = fmix32(key), h_cnt_r / h_cnt_s = its tuple counts, h_chk[k] = C_k =
+ * sum of pair_hash over R_k x S_k mod 2^64 (host arrays of cap entries); *h_n = number of
+ * skewed keys.  With gsh_result.normal_count / normal_checksum this splits the result into the
+ * NM-join's share and one term per skewed key: count = normal_count + sum cnt_r * cnt_s,
+ * checksum = normal_checksum + sum C_k.  n_r, n_s and cfg must be those of the join.
+ * GSH_ERR_INVALID if more than cap keys or the join did not run with heavy_detail. */
+GSH_API gsh_status gsh_heavy_detail(uint64_t n_r, uint64_t n_s, const gsh_config *cfg,
+                                    void *workspace, size_t workspace_bytes, void *stream,
+                                    uint32_t *h_keys, uint32_t *h_cnt_r, uint32_t *h_cnt_s,
+                                    uint64_t *h_chk, uint64_t cap, uint64_t *h_n);
 
 /* ---------------------------------------------------------------- step entry points --
  * Individual phases exposed for per-kernel parity tests and the multi-GPU driver.

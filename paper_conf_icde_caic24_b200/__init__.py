@@ -14,6 +14,7 @@ from .join import (  # noqa: F401
     detect,
     hash_keys,
     join,
+    join_detail,
     join_host,
     make_config,
     partition,

@@ -48,6 +48,7 @@ class GshConfig(ctypes.Structure):
         ("sample_stride", u32),
         ("top_k", u32),
         ("prepass_bits", i32),
+        ("heavy_detail", i32),
         ("input_side_only", i32),
     ]
 
@@ -118,6 +119,8 @@ _PROTOS = [
     ("gsh_join_host", ctypes.c_int, [ctypes.POINTER(GshRelation), ctypes.POINTER(GshRelation), ctypes.c_int,
                                      ctypes.POINTER(GshOutput), vp, ctypes.c_size_t, ctypes.POINTER(GshConfig), vp,
                                      ctypes.POINTER(GshResult)]),
+    ("gsh_heavy_detail", ctypes.c_int, [u64, u64, ctypes.POINTER(GshConfig), vp, ctypes.c_size_t, vp, p32, p32, p32,
+                                        p64, u64, p64]),
     ("gsh_hash_keys", ctypes.c_int, [vp, vp, u64, vp]),
     ("gsh_radix_histogram", ctypes.c_int, [vp, u64, u32, u32, vp, vp, ctypes.c_size_t, vp]),
     ("gsh_partition", ctypes.c_int, [ctypes.POINTER(GshRelation), ctypes.POINTER(GshRelation),

@@ -121,6 +121,7 @@ bool plan_build(Plan& p, uint64_t nR, uint64_t nS, const gsh_config* cfg_in, voi
     }
     p.force_normal = cfg.force_all_normal;
     p.input_only = cfg.input_side_only;
+    p.detail = cfg.heavy_detail;
     p.force_heavy = cfg.force_all_heavy;
     p.timing = cfg.timing;
     if (cfg.nm_table < 0 || cfg.nm_table > 2) return false;
@@ -210,6 +211,7 @@ bool plan_build(Plan& p, uint64_t nR, uint64_t nS, const gsh_config* cfg_in, voi
     p.H = c.take<HeavyKey>(p.h_max);
     p.h_off = c.take<uint64_t>(2 * (p.h_max + 1));
     p.h_tiles = c.take<uint64_t>(p.h_max + 1);
+    p.h_chk = c.take<unsigned long long>(p.detail ? p.h_max : 0);
     p.h_cur = c.take<uint32_t>(2 * p.h_max);
     p.nm = c.take<NmPart>(F);
     p.nm_prefix = c.take<uint64_t>(F + 1);
@@ -474,6 +476,7 @@ static gsh_status join_direct(const gsh_relation* R, const gsh_relation* S, gsh_
         n_heavy = hs.n_heavy;
         if (hs.heavy_overflow || n_heavy > p.h_max) return fail(GSH_ERR_INTERNAL, "skewed-key list overflow");
         launches += launch_heavy_prefix(p, n_heavy, n_large, s);
+        if (p.detail && n_heavy) cudaMemsetAsync(p.h_chk, 0, size_t(n_heavy) * 8, s);
         launches += launch_split(p, n_large, (uint32_t)gcap, s);
         e5 = tm.mark();
     }
@@ -554,6 +557,7 @@ gsh_status gsh_join(const gsh_relation* R, const gsh_relation* S, gsh_out_mode m
     if (r < 0) return fail(GSH_ERR_INVALID, "invalid gsh_config (prepass_bits)");
     if (r == 0 || R->n == 0 || S->n == 0)
         return join_direct(R, S, mode, out, workspace, workspace_bytes, cfg, stream, res);
+    if (cfg && cfg->heavy_detail) return fail(GSH_ERR_INVALID, "heavy_detail is not available with the pre-partition pass");
     if (mode != GSH_OUT_COUNT && mode != GSH_OUT_MATERIALIZE) return fail(GSH_ERR_INVALID, "bad mode");
     const bool mat = (mode == GSH_OUT_MATERIALIZE);
     if (mat && (!out || (!out->pairs && out->capacity > 0)))
@@ -718,6 +722,42 @@ gsh_status gsh_join_host(const gsh_relation* R, const gsh_relation* S, gsh_out_m
         ce = cudaMemcpyAsync(out->pairs, dp, res->written * 8, cudaMemcpyDeviceToHost, s);
         if (ce == cudaSuccess) ce = cudaStreamSynchronize(s);
         if (ce != cudaSuccess) return cuda_fail(ce, "D2H");
+    }
+    return GSH_OK;
+}
+
+gsh_status gsh_heavy_detail(uint64_t n_r, uint64_t n_s, const gsh_config* cfg, void* workspace, size_t workspace_bytes,
+                            void* stream, uint32_t* h_keys, uint32_t* h_cnt_r, uint32_t* h_cnt_s, uint64_t* h_chk,
+                            uint64_t cap, uint64_t* h_n) {
+    if (!cfg || !cfg->heavy_detail || !h_n || (cap && (!h_keys || !h_cnt_r || !h_cnt_s || !h_chk)))
+        return fail(GSH_ERR_INVALID, "heavy_detail config and output arrays required");
+    if (prepass_bits_for(n_r, n_s, cfg) > 0) return fail(GSH_ERR_INVALID, "heavy_detail: pre-partition pass active");
+    Plan p;
+    if (!plan_build(p, n_r, n_s, cfg, nullptr, device_sms())) return fail(GSH_ERR_INVALID, "invalid gsh_config");
+    if (!workspace || workspace_bytes < p.bytes || (reinterpret_cast<uintptr_t>(workspace) & 255u))
+        return fail(GSH_ERR_INVALID, "workspace NULL, misaligned or too small");
+    plan_build(p, n_r, n_s, cfg, workspace, device_sms());
+    cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+    DevState hs;
+    cudaError_t ce = cudaMemcpyAsync(&hs, p.st, sizeof(DevState), cudaMemcpyDeviceToHost, s);
+    if (ce == cudaSuccess) ce = cudaStreamSynchronize(s);
+    if (ce != cudaSuccess) return cuda_fail(ce, "detail sync");
+    const uint32_t nh = hs.n_large ? hs.n_heavy : 0u;
+    *h_n = nh;
+    if (nh > cap) return fail(GSH_ERR_INVALID, "capacity too small (see *h_n)");
+    if (nh) {
+        std::vector<HeavyKey> hk(nh);
+        std::vector<unsigned long long> ck(nh);
+        ce = cudaMemcpyAsync(hk.data(), p.H, nh * sizeof(HeavyKey), cudaMemcpyDeviceToHost, s);
+        if (ce == cudaSuccess) ce = cudaMemcpyAsync(ck.data(), p.h_chk, nh * 8, cudaMemcpyDeviceToHost, s);
+        if (ce == cudaSuccess) ce = cudaStreamSynchronize(s);
+        if (ce != cudaSuccess) return cuda_fail(ce, "detail copy");
+        for (uint32_t i = 0; i < nh; ++i) {
+            h_keys[i] = hk[i].h;
+            h_cnt_r[i] = hk[i].cnt_r;
+            h_cnt_s[i] = hk[i].cnt_s;
+            h_chk[i] = ck[i];
+        }
     }
     return GSH_OK;
 }

@@ -129,7 +129,7 @@ struct Plan {
     uint32_t C = 4096, Th = 64, L = 4096;  // NM capacity, skew-key threshold, large-partition threshold
     uint32_t nm_slots = 0;          // NM build-table slots (set after classification; 0 = from C)
     uint32_t F = 1;                 // 1 << (b1 + b2)
-    int force_normal = 0, force_heavy = 0, timing = 0, input_only = 0;
+    int force_normal = 0, force_heavy = 0, timing = 0, input_only = 0, detail = 0;
     int nm_table = 0;               // config: 0 auto, 1 CSR, 2 chained where possible
     int nm_chain = 0;               // chosen for this call (nm_ring.cu)
     int detect_mode = 0;            // 0 exact counts, 1 sampled top-k (L107, L112)
@@ -172,6 +172,7 @@ struct Plan {
     HeavyKey* H = nullptr;                    // [h_max]
     uint64_t* h_off = nullptr;                // [2][h_max + 1]
     uint64_t* h_tiles = nullptr;              // [h_max + 1]
+    unsigned long long* h_chk = nullptr;      // [h_max] per skewed key checksum share (heavy_detail)
     uint32_t* h_cur = nullptr;                // [2][h_max] split cursors
     uint32_t* nrm_cur = nullptr;              // [2][F]     split cursors (normal)
     NmPart* nm = nullptr;                     // [F]
@@ -202,7 +203,7 @@ int launch_nm_setup(const Plan& p, uint32_t n_large, cudaStream_t s);
 int launch_nmjoin(const Plan& p, int materialize, uint32_t* pairs, uint64_t cap, cudaStream_t s);
 int launch_nmjoin_ring(const Plan& p, int materialize, uint32_t* pairs, uint64_t cap, cudaStream_t s);
 int launch_skewjoin(const Plan& p, uint32_t n_heavy, int materialize, uint32_t* pairs, uint64_t cap,
-                    cudaStream_t s);
+                    cudaStream_t s);   // p.detail: also per-key checksum shares into p.h_chk
 
 // Routing (multi-GPU)
 int launch_route_count(const uint32_t* keys, uint64_t n, uint32_t rb, const uint32_t* hk, uint64_t nh,

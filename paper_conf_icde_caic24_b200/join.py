@@ -19,7 +19,8 @@ from ._lib import GshConfig, GshOutput, GshRelation, GshResult, check, load
 def make_config(capacity: int = 0, pass_bits=None, heavy_threshold: int = 0, route_bits: int = 0,
                 force_all_normal: bool = False, force_all_heavy: bool = False, timing: bool = False,
                 large_threshold: int = 0, nm_table: int = 0, detect_mode: int = 0, sample_stride: int = 0,
-                top_k: int = 0, prepass_bits: int = 0, input_side_only: bool = False) -> GshConfig:
+                top_k: int = 0, prepass_bits: int = 0, input_side_only: bool = False,
+                heavy_detail: bool = False) -> GshConfig:
     """Build a gsh_config (see include/gsh.h for each field's meaning)."""
     cfg = _lib.default_config()
     cfg.capacity = int(capacity)
@@ -38,6 +39,7 @@ def make_config(capacity: int = 0, pass_bits=None, heavy_threshold: int = 0, rou
     cfg.top_k = int(top_k)
     cfg.prepass_bits = int(prepass_bits)
     cfg.input_side_only = int(bool(input_side_only))
+    cfg.heavy_detail = int(bool(heavy_detail))
     return cfg
 
 
@@ -278,3 +280,30 @@ def detect(r_keys, r_payloads, s_keys, s_payloads, config: GshConfig | None = No
     b = torch.tensor(list(cs[:m]), dtype=torch.int64)
     order = torch.argsort(h)
     return h[order], a[order], b[order], res.as_dict()
+
+
+def join_detail(r_keys, r_payloads, s_keys, s_payloads, config: GshConfig | None = None, stream=None):
+    """COUNT join with the skewed-key decomposition (gsh_config.heavy_detail +
+    gsh_heavy_detail): returns (JoinResult, detail) where detail = dict of int64 CPU tensors
+    h, cnt_r, cnt_s and uint64-valued checksum (C_k as Python ints in a list), one entry per
+    skewed key.  result.count == normal_count + sum(cnt_r * cnt_s) and result.checksum ==
+    normal_checksum + sum(C_k) mod 2^64."""
+    lib = load()
+    cfg = make_config(heavy_detail=True) if config is None else config
+    cfg.heavy_detail = 1
+    rk, rp = _check_dev(r_keys, "r_keys"), _check_dev(r_payloads, "r_payloads")
+    sk, sp = _check_dev(s_keys, "s_keys"), _check_dev(s_payloads, "s_payloads")
+    dev = rk.device
+    ws = torch.empty(workspace_bytes(rk.numel(), sk.numel(), cfg), dtype=torch.uint8, device=dev)
+    r = join(rk, rp, sk, sp, config=cfg, stream=stream, workspace=ws)
+    cap = max(1, int(r.stats["n_heavy"]))
+    hk, cr, cs = (ctypes.c_uint32 * cap)(), (ctypes.c_uint32 * cap)(), (ctypes.c_uint32 * cap)()
+    ck = (ctypes.c_uint64 * cap)()
+    n = ctypes.c_uint64(0)
+    with torch.cuda.device(dev):
+        check(lib.gsh_heavy_detail(rk.numel(), sk.numel(), ctypes.byref(cfg), ws.data_ptr(), ws.numel(),
+                                   _stream_handle(stream, dev), hk, cr, cs, ck, cap, ctypes.byref(n)), "gsh_heavy_detail")
+    m = int(n.value)
+    detail = {"h": torch.tensor(list(hk[:m]), dtype=torch.int64), "cnt_r": torch.tensor(list(cr[:m]), dtype=torch.int64),
+              "cnt_s": torch.tensor(list(cs[:m]), dtype=torch.int64), "checksum": [int(x) for x in ck[:m]]}
+    return r, detail
