@@ -70,7 +70,7 @@ constexpr uint32_t kRingItemMax = kRingBytes / 2;
 constexpr uint32_t kRingMaxRChain = 8190;
 __host__ __device__ __forceinline__ bool ring_eligible(uint32_t rl, uint32_t sl, bool chain) {
     return rl > 0 && sl > 0 && rl <= (chain ? kRingMaxRChain : kRingMaxR) &&
-           (uint64_t(rl) + sl) * 8 + 32 <= kRingItemMax;
+           (uint64_t(rl) + sl) * 8 + 32 + 48 <= kRingItemMax;   // + alignment + per-item slack
 }
 constexpr int kSkewBlock = 256;                 // skewed-key join CTA
 constexpr int kSkewSpt = 4;                     // S payloads per thread (registers)

@@ -589,6 +589,7 @@ __global__ void __launch_bounds__(BLOCK, 2) k_scatter(ScatterArgs a) {
     }
     __syncthreads();
     uint32_t u = S.claim;
+    __syncthreads();   // every thread has read the first claim before thread 0 claims again
     uint32_t par = 0;
     bool issued = false;   // first tile of unit u already in flight
     while (u < total) {

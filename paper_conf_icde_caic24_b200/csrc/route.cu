@@ -303,19 +303,26 @@ __global__ void __launch_bounds__(kSplitBlock, 2) k_split_scatter_tiles(
             for (int g = 0; g < G; ++g) s_wc[warp][g] = wc[g];
         }
         __syncthreads();
-        if (threadIdx.x < G) {
+        if (threadIdx.x < G) {   // bucket g: per-warp counts -> per-warp bases, and the total
             const uint32_t g = threadIdx.x;
-            uint32_t before = 0;   // tuples of the tile in buckets < g
-            for (uint32_t h = 0; h < g; ++h)
-                for (int w = 0; w < kSplitWarps; ++w) before += s_wc[w][h];
-            pre[g] = before;
             uint32_t acc = 0;
             for (int w = 0; w < kSplitWarps; ++w) {
                 const uint32_t c = s_wc[w][g];
                 s_wc[w][g] = acc;
                 acc += c;
             }
+            pre[g] = acc;
             base[g] = off[g] + (tpfx[uint64_t(g) * ntiles + t] - tpfx[uint64_t(g) * ntiles]);
+        }
+        __syncthreads();
+        if (threadIdx.x == 0) {   // totals -> tile-local bucket starts (G <= 8)
+            uint32_t run = 0;
+#pragma unroll
+            for (int g = 0; g < G; ++g) {
+                const uint32_t c = pre[g];
+                pre[g] = run;
+                run += c;
+            }
         }
         __syncthreads();
 #pragma unroll
