@@ -365,3 +365,4 @@ def test_join_sampled_detection_exact(kind, n, theta, nmat):
     m = gsh.join(*d, mode="materialize", out_capacity=on, config=cfg)
     assert (m.count, m.checksum, m.written) == (on, oc, on)
     assert np.array_equal(_sorted_pairs(m.pairs), op)
+
