@@ -48,6 +48,7 @@ WORKLOADS = {
     "pkfk28": ("pkfk", 1 << 28, 0.0, "scale point: |R|=|S|=2^28 uniform 1:1 PK-FK (cfg5's per-GPU share at G=8), COUNT"),
     "pkfk29": ("pkfk", 1 << 29, 0.0, "scale point: |R|=|S|=2^29 uniform 1:1 PK-FK (4x cfg2; 2^30 input tuples), COUNT"),
     "pkfk30": ("pkfk", 1 << 30, 0.0, "scale point: |R|=|S|=2^30 uniform 1:1 PK-FK (8x cfg2; 2^31 input tuples), COUNT"),
+    "zipf07_29": ("zipf", 1 << 29, 0.7, "NEXT-3 (PAPER.md L170: 560M x 560M, theta=0.7) on one B200: |R|=|S|=2^29 Zipf theta=0.7 both sides, COUNT"),
     "pkfkzipf": ("pkfk_zipf", 1 << 27, 1.0, "skewed-FK PK-FK: |R|=|S|=2^27, R unique, S Zipf theta=1.0 over R's rows, COUNT"),
 }
 

@@ -4,6 +4,8 @@
 // (S_k stays local, R_k is all-gathered by the driver), so no GPU receives a skewed key's S.
 //
 // Skewed keys are identified by their hash h (fmix32 is a bijection), sorted ascending.
+#include <type_traits>
+
 #include "gsh_device.cuh"
 #include "gsh_internal.h"
 #include "gsh_scan.cuh"
@@ -20,7 +22,7 @@ namespace gsh {
 // (warp, bucket) and one global cursor atomic per (tile, bucket).
 
 __device__ __forceinline__ uint32_t split_dest(uint32_t k, uint32_t skip, uint32_t rb) {
-    return (hash32(k) << skip) >> (32 - rb);
+    return (hash32_top(k) << skip) >> (32 - rb);   // skip + rb <= 16: the top half of h
 }
 
 // lanes of this warp holding the same bucket d (valid lanes only)
@@ -73,7 +75,7 @@ __global__ void __launch_bounds__(kSplitBlock) k_split_count(const uint32_t* __r
 // atomic per (warp, bucket)), reserve each bucket's run with one global atomic, permute the tile
 // into shared memory grouped by bucket, then write it out with consecutive threads on consecutive
 // addresses of a run (coalesced; only run ends touch partial sectors).
-constexpr size_t kSplitSmem = kSplitTile * (4 + 4 + 1);
+constexpr size_t kSplitSmem = kSplitTile * (4 + 4 + 1);   // k_split_scatter: keys, payloads, buckets
 
 __global__ void __launch_bounds__(kSplitBlock, 2) k_split_scatter(const uint32_t* __restrict__ keys,
                                                               const uint32_t* __restrict__ pays, uint64_t n,
@@ -208,138 +210,176 @@ __device__ __forceinline__ void split_load(const uint32_t* __restrict__ src, uin
 
 constexpr int kSplitWarps = kSplitBlock / 32;
 
+// Per-thread bucket counts of a tile live in one u64 of eight 8-bit fields (<= 16 elements per
+// thread): an element costs its hash, one shift and one add -- no ballots or popcounts.  Sums over
+// a warp or the tile widen the fields to 16 bits: word q of wide16() holds buckets 2q' and 2q'+2
+// (even bytes) or 2q'+1 and 2q'+3 (odd bytes) of each half.
+__device__ __forceinline__ void wide16(uint64_t c, uint32_t (&w)[4]) {
+    const uint32_t lo = uint32_t(c), hi = uint32_t(c >> 32);
+    w[0] = lo & 0x00ff00ffu;          // buckets 0, 2
+    w[1] = (lo >> 8) & 0x00ff00ffu;   // buckets 1, 3
+    w[2] = hi & 0x00ff00ffu;          // buckets 4, 6
+    w[3] = (hi >> 8) & 0x00ff00ffu;   // buckets 5, 7
+}
+// word and bit offset of bucket g in wide16()'s layout
+__device__ __forceinline__ uint32_t w16_word(uint32_t g) { return (g & 1u) | ((g >> 2) << 1); }
+__device__ __forceinline__ uint32_t w16_shift(uint32_t g) { return ((g >> 1) & 1u) << 4; }
+
 template <int RB, bool VEC>
 __global__ void __launch_bounds__(kSplitBlock, 2) k_split_count_tiles(const uint32_t* __restrict__ keys, uint64_t n,
                                                                      uint32_t skip, uint32_t* __restrict__ tile_cnt,
                                                                      unsigned long long* counts) {
     constexpr int G = 1 << RB;
-    __shared__ uint32_t s_wc[kSplitWarps][G];
+    constexpr int NWD = G <= 4 ? 2 : 4;   // 16-bit-field words in use
+    __shared__ uint32_t s_c[2][G];        // tile totals, double-buffered by tile parity
     const uint64_t ntiles = (n + kSplitTile - 1) / kSplitTile;
-    const uint32_t warp = threadIdx.x >> 5;
+    if (threadIdx.x < 2 * G) (&s_c[0][0])[threadIdx.x] = 0;
+    __syncthreads();
     // the next tile's keys are loaded while this tile's counts are reduced (k[] is free by then)
     uint32_t k[kSplitIpt];
     auto load = [&](uint64_t tt) {
         if (tt < ntiles) split_load<VEC>(keys, tt * kSplitTile, n, k);
     };
     load(blockIdx.x);
-    for (uint64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
+    for (uint64_t t = blockIdx.x, par = 0; t < ntiles; t += gridDim.x, par ^= 1) {
         const uint64_t t0 = t * kSplitTile;
-        uint32_t wc[G];
-#pragma unroll
-        for (int g = 0; g < G; ++g) wc[g] = 0;
+        using C = typename std::conditional<(G <= 4), uint32_t, uint64_t>::type;   // 8-bit fields
+        C c = 0;
 #pragma unroll
         for (int j = 0; j < kSplitIpt; ++j) {
             const bool v = split_elem<VEC>(t0, j) < n;
-            uint32_t eq[G];
-            split_masks<RB>(v, v ? split_dest(k[j], skip, RB) : 0u, eq);
-#pragma unroll
-            for (int g = 0; g < G; ++g) wc[g] += __popc(eq[g]);
+            c += v ? (C(1) << (8 * split_dest(k[j], skip, RB))) : C(0);
         }
         load(t + gridDim.x);
+        uint32_t w[4];
+        wide16(c, w);
+#pragma unroll
+        for (int q = 0; q < NWD; ++q) w[q] = __reduce_add_sync(kFull, w[q]);
         if (lane_id() == 0) {
 #pragma unroll
-            for (int g = 0; g < G; ++g) s_wc[warp][g] = wc[g];
+            for (int g = 0; g < G; ++g) {
+                const uint32_t x = (w[w16_word(g)] >> w16_shift(g)) & 0xffffu;
+                if (x) atomicAdd(&s_c[par][g], x);
+            }
         }
         __syncthreads();
-        if (threadIdx.x < G) {
-            uint32_t c = 0;
-            for (int w = 0; w < kSplitWarps; ++w) c += s_wc[w][threadIdx.x];
-            tile_cnt[uint64_t(threadIdx.x) * ntiles + t] = c;
-            if (c) atomicAdd(&counts[threadIdx.x], (unsigned long long)c);
+        if (threadIdx.x < G) {   // read and reset this parity's totals (reused two tiles later)
+            const uint32_t cg = s_c[par][threadIdx.x];
+            s_c[par][threadIdx.x] = 0;
+            tile_cnt[uint64_t(threadIdx.x) * ntiles + t] = cg;
+            if (cg) atomicAdd(&counts[threadIdx.x], (unsigned long long)cg);
         }
-        __syncthreads();
     }
 }
 
+// Scatter of one 8192-tuple tile: every element's bucket and its rank among the thread's own
+// elements of that bucket come from the packed counter; a block scan of the widened counters
+// gives each thread's offset per bucket; the tile is permuted into shared memory (bucket-grouped)
+// and written out with consecutive threads on consecutive addresses of each bucket's run (the
+// bucket of a staged position is found from the tile's bucket starts, so none is stored).
 template <int RB, bool VEC>
 __global__ void __launch_bounds__(kSplitBlock, 2) k_split_scatter_tiles(
     const uint32_t* __restrict__ keys, const uint32_t* __restrict__ pays, uint64_t n, uint32_t skip,
     const uint64_t* __restrict__ off, const uint64_t* __restrict__ tpfx, uint32_t* __restrict__ ok,
     uint32_t* __restrict__ op) {
     constexpr int G = 1 << RB;
+    constexpr int NWD = G <= 4 ? 2 : 4;
     extern __shared__ uint4 split_dyn[];
     uint32_t* s_k = reinterpret_cast<uint32_t*>(split_dyn);
     uint32_t* s_p = s_k + kSplitTile;
-    uint8_t* s_d = reinterpret_cast<uint8_t*>(s_p + kSplitTile);
-    __shared__ uint32_t s_wc[kSplitWarps][G];   // per-warp counts, then per-warp bases within the tile
-    __shared__ uint32_t pre[G];
+    __shared__ uint32_t s_wt[kSplitWarps][4];   // per-warp widened totals
+    __shared__ uint32_t pre[G + 1];
     __shared__ unsigned long long base[G];
     const uint64_t ntiles = (n + kSplitTile - 1) / kSplitTile;
-    const uint32_t warp = threadIdx.x >> 5;
+    const uint32_t warp = threadIdx.x >> 5, lane = lane_id();
     // the next tile is loaded into k[] / p[] before this tile's write-out (they are free once the
     // tile sits permuted in shared memory), so its load latency overlaps the stores
-    uint32_t k[kSplitIpt], p[kSplitIpt], dr[kSplitIpt];  // dr = bucket << 16 | rank in the warp
+    uint32_t k[kSplitIpt], p[kSplitIpt];
+    uint32_t dr[kSplitIpt / 4];   // byte j: bucket << 5 | rank among the thread's elements of that bucket
+    static_assert(kSplitIpt % 4 == 0 && kSplitIpt <= 31, "ranks fit 5 bits, four per word");
     auto load = [&](uint64_t tt) {
         if (tt < ntiles) {
             split_load<VEC>(keys, tt * kSplitTile, n, k);
             split_load<VEC>(pays, tt * kSplitTile, n, p);
         }
     };
-    const uint32_t lt = lanemask_lt();
     load(blockIdx.x);
     for (uint64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
         const uint64_t t0 = t * kSplitTile;
-        uint32_t wc[G];
-#pragma unroll
-        for (int g = 0; g < G; ++g) wc[g] = 0;
+        using C = typename std::conditional<(G <= 4), uint32_t, uint64_t>::type;   // 8-bit fields
+        C c = 0;
 #pragma unroll
         for (int j = 0; j < kSplitIpt; ++j) {
             const bool v = split_elem<VEC>(t0, j) < n;
-            const uint32_t d = v ? split_dest(k[j], skip, RB) : 0u;
-            uint32_t eq[G];
-            split_masks<RB>(v, d, eq);
-            uint32_t mine = 0, r0 = 0;
-#pragma unroll
-            for (int g = 0; g < G; ++g) {
-                const bool is = (uint32_t)g == d;
-                mine = is ? eq[g] : mine;
-                r0 = is ? wc[g] : r0;
-                wc[g] += __popc(eq[g]);
-            }
-            dr[j] = v ? (d << 16 | (r0 + __popc(mine & lt))) : 0xffffffffu;
+            const uint32_t d = split_dest(k[j], skip, RB);
+            const uint32_t b = d << 5 | uint32_t((c >> (8 * d)) & 0xffu);
+            if ((j & 3) == 0) dr[j >> 2] = 0;
+            dr[j >> 2] |= b << (8 * (j & 3));
+            c += v ? (C(1) << (8 * d)) : C(0);
         }
-        if (lane_id() == 0) {
+        // block exclusive scan of the widened counters (thread order)
+        uint32_t ex[4] = {0, 0, 0, 0};   // this thread's exclusive prefix per bucket (16-bit fields)
+        {
+            uint32_t w[4];
+            wide16(c, w);
 #pragma unroll
-            for (int g = 0; g < G; ++g) s_wc[warp][g] = wc[g];
+            for (int q = 0; q < NWD; ++q) {
+                uint32_t x = w[q];
+#pragma unroll
+                for (int o = 1; o < 32; o <<= 1) {
+                    const uint32_t y = __shfl_up_sync(kFull, x, o);
+                    if (lane >= (uint32_t)o) x += y;
+                }
+                ex[q] = x - w[q];
+                if (lane == 31) s_wt[warp][q] = x;
+            }
         }
         __syncthreads();
-        if (threadIdx.x < G) {   // bucket g: per-warp counts -> per-warp bases, and the total
-            const uint32_t g = threadIdx.x;
-            uint32_t acc = 0;
-            for (int w = 0; w < kSplitWarps; ++w) {
-                const uint32_t c = s_wc[w][g];
-                s_wc[w][g] = acc;
-                acc += c;
-            }
-            pre[g] = acc;
-            base[g] = off[g] + (tpfx[uint64_t(g) * ntiles + t] - tpfx[uint64_t(g) * ntiles]);
+        for (uint32_t v2 = 0; v2 < warp; ++v2) {
+#pragma unroll
+            for (int q = 0; q < NWD; ++q) ex[q] += s_wt[v2][q];
         }
-        __syncthreads();
-        if (threadIdx.x == 0) {   // totals -> tile-local bucket starts (G <= 8)
+        if (threadIdx.x == 0) {   // bucket starts inside the tile
+            uint32_t tot[4] = {0, 0, 0, 0};
+            for (int v2 = 0; v2 < kSplitWarps; ++v2) {
+#pragma unroll
+                for (int q = 0; q < NWD; ++q) tot[q] += s_wt[v2][q];
+            }
             uint32_t run = 0;
 #pragma unroll
             for (int g = 0; g < G; ++g) {
-                const uint32_t c = pre[g];
                 pre[g] = run;
-                run += c;
+                run += (tot[w16_word(g)] >> w16_shift(g)) & 0xffffu;
             }
+            pre[G] = run;
+        }
+        if (threadIdx.x < G) {
+            const uint32_t g = threadIdx.x;
+            base[g] = off[g] + (tpfx[uint64_t(g) * ntiles + t] - tpfx[uint64_t(g) * ntiles]);
         }
         __syncthreads();
 #pragma unroll
         for (int j = 0; j < kSplitIpt; ++j) {
-            if (dr[j] != 0xffffffffu) {
-                const uint32_t d = dr[j] >> 16, q = pre[d] + s_wc[warp][d] + (dr[j] & 0xffffu);
+            if (split_elem<VEC>(t0, j) < n) {
+                const uint32_t b = (dr[j >> 2] >> (8 * (j & 3))) & 0xffu, d = b >> 5;
+                const uint32_t wd = w16_word(d);   // register select, not a dynamically indexed array
+                const uint32_t e4 = wd == 0 ? ex[0] : wd == 1 ? ex[1] : wd == 2 ? ex[2] : ex[3];
+                const uint32_t q = pre[d] + ((e4 >> w16_shift(d)) & 0xffffu) + (b & 31u);
                 s_k[q] = k[j];
                 s_p[q] = p[j];
-                s_d[q] = (uint8_t)d;
             }
         }
         __syncthreads();
         load(t + gridDim.x);
         const uint32_t tn = (uint32_t)umin64(kSplitTile, n - t0);
+        uint32_t pr[G + 1];
+#pragma unroll
+        for (int g = 0; g <= G; ++g) pr[g] = pre[g];
         for (uint32_t i = threadIdx.x; i < tn; i += kSplitBlock) {
-            const uint32_t d = s_d[i];
-            const uint64_t pos = base[d] + (i - pre[d]);
+            uint32_t d = 0;
+#pragma unroll
+            for (int g = 1; g < G; ++g) d += i >= pr[g] ? 1u : 0u;
+            const uint64_t pos = base[d] + (i - pr[d]);
             ok[pos] = s_k[i];
             op[pos] = s_p[i];
         }

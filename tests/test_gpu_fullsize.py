@@ -152,3 +152,33 @@ def test_cfg3_theta075_count_fullsize():
     assert r.stats["n_heavy"] > 0 and r.stats["n_large"] > 0
     r2 = gsh.join(rk, rp, sk, sp, config=gsh.make_config(force_all_normal=True))
     assert (r2.count, r2.checksum) == (r.count, r.checksum)
+
+
+def _closed_form_gpu(rk, sk):
+    """sum_k cnt_R(k) cnt_S(k) from exact key histograms (torch.unique on the device: a library
+    sort, independent of the join's kernels)."""
+    ur, cr = torch.unique(rk.long() & 0xFFFFFFFF, return_counts=True)
+    us, cs = torch.unique(sk.long() & 0xFFFFFFFF, return_counts=True)
+    pos = torch.searchsorted(us, ur).clamp(max=us.numel() - 1)
+    hit = us[pos] == ur
+    return int((cr[hit] * cs[pos[hit]]).sum().item())
+
+
+def test_next3_theta07_2e29():
+    """the paper's large-input experiment (§V-B: 560 million
+    tuples per side, Zipf theta = 0.7) scaled to one B200: |R| = |S| = 2^29 (537M), both sides
+    Zipf theta = 0.7 with N = n.  Beyond 2^28 per side the pre-partition pass runs (auto 1 bit).
+    count = the closed form from exact histograms; the checksum is identical when the input is
+    split into 8 sub-problems instead (prepass_bits = 3): the same pairs through a different
+    decomposition."""
+    if torch.cuda.get_device_properties(0).total_memory < (96 << 30):
+        pytest.skip("needs a GPU with >= 96 GB")
+    n = 1 << 29
+    rk, rp, sk, sp = datagen.zipf_pair(n, n, 0.7, seed=0x6A5, device="cuda")
+    expect = _closed_form_gpu(rk, sk)
+    torch.cuda.empty_cache()
+    r = gsh.join(rk, rp, sk, sp)
+    assert r.count == expect
+    assert r.stats["prepass_bits"] == 1 and r.stats["n_heavy"] > 0
+    r2 = gsh.join(rk, rp, sk, sp, config=gsh.make_config(prepass_bits=3))
+    assert (r2.count, r2.checksum) == (r.count, r.checksum)
