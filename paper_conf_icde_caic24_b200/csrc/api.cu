@@ -206,6 +206,10 @@ bool plan_build(Plan& p, uint64_t nR, uint64_t nS, const gsh_config* cfg_in, voi
     p.part_heavy = c.take<uint32_t>(2 * F);
     p.det_prefix = c.take<uint64_t>(F + 1);
     p.det_prefix2 = c.take<uint64_t>(F + 1);
+    p.item_cap = (nR + nS) / kDetectChunk + F + 1;        // bound on split items (any large set)
+    p.item_cap2 = (nR + nS) / kDetectItem + F + 1;        // bound on exact-detect items
+    p.item_li = c.take<uint32_t>(p.item_cap);
+    p.item_li2 = c.take<uint32_t>(p.item_cap2);
     p.nrm_off = c.take<uint64_t>(2 * (F + 1));
     p.nrm_cur = c.take<uint32_t>(2 * F);
     p.H = c.take<HeavyKey>(p.h_max);
@@ -290,8 +294,8 @@ gsh_status check_launch(const char* where) {
 // Skew detection over the large partitions (L107, L112): exact counts of every key (detect_mode
 // 0), or the paper's sample + top-k per partition followed by exact counts of the chosen keys
 // (detect_mode 1); then the threshold pass that builds H.
-int run_detect(const Plan& p, uint32_t n_large, uint32_t gcap, cudaStream_t s) {
-    int l = launch_detect_prefix(p, n_large, s);
+int run_detect(const Plan& p, uint32_t n_large, uint64_t large_tuples, uint32_t gcap, cudaStream_t s) {
+    int l = launch_detect_prefix(p, n_large, large_tuples, s);
     if (p.detect_mode == 1) l += launch_sample_topk(p, n_large, gcap, s);
     l += launch_detect(p, n_large, gcap, s);
     l += launch_select(p, gcap, s);
@@ -467,7 +471,7 @@ static gsh_status join_direct(const gsh_relation* R, const gsh_relation* S, gsh_
         uint64_t gcap = next_pow2_u64(2 * (hs.large_tuples[0] + hs.large_tuples[1]));
         if (gcap < 1024) gcap = 1024;
         if (gcap > p.gt_cap_alloc) gcap = p.gt_cap_alloc;
-        launches += run_detect(p, n_large, (uint32_t)gcap, s);
+        launches += run_detect(p, n_large, hs.large_tuples[0] + hs.large_tuples[1], (uint32_t)gcap, s);
         e4 = tm.mark();
         if ((st = check_launch("detect")) != GSH_OK) return st;
         ce = cudaMemcpyAsync(&hs, p.st, sizeof(DevState), cudaMemcpyDeviceToHost, s);
@@ -824,7 +828,7 @@ gsh_status gsh_detect(const gsh_relation* R, const gsh_relation* S, const gsh_co
         uint64_t gcap = next_pow2_u64(2 * (hs.large_tuples[0] + hs.large_tuples[1]));
         if (gcap < 1024) gcap = 1024;
         if (gcap > p.gt_cap_alloc) gcap = p.gt_cap_alloc;
-        run_detect(p, hs.n_large, (uint32_t)gcap, s);
+        run_detect(p, hs.n_large, hs.large_tuples[0] + hs.large_tuples[1], (uint32_t)gcap, s);
         if ((st = check_launch("detect")) != GSH_OK) return st;
         ce = cudaMemcpyAsync(&hs, p.st, sizeof(DevState), cudaMemcpyDeviceToHost, s);
         if (ce == cudaSuccess) ce = cudaStreamSynchronize(s);

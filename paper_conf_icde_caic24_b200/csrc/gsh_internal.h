@@ -77,6 +77,7 @@ constexpr int kSkewSpt = 4;                     // S payloads per thread (regist
 constexpr int kSkewTileS = kSkewBlock * kSkewSpt;  // 1024
 constexpr int kSkewTileR = 64;                  // R payloads per tile (shared memory)
 constexpr uint32_t kDetectChunk = 2048;         // tuples per split (and sampled-detect) work item
+constexpr uint32_t kDetectItem = 16384;         // tuples per exact-detect work item
 constexpr uint32_t kNoHeavy = 0xffffffffu;
 constexpr int kDetectMaxProbe = 64;   // a full table degrades to "normal", never to a long probe
 
@@ -168,6 +169,9 @@ struct Plan {
     uint32_t* part_heavy = nullptr;           // [2][F]  skewed tuples per partition
     uint64_t* det_prefix = nullptr;           // [F + 1] split (and sampled-detect) items per large partition
     uint64_t* det_prefix2 = nullptr;          // [F + 1] exact-detect items per large partition
+    uint32_t* item_li = nullptr;              // [item_cap]  split item -> large partition index
+    uint32_t* item_li2 = nullptr;             // [item_cap2] exact-detect item -> large partition index
+    uint64_t item_cap = 0, item_cap2 = 0;
     uint64_t* nrm_off = nullptr;              // [2][F + 1] normal remainder offsets (large idx)
     HeavyKey* H = nullptr;                    // [h_max]
     uint64_t* h_off = nullptr;                // [2][h_max + 1]
@@ -193,7 +197,7 @@ int launch_hist_reduce_scan(const Plan& p, cudaStream_t s);
 int launch_scatter(const Plan& p, int pass, const uint32_t* const keys[2], const uint32_t* const pays[2],
                    cudaStream_t s);
 int launch_classify(const Plan& p, cudaStream_t s);
-int launch_detect_prefix(const Plan& p, uint32_t n_large, cudaStream_t s);
+int launch_detect_prefix(const Plan& p, uint32_t n_large, uint64_t large_tuples, cudaStream_t s);
 int launch_detect(const Plan& p, uint32_t n_large, uint32_t gt_cap, cudaStream_t s);
 int launch_sample_topk(const Plan& p, uint32_t n_large, uint32_t gt_cap, cudaStream_t s);
 int launch_select(const Plan& p, uint32_t gt_cap, cudaStream_t s);

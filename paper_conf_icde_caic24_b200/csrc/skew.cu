@@ -56,7 +56,6 @@ int launch_classify(const Plan& p, cudaStream_t s) {
 // Work items of detect / split: ceil((|R_p| + |S_p|) / chunk) per large partition, never spanning
 // two partitions.  Detect uses kDetectItem-tuple items (one shared-memory count table flush per
 // item), split kDetectChunk-tuple items (every tuple held in registers across its two phases).
-constexpr uint32_t kDetectItem = 16384;
 
 struct DetectItems {
     const uint32_t* cnt;
@@ -69,21 +68,36 @@ struct DetectItems {
     }
 };
 
-int launch_detect_prefix(const Plan& p, uint32_t n_large, cudaStream_t s) {
-    return launch_scan(DetectItems{p.cnt, p.large_list, p.F, kDetectChunk}, n_large, p.det_prefix, p.scan_scratch,
-                       s) +
-           launch_scan(DetectItems{p.cnt, p.large_list, p.F, kDetectItem}, n_large, p.det_prefix2, p.scan_scratch, s);
+// item -> large partition index, one thread per item (a binary search over the item prefix, done
+// once here instead of by every thread of every claiming CTA: ~16 dependent loads per item)
+__global__ void k_item_map(const uint64_t* __restrict__ prefix, uint32_t n_large, uint64_t bound,
+                           uint32_t* __restrict__ item_li) {
+    const uint64_t total = prefix[n_large];
+    for (uint64_t it = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; it < umin64(total, bound);
+         it += uint64_t(gridDim.x) * blockDim.x) {
+        uint32_t lo = 0, hi = n_large;
+        while (hi - lo > 1) {
+            const uint32_t mid = (lo + hi) >> 1;
+            if (prefix[mid] <= it) lo = mid; else hi = mid;
+        }
+        item_li[it] = lo;
+    }
 }
 
-// Locate item `it` among large partitions: returns large index li and chunk c.
-__device__ __forceinline__ uint32_t find_prefix(const uint64_t* prefix, uint32_t n, uint64_t it) {
-    // largest i with prefix[i] <= it, i < n
-    uint32_t lo = 0, hi = n;
-    while (hi - lo > 1) {
-        uint32_t mid = (lo + hi) >> 1;
-        if (prefix[mid] <= it) lo = mid; else hi = mid;
-    }
-    return lo;
+uint64_t detect_items_bound(uint64_t large_tuples, uint32_t n_large, uint32_t chunk) {
+    return large_tuples / chunk + n_large + 1;
+}
+
+int launch_detect_prefix(const Plan& p, uint32_t n_large, uint64_t large_tuples, cudaStream_t s) {
+    int l = launch_scan(DetectItems{p.cnt, p.large_list, p.F, kDetectChunk}, n_large, p.det_prefix, p.scan_scratch, s) +
+            launch_scan(DetectItems{p.cnt, p.large_list, p.F, kDetectItem}, n_large, p.det_prefix2, p.scan_scratch, s);
+    const uint64_t b1 = umin64(detect_items_bound(large_tuples, n_large, kDetectChunk), p.item_cap);
+    const uint64_t b2 = umin64(detect_items_bound(large_tuples, n_large, kDetectItem), p.item_cap2);
+    k_item_map<<<(unsigned)umin64((b1 + 255) / 256, uint64_t(p.num_sms) * 16), 256, 0, s>>>(p.det_prefix, n_large, b1,
+                                                                                             p.item_li);
+    k_item_map<<<(unsigned)umin64((b2 + 255) / 256, uint64_t(p.num_sms) * 16), 256, 0, s>>>(p.det_prefix2, n_large, b2,
+                                                                                             p.item_li2);
+    return l + 2;
 }
 
 struct LargeView {
@@ -93,6 +107,7 @@ struct LargeView {
     const uint32_t* large_list;
     const uint64_t* det_prefix;
     uint32_t F, n_large, chunk;
+    const uint32_t* item_li;   // item -> large partition index (k_item_map)
 };
 
 // The element range of one item: tuples [e0, e1) of the concatenation R_p ++ S_p.
@@ -103,7 +118,7 @@ struct ItemRange {
 
 __device__ __forceinline__ ItemRange item_range(const LargeView& v, uint64_t it) {
     ItemRange r;
-    r.li = find_prefix(v.det_prefix, v.n_large, it);
+    r.li = v.item_li[it];
     r.p = v.large_list[r.li];
     r.cr = v.cnt[r.p];
     r.cs = v.cnt[v.F + r.p];
@@ -302,7 +317,8 @@ int launch_detect(const Plan& p, uint32_t n_large, uint32_t gt_cap, cudaStream_t
     if (p.detect_mode == 0) cudaMemsetAsync(p.gt_key, 0, size_t(gt_cap) * sizeof(unsigned long long), s);
     cudaMemsetAsync(p.gt_cnt, 0, size_t(gt_cap) * sizeof(uint32_t), s);
     cudaMemsetAsync(p.gt_cnt + p.gt_cap_alloc, 0, size_t(gt_cap) * sizeof(uint32_t), s);
-    LargeView v{{p.bufB[0], p.bufB[1]}, p.start, p.cnt, p.large_list, p.det_prefix, p.F, n_large, kDetectChunk};
+    LargeView v{{p.bufB[0], p.bufB[1]}, p.start, p.cnt, p.large_list, p.det_prefix, p.F, n_large, kDetectChunk,
+                p.item_li};
     if (p.detect_mode == 1)
         k_detect<true><<<p.num_sms * 8, kDetBlock, 0, s>>>(v, p.gt_key, p.gt_cnt, p.gt_cap_alloc, logcap, p.st,
                                                            &p.st->claim[2]);
@@ -314,6 +330,7 @@ int launch_detect(const Plan& p, uint32_t n_large, uint32_t gt_cap, cudaStream_t
         LargeView v2 = v;
         v2.det_prefix = p.det_prefix2;
         v2.chunk = kDetectItem;
+        v2.item_li = p.item_li2;
         k_detect_smem<<<p.num_sms * 3, kDetBlock, kDetSmemBytes, s>>>(v2, p.gt_key, p.gt_cnt, p.gt_cap_alloc, logcap,
                                                                       p.Th, p.force_heavy, p.st, &p.st->claim[2]);
     }
@@ -404,7 +421,8 @@ int launch_sample_topk(const Plan& p, uint32_t n_large, uint32_t gt_cap, cudaStr
     uint32_t logcap = 0;
     while ((1u << logcap) < gt_cap) ++logcap;
     cudaMemsetAsync(p.gt_key, 0, size_t(gt_cap) * sizeof(unsigned long long), s);
-    LargeView v{{p.bufB[0], p.bufB[1]}, p.start, p.cnt, p.large_list, p.det_prefix, p.F, n_large, kDetectChunk};
+    LargeView v{{p.bufB[0], p.bufB[1]}, p.start, p.cnt, p.large_list, p.det_prefix, p.F, n_large, kDetectChunk,
+                p.item_li};
     const unsigned grid = (unsigned)umin64(n_large, uint64_t(p.num_sms) * 8);
     k_sample_topk<<<grid, kSampleBlock, 0, s>>>(v, p.sample_stride, p.top_k, p.gt_key, logcap, p.st);
     return 1;
@@ -662,7 +680,8 @@ int launch_split(const Plan& p, uint32_t n_large, uint32_t gt_cap, cudaStream_t 
     once_per_device(attr_once, [] {
         cudaFuncSetAttribute(k_split, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSplitSmemBytes);
     });
-    LargeView v{{p.bufB[0], p.bufB[1]}, p.start, p.cnt, p.large_list, p.det_prefix, p.F, n_large, kDetectChunk};
+    LargeView v{{p.bufB[0], p.bufB[1]}, p.start, p.cnt, p.large_list, p.det_prefix, p.F, n_large, kDetectChunk,
+                p.item_li};
     k_split<<<p.num_sms * 4, kDetBlock, kSplitSmemBytes, s>>>(v, p.gt_key, p.gt_hid, logcap, p.h_off, p.h_max + 1,
                                                              p.h_cur, (uint32_t)p.h_max, p.heavy_pay[0],
                                                              p.heavy_pay[1], p.nrm_off, p.nrm_cur, p.bufA[0],
