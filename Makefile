@@ -17,7 +17,7 @@ $(OBJ_DIR)/%.o: $(SRC_DIR)/%.cu $(HDR)
 
 $(LIB): $(OBJ)
 	@mkdir -p $(dir $(LIB))
-	$(NVCC) $(ARCH) -shared -cudart static -o $@ $(OBJ)
+	$(NVCC) $(ARCH) -shared -cudart static -o $@ $(OBJ) -ldl
 
 oracle/liboracle.so: oracle/join_oracle.c
 	gcc -O2 -std=c11 -shared -fPIC -pthread $< -o $@

@@ -70,6 +70,8 @@ def parse():
     ap.add_argument("--no-sweep", action="store_true", help="skip the theta_sweep sub-object (N=1 only)")
     ap.add_argument("--input-side", action="store_true",
                     help="time only the input side (partition, detect, split): gsh_config.input_side_only")
+    ap.add_argument("--exchange", default="a2a", choices=["a2a", "p2p"],
+                    help="multi-GPU exchange: NCCL all_to_all (a2a) or the route kernel's direct peer stores (p2p)")
     ap.add_argument("--fake-ranks", type=int, default=0,
                     help="run the sharded step for G logical ranks on one GPU (code-path check, not a headline)")
     return ap.parse_args()
@@ -431,14 +433,14 @@ def main():
         rk, rp, sk, sp = full
 
         def step():
-            rs = sharded.run_local(fake, shards, config=cfg)
+            rs = sharded.run_local(fake, shards, config=cfg, exchange=args.exchange)
             rs[0].stats["launches"] = sum(x.stats.get("launches", 0) for x in rs)
             return rs[0]
     elif world > 1:
         rk, rp, sk, sp = make_data(kind, n, theta, args.seed, dev, rank)
 
         def step():
-            return sharded.join_sharded(rk, rp, sk, sp, config=cfg)
+            return sharded.join_sharded(rk, rp, sk, sp, config=cfg, exchange=args.exchange)
     else:
         rk, rp, sk, sp = make_data(kind, n, theta, args.seed, dev, rank)
         ws = torch.empty(gsh.workspace_bytes(n, n, cfg), dtype=torch.uint8, device=dev)
@@ -544,6 +546,7 @@ def main():
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32",
             "data": "synthetic (datagen, seeded)",
             "config": {"workload": desc, "n_r": n * world, "n_s": n * world, "mode": args.mode, "detect": args.detect,
+                       "exchange": args.exchange if multi else None,
                        "parallelism": (f"hash-sharded x{world} (NCCL)" if world > 1 else
                                        f"{fake} logical ranks on one GPU (code-path check)" if fake >= 1 else
                                        "single GPU"),

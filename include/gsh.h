@@ -335,13 +335,28 @@ GSH_API gsh_status gsh_route_count(const uint32_t *d_keys, uint64_t n, uint32_t 
                                    const void *d_set, size_t set_bytes, uint64_t *d_counts,
                                    void *stream);
 
-/* Scatter every tuple to its destination (as gsh_route_count).  d_dst: device u64[2 (G + 1)],
- * d_dst[2d] / d_dst[2d + 1] = device addresses of destination d's key / payload arrays, each
- * with room for its count; d_cursor: device u64[G + 1] scratch (overwritten).  The order of
- * tuples inside a destination is unspecified. */
+/* Scatter every tuple to its destination (as gsh_route_count).  d_dst: device
+ * u64[2 (G + heavy_copies)]: d_dst[2d] / d_dst[2d + 1] = device addresses of destination d's
+ * key / payload arrays (d < G: normal routes, d = G: the skewed tuples), each with room for its
+ * count; heavy_copies >= 1 -- with more than one, every skewed tuple is also stored at the same
+ * position in the arrays d_dst[2 (G + c)], d_dst[2 (G + c) + 1], c = 1 .. heavy_copies - 1 (the
+ * all-gather of skewed R done by the scatter itself).  The addresses may be peer memory (another
+ * GPU's buffer opened with gsh_ipc_open, or under peer access): the kernel then IS the exchange,
+ * its stores travelling over NVLink.  d_cursor: device u64[G + 1] scratch (overwritten).  The
+ * order of tuples inside a destination is unspecified. */
 GSH_API gsh_status gsh_route_scatter(const uint32_t *d_keys, const uint32_t *d_payloads, uint64_t n,
                                      uint32_t route_bits, const void *d_set, size_t set_bytes,
-                                     const uint64_t *d_dst, uint64_t *d_cursor, void *stream);
+                                     const uint64_t *d_dst, uint32_t heavy_copies, uint64_t *d_cursor,
+                                     void *stream);
+
+/* CUDA IPC for the peer-store exchange: *handle (host, 64 bytes) names the device allocation
+ * holding d_ptr for other processes, d_ptr = that allocation's base + *offset; gsh_ipc_open maps
+ * such a handle into this process (*d_ptr = the base, a device address usable by kernels: a peer
+ * GPU's memory over NVLink, or the same GPU's memory from another process); gsh_ipc_close unmaps
+ * it.  GSH_ERR_CUDA with the CUDA message on failure. */
+GSH_API gsh_status gsh_ipc_handle(const void *d_ptr, void *handle, uint64_t *offset);
+GSH_API gsh_status gsh_ipc_open(const void *handle, void **d_ptr);
+GSH_API gsh_status gsh_ipc_close(void *d_ptr);
 
 /* ------------------------------------------------------------------- diagnostics -- */
 GSH_API const char *gsh_status_string(gsh_status s);

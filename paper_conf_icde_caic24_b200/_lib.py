@@ -143,7 +143,10 @@ _PROTOS = [
     ("gsh_heavy_set_bytes", ctypes.c_size_t, [u64]),
     ("gsh_heavy_set_build", ctypes.c_int, [vp, u64, vp, ctypes.c_size_t, vp]),
     ("gsh_route_count", ctypes.c_int, [vp, u64, u32, vp, ctypes.c_size_t, vp, vp]),
-    ("gsh_route_scatter", ctypes.c_int, [vp, vp, u64, u32, vp, ctypes.c_size_t, vp, vp, vp]),
+    ("gsh_route_scatter", ctypes.c_int, [vp, vp, u64, u32, vp, ctypes.c_size_t, vp, u32, vp, vp]),
+    ("gsh_ipc_handle", ctypes.c_int, [vp, vp, p64]),
+    ("gsh_ipc_open", ctypes.c_int, [vp, ctypes.POINTER(vp)]),
+    ("gsh_ipc_close", ctypes.c_int, [vp]),
     ("gsh_status_string", ctypes.c_char_p, [ctypes.c_int]),
     ("gsh_last_error", ctypes.c_char_p, []),
     ("gsh_version", ctypes.c_int, []),

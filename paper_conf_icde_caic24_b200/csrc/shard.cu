@@ -20,6 +20,7 @@
 //                      into per-destination buffers the driver lays out (its own received segment,
 //                      the all-gathered R_H buffer, the send buffer), so no copy follows.
 #include <cstring>
+#include <dlfcn.h>
 
 #include "gsh_device.cuh"
 #include "gsh_internal.h"
@@ -219,7 +220,7 @@ __global__ void __launch_bounds__(kRouteBlock, 1) k_route_scatter(const uint32_t
                                                               const uint32_t* __restrict__ pays, uint64_t n,
                                                               uint32_t rb, HeavySet hs,
                                                               const unsigned long long* __restrict__ dst,
-                                                              unsigned long long* cur) {
+                                                              uint32_t heavy_copies, unsigned long long* cur) {
     extern __shared__ uint4 route_dyn[];
     uint32_t* s_k = reinterpret_cast<uint32_t*>(route_dyn);
     uint32_t* s_p = s_k + kRouteTile;
@@ -292,8 +293,14 @@ __global__ void __launch_bounds__(kRouteBlock, 1) k_route_scatter(const uint32_t
         for (uint32_t i = threadIdx.x; i < tn; i += kRouteBlock) {
             const uint32_t d = s_d[i];
             const uint64_t pos = base[d] + (i - pre[d]);
-            reinterpret_cast<uint32_t*>(dst[2 * d])[pos] = s_k[i];
-            reinterpret_cast<uint32_t*>(dst[2 * d + 1])[pos] = s_p[i];
+            const uint32_t kk = s_k[i], pp = s_p[i];
+            reinterpret_cast<uint32_t*>(dst[2 * d])[pos] = kk;
+            reinterpret_cast<uint32_t*>(dst[2 * d + 1])[pos] = pp;
+            if (d == G1 - 1)   // the heavy destination: further copies (one per peer GPU's R_H buffer)
+                for (uint32_t c = 1; c < heavy_copies; ++c) {
+                    reinterpret_cast<uint32_t*>(dst[2 * (d + c)])[pos] = kk;
+                    reinterpret_cast<uint32_t*>(dst[2 * (d + c) + 1])[pos] = pp;
+                }
         }
         __syncthreads();
     }
@@ -540,9 +547,10 @@ gsh_status gsh_route_count(const uint32_t* d_keys, uint64_t n, uint32_t route_bi
 }
 
 gsh_status gsh_route_scatter(const uint32_t* d_keys, const uint32_t* d_payloads, uint64_t n, uint32_t route_bits,
-                             const void* d_set, size_t set_bytes, const uint64_t* d_dst, uint64_t* d_cursor,
-                             void* stream) {
+                             const void* d_set, size_t set_bytes, const uint64_t* d_dst, uint32_t heavy_copies,
+                             uint64_t* d_cursor, void* stream) {
     if (route_bits > 8) return api_fail(GSH_ERR_INVALID, "route_bits > 8");
+    if (heavy_copies < 1 || heavy_copies > kMaxShardWorld) return api_fail(GSH_ERR_INVALID, "bad heavy_copies");
     if (n && (!d_keys || !d_payloads || !d_dst || !d_cursor)) return api_fail(GSH_ERR_INVALID, "NULL pointer");
     if (n == 0) return GSH_OK;
     cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
@@ -552,8 +560,67 @@ gsh_status gsh_route_scatter(const uint32_t* d_keys, const uint32_t* d_payloads,
     k_route_scatter<<<grid, kRouteBlock, kRouteSmem, s>>>(d_keys, d_payloads, n, route_bits,
                                                           heavy_set_view(d_set, set_bytes),
                                                           reinterpret_cast<const unsigned long long*>(d_dst),
+                                                          heavy_copies,
                                                           reinterpret_cast<unsigned long long*>(d_cursor));
     return api_cuda("route_scatter");
+}
+
+// CUDA IPC: a device allocation shared with the other processes of the node (peer GPUs over
+// NVLink, or another process on the same GPU), for the route kernel's direct peer stores.  A
+// handle names a whole cudaMalloc allocation; the caller's buffer (a caching-allocator
+// sub-range) is its base + *offset, found with the driver's cuMemGetAddressRange (looked up at
+// run time, so libgsh loads without a driver, e.g. for the CPU tests).
+typedef int (*CuMemGetAddressRange)(unsigned long long*, size_t*, unsigned long long);
+static CuMemGetAddressRange cu_range() {
+    static CuMemGetAddressRange fn = nullptr;
+    static std::once_flag once;
+    std::call_once(once, [] {
+        void* h = dlopen("libcuda.so.1", RTLD_NOW | RTLD_NOLOAD);
+        if (!h) h = dlopen("libcuda.so.1", RTLD_NOW);
+        if (h) fn = reinterpret_cast<CuMemGetAddressRange>(dlsym(h, "cuMemGetAddressRange_v2"));
+    });
+    return fn;
+}
+
+gsh_status gsh_ipc_handle(const void* d_ptr, void* handle, uint64_t* offset) {
+    if (!d_ptr || !handle || !offset) return api_fail(GSH_ERR_INVALID, "NULL pointer");
+    const CuMemGetAddressRange range = cu_range();
+    if (!range) return api_fail(GSH_ERR_CUDA, "cuMemGetAddressRange unavailable (no CUDA driver)");
+    unsigned long long base = 0;
+    size_t size = 0;
+    if (range(&base, &size, reinterpret_cast<unsigned long long>(d_ptr)) != 0)
+        return api_fail(GSH_ERR_CUDA, "cuMemGetAddressRange failed");
+    cudaIpcMemHandle_t h;
+    const cudaError_t e = cudaIpcGetMemHandle(&h, reinterpret_cast<void*>(base));
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        return api_fail(GSH_ERR_CUDA, cudaGetErrorString(e));
+    }
+    std::memcpy(handle, &h, sizeof(h));
+    *offset = reinterpret_cast<unsigned long long>(d_ptr) - base;
+    return GSH_OK;
+}
+
+gsh_status gsh_ipc_open(const void* handle, void** d_ptr) {
+    if (!handle || !d_ptr) return api_fail(GSH_ERR_INVALID, "NULL pointer");
+    cudaIpcMemHandle_t h;
+    std::memcpy(&h, handle, sizeof(h));
+    const cudaError_t e = cudaIpcOpenMemHandle(d_ptr, h, cudaIpcMemLazyEnablePeerAccess);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        return api_fail(GSH_ERR_CUDA, cudaGetErrorString(e));
+    }
+    return GSH_OK;
+}
+
+gsh_status gsh_ipc_close(void* d_ptr) {
+    if (!d_ptr) return GSH_OK;
+    const cudaError_t e = cudaIpcCloseMemHandle(d_ptr);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        return api_fail(GSH_ERR_CUDA, cudaGetErrorString(e));
+    }
+    return GSH_OK;
 }
 
 }  // extern "C"

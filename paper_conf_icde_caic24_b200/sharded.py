@@ -51,26 +51,36 @@ class TorchComm:
         self.rank = dist.get_rank(group)
         self.world = dist.get_world_size(group)
         self.device = device
+        # gloo moves host tensors: device tensors travel through host copies (control-size data;
+        # the bulk exchange of the p2p mode never goes through a collective)
+        self.host_only = dist.get_backend(group) == "gloo"
+        self.ctl = torch.device("cpu") if self.host_only else device
 
     def _src(self, g: int) -> int:
         return dist.get_global_rank(self.group, g) if self.group is not None else g
 
     def all_reduce_(self, t: torch.Tensor) -> None:
-        dist.all_reduce(t, group=self.group)
+        if self.host_only and t.is_cuda:
+            h = t.cpu()
+            dist.all_reduce(h, group=self.group)
+            t.copy_(h)
+        else:
+            dist.all_reduce(t, group=self.group)
 
     def all_gather_sizes(self, n: int) -> list[int]:
-        t = torch.tensor([n], dtype=torch.int64, device=self.device)
+        t = torch.tensor([n], dtype=torch.int64, device=self.ctl)
         out = [torch.zeros_like(t) for _ in range(self.world)]
         dist.all_gather(out, t, group=self.group)
         return [int(x.item()) for x in out]
 
     def all_gather_pad(self, t: torch.Tensor, m: int) -> torch.Tensor:
         """[world * m] buffer; rank g's tensor at [g * m, g * m + len)."""
-        out = torch.zeros(self.world * max(m, 1), dtype=t.dtype, device=t.device)
-        pad = torch.zeros(max(m, 1), dtype=t.dtype, device=t.device)
-        pad[: t.numel()] = t
+        dev = self.ctl if self.host_only else t.device
+        out = torch.zeros(self.world * max(m, 1), dtype=t.dtype, device=dev)
+        pad = torch.zeros(max(m, 1), dtype=t.dtype, device=dev)
+        pad[: t.numel()] = t.to(dev)
         dist.all_gather(list(out.view(self.world, -1).unbind(0)), pad, group=self.group)
-        return out
+        return out.to(t.device)
 
     def all_to_all_v(self, out: torch.Tensor, inp: torch.Tensor, out_splits: list[int], in_splits: list[int]) -> None:
         if sum(out_splits) == 0 and sum(in_splits) == 0 and self.world == 1:
@@ -85,6 +95,71 @@ class TorchComm:
             if n:
                 dist.broadcast(buf[off: off + n], src=self._src(g), group=self.group)
             off += n
+
+    def all_gather_rows(self, row: list[int]) -> list[list[int]]:
+        t = torch.tensor(row, dtype=torch.int64, device=self.ctl)
+        out = [torch.zeros_like(t) for _ in range(self.world)]
+        dist.all_gather(out, t, group=self.group)
+        return [[int(v) for v in x.tolist()] for x in out]
+
+    def space_key(self):
+        return ("torch", id(self.group), str(self.device))
+
+    def barrier(self) -> None:
+        """Every rank's queued device work (e.g. peer stores) is complete before any returns."""
+        if torch.cuda.is_available():
+            torch.cuda.current_stream().synchronize()
+        dist.barrier(group=self.group)
+
+    def peer_views(self, bufs: dict) -> list[dict]:
+        """The other ranks' buffers of the same names, mapped into this process through CUDA IPC
+        (NVLink peer memory; the same GPU's memory when ranks share one): {name: PeerPtr}."""
+        lib = load()
+        mine = []
+        for name in sorted(bufs):
+            h = (ctypes.c_uint8 * 64)()
+            off = ctypes.c_uint64(0)
+            check(lib.gsh_ipc_handle(bufs[name].data_ptr(), h, ctypes.byref(off)), "gsh_ipc_handle")
+            mine.append(list(bytes(h)) + [off.value & 0xFF_FFFF_FFFF_FFFF, bufs[name].numel()])
+        flat = [v for rec in mine for v in rec]
+        rows = self.all_gather_rows(flat)
+        per = len(flat) // max(len(bufs), 1)
+        views = []
+        for g, row in enumerate(rows):
+            if g == self.rank:
+                views.append(dict(bufs))
+                continue
+            d = {}
+            for i, name in enumerate(sorted(bufs)):
+                rec = row[i * per: (i + 1) * per]
+                d[name] = PeerPtr.open(bytes(v & 0xFF for v in rec[:64]), rec[64], rec[65])
+            views.append(d)
+        return views
+
+
+class PeerPtr:
+    """A peer process's device buffer mapped with gsh_ipc_open (base of its allocation + offset)."""
+
+    _open: dict = {}   # handle bytes -> mapped base (one mapping per allocation and process)
+
+    def __init__(self, ptr: int, n: int):
+        self.ptr, self.n = ptr, n
+
+    def data_ptr(self) -> int:
+        return self.ptr
+
+    def numel(self) -> int:
+        return self.n
+
+    @classmethod
+    def open(cls, handle: bytes, offset: int, n: int) -> "PeerPtr":
+        base = cls._open.get(handle)
+        if base is None:
+            p = ctypes.c_void_p(0)
+            h = (ctypes.c_uint8 * 64).from_buffer_copy(handle)
+            check(load().gsh_ipc_open(h, ctypes.byref(p)), "gsh_ipc_open")
+            base = cls._open[handle] = p.value
+        return cls(base + offset, n)
 
 
 class LocalWorld:
@@ -159,6 +234,19 @@ class LocalComm:
                     buf[off: off + sizes[g]].copy_(x[off: off + sizes[g]])
                 off += sizes[g]
         self._round(buf, fn)
+
+    def all_gather_rows(self, row):
+        return self._round(list(row), lambda xs: [list(x) for x in xs])
+
+    def space_key(self):
+        return ("local", id(self.w), self.rank)
+
+    def barrier(self) -> None:
+        self._round(None, lambda xs: None)
+
+    def peer_views(self, bufs: dict) -> list[dict]:
+        """In one process the peers' buffers are directly addressable: their tensors."""
+        return self._round(dict(bufs), lambda xs: [dict(x) for x in xs])
 
 
 # ------------------------------------------------------------------------------- CUDA ops
@@ -264,18 +352,21 @@ class CudaOps:
         self.launches += keys.numel() > 0
         return [int(x) for x in c.cpu().tolist()]
 
-    def route_scatter(self, state, keys, pays, rb, dst):
-        """dst[d] = (keys_tensor, pays_tensor, offset): destination d's run starts at offset."""
+    def route_scatter(self, state, keys, pays, rb, dst, heavy_copies: int = 1):
+        """dst[d] = (keys_buffer, pays_buffer, offset): destination d's run starts at offset (d = G:
+        skewed tuples; heavy_copies > 1: further copies of them follow in dst).  A buffer is a
+        tensor or a PeerPtr (another rank's memory)."""
         if keys.numel() == 0:
             return
         ptrs = []
         for k, p, off in dst:
             ptrs += [k.data_ptr() + 4 * off if k.numel() else 0, p.data_ptr() + 4 * off if p.numel() else 0]
         d_dst = self.tensor([x - (1 << 64) if x >= (1 << 63) else x for x in ptrs])
-        cur = torch.empty(len(dst), dtype=torch.int64, device=self.dev)
+        cur = torch.empty(len(dst) - heavy_copies + 1, dtype=torch.int64, device=self.dev)
         check(load().gsh_route_scatter(keys.data_ptr(), pays.data_ptr(), keys.numel(), rb,
                                        state["set"].data_ptr() if state["set_bytes"] else None, state["set_bytes"],
-                                       d_dst.data_ptr(), cur.data_ptr(), self.stream()), "gsh_route_scatter")
+                                       d_dst.data_ptr(), heavy_copies, cur.data_ptr(), self.stream()),
+              "gsh_route_scatter")
         state.setdefault("keep", []).append(d_dst)
         self.launches += 1
 
@@ -284,6 +375,76 @@ class CudaOps:
         r = join(rk, rp, sk, sp, mode=mode, out=out, config=config)
         self.launches += r.stats.get("launches", 0)
         return r.count, r.checksum, r.written, r.stats
+
+
+# --------------------------------------------------------------------- peer-store exchange
+_SPACES: dict = {}   # communicator identity -> PeerSpace (the IPC mappings outlive a call)
+
+
+class PeerSpace:
+    """A rank's receive buffers for the peer-store exchange, kept across calls (their IPC
+    mappings are set up once): normal R / S keys and payloads, and the all-gathered skewed R.
+    Capacities are decided from the all-gathered count matrix (identical on every rank), so
+    all ranks grow together and re-share their buffers."""
+
+    NAMES = ("rn_k", "rn_p", "sn_k", "sn_p", "rh_k", "rh_p")
+
+    def __init__(self, ops):
+        self.ops = ops
+        self.caps = (-1, -1, -1)
+        self.bufs: dict = {}
+        self.views: list = []
+
+    def ensure(self, comm, cap_rn: int, cap_sn: int, cap_rh: int) -> None:
+        if cap_rn <= self.caps[0] and cap_sn <= self.caps[1] and cap_rh <= self.caps[2]:
+            return
+        grow = lambda c, old: max(c + (c >> 3) + 1024, old)   # noqa: E731  (headroom against regrowth)
+        caps = (grow(cap_rn, self.caps[0]), grow(cap_sn, self.caps[1]), grow(cap_rh, self.caps[2]))
+        comm.barrier()   # every peer is done with the old buffers
+        self.bufs = {}
+        for name, c in zip(self.NAMES, (caps[0], caps[0], caps[1], caps[1], caps[2], caps[2])):
+            self.bufs[name] = self.ops.empty(c)
+        self.caps = caps
+        self.views = comm.peer_views(self.bufs)
+
+
+def _route_p2p(rk, rp, sk, sp, rb, rc, sc, comm, ops, state):
+    """Steps 2-3 with the exchange inside the route kernel: every tuple is stored straight into its
+    destination rank's receive buffer (skewed R into every rank's), at an offset fixed by the
+    all-gathered count matrix; a barrier then makes all peers' stores visible.  Returns this
+    rank's (normal R, normal S, all skewed R, local skewed S) and the bytes it stored remotely."""
+    G, me = comm.world, comm.rank
+    M = comm.all_gather_rows(list(rc) + list(sc))          # row g: rank g's R counts, then S counts
+    rcm = [row[: G + 1] for row in M]
+    scm = [row[G + 1:] for row in M]
+    need_rn = [sum(rcm[g][d] for g in range(G)) for d in range(G)]
+    need_sn = [sum(scm[g][d] for g in range(G)) for d in range(G)]
+    need_rh = sum(rcm[g][G] for g in range(G))
+    key = comm.space_key()
+    space = _SPACES.get(key)
+    if space is None:
+        space = _SPACES[key] = PeerSpace(ops)
+    space.ensure(comm, max(need_rn), max(need_sn), need_rh)
+    V = space.views
+    off_rn = [sum(rcm[g][d] for g in range(me)) for d in range(G)]   # my run in each destination
+    off_sn = [sum(scm[g][d] for g in range(me)) for d in range(G)]
+    off_rh = sum(rcm[g][G] for g in range(me))
+    Sh = (ops.empty(sc[G]), ops.empty(sc[G]))
+    dst_r = [(V[d]["rn_k"], V[d]["rn_p"], off_rn[d]) for d in range(G)]
+    dst_r += [(V[d]["rh_k"], V[d]["rh_p"], off_rh) for d in range(G)]     # skewed R: every rank
+    dst_s = [(V[d]["sn_k"], V[d]["sn_p"], off_sn[d]) for d in range(G)] + [(Sh[0], Sh[1], 0)]
+    ops.route_scatter(state, rk, rp, rb, dst_r, heavy_copies=G)
+    ops.route_scatter(state, sk, sp, rb, dst_s)
+    ops.mark("route")
+    comm.barrier()
+    ops.mark("exchange")
+    B = space.bufs
+    Rn = (B["rn_k"][: need_rn[me]], B["rn_p"][: need_rn[me]])
+    Sn = (B["sn_k"][: need_sn[me]], B["sn_p"][: need_sn[me]])
+    Rh = (B["rh_k"][:need_rh], B["rh_p"][:need_rh])
+    remote = 8 * (sum(rc[d] for d in range(G) if d != me) + sum(sc[d] for d in range(G) if d != me)
+                  + (G - 1) * rc[G])
+    return Rn, Sn, Rh, Sh, remote, rcm
 
 
 # ------------------------------------------------------------------------------- protocol
@@ -329,37 +490,11 @@ def agree_heavy(rk, rp, sk, sp, P, comm, ops, state):
     return ops.select(state, uni, cnt, P)
 
 
-def join_sharded(rk, rp, sk, sp, config=None, group=None, ops=None, comm=None, mode: str = "count", out=None):
-    """Hash-sharded GSH join of this rank's shards (any positional split of R and S over the ranks).
-
-    Returns a JoinResult whose count / checksum are GLOBAL (identical on all ranks); in
-    "materialize" mode `out` ((capacity, 2) int32 CUDA tensor) receives this rank's pairs and
-    `written` counts them.  stats: per-phase ms, exchanged bytes and their NVLink fraction."""
-    if ops is None:
-        rk, rp = _check_dev(rk, "r_keys"), _check_dev(rp, "r_payloads")
-        sk, sp = _check_dev(sk, "s_keys"), _check_dev(sp, "s_payloads")
-        ops = CudaOps(rk.device)
-    if comm is None:
-        comm = TorchComm(group, rk.device)
+def _route_a2a(rk, rp, sk, sp, rb, rc, sc, comm, ops, state):
+    """Steps 2-3 with collectives: the route kernel writes this rank's own normal tuples to the end
+    of its receive buffer, its skewed R to its offset in the all-gathered R_H buffer, the rest to
+    send buffers; then all_to_all of the normal tuples and the in-place all-gather of R_H."""
     G, me = comm.world, comm.rank
-    if G & (G - 1):
-        raise ValueError("world size must be a power of two (route bits)")
-    if mode not in ("count", "materialize"):
-        raise ValueError("mode must be 'count' or 'materialize'")
-    state: dict = {}
-    ops.mark("start")
-    n = ops.tensor([rk.numel(), sk.numel()])
-    comm.all_reduce_(n)
-    n_r, n_s = (int(x) for x in n.tolist())
-    P = shard_plan(n_r, n_s, G, config)
-    rb = int(P.route_bits)
-    heavy = agree_heavy(rk, rp, sk, sp, P, comm, ops, state)
-    ops.mark("agree")
-
-    # routing plan: destination counts, then every buffer laid out so the route kernel writes
-    # each tuple to its final place
-    rc = ops.route_count(state, rk, rb)
-    sc = ops.route_count(state, sk, rb)
     send = ops.tensor([[rc[d], sc[d]] for d in range(G)]).reshape(-1)
     recv = ops.tensor([0] * (2 * G))
     comm.all_to_all_v(recv, send, [2] * G, [2] * G)
@@ -398,7 +533,57 @@ def join_sharded(rk, rp, sk, sp, config=None, group=None, ops=None, comm=None, m
     for i in range(2):
         comm.all_gather_v_(Rh[i], rh_sizes)
     ops.mark("broadcast")
+    xbytes = 8 * (sum(rsend) + sum(ssend))
+    bbytes = 8 * (sum(rh_sizes) - rh_sizes[me])
+    return Rn, Sn, Rh, Sh, xbytes, bbytes, rh_sizes
 
+
+def join_sharded(rk, rp, sk, sp, config=None, group=None, ops=None, comm=None, mode: str = "count", out=None,
+                 exchange: str = "a2a"):
+    """Hash-sharded GSH join of this rank's shards (any positional split of R and S over the ranks).
+
+    exchange: "a2a" -- the route kernel fills send buffers, then all_to_all / all-gather
+    collectives (NCCL); "p2p" -- the route kernel stores every tuple straight into its
+    destination rank's receive buffer (peer memory: CUDA IPC over NVLink, or in-process), skewed R
+    into every rank's, so the scatter IS the exchange and no send buffer exists.
+
+    Returns a JoinResult whose count / checksum are GLOBAL (identical on all ranks); in
+    "materialize" mode `out` ((capacity, 2) int32 CUDA tensor) receives this rank's pairs and
+    `written` counts them.  stats: per-phase ms, exchanged bytes and their NVLink fraction."""
+    if exchange not in ("a2a", "p2p"):
+        raise ValueError("exchange must be 'a2a' or 'p2p'")
+    if ops is None:
+        rk, rp = _check_dev(rk, "r_keys"), _check_dev(rp, "r_payloads")
+        sk, sp = _check_dev(sk, "s_keys"), _check_dev(sp, "s_payloads")
+        ops = CudaOps(rk.device)
+    if comm is None:
+        comm = TorchComm(group, rk.device)
+    G, me = comm.world, comm.rank
+    if G & (G - 1):
+        raise ValueError("world size must be a power of two (route bits)")
+    if mode not in ("count", "materialize"):
+        raise ValueError("mode must be 'count' or 'materialize'")
+    state: dict = {}
+    ops.mark("start")
+    n = ops.tensor([rk.numel(), sk.numel()])
+    comm.all_reduce_(n)
+    n_r, n_s = (int(x) for x in n.tolist())
+    P = shard_plan(n_r, n_s, G, config)
+    rb = int(P.route_bits)
+    heavy = agree_heavy(rk, rp, sk, sp, P, comm, ops, state)
+    ops.mark("agree")
+
+    # routing plan: destination counts, then every buffer laid out so the route kernel writes
+    # each tuple to its final place
+    rc = ops.route_count(state, rk, rb)
+    sc = ops.route_count(state, sk, rb)
+    if exchange == "p2p":
+        Rn, Sn, Rh, Sh, xbytes, rcm = _route_p2p(rk, rp, sk, sp, rb, rc, sc, comm, ops, state)
+        rh_sizes = [row[G] for row in rcm]
+        bbytes = 0   # the skewed R copies are part of the peer stores (xbytes)
+        ops.mark("broadcast")
+    else:
+        Rn, Sn, Rh, Sh, xbytes, bbytes, rh_sizes = _route_a2a(rk, rp, sk, sp, rb, rc, sc, comm, ops, state)
     # local joins: the routed normal shard under route_bits = rb, the skewed keys under 0
     cfg_n = _copy_cfg(config, route_bits=rb, timing=1)
     cfg_h = _copy_cfg(config, route_bits=0, timing=1)
@@ -417,8 +602,6 @@ def join_sharded(rk, rp, sk, sp, config=None, group=None, ops=None, comm=None, m
     gc, gk = (int(x) & M64 for x in t.tolist())
     ops.mark("reduce")
     phases = ops.phase_ms()
-    xbytes = 8 * (sum(rsend) + sum(ssend))
-    bbytes = 8 * (sum(rh_sizes) - rh_sizes[me])
     stats = {
         "world": G, "rank": me, "route_bits": rb, "part_bits": int(P.part_bits),
         "large_threshold": int(P.large_threshold), "heavy_threshold": int(P.heavy_threshold),
@@ -427,7 +610,7 @@ def join_sharded(rk, rp, sk, sp, config=None, group=None, ops=None, comm=None, m
         "candidate_table_overflow": bool(state.get("cand_overflow", False)),
         "local_r": rk.numel(), "local_s": sk.numel(),
         "normal_r": Rn[0].numel(), "normal_s": Sn[0].numel(), "heavy_r": Rh[0].numel(), "heavy_s": Sh[0].numel(),
-        "exchange_send_bytes": xbytes, "broadcast_recv_bytes": bbytes,
+        "exchange": exchange, "exchange_send_bytes": xbytes, "broadcast_recv_bytes": bbytes,
         "count_normal": c1, "count_heavy": c2, "written": w1 + w2,
         "join_normal": st1, "join_heavy": st2, "launches": getattr(ops, "launches", 0),
     }
@@ -442,7 +625,8 @@ def join_sharded(rk, rp, sk, sp, config=None, group=None, ops=None, comm=None, m
                       pairs=(out[: w1 + w2] if mat else None), stats=stats)
 
 
-def run_local(world: int, shards, config=None, mode: str = "count", out_capacity: int = 0, device=None):
+def run_local(world: int, shards, config=None, mode: str = "count", out_capacity: int = 0, device=None,
+              exchange: str = "a2a"):
     """Run join_sharded for `world` logical ranks on ONE device (threads + LocalWorld): the
     one-GPU multi-rank harness.  shards[g] = (rk, rp, sk, sp) CUDA tensors of rank g.  Returns the
     per-rank JoinResults (rank order)."""
@@ -458,7 +642,8 @@ def run_local(world: int, shards, config=None, mode: str = "count", out_capacity
                 with torch.cuda.stream(s):
                     out = (torch.empty((out_capacity, 2), dtype=torch.int32, device=dev)
                            if mode == "materialize" else None)
-                    res[g] = join_sharded(*shards[g], config=config, comm=lw.comm(g), mode=mode, out=out)
+                    res[g] = join_sharded(*shards[g], config=config, comm=lw.comm(g), mode=mode, out=out,
+                                          exchange=exchange)
                 s.synchronize()
         except BaseException as e:  # surface the first failure, release the other ranks
             err.append(e)

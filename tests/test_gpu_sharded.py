@@ -81,7 +81,7 @@ def test_route_kernels_vs_oracle(rb, n_heavy):
     d_dst = torch.tensor(ptrs, dtype=torch.int64, device=dev)
     cur = torch.empty(G + 1, dtype=torch.int64, device=dev)
     assert lib.gsh_route_scatter(dk.data_ptr(), dp.data_ptr(), dk.numel(), rb, setbuf.data_ptr() if nb else None,
-                                 nb, d_dst.data_ptr(), cur.data_ptr(), s) == 0
+                                 nb, d_dst.data_ptr(), 1, cur.data_ptr(), s) == 0
     torch.cuda.synchronize()
     pays = _u32(rp)
     for d, (k, p) in enumerate(outs):
@@ -263,3 +263,67 @@ def test_sharded_single_rank_nccl(kind, n, theta):
     assert (cnt, chk) == (on, oc)
     if theta >= 1.0:
         assert nh > 0
+
+
+@pytest.mark.parametrize("world,kind,n,theta,kw", [
+    (2, "zipf", 1 << 18, 1.0, {}),
+    (4, "pkfk_zipf", 1 << 18, 1.0, dict(heavy_threshold=64)),
+    (8, "graph", 1 << 17, 0.909, {}),
+    (4, "uniform", 1 << 18, 0.0, {}),
+])
+def test_sharded_p2p_local_world_vs_oracle(world, kind, n, theta, kw):
+    """exchange="p2p": the route kernel stores every tuple straight into its destination rank's
+    receive buffer (skewed R into every rank's), so the scatter IS the exchange -- here the G
+    logical ranks' buffers share the one GPU.  Twice in a row: the second call reuses the buffers."""
+    from paper_conf_icde_caic24_b200 import make_config, sharded
+    dev = torch.device("cuda", 0)
+    full = datagen.make_workload(kind, n, theta, seed=41)
+    on, oc, _ = oracle.join(*(t.numpy().view(np.uint32) for t in full))
+    cfg = make_config(**kw)
+    shards = [tuple(_shard(t, g, world).to(dev) for t in full) for g in range(world)]
+    for _ in range(2):
+        res = sharded.run_local(world, shards, config=cfg, exchange="p2p")
+        for r in res:
+            assert (r.count, r.checksum) == (on, oc), r.stats
+            assert r.stats["exchange"] == "p2p"
+        assert sum(r.stats["normal_s"] + r.stats["heavy_s"] for r in res) == n
+
+
+def _p2p_worker(rank, world, port, kind, n, theta, q):
+    import torch.distributed as dist
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    torch.cuda.set_device(0)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        from paper_conf_icde_caic24_b200 import sharded
+        full = datagen.make_workload(kind, n, theta, seed=43)
+        rk, rp, sk, sp = (_shard(t, rank, world).cuda() for t in full)
+        out = []
+        for _ in range(2):
+            r = sharded.join_sharded(rk, rp, sk, sp, exchange="p2p")
+            out.append((r.count, r.checksum))
+        q.put((rank, out))
+    finally:
+        dist.destroy_process_group()
+
+
+def test_sharded_p2p_two_processes_ipc():
+    """The peer-store exchange across PROCESSES: two ranks on the one GPU, receive buffers shared
+    through CUDA IPC (gsh_ipc_handle / gsh_ipc_open -- the same calls that map a peer GPU's memory
+    over NVLink), host-side collectives on gloo.  Exact vs the oracle, and again on reused buffers."""
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    world, kind, n, theta = 2, "zipf", 1 << 17, 1.0
+    procs = [ctx.Process(target=_p2p_worker, args=(r, world, port, kind, n, theta, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    out = [q.get(timeout=300) for _ in range(world)]
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    full = datagen.make_workload(kind, n, theta, seed=43)
+    on, oc, _ = oracle.join(*(t.numpy().view(np.uint32) for t in full))
+    for _, res in out:
+        assert res == [(on, oc), (on, oc)]

@@ -97,10 +97,11 @@ class OracleOps:
     def route_count(self, state, keys, rb):
         return np.bincount(self._dest(state, keys, rb), minlength=(1 << rb) + 1).tolist()
 
-    def route_scatter(self, state, keys, pays, rb, dst):
+    def route_scatter(self, state, keys, pays, rb, dst, heavy_copies=1):
         dest = self._dest(state, keys, rb)
+        G = 1 << rb
         for d, (kb, pb, off) in enumerate(dst):
-            sel = torch.from_numpy(np.nonzero(dest == d)[0])
+            sel = torch.from_numpy(np.nonzero(dest == min(d, G))[0])   # d >= G: copies of the skewed tuples
             n = sel.numel()
             if n:
                 kb[off: off + n] = keys[sel]
@@ -181,12 +182,13 @@ def test_sharded_gloo_matches_oracle(world, kind, n, theta):
         assert len(oh) > 0 and out[0][4] > 0
 
 
+@pytest.mark.parametrize("exchange", ["a2a", "p2p"])
 @pytest.mark.parametrize("world,kind,n,theta,mode", [(2, "zipf", 1 << 13, 1.0, "count"),
                                                      (4, "zipf", 1 << 13, 1.5, "count"),
                                                      (8, "graph", 1 << 13, 0.909, "count"),
                                                      (4, "zipf", 1 << 12, 0.75, "materialize"),
                                                      (8, "uniform", 1 << 12, 0.0, "count")])
-def test_sharded_localworld_cpu(world, kind, n, theta, mode):
+def test_sharded_localworld_cpu(world, kind, n, theta, mode, exchange):
     """The LocalWorld communicator (threads, the one-GPU harness's exchange) on CPU tensors."""
     import threading
 
@@ -201,7 +203,7 @@ def test_sharded_localworld_cpu(world, kind, n, theta, mode):
     def worker(g):
         out = torch.zeros((cap, 2), dtype=torch.int32) if mode == "materialize" else None
         res[g] = sharded.join_sharded(*(_shard(t, g, world) for t in (rk, rp, sk, sp)), config=cfg, ops=OracleOps(),
-                                      comm=lw.comm(g), mode=mode, out=out)
+                                      comm=lw.comm(g), mode=mode, out=out, exchange=exchange)
 
     th = [threading.Thread(target=worker, args=(g,)) for g in range(world)]
     for t in th:
