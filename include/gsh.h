@@ -358,6 +358,112 @@ GSH_API gsh_status gsh_ipc_handle(const void *d_ptr, void *handle, uint64_t *off
 GSH_API gsh_status gsh_ipc_open(const void *handle, void **d_ptr);
 GSH_API gsh_status gsh_ipc_close(void *d_ptr);
 
+/* ------------------------------------------------- native multi-GPU driver --
+ * gsh_join_sharded runs the whole per-rank protocol above (agreement, routing, exchange, the two
+ * local joins, the result reduction) in the library, over a communicator given as a table of
+ * collectives.  SURVEY.md §8(b) "gsh_join_sharded(..., ncclComm_t)", §8(e).  Three communicators
+ * are provided: an existing ncclComm_t (e.g. the one a torch.distributed NCCL process group
+ * owns), a new NCCL communicator from a unique id, and an in-process "local world" in which G
+ * host threads act as G ranks on any devices (the one-GPU multi-rank test harness).
+ * Every callback enqueues on / synchronises `stream` and returns a gsh_status. */
+typedef struct gsh_comm {
+    uint32_t rank, world;      /* this rank, number of ranks */
+    uint32_t same_process;     /* 1: every rank lives in this process (device pointers are valid
+                                  across ranks); 0: ranks are processes (buffers shared via CUDA IPC) */
+    uint32_t reserved;
+    void *ctx;                 /* the implementation's state */
+    /* d_buf[0..n) (device u64) := sum over ranks mod 2^64, in place */
+    gsh_status (*all_reduce_u64)(void *ctx, uint64_t *d_buf, uint64_t n, void *stream);
+    /* d_recv[g * bytes .. +bytes) := rank g's d_send[0..bytes) (device buffers) */
+    gsh_status (*all_gather)(void *ctx, const void *d_send, void *d_recv, uint64_t bytes, void *stream);
+    /* variable all-to-all of bytes: rank g receives h_send_bytes[g] bytes from d_send + h_send_off[g]
+       of every rank at d_recv + h_recv_off[src] (its h_recv_bytes[src] must match; host arrays of
+       world entries; zero-byte pairs are skipped) */
+    gsh_status (*all_to_all_v)(void *ctx, const void *d_send, const uint64_t *h_send_off,
+                               const uint64_t *h_send_bytes, void *d_recv, const uint64_t *h_recv_off,
+                               const uint64_t *h_recv_bytes, void *stream);
+    /* returns once every rank's work enqueued on its stream before the call is complete */
+    gsh_status (*barrier)(void *ctx, void *stream);
+    /* optional (may be NULL): release ranks blocked in a collective after this rank failed */
+    void (*abort)(void *ctx);
+} gsh_comm;
+
+/* NCCL communicators (libnccl.so.2 is looked up at run time: the copy already loaded in the
+ * process, e.g. torch's, else the system one; GSH_ERR_NCCL if none).  gsh_comm_nccl wraps an
+ * existing ncclComm_t (passed as void*, not owned); gsh_nccl_unique_id fills 128 bytes on one
+ * rank, which every rank passes to gsh_comm_nccl_init (collective over the world's ranks, with
+ * `device` current) to create an owned communicator.  gsh_comm_destroy frees what the
+ * constructor allocated (an owned NCCL communicator, or nothing). */
+GSH_API gsh_status gsh_comm_nccl(void *nccl_comm, gsh_comm *out);
+GSH_API gsh_status gsh_nccl_unique_id(void *id128);
+GSH_API gsh_status gsh_comm_nccl_init(const void *id128, uint32_t world, uint32_t rank, int device,
+                                      gsh_comm *out);
+GSH_API gsh_status gsh_comm_destroy(gsh_comm *comm);
+
+/* In-process world of `world` ranks (one host thread each): collectives are device copies
+ * between the ranks' buffers behind host barriers.  gsh_comm_local fills rank r's table; the
+ * world outlives every use of its tables. */
+GSH_API gsh_status gsh_local_world_create(uint32_t world, void **lw);
+GSH_API gsh_status gsh_comm_local(void *lw, uint32_t rank, gsh_comm *out);
+GSH_API gsh_status gsh_local_world_destroy(void *lw);
+
+/* Per-rank driver state: the comm table (copied), the device, and the grow-only device buffers of
+ * the protocol (receive / send buffers, the two local joins' workspaces, IPC mappings of the
+ * peers' receive buffers).  The receive sizes depend on the data, so -- unlike gsh_join -- the
+ * driver allocates (cudaMalloc) and keeps its buffers across calls; gsh_sharded_destroy frees
+ * them (call it on every rank after the last join, no collective involved). */
+typedef struct gsh_sharded gsh_sharded;
+GSH_API gsh_status gsh_sharded_create(const gsh_comm *comm, int device, gsh_sharded **ctx);
+GSH_API gsh_status gsh_sharded_destroy(gsh_sharded *ctx);
+
+typedef enum {
+    GSH_EXCHANGE_A2A = 0,      /* route into send buffers, then all_to_all_v of normal tuples and an
+                                  all-gather of skewed R; the normal exchange runs on a second stream
+                                  while the skewed-key join computes */
+    GSH_EXCHANGE_P2P = 1       /* the route kernel stores every tuple straight into its destination
+                                  rank's receive buffer (skewed R into every rank's): the scatter IS
+                                  the exchange (NVLink peer stores), then one barrier */
+} gsh_exchange;
+
+typedef struct {
+    uint64_t count;            /* GLOBAL |M| (identical on every rank) */
+    uint64_t checksum;         /* GLOBAL checksum mod 2^64 */
+    uint64_t written;          /* pairs written to this rank's out (MATERIALIZE) */
+    uint32_t overflow;         /* this rank's out was too small */
+    uint32_t n_heavy;          /* agreed skewed keys */
+    uint32_t route_bits, part_bits, large_threshold, heavy_threshold, cand_threshold;
+    uint32_t cand_overflow;    /* some rank's candidate table filled (exact, skew handling lost) */
+    uint64_t n_candidates;     /* candidates gathered over all ranks */
+    uint64_t n_union;          /* distinct candidates */
+    uint64_t local_r, local_s; /* this rank's input shard */
+    uint64_t normal_r, normal_s, heavy_r, heavy_s;   /* this rank's local join inputs */
+    uint64_t count_normal, count_heavy;               /* this rank's share of count */
+    uint64_t exchange_bytes;   /* bytes this rank moved to other ranks (a2a: normal tuples sent;
+                                  p2p: every remote store, skewed-R copies included) */
+    uint64_t broadcast_bytes;  /* a2a: skewed-R bytes received from the other ranks */
+    uint32_t launches;         /* libgsh kernels this call launched (local joins included) */
+    uint32_t exchange;         /* gsh_exchange used */
+    float ms_agree, ms_route, ms_exchange, ms_join_heavy, ms_join_normal, ms_reduce, ms_total;
+    gsh_result normal;         /* the local join of the routed normal shard */
+    gsh_result heavy;          /* the local join of all ranks' skewed R x this rank's skewed S */
+} gsh_sharded_result;
+
+/*
+ * gsh_join_sharded -- the hash-sharded GSH join; every rank calls it with its shards R, S (device
+ * SoA, any positional split of the global relations).  Steps: gsh_shard_plan on the all-reduced
+ * sizes, histogram -> all_reduce, candidates -> all_gather, agree -> all_reduce, select (the
+ * single-GPU skew rule on the whole input), route counts -> all_gather (the G x 2(G+1) count
+ * matrix fixes every buffer offset), route scatter + exchange (`exchange`), gsh_join of the
+ * normal shard (cfg->route_bits := log2 G) and of all skewed R x local skewed S (route_bits 0),
+ * all_reduce of (count, checksum).  The result equals gsh_join on the whole input bit-exactly.
+ * cfg: NULL = defaults (route_bits must be 0).  out: NULL iff COUNT; this rank's pairs.
+ * Returns GSH_ERR_INVALID for bad arguments (detected before any collective only when local), and
+ * any status a collective returns; after an error the comm's abort (if any) has been called.
+ */
+GSH_API gsh_status gsh_join_sharded(gsh_sharded *ctx, const gsh_relation *R, const gsh_relation *S,
+                                    gsh_out_mode mode, const gsh_output *out, const gsh_config *cfg,
+                                    gsh_exchange exchange, void *stream, gsh_sharded_result *res);
+
 /* ------------------------------------------------------------------- diagnostics -- */
 GSH_API const char *gsh_status_string(gsh_status s);
 GSH_API const char *gsh_last_error(void);

@@ -23,6 +23,7 @@ p64 = ctypes.POINTER(ctypes.c_uint64)
 
 GSH_OK, GSH_ERR_INVALID, GSH_ERR_NOMEM, GSH_ERR_CUDA, GSH_ERR_NCCL, GSH_ERR_INTERNAL = range(6)
 GSH_OUT_COUNT, GSH_OUT_MATERIALIZE = 0, 1
+GSH_EXCHANGE_A2A, GSH_EXCHANGE_P2P = 0, 1
 
 
 class GshRelation(ctypes.Structure):
@@ -108,6 +109,35 @@ class GshShardParams(ctypes.Structure):
     ]
 
 
+class GshComm(ctypes.Structure):
+    """gsh_comm: a table of collectives (function pointers kept opaque: filled by the library's
+    constructors gsh_comm_nccl / gsh_comm_nccl_init / gsh_comm_local)."""
+    _fields_ = [("rank", u32), ("world", u32), ("same_process", u32), ("reserved", u32), ("ctx", vp),
+                ("all_reduce_u64", vp), ("all_gather", vp), ("all_to_all_v", vp), ("barrier", vp), ("abort", vp)]
+
+
+class GshShardedResult(ctypes.Structure):
+    _fields_ = [
+        ("count", u64), ("checksum", u64), ("written", u64), ("overflow", u32), ("n_heavy", u32),
+        ("route_bits", u32), ("part_bits", u32), ("large_threshold", u32), ("heavy_threshold", u32),
+        ("cand_threshold", u32), ("cand_overflow", u32), ("n_candidates", u64), ("n_union", u64),
+        ("local_r", u64), ("local_s", u64), ("normal_r", u64), ("normal_s", u64), ("heavy_r", u64), ("heavy_s", u64),
+        ("count_normal", u64), ("count_heavy", u64), ("exchange_bytes", u64), ("broadcast_bytes", u64),
+        ("launches", u32), ("exchange", u32),
+        ("ms_agree", ctypes.c_float), ("ms_route", ctypes.c_float), ("ms_exchange", ctypes.c_float),
+        ("ms_join_heavy", ctypes.c_float), ("ms_join_normal", ctypes.c_float), ("ms_reduce", ctypes.c_float),
+        ("ms_total", ctypes.c_float),
+        ("normal", GshResult), ("heavy", GshResult),
+    ]
+
+    def as_dict(self) -> dict:
+        d = {}
+        for name, _ in self._fields_:
+            v = getattr(self, name)
+            d[name] = v.as_dict() if isinstance(v, GshResult) else v
+        return d
+
+
 # (name, restype, argtypes) for every entry point declared in include/gsh.h
 _PROTOS = [
     ("gsh_config_default", None, [ctypes.POINTER(GshConfig)]),
@@ -147,6 +177,18 @@ _PROTOS = [
     ("gsh_ipc_handle", ctypes.c_int, [vp, vp, p64]),
     ("gsh_ipc_open", ctypes.c_int, [vp, ctypes.POINTER(vp)]),
     ("gsh_ipc_close", ctypes.c_int, [vp]),
+    ("gsh_comm_nccl", ctypes.c_int, [vp, ctypes.POINTER(GshComm)]),
+    ("gsh_nccl_unique_id", ctypes.c_int, [vp]),
+    ("gsh_comm_nccl_init", ctypes.c_int, [vp, u32, u32, ctypes.c_int, ctypes.POINTER(GshComm)]),
+    ("gsh_comm_destroy", ctypes.c_int, [ctypes.POINTER(GshComm)]),
+    ("gsh_local_world_create", ctypes.c_int, [u32, ctypes.POINTER(vp)]),
+    ("gsh_comm_local", ctypes.c_int, [vp, u32, ctypes.POINTER(GshComm)]),
+    ("gsh_local_world_destroy", ctypes.c_int, [vp]),
+    ("gsh_sharded_create", ctypes.c_int, [ctypes.POINTER(GshComm), ctypes.c_int, ctypes.POINTER(vp)]),
+    ("gsh_sharded_destroy", ctypes.c_int, [vp]),
+    ("gsh_join_sharded", ctypes.c_int, [vp, ctypes.POINTER(GshRelation), ctypes.POINTER(GshRelation), ctypes.c_int,
+                                        ctypes.POINTER(GshOutput), ctypes.POINTER(GshConfig), ctypes.c_int, vp,
+                                        ctypes.POINTER(GshShardedResult)]),
     ("gsh_status_string", ctypes.c_char_p, [ctypes.c_int]),
     ("gsh_last_error", ctypes.c_char_p, []),
     ("gsh_version", ctypes.c_int, []),

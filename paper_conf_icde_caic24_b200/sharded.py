@@ -660,3 +660,276 @@ def run_local(world: int, shards, config=None, mode: str = "count", out_capacity
     for r in res:
         r.stats["wall_s"] = time.perf_counter() - t0
     return res
+
+
+# ------------------------------------------------------- native driver (gsh_join_sharded)
+EXCHANGES = {"a2a": _lib.GSH_EXCHANGE_A2A, "p2p": _lib.GSH_EXCHANGE_P2P}
+
+
+class NativeComm:
+    """A gsh_comm table (include/gsh.h) for the native driver: an NCCL communicator or one rank of
+    a NativeLocalWorld.  close() releases what the library allocated for it."""
+
+    def __init__(self, comm: _lib.GshComm, owner=None, destroy: bool = True):
+        self.c, self._owner, self._destroy = comm, owner, destroy
+
+    @property
+    def rank(self) -> int:
+        return int(self.c.rank)
+
+    @property
+    def world(self) -> int:
+        return int(self.c.world)
+
+    def close(self) -> None:
+        if self._destroy and self.c.ctx:
+            check(load().gsh_comm_destroy(ctypes.byref(self.c)), "gsh_comm_destroy")
+
+    def abort(self) -> None:
+        """Release the peers blocked in a collective (the comm's abort, when it has one)."""
+        if self.c.abort:
+            ctypes.CFUNCTYPE(None, ctypes.c_void_p)(self.c.abort)(self.c.ctx)
+
+
+class NativeLocalWorld:
+    """gsh_local_world_create: `world` ranks in this process, one host thread each (the one-GPU
+    multi-rank harness of the native driver)."""
+
+    def __init__(self, world: int):
+        lw = ctypes.c_void_p(0)
+        check(load().gsh_local_world_create(world, ctypes.byref(lw)), "gsh_local_world_create")
+        self.ptr, self.world = lw.value, world
+
+    def comm(self, rank: int) -> NativeComm:
+        c = _lib.GshComm()
+        check(load().gsh_comm_local(self.ptr, rank, ctypes.byref(c)), "gsh_comm_local")
+        return NativeComm(c, owner=self, destroy=False)
+
+    def close(self) -> None:
+        if self.ptr:
+            load().gsh_local_world_destroy(self.ptr)
+            self.ptr = None
+
+
+def nccl_comm(group=None, device=None, use_group_comm: bool = False) -> NativeComm:
+    """An NCCL gsh_comm for this rank of `group` (default: the world).  use_group_comm=True wraps the
+    process group's own ncclComm_t (gsh_comm_nccl; the group must be an initialised NCCL group);
+    otherwise a new communicator is created (gsh_nccl_unique_id on the group's rank 0, broadcast over
+    the group, gsh_comm_nccl_init on every rank)."""
+    lib = load()
+    pg = group if group is not None else dist.distributed_c10d._get_default_group()
+    dev = torch.device(device) if device is not None else torch.device("cuda", torch.cuda.current_device())
+    if use_group_comm:
+        ptr = pg._get_backend(torch.device("cuda", dev.index))._comm_ptr()
+        if not ptr:
+            raise RuntimeError("the process group has no initialised NCCL communicator")
+        c = _lib.GshComm()
+        check(lib.gsh_comm_nccl(ptr, ctypes.byref(c)), "gsh_comm_nccl")
+        return NativeComm(c)
+    rank, world = dist.get_rank(pg), dist.get_world_size(pg)
+    uid = (ctypes.c_uint8 * 128)()
+    if rank == 0:
+        check(lib.gsh_nccl_unique_id(uid), "gsh_nccl_unique_id")
+    box = [bytes(uid)]
+    dist.broadcast_object_list(box, src=dist.get_global_rank(pg, 0) if group is not None else 0, group=pg)
+    uid = (ctypes.c_uint8 * 128).from_buffer_copy(box[0])
+    c = _lib.GshComm()
+    check(lib.gsh_comm_nccl_init(uid, world, rank, dev.index, ctypes.byref(c)), "gsh_comm_nccl_init")
+    return NativeComm(c)
+
+
+class ShardedJoin:
+    """The native per-rank driver (gsh_sharded_create / gsh_join_sharded): the whole protocol of
+    join_sharded -- agreement, routing, exchange, the two local joins, the reduction -- runs inside
+    libgsh.so over the collectives of `comm`.  Buffers persist across calls (close() frees them)."""
+
+    def __init__(self, comm: NativeComm, device=None):
+        self.comm = comm
+        self.device = torch.device(device) if device is not None else torch.device("cuda", torch.cuda.current_device())
+        ctx = ctypes.c_void_p(0)
+        check(load().gsh_sharded_create(ctypes.byref(comm.c), self.device.index, ctypes.byref(ctx)),
+              "gsh_sharded_create")
+        self.ctx = ctx.value
+
+    def join(self, rk, rp, sk, sp, config=None, mode: str = "count", out=None, exchange: str = "p2p",
+             stream=None) -> JoinResult:
+        """This rank's shards in; the GLOBAL count / checksum out (identical on every rank); in
+        "materialize" mode `out` ((capacity, 2) int32 CUDA tensor) receives this rank's pairs."""
+        if exchange not in EXCHANGES:
+            raise ValueError("exchange must be 'a2a' or 'p2p'")
+        if mode not in ("count", "materialize"):
+            raise ValueError("mode must be 'count' or 'materialize'")
+        rk, rp = _check_dev(rk, "r_keys"), _check_dev(rp, "r_payloads")
+        sk, sp = _check_dev(sk, "s_keys"), _check_dev(sp, "s_payloads")
+        R, S = _rel(rk, rp, "R"), _rel(sk, sp, "S")
+        o = None
+        if mode == "materialize":
+            if out is None or out.dim() != 2 or out.shape[1] != 2 or not out.is_cuda:
+                raise ValueError("materialize needs out: a (capacity, 2) int32 CUDA tensor")
+            o = _lib.GshOutput(out.data_ptr() if out.numel() else None, out.shape[0])
+        res = _lib.GshShardedResult()
+        st = load().gsh_join_sharded(self.ctx, ctypes.byref(R), ctypes.byref(S), int(mode == "materialize"),
+                                     ctypes.byref(o) if o is not None else None,
+                                     ctypes.byref(config) if config is not None else None, EXCHANGES[exchange],
+                                     _stream_handle(stream, self.device), ctypes.byref(res))
+        check(st, "gsh_join_sharded")
+        w = int(res.written)
+        stats = res.as_dict()
+        stats.update(world=self.comm.world, rank=self.comm.rank, exchange=exchange, driver="native")
+        for name, nbytes in (("exchange", int(res.exchange_bytes)), ("broadcast", int(res.broadcast_bytes))):
+            ms = stats.get(f"ms_{name}", 0.0)
+            gbs = nbytes / (ms * 1e6) if ms > 0 else None
+            stats[f"{name}_GBps"] = gbs
+            stats[f"{name}_nvlink_frac"] = gbs / NVLINK_GBS if gbs is not None else None
+        return JoinResult(count=int(res.count), checksum=int(res.checksum), written=w, overflow=bool(res.overflow),
+                          pairs=(out[:w] if mode == "materialize" else None), stats=stats)
+
+    def close(self) -> None:
+        if self.ctx:
+            load().gsh_sharded_destroy(self.ctx)
+            self.ctx = None
+
+
+def run_local_native(world: int, shards, config=None, mode: str = "count", out_capacity: int = 0, device=None,
+                     exchange: str = "p2p", repeat: int = 1, calls=None, configs=None):
+    """The native driver for `world` logical ranks on ONE device (host threads + a native local
+    world).  shards[g] = (rk, rp, sk, sp) CUDA tensors of rank g; returns the per-rank JoinResults of
+    the last of `repeat` calls (rank order).  calls: a list of such shard lists, joined one after
+    another by the same per-rank drivers (buffer reuse and growth); the per-call results are then
+    returned.  configs: per-rank configs (default `config` everywhere)."""
+    lw = NativeLocalWorld(world)
+    seq = list(calls) if calls is not None else [shards] * repeat
+    dev = torch.device(device) if device is not None else seq[0][0][0].device
+    res: list = [[None] * world for _ in seq]
+    err: list = []
+
+    def worker(g):
+        drv = None
+        comm = lw.comm(g)
+        try:
+            with torch.cuda.device(dev):
+                s = torch.cuda.Stream(dev)
+                with torch.cuda.stream(s):
+                    drv = ShardedJoin(comm, dev)
+                    out = (torch.empty((out_capacity, 2), dtype=torch.int32, device=dev)
+                           if mode == "materialize" else None)
+                    cfg = configs[g] if configs is not None else config
+                    for i, sh in enumerate(seq):
+                        res[i][g] = drv.join(*sh[g], config=cfg, mode=mode, out=out, exchange=exchange)
+                s.synchronize()
+        except BaseException as e:  # the library aborted the world (or we do): the other ranks return too
+            err.append((g, e))
+            comm.abort()
+        finally:
+            if drv is not None:
+                drv.close()
+
+    th = [threading.Thread(target=worker, args=(g,)) for g in range(world)]
+    for t in th:
+        t.start()
+    for t in th:
+        t.join()
+    lw.close()
+    if err:
+        err.sort(key=lambda x: "peer rank failed" in str(x[1]))   # the root cause first
+        raise err[0][1]
+    return res if calls is not None else res[-1]
+
+
+class _DevBytes:
+    """A zero-copy uint8 view of raw device memory (CUDA array interface) for the callback comm."""
+
+    def __init__(self, ptr: int, n: int):
+        self.__cuda_array_interface__ = {"shape": (n,), "typestr": "|u1", "data": (ptr, False), "version": 3,
+                                         "strides": None}
+
+
+def _dev_bytes(ptr, n: int) -> torch.Tensor:
+    if n == 0:
+        return torch.empty(0, dtype=torch.uint8, device="cuda")
+    return torch.as_tensor(_DevBytes(int(ptr), int(n)), device="cuda")
+
+
+_ALLRED = ctypes.CFUNCTYPE(ctypes.c_int, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_uint64, ctypes.c_void_p)
+_ALLGATHER = ctypes.CFUNCTYPE(ctypes.c_int, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_uint64,
+                              ctypes.c_void_p)
+_P64 = ctypes.POINTER(ctypes.c_uint64)
+_A2AV = ctypes.CFUNCTYPE(ctypes.c_int, ctypes.c_void_p, ctypes.c_void_p, _P64, _P64, ctypes.c_void_p, _P64, _P64,
+                         ctypes.c_void_p)
+_BARRIER = ctypes.CFUNCTYPE(ctypes.c_int, ctypes.c_void_p, ctypes.c_void_p)
+
+
+class TorchGroupComm(NativeComm):
+    """A gsh_comm whose collectives are torch.distributed calls on `group` (any backend; payloads
+    staged through host memory, so meant for gloo process groups, e.g. several processes sharing
+    one GPU, where NCCL refuses to run).  The library calls back into Python for every collective;
+    the peer-store exchange still shares its receive buffers through CUDA IPC."""
+
+    def __init__(self, group=None):
+        self.group = group
+        rank, world = dist.get_rank(group), dist.get_world_size(group)
+        self._cbs = (_ALLRED(self._all_reduce), _ALLGATHER(self._all_gather), _A2AV(self._a2a),
+                     _BARRIER(self._barrier))
+        c = _lib.GshComm()
+        c.rank, c.world, c.same_process = rank, world, 0
+        c.ctx = None
+        c.all_reduce_u64, c.all_gather, c.all_to_all_v, c.barrier = (ctypes.cast(f, ctypes.c_void_p) for f in self._cbs)
+        super().__init__(c, destroy=False)
+
+    @staticmethod
+    def _sync(stream):
+        torch.cuda.ExternalStream(int(stream or 0)).synchronize() if stream else torch.cuda.synchronize()
+
+    def _guard(self, fn):
+        try:
+            fn()
+            return _lib.GSH_OK
+        except Exception:   # noqa: BLE001  (reported as a collective failure through the ABI)
+            import traceback
+            traceback.print_exc()
+            return _lib.GSH_ERR_NCCL
+
+    def _all_reduce(self, ctx, d, n, stream):
+        def go():
+            self._sync(stream)
+            t = _dev_bytes(d, 8 * n)
+            h = t.cpu().view(torch.int64)
+            dist.all_reduce(h, group=self.group)
+            t.copy_(h.view(torch.uint8))
+            torch.cuda.synchronize()
+        return self._guard(go)
+
+    def _all_gather(self, ctx, send, recv, nbytes, stream):
+        def go():
+            self._sync(stream)
+            src = _dev_bytes(send, nbytes).cpu()
+            out = [torch.empty_like(src) for _ in range(self.c.world)]
+            dist.all_gather(out, src, group=self.group)
+            _dev_bytes(recv, nbytes * self.c.world).copy_(torch.cat(out))
+            torch.cuda.synchronize()
+        return self._guard(go)
+
+    def _a2a(self, ctx, send, soff, sbytes, recv, roff, rbytes, stream):
+        def go():
+            self._sync(stream)
+            G = self.c.world
+            so, sb = [soff[g] for g in range(G)], [sbytes[g] for g in range(G)]
+            ro, rbn = [roff[g] for g in range(G)], [rbytes[g] for g in range(G)]
+            parts = [(_dev_bytes(send + so[g], sb[g]).cpu() if sb[g] else torch.empty(0, dtype=torch.uint8))
+                     for g in range(G)]
+            inp = torch.cat(parts)
+            out = torch.empty(sum(rbn), dtype=torch.uint8)
+            dist.all_to_all_single(out, inp, rbn, sb, group=self.group)
+            o = 0
+            for g in range(G):
+                if rbn[g]:
+                    _dev_bytes(recv + ro[g], rbn[g]).copy_(out[o: o + rbn[g]])
+                o += rbn[g]
+            torch.cuda.synchronize()
+        return self._guard(go)
+
+    def _barrier(self, ctx, stream):
+        def go():
+            self._sync(stream)
+            dist.barrier(group=self.group)
+        return self._guard(go)

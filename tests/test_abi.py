@@ -45,7 +45,10 @@ def test_status_strings_and_struct_sizes():
     assert lib.gsh_status_string(1) == b"GSH_ERR_INVALID"
     # the ctypes mirrors match the C compiler's layout of include/gsh.h field by field
     src = "#include <stdio.h>\n#include <stddef.h>\n#include \"gsh.h\"\nint main(void){\n"
-    for cname, cls in (("gsh_config", _lib.GshConfig), ("gsh_result", _lib.GshResult)):
+    structs = (("gsh_config", _lib.GshConfig), ("gsh_result", _lib.GshResult),
+               ("gsh_shard_params", _lib.GshShardParams), ("gsh_comm", _lib.GshComm),
+               ("gsh_sharded_result", _lib.GshShardedResult))
+    for cname, cls in structs:
         src += f'printf("%zu\\n", sizeof({cname}));\n'
         for f, _ in cls._fields_:
             src += f'printf("%zu\\n", offsetof({cname}, {f}));\n'
@@ -56,7 +59,7 @@ def test_status_strings_and_struct_sizes():
         subprocess.check_call(["gcc", "-std=c11", "-I", os.path.join(ROOT, "include"), c, "-o", exe])
         got = [int(x) for x in subprocess.check_output([exe]).split()]
     want = []
-    for cls in (_lib.GshConfig, _lib.GshResult):
+    for _, cls in structs:
         want.append(ctypes.sizeof(cls))
         want += [getattr(cls, f).offset for f, _ in cls._fields_]
     assert got == want
