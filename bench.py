@@ -9,10 +9,12 @@ the 126 MB L2, so no flush is needed between steps.
 
   python bench.py [--gpus N] [--steps K] [--warmup W] [--impl gsh|reference] [--workload cfg2|cfg1|zipf]
   N > 1: one process per GPU under torch.distributed.run (started here when WORLD_SIZE is unset);
-  hash-sharded join over NCCL (sharded.join_sharded; weak scaling: each rank holds a shard of the
-  workload's per-GPU size, so the job joins N x that size per side).
-  --fake-ranks G: the same sharded step for G logical ranks sharing ONE GPU (threads, device-copy
-  exchange): exercises the multi-GPU code path on a one-GPU box; never the headline number.
+  hash-sharded join: gsh_join_sharded (the native driver in libgsh) over an NCCL communicator,
+  the route kernel storing straight into the peers' receive buffers (--exchange p2p, default) or
+  NCCL all-to-all (--exchange a2a); --driver python runs sharded.join_sharded instead.  Weak
+  scaling: each rank holds a shard of the workload's per-GPU size, so the job joins N x that size.
+  --fake-ranks G: the same sharded step for G logical ranks sharing ONE GPU (threads, the
+  library's local world): exercises the multi-GPU code path on a one-GPU box; never the headline.
 """
 from __future__ import annotations
 
@@ -70,8 +72,12 @@ def parse():
     ap.add_argument("--no-sweep", action="store_true", help="skip the theta_sweep sub-object (N=1 only)")
     ap.add_argument("--input-side", action="store_true",
                     help="time only the input side (partition, detect, split): gsh_config.input_side_only")
-    ap.add_argument("--exchange", default="a2a", choices=["a2a", "p2p"],
-                    help="multi-GPU exchange: NCCL all_to_all (a2a) or the route kernel's direct peer stores (p2p)")
+    ap.add_argument("--exchange", default="p2p", choices=["a2a", "p2p"],
+                    help="multi-GPU exchange: the route kernel's direct peer stores (p2p) or NCCL all_to_all (a2a)")
+    ap.add_argument("--sharded", action="store_true",
+                    help="run the hash-sharded step over NCCL even with one GPU (world of one)")
+    ap.add_argument("--driver", default="native", choices=["native", "python"],
+                    help="multi-GPU protocol: gsh_join_sharded inside libgsh (native) or sharded.join_sharded")
     ap.add_argument("--fake-ranks", type=int, default=0,
                     help="run the sharded step for G logical ranks on one GPU (code-path check, not a headline)")
     return ap.parse_args()
@@ -333,7 +339,8 @@ def flatten(r, world):
     st = r.stats
     if world == 1 and "join_normal" not in st:
         return {k: v for k, v in st.items() if k.startswith("ms_")}, st.get("launches", 0), st
-    jn, jh = st.get("join_normal") or {}, st.get("join_heavy") or {}
+    jn = st.get("join_normal") or st.get("normal") or {}   # python driver / native driver
+    jh = st.get("join_heavy") or st.get("heavy") or {}
     ph = {k: v for k, v in st.items() if k.startswith("ms_")}
     for k, v in jn.items():
         if k.startswith("ms_") and k != "ms_total":
@@ -385,7 +392,9 @@ def sharded_summary(phases, st, world):
     (900 GB/s per direction per GPU)."""
     keys = ("ms_agree", "ms_route", "ms_exchange", "ms_broadcast", "ms_join_normal", "ms_join_heavy", "ms_reduce")
     out = {k: phases.get(k) for k in keys}
-    for name, nb in (("exchange", st.get("exchange_send_bytes", 0)), ("broadcast", st.get("broadcast_recv_bytes", 0))):
+    xb = st.get("exchange_send_bytes", st.get("exchange_bytes", 0))
+    bb = st.get("broadcast_recv_bytes", st.get("broadcast_bytes", 0))
+    for name, nb in (("exchange", xb), ("broadcast", bb)):
         ms = phases.get(f"ms_{name}") or 0.0
         gbs = nb / (ms * 1e6) if ms > 0 else None
         out[f"{name}_bytes_per_rank"] = nb
@@ -414,8 +423,11 @@ def main():
     if args.mode == "materialize":
         desc = desc.replace("COUNT", "MATERIALIZE")
     dist = None
-    if world > 1:
+    nccl_world = world > 1 or args.sharded
+    if nccl_world:
         import torch.distributed as dist
+        for k, v in (("MASTER_ADDR", "127.0.0.1"), ("MASTER_PORT", "29541"), ("RANK", "0"), ("WORLD_SIZE", "1")):
+            os.environ.setdefault(k, v)
         dist.init_process_group("nccl", device_id=dev)
     extra = json.loads(os.environ.get("GSH_BENCH_CFG", "{}"))  # experiments only
     if args.detect == "sampled":
@@ -426,20 +438,30 @@ def main():
         extra["input_side_only"] = True
     cfg = gsh.make_config(timing=True, **extra)
     fake = args.fake_ranks if world == 1 else 0   # 1 = the sharded protocol with one rank
+    native = args.driver == "native"
     if fake >= 1:
         # G logical ranks on this one GPU: each holds a 1/G positional shard of ONE workload
         full = make_data(kind, n, theta, args.seed, dev, 0)
         shards = [tuple(t[g * n // fake:(g + 1) * n // fake] for t in full) for g in range(fake)]
         rk, rp, sk, sp = full
+        runner = sharded.LocalNativeRunner(fake, dev) if native else None
 
         def step():
-            rs = sharded.run_local(fake, shards, config=cfg, exchange=args.exchange)
+            if native:
+                t0 = time.perf_counter()
+                rs = runner.run(shards, config=cfg, exchange=args.exchange)
+                rs[0].stats["wall_s"] = time.perf_counter() - t0
+            else:
+                rs = sharded.run_local(fake, shards, config=cfg, exchange=args.exchange)
             rs[0].stats["launches"] = sum(x.stats.get("launches", 0) for x in rs)
             return rs[0]
-    elif world > 1:
+    elif nccl_world:
         rk, rp, sk, sp = make_data(kind, n, theta, args.seed, dev, rank)
+        drv = sharded.ShardedJoin(sharded.nccl_comm(device=dev), dev) if native else None
 
         def step():
+            if native:
+                return drv.join(rk, rp, sk, sp, config=cfg, exchange=args.exchange)
             return sharded.join_sharded(rk, rp, sk, sp, config=cfg, exchange=args.exchange)
     else:
         rk, rp, sk, sp = make_data(kind, n, theta, args.seed, dev, rank)
@@ -449,7 +471,7 @@ def main():
         def step():
             return gsh.join(rk, rp, sk, sp, mode=args.mode, out=out, config=cfg, workspace=ws)
     torch.cuda.synchronize()
-    multi = world > 1 or fake >= 1
+    multi = nccl_world or fake >= 1
 
     for _ in range(max(3, args.warmup)):
         r = step()
@@ -494,7 +516,7 @@ def main():
     if not args.no_e2e and not fake:
         hk = [t.cpu().pin_memory() for t in (rk, rp, sk, sp)]
         ke = max(2, min(args.steps, 5))
-        if world == 1:
+        if not multi:
             ws_h = torch.empty(gsh._lib.load().gsh_host_workspace_bytes(n, n, 0, 0, None), dtype=torch.uint8,
                                device=dev)
 
@@ -504,8 +526,11 @@ def main():
         else:
             def estep():
                 d = [h.to(dev, non_blocking=True) for h in hk]
-                return sharded.join_sharded(*d, config=cfg)
-            api, d2h = "H2D of the rank's pinned shard + sharded.join_sharded", 16
+                if native:
+                    return drv.join(*d, config=cfg, exchange=args.exchange)
+                return sharded.join_sharded(*d, config=cfg, exchange=args.exchange)
+            api, d2h = ("H2D of the rank's pinned shard + " +
+                        ("gsh_join_sharded" if native else "sharded.join_sharded")), 16
         for _ in range(2):
             estep()
         if dist:
@@ -529,14 +554,14 @@ def main():
         del hk
 
     sweep = None
-    if world == 1 and not fake and not args.no_sweep and args.workload == "cfg2" and args.mode == "count":
+    if not multi and not args.no_sweep and args.workload == "cfg2" and args.mode == "count":
         del rk, rp, sk, sp, ws
         torch.cuda.empty_cache()
         sweep = theta_sweep(gsh, dev, args.seed)
         rk, rp, sk, sp = make_data(kind, n, theta, args.seed, dev, rank)
 
     base = None
-    if rank == 0 and world == 1 and not fake and not args.no_cpu_baseline:
+    if rank == 0 and not multi and not args.no_cpu_baseline:
         base = cpu_baseline(kind, n, theta, args.seed, rk, rp, sk, sp, r)
 
     if rank == 0:
@@ -547,7 +572,8 @@ def main():
             "data": "synthetic (datagen, seeded)",
             "config": {"workload": desc, "n_r": n * world, "n_s": n * world, "mode": args.mode, "detect": args.detect,
                        "exchange": args.exchange if multi else None,
-                       "parallelism": (f"hash-sharded x{world} (NCCL)" if world > 1 else
+                       "driver": (("gsh_join_sharded" if native else "sharded.join_sharded") if multi else None),
+                       "parallelism": (f"hash-sharded x{world} (NCCL)" if nccl_world else
                                        f"{fake} logical ranks on one GPU (code-path check)" if fake >= 1 else
                                        "single GPU"),
                        "l2": "inputs 2 GiB per GPU > 126 MB L2: no flush needed" if n >= (1 << 24) else

@@ -231,5 +231,12 @@ int launch_count_keys(const uint32_t* keys, uint64_t n, const uint32_t* q, uint6
                       cudaStream_t s);
 int launch_radix_hist(const uint32_t* keys, uint64_t n, uint32_t hi_bits, uint32_t nbits, uint64_t* hist,
                       cudaStream_t s);
+// shard.cu: this rank's route counts without reading the keys again (native driver, route_bits <=
+// part_bits): destination sums of the LOCAL partition histogram, minus the local counts of the
+// skewed keys (exact: every skewed key lies in a large partition, where the local table counts
+// every key), which go to destination G.  out = [R counts (G+1) | S counts (G+1)].
+int launch_route_counts_from_hist(const uint64_t* hist_local, uint32_t part_bits, uint32_t route_bits,
+                                  const uint32_t* uni, const uint64_t* cnt_global, const uint64_t* cnt_local,
+                                  uint64_t m, uint32_t heavy_threshold, uint64_t* out, cudaStream_t s);
 
 }  // namespace gsh

@@ -933,30 +933,34 @@ int launch_scatter(const Plan& p, int pass, const uint32_t* const keys[2], const
 }
 
 // ----------------------------------------------- standalone radix histogram (ABI) --
-// Shared-memory bins for up to 2^14 digits; wider histograms aggregate per warp and go
-// straight to global atomics.
-__global__ void k_radix_hist(const uint32_t* __restrict__ keys, uint64_t n, uint32_t shift, uint32_t mask,
-                             unsigned long long* __restrict__ hist, int use_smem) {
+// Shared-memory bins, one window of up to 2^15 digits per CTA (128 KB of u32 counters): a
+// 16-bit histogram runs as two windows (blockIdx.y), each CTA reading its key range once per
+// window and counting the keys whose digit falls in it.  atomicAdd(.., 1) without a return value
+// is the hardware-aggregated ATOMS.POPC.INC (no __match_any_sync: ~64 cycles per call).
+constexpr uint32_t kHistWindowBits = 15;
+
+__global__ void __launch_bounds__(1024, 1) k_radix_hist(const uint32_t* __restrict__ keys, uint64_t n,
+                                                        uint32_t shift, uint32_t mask,
+                                                        unsigned long long* __restrict__ hist) {
     extern __shared__ uint32_t hs[];
-    if (use_smem) {
-        for (uint32_t i = threadIdx.x; i <= mask; i += blockDim.x) hs[i] = 0;
-        __syncthreads();
-    }
-    for (uint64_t i = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; i - threadIdx.x < n;
-         i += uint64_t(gridDim.x) * blockDim.x) {
-        bool v = i < n;
-        uint32_t bin = v ? ((hash32(keys[i]) >> shift) & mask) : (0x80000000u | lane_id());
-        uint32_t peers = __match_any_sync(kFull, bin);
-        if (v && (peers & lanemask_lt()) == 0) {
-            if (use_smem) atomicAdd(&hs[bin], (uint32_t)__popc(peers));
-            else atomicAdd(&hist[bin], (unsigned long long)__popc(peers));
+    const uint32_t wlen = umin64(uint64_t(mask) + 1, 1u << kHistWindowBits);
+    const uint32_t wlo = blockIdx.y * wlen;
+    for (uint32_t i = threadIdx.x; i < wlen; i += blockDim.x) hs[i] = 0;
+    __syncthreads();
+    const uint64_t stride = uint64_t(gridDim.x) * blockDim.x;
+    for (uint64_t i = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; i < n; i += 4 * stride) {
+        uint32_t k[4];
+#pragma unroll
+        for (int j = 0; j < 4; ++j) k[j] = i + j * stride < n ? __ldcs(keys + i + j * stride) : 0u;
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+            const uint32_t bin = ((hash32(k[j]) >> shift) & mask) - wlo;
+            if (i + j * stride < n && bin < wlen) atomicAdd(&hs[bin], 1u);
         }
     }
-    if (use_smem) {
-        __syncthreads();
-        for (uint32_t i = threadIdx.x; i <= mask; i += blockDim.x)
-            if (hs[i]) atomicAdd(&hist[i], (unsigned long long)hs[i]);
-    }
+    __syncthreads();
+    for (uint32_t i = threadIdx.x; i < wlen; i += blockDim.x)
+        if (hs[i]) atomicAdd(&hist[wlo + i], (unsigned long long)hs[i]);
 }
 
 int launch_radix_hist(const uint32_t* keys, uint64_t n, uint32_t hi_bits, uint32_t nbits, uint64_t* hist,
@@ -964,15 +968,14 @@ int launch_radix_hist(const uint32_t* keys, uint64_t n, uint32_t hi_bits, uint32
     if (n == 0) return 0;
     const uint32_t F = 1u << nbits;
     const uint32_t shift = nbits ? (32 - hi_bits - nbits) : 0;
-    const int use_smem = nbits <= 14;
-    size_t smem = use_smem ? size_t(F) * 4 : 0;
+    const uint32_t wlen = F < (1u << kHistWindowBits) ? F : (1u << kHistWindowBits);
     static std::once_flag attr_once[kMaxDevices];   // > 48 KB of dynamic shared memory: opt in once per device
     once_per_device(attr_once, [&] {
-        cudaFuncSetAttribute(k_radix_hist, cudaFuncAttributeMaxDynamicSharedMemorySize, 64 * 1024);
+        cudaFuncSetAttribute(k_radix_hist, cudaFuncAttributeMaxDynamicSharedMemorySize, (4u << kHistWindowBits));
     });
-    unsigned grid = (unsigned)umin64((n + 1023) / 1024, 148);
-    k_radix_hist<<<grid, 1024, smem, s>>>(keys, n, shift, F - 1, reinterpret_cast<unsigned long long*>(hist),
-                                          use_smem);
+    const dim3 grid((unsigned)umin64((n + 4095) / 4096, 148), F / wlen);
+    k_radix_hist<<<grid, 1024, size_t(wlen) * 4, s>>>(keys, n, shift, F - 1,
+                                                      reinterpret_cast<unsigned long long*>(hist));
     return 1;
 }
 

@@ -34,11 +34,16 @@ constexpr uint64_t kCandMaxSlots = 1ull << 27;
 
 // ------------------------------------------------------------------ large partitions --
 __global__ void k_shard_large(const unsigned long long* __restrict__ hist, uint32_t F, uint32_t L, int force_normal,
-                              uint8_t* __restrict__ large) {
+                              uint8_t* __restrict__ large, unsigned long long* __restrict__ nlarge) {
+    unsigned long long t = 0;   // global tuples in large partitions (sizes the local count table)
     for (uint32_t p = blockIdx.x * blockDim.x + threadIdx.x; p < F; p += gridDim.x * blockDim.x) {
         const unsigned long long cr = hist[p], cs = hist[F + p];
-        large[p] = (!force_normal && cr > 0 && cs > 0 && (cr > L || cs > L)) ? 1 : 0;
+        const bool lg = !force_normal && cr > 0 && cs > 0 && (cr > L || cs > L);
+        large[p] = lg ? 1 : 0;
+        if (lg) t += cr + cs;
     }
+    for (int o = 16; o > 0; o >>= 1) t += __shfl_xor_sync(kFull, t, o);
+    if (lane_id() == 0 && t) atomicAdd(nlarge, t);
 }
 
 // -------------------------------------------------- exact local counts of large keys --
@@ -78,6 +83,7 @@ struct CandWs {
     unsigned long long* nout;
     unsigned int* overflow;
     uint32_t* slots_used;   // T's slot count (log2 in the high byte is recomputed from it)
+    unsigned long long* nlarge;   // global tuples in large partitions
     uint8_t* large;
     unsigned long long* key;
     uint32_t* cnt;
@@ -96,6 +102,7 @@ static CandWs cand_ws(void* ws, uint32_t cap) {
     w.nout = reinterpret_cast<unsigned long long*>(b);
     w.overflow = reinterpret_cast<unsigned int*>(b + 8);
     w.slots_used = reinterpret_cast<uint32_t*>(b + 12);
+    w.nlarge = reinterpret_cast<unsigned long long*>(b + 16);
     w.large = b + 256;
     w.key = reinterpret_cast<unsigned long long*>(b + 256 + 65536);
     w.cnt = reinterpret_cast<uint32_t*>(w.key + cap);
@@ -195,12 +202,8 @@ __global__ void k_route_count(const uint32_t* __restrict__ keys, uint64_t n, uin
     const uint32_t G1 = (1u << rb) + 1;
     for (uint32_t i = threadIdx.x; i < G1; i += blockDim.x) c[i] = 0;
     __syncthreads();
-    for (uint64_t i = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; i - threadIdx.x < n;
-         i += uint64_t(gridDim.x) * blockDim.x) {
-        const bool v = i < n;
-        const uint32_t d = v ? route_dest(hash32(__ldcs(keys + i)), rb, hs) : (0x10000u | lane_id());
-        const uint32_t peers = __match_any_sync(kFull, d);
-        if (v && (peers & lanemask_lt()) == 0) atomicAdd(&c[d], (uint32_t)__popc(peers));
+    for (uint64_t i = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; i < n; i += uint64_t(gridDim.x) * blockDim.x) {
+        if (i < n) atomicAdd(&c[route_dest(hash32(__ldcs(keys + i)), rb, hs)], 1u);   // ATOMS.POPC.INC
     }
     __syncthreads();
     for (uint32_t i = threadIdx.x; i < G1; i += blockDim.x)
@@ -212,11 +215,11 @@ __global__ void k_route_count(const uint32_t* __restrict__ keys, uint64_t n, uin
 // atomic on its cursor, permute the tile into shared memory grouped by destination, then write
 // runs with consecutive threads on consecutive addresses of the destination buffer.
 constexpr int kRouteBlock = 512;
-constexpr int kRouteIpt = 16;
+constexpr int kRouteIpt = 8;
 constexpr uint32_t kRouteTile = kRouteBlock * kRouteIpt;
 constexpr size_t kRouteSmem = size_t(kRouteTile) * (4 + 4 + 2);
 
-__global__ void __launch_bounds__(kRouteBlock, 1) k_route_scatter(const uint32_t* __restrict__ keys,
+__global__ void __launch_bounds__(kRouteBlock, 2) k_route_scatter(const uint32_t* __restrict__ keys,
                                                               const uint32_t* __restrict__ pays, uint64_t n,
                                                               uint32_t rb, HeavySet hs,
                                                               const unsigned long long* __restrict__ dst,
@@ -226,8 +229,9 @@ __global__ void __launch_bounds__(kRouteBlock, 1) k_route_scatter(const uint32_t
     uint32_t* s_p = s_k + kRouteTile;
     uint16_t* s_d = reinterpret_cast<uint16_t*>(s_p + kRouteTile);
     __shared__ uint32_t cnt[kMaxShardWorld + 1], pre[kMaxShardWorld + 1];
-    __shared__ unsigned long long base[kMaxShardWorld + 1];
+    __shared__ unsigned long long base[kMaxShardWorld + 1], wk[kMaxShardWorld + 1], wp[kMaxShardWorld + 1];
     const uint32_t G1 = (1u << rb) + 1;
+    const uint32_t dbits = rb + 2;   // destinations 0..G (normal, heavy) and G1 (invalid) fit
     const uint64_t ntiles = (n + kRouteTile - 1) / kRouteTile;
     for (uint64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
         for (uint32_t i = threadIdx.x; i < G1; i += blockDim.x) cnt[i] = 0;
@@ -244,8 +248,16 @@ __global__ void __launch_bounds__(kRouteBlock, 1) k_route_scatter(const uint32_t
 #pragma unroll
         for (int j = 0; j < kRouteIpt; ++j) {
             const bool v = t0 + uint64_t(j) * kRouteBlock + threadIdx.x < n;
-            const uint32_t d = v ? route_dest(hash32(k[j]), rb, hs) : (0x10000u | lane_id());
-            const uint32_t peers = __match_any_sync(kFull, d);
+            const uint32_t d = v ? route_dest(hash32(k[j]), rb, hs) : G1;   // G1: invalid lanes' own class
+            // lanes with the same destination: AND of rb + 2 bit ballots (cheaper than match_any)
+            uint32_t peers = kFull;
+#pragma unroll
+            for (uint32_t b = 0; b < 10; ++b) {
+                if (b < dbits) {
+                    const uint32_t m = __ballot_sync(kFull, (d >> b) & 1u);
+                    peers &= ((d >> b) & 1u) ? m : ~m;
+                }
+            }
             const uint32_t leader = __ffs(peers) - 1;
             uint32_t b = 0;
             if (v && lane_id() == leader) b = atomicAdd(&cnt[d], (uint32_t)__popc(peers));
@@ -276,9 +288,16 @@ __global__ void __launch_bounds__(kRouteBlock, 1) k_route_scatter(const uint32_t
                 e += c[q];
             }
         }
-        for (uint32_t i = threadIdx.x; i < G1; i += blockDim.x)
-            base[i] = cnt[i] ? atomicAdd(&cur[i], (unsigned long long)cnt[i]) : 0ull;
         __syncthreads();
+        // reserve each destination's run; wk / wp: write addresses biased so that tile position i of
+        // destination d's run lands at wk[d] + 4 i (unsigned wrap-around is intended)
+        for (uint32_t i = threadIdx.x; i < G1; i += blockDim.x) {
+            const unsigned long long b = cnt[i] ? atomicAdd(&cur[i], (unsigned long long)cnt[i]) : 0ull;
+            const unsigned long long bias = 4ull * (b - pre[i]);
+            wk[i] = dst[2 * i] + bias;
+            wp[i] = dst[2 * i + 1] + bias;
+            base[i] = b;
+        }
 #pragma unroll
         for (int j = 0; j < kRouteIpt; ++j) {
             if (dr[j] != 0xffffffffu) {
@@ -292,18 +311,78 @@ __global__ void __launch_bounds__(kRouteBlock, 1) k_route_scatter(const uint32_t
         const uint32_t tn = (uint32_t)umin64(kRouteTile, n - t0);
         for (uint32_t i = threadIdx.x; i < tn; i += kRouteBlock) {
             const uint32_t d = s_d[i];
-            const uint64_t pos = base[d] + (i - pre[d]);
-            const uint32_t kk = s_k[i], pp = s_p[i];
-            reinterpret_cast<uint32_t*>(dst[2 * d])[pos] = kk;
-            reinterpret_cast<uint32_t*>(dst[2 * d + 1])[pos] = pp;
-            if (d == G1 - 1)   // the heavy destination: further copies (one per peer GPU's R_H buffer)
-                for (uint32_t c = 1; c < heavy_copies; ++c) {
-                    reinterpret_cast<uint32_t*>(dst[2 * (d + c)])[pos] = kk;
-                    reinterpret_cast<uint32_t*>(dst[2 * (d + c) + 1])[pos] = pp;
+            *reinterpret_cast<uint32_t*>(wk[d] + 4ull * i) = s_k[i];
+            *reinterpret_cast<uint32_t*>(wp[d] + 4ull * i) = s_p[i];
+        }
+        if (heavy_copies > 1) {   // the skewed run again into every further R_H buffer (peer GPUs')
+            const uint32_t h0 = pre[G1 - 1], hn = cnt[G1 - 1];
+            const unsigned long long hb = base[G1 - 1];
+            for (uint32_t c = 1; c < heavy_copies; ++c)
+                for (uint32_t i = threadIdx.x; i < hn; i += kRouteBlock) {
+                    reinterpret_cast<uint32_t*>(dst[2 * (G1 - 1 + c)])[hb + i] = s_k[h0 + i];
+                    reinterpret_cast<uint32_t*>(dst[2 * (G1 - 1 + c) + 1])[hb + i] = s_p[h0 + i];
                 }
         }
         __syncthreads();
     }
+}
+
+__global__ void __launch_bounds__(1024, 1)
+k_route_from_hist(const unsigned long long* __restrict__ hist, uint32_t B, uint32_t rb,
+                  const uint32_t* __restrict__ uni, IsHeavy global, const unsigned long long* __restrict__ cloc,
+                  uint64_t m, unsigned long long* __restrict__ out) {
+    __shared__ unsigned long long acc[2][kMaxShardWorld + 1];
+    const uint32_t G = 1u << rb, F = 1u << B;
+    for (uint32_t i = threadIdx.x; i <= G; i += blockDim.x) acc[0][i] = acc[1][i] = 0;
+    __syncthreads();
+    const uint32_t dshift = B - rb;   // partition p = top B bits of h; its destination = top rb bits
+    {   // each thread sums a contiguous range of partitions, flushing when the destination changes
+        const uint32_t per = (F + blockDim.x - 1) / blockDim.x, p0 = threadIdx.x * per, p1 = min(F, p0 + per);
+        unsigned long long sr = 0, ss = 0;
+        uint32_t dcur = p0 >> dshift;
+        for (uint32_t p = p0; p < p1; ++p) {
+            if ((p >> dshift) != dcur) {
+                atomicAdd(&acc[0][dcur], sr);
+                atomicAdd(&acc[1][dcur], ss);
+                sr = ss = 0;
+                dcur = p >> dshift;
+            }
+            sr += hist[p];
+            ss += hist[F + p];
+        }
+        if (p0 < p1) {
+            atomicAdd(&acc[0][dcur], sr);
+            atomicAdd(&acc[1][dcur], ss);
+        }
+    }
+    for (uint64_t u = threadIdx.x; u < m; u += blockDim.x) {
+        if (!global(u)) continue;
+        const uint32_t d = rb ? (uni[u] >> (32 - rb)) : 0u;
+        const unsigned long long cr = cloc[2 * u], cs = cloc[2 * u + 1];
+        if (cr) {
+            atomicAdd(&acc[0][d], 0ull - cr);
+            atomicAdd(&acc[0][G], cr);
+        }
+        if (cs) {
+            atomicAdd(&acc[1][d], 0ull - cs);
+            atomicAdd(&acc[1][G], cs);
+        }
+    }
+    __syncthreads();
+    for (uint32_t i = threadIdx.x; i <= G; i += blockDim.x) {
+        out[i] = acc[0][i];
+        out[G + 1 + i] = acc[1][i];
+    }
+}
+
+int launch_route_counts_from_hist(const uint64_t* hist_local, uint32_t part_bits, uint32_t route_bits,
+                                  const uint32_t* uni, const uint64_t* cnt_global, const uint64_t* cnt_local,
+                                  uint64_t m, uint32_t heavy_threshold, uint64_t* out, cudaStream_t s) {
+    IsHeavy f{reinterpret_cast<const unsigned long long*>(cnt_global), heavy_threshold};
+    k_route_from_hist<<<1, 1024, 0, s>>>(reinterpret_cast<const unsigned long long*>(hist_local), part_bits,
+                                         route_bits, uni, f, reinterpret_cast<const unsigned long long*>(cnt_local),
+                                         m, reinterpret_cast<unsigned long long*>(out));
+    return 1;
 }
 
 // Per-device one-time opt-in for > 48 KB of dynamic shared memory.
@@ -382,23 +461,38 @@ gsh_status gsh_shard_candidates(const gsh_relation* R, const gsh_relation* S, co
     if (!workspace || workspace_bytes < cand_ws_bytes(cap_t) || (reinterpret_cast<uintptr_t>(workspace) & 255u))
         return api_fail(GSH_ERR_INVALID, "workspace NULL, misaligned or smaller than gsh_shard_workspace_bytes");
     cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
-    CandWs w = cand_ws(workspace, cap_t);
-    const uint32_t F = 1u << p->part_bits, logcap = log2_pow2(cap_t);
+    const uint32_t F = 1u << p->part_bits;
     cudaMemsetAsync(workspace, 0, 256, s);
-    cudaMemsetAsync(w.key, 0, size_t(cap_t) * 16, s);
-    cudaMemcpyAsync(w.slots_used, &cap_t, 4, cudaMemcpyHostToDevice, s);
     k_shard_large<<<(F + 255) / 256, 256, 0, s>>>(reinterpret_cast<const unsigned long long*>(d_hist_global), F,
-                                                  p->large_threshold, p->force_all_normal, w.large);
+                                                  p->large_threshold, p->force_all_normal,
+                                                  cand_ws(workspace, cap_t).large, cand_ws(workspace, cap_t).nlarge);
+    // the count table only needs room for this rank's tuples of large partitions (<= the global
+    // number): size it from the global count, so a skew-free input clears and scans ~nothing
+    unsigned long long nlarge = 0;
+    cudaError_t ce = cudaMemcpyAsync(&nlarge, cand_ws(workspace, cap_t).nlarge, 8, cudaMemcpyDeviceToHost, s);
+    if (ce == cudaSuccess) ce = cudaStreamSynchronize(s);
+    if (ce != cudaSuccess) return api_cuda("shard_candidates large count");
+    uint32_t cap_u = 1024;
+    const uint64_t local_large = umin64(nlarge, R->n + S->n);
+    while (cap_u < 2 * local_large && cap_u < cap_t) cap_u <<= 1;
+    CandWs w = cand_ws(workspace, cap_u);
+    const uint32_t logcap = log2_pow2(cap_u);
+    cudaMemsetAsync(w.key, 0, size_t(cap_u) * 16, s);
+    cudaMemcpyAsync(w.slots_used, &cap_u, 4, cudaMemcpyHostToDevice, s);
     const uint32_t pshift = p->part_bits ? 32 - p->part_bits : 32;
-    if (R->n)
-        k_cand_count<<<148 * 8, 512, 0, s>>>(R->keys, R->n, 0, pshift, w.large, w.key, w.cnt, cap_t, logcap, w.overflow);
-    if (S->n)
-        k_cand_count<<<148 * 8, 512, 0, s>>>(S->keys, S->n, 1, pshift, w.large, w.key, w.cnt, cap_t, logcap, w.overflow);
-    k_cand_select<<<148 * 4, 256, 0, s>>>(w.key, w.cnt, cap_t, p->cand_threshold, d_cand, cap, w.nout);
+    if (nlarge) {
+        if (R->n)
+            k_cand_count<<<148 * 8, 512, 0, s>>>(R->keys, R->n, 0, pshift, w.large, w.key, w.cnt, cap_u, logcap,
+                                                 w.overflow);
+        if (S->n)
+            k_cand_count<<<148 * 8, 512, 0, s>>>(S->keys, S->n, 1, pshift, w.large, w.key, w.cnt, cap_u, logcap,
+                                                 w.overflow);
+        k_cand_select<<<148 * 4, 256, 0, s>>>(w.key, w.cnt, cap_u, p->cand_threshold, d_cand, cap, w.nout);
+    }
     gsh_status st = api_cuda("shard_candidates");
     if (st != GSH_OK) return st;
     unsigned long long hs[2] = {0, 0};
-    cudaError_t ce = cudaMemcpyAsync(hs, workspace, 16, cudaMemcpyDeviceToHost, s);
+    ce = cudaMemcpyAsync(hs, workspace, 16, cudaMemcpyDeviceToHost, s);
     if (ce == cudaSuccess) ce = cudaStreamSynchronize(s);
     if (ce != cudaSuccess) return api_cuda("shard_candidates sync");
     *h_n = hs[0];

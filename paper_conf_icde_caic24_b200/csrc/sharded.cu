@@ -331,7 +331,7 @@ struct gsh_sharded {
     int dev = 0;
     cudaStream_t xs = nullptr;     // exchange stream (a2a: normal all_to_all_v beside the skewed join)
     cudaEvent_t ev[10] = {};
-    Buf ctl, hist, candws, cand, gathered, agreews, uni, cnt, heavy, set, mat, sh, rx, sx, wsn, wsh;
+    Buf ctl, hist, hloc, cloc, candws, cand, gathered, agreews, uni, cnt, heavy, set, mat, sh, rx, sx, wsn, wsh;
     Buf rn, sn, rh;                // receive buffers: keys [0, cap), payloads [cap, 2 cap)
     uint64_t cap_rn = 0, cap_sn = 0, cap_rh = 0;   // p2p: the world-wide capacities (tuples)
     bool shared = false;           // p2p: rn / sn / rh are known to the peers
@@ -491,6 +491,11 @@ gsh_status run_sharded(gsh_sharded* x, const gsh_relation* R, const gsh_relation
     CK(ensure(x->hist, 2 * F * 8, s));
     CK(gsh_shard_histogram(R, S, &P, at<uint64_t>(x->hist), s));
     launches += (R->n > 0) + (S->n > 0);
+    const bool counts_from_hist = rb <= P.part_bits;   // route counts from the local histogram
+    if (counts_from_hist) {
+        CK(ensure(x->hloc, 2 * F * 8, s));
+        CK(cuda_status(cudaMemcpyAsync(x->hloc.p, x->hist.p, 2 * F * 8, cudaMemcpyDeviceToDevice, s), "local hist"));
+    }
     CK(c.all_reduce_u64(c.ctx, at<uint64_t>(x->hist), 2 * F, s));
     const size_t cws = gsh_shard_workspace_bytes(R->n, S->n);
     CK(ensure(x->candws, cws, s));
@@ -524,7 +529,7 @@ gsh_status run_sharded(gsh_sharded* x, const gsh_relation* R, const gsh_relation
         res->cand_overflow |= gs[2 * g + 1] ? 1u : 0u;
     }
     res->n_candidates = total;
-    uint64_t nh = 0;
+    uint64_t nh = 0, m = 0;
     if (stride) {
         CK(ensure(x->cand, stride * 4, s, /*keep=*/true));
         CK(ensure(x->gathered, G * stride * 4, s));
@@ -532,11 +537,14 @@ gsh_status run_sharded(gsh_sharded* x, const gsh_relation* R, const gsh_relation
         CK(ensure(x->agreews, gsh_shard_agree_workspace_bytes(uint64_t(G) * stride), s));
         CK(ensure(x->uni, total * 4, s));
         CK(ensure(x->cnt, total * 16, s));
-        uint64_t m = 0;
         CK(gsh_shard_agree(x->candws.p, x->candws.cap, at<uint32_t>(x->gathered), G, stride, sizes.data(),
                            x->agreews.p, x->agreews.cap, s, at<uint32_t>(x->uni), at<uint64_t>(x->cnt), total, &m));
         launches += 5;
         res->n_union = m;
+        if (counts_from_hist) {
+            CK(ensure(x->cloc, std::max<uint64_t>(m, 1) * 16, s));
+            CK(cuda_status(cudaMemcpyAsync(x->cloc.p, x->cnt.p, m * 16, cudaMemcpyDeviceToDevice, s), "local counts"));
+        }
         CK(c.all_reduce_u64(c.ctx, at<uint64_t>(x->cnt), 2 * m, s));
         CK(ensure(x->heavy, std::max<uint64_t>(m, 1) * 4, s));
         CK(gsh_shard_select(at<uint32_t>(x->uni), at<uint64_t>(x->cnt), m, &P, x->agreews.p, x->agreews.cap, s,
@@ -557,9 +565,19 @@ gsh_status run_sharded(gsh_sharded* x, const gsh_relation* R, const gsh_relation
     const uint32_t W = 2 * (G + 1);
     CK(ensure(x->mat, size_t(W) * (G + 1) * 8, s));
     uint64_t* d_mat = at<uint64_t>(x->mat);
-    CK(gsh_route_count(R->keys, R->n, rb, set, sb, d_mat + size_t(W) * G, s));
-    CK(gsh_route_count(S->keys, S->n, rb, set, sb, d_mat + size_t(W) * G + G + 1, s));
-    launches += (R->n > 0) + (S->n > 0);
+    if (counts_from_hist && !covf) {
+        // no second read of the keys: the local histogram's destination sums minus the skewed keys'
+        // exact local counts (this rank's count table did not overflow)
+        launch_route_counts_from_hist(at<uint64_t>(x->hloc), P.part_bits, rb, m ? at<uint32_t>(x->uni) : nullptr,
+                                      m ? at<uint64_t>(x->cnt) : nullptr, m ? at<uint64_t>(x->cloc) : nullptr, m,
+                                      P.heavy_threshold, d_mat + size_t(W) * G, s);
+        launches += 1;
+        CK(api_cuda("route counts"));
+    } else {
+        CK(gsh_route_count(R->keys, R->n, rb, set, sb, d_mat + size_t(W) * G, s));
+        CK(gsh_route_count(S->keys, S->n, rb, set, sb, d_mat + size_t(W) * G + G + 1, s));
+        launches += (R->n > 0) + (S->n > 0);
+    }
     CK(c.all_gather(c.ctx, d_mat + size_t(W) * G, d_mat, W * 8, s));
     std::vector<uint64_t> M(size_t(W) * G);
     CK(cuda_status(cudaMemcpyAsync(M.data(), d_mat, M.size() * 8, cudaMemcpyDeviceToHost, s), "count matrix"));
@@ -923,7 +941,7 @@ gsh_status gsh_sharded_destroy(gsh_sharded* x) {
     if (!x) return GSH_OK;
     cudaSetDevice(x->dev);
     close_peers(x);
-    for (gsh_sharded::Buf* b : {&x->ctl, &x->hist, &x->candws, &x->cand, &x->gathered, &x->agreews, &x->uni, &x->cnt,
+    for (gsh_sharded::Buf* b : {&x->ctl, &x->hist, &x->hloc, &x->cloc, &x->candws, &x->cand, &x->gathered, &x->agreews, &x->uni, &x->cnt,
                                 &x->heavy, &x->set, &x->mat, &x->sh, &x->rx, &x->sx, &x->wsn, &x->wsh, &x->rn, &x->sn,
                                 &x->rh})
         release(*b);

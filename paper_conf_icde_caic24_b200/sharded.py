@@ -790,50 +790,76 @@ class ShardedJoin:
             self.ctx = None
 
 
+class LocalNativeRunner:
+    """`world` logical ranks of the native driver on ONE device: a native local world, one
+    ShardedJoin (persistent buffers) and one stream per rank; run() joins one set of shards with a
+    host thread per rank (ctypes releases the GIL, so the ranks' protocol steps run concurrently)."""
+
+    def __init__(self, world: int, device=None):
+        self.world = world
+        self.dev = torch.device(device) if device is not None else torch.device("cuda", torch.cuda.current_device())
+        self.lw = NativeLocalWorld(world)
+        self.comms = [self.lw.comm(g) for g in range(world)]
+        with torch.cuda.device(self.dev):
+            self.drv = [ShardedJoin(c, self.dev) for c in self.comms]
+            self.streams = [torch.cuda.Stream(self.dev) for _ in range(world)]
+
+    def run(self, shards, config=None, mode: str = "count", outs=None, exchange: str = "p2p", configs=None):
+        """shards[g] = (rk, rp, sk, sp) of rank g; outs[g]: rank g's (capacity, 2) output (materialize).
+        Returns the per-rank JoinResults.  A failing rank aborts the world (the runner is then dead)."""
+        res: list = [None] * self.world
+        err: list = []
+        ready = torch.cuda.Event()
+        ready.record(torch.cuda.current_stream(self.dev))   # the shards are ready on the caller's stream
+
+        def worker(g):
+            try:
+                with torch.cuda.device(self.dev), torch.cuda.stream(self.streams[g]):
+                    self.streams[g].wait_event(ready)
+                    cfg = configs[g] if configs is not None else config
+                    res[g] = self.drv[g].join(*shards[g], config=cfg, mode=mode,
+                                              out=outs[g] if outs is not None else None, exchange=exchange)
+            except BaseException as e:  # noqa: BLE001  (the library aborted the world, or we do)
+                err.append((g, e))
+                self.comms[g].abort()
+
+        th = [threading.Thread(target=worker, args=(g,)) for g in range(self.world)]
+        for t in th:
+            t.start()
+        for t in th:
+            t.join()
+        done = torch.cuda.current_stream(self.dev)
+        for s in self.streams:
+            done.wait_stream(s)
+        if err:
+            err.sort(key=lambda x: "peer rank failed" in str(x[1]))   # the root cause first
+            raise err[0][1]
+        return res
+
+    def close(self) -> None:
+        for d in self.drv:
+            d.close()
+        self.drv = []
+        self.lw.close()
+
+
 def run_local_native(world: int, shards, config=None, mode: str = "count", out_capacity: int = 0, device=None,
                      exchange: str = "p2p", repeat: int = 1, calls=None, configs=None):
-    """The native driver for `world` logical ranks on ONE device (host threads + a native local
-    world).  shards[g] = (rk, rp, sk, sp) CUDA tensors of rank g; returns the per-rank JoinResults of
-    the last of `repeat` calls (rank order).  calls: a list of such shard lists, joined one after
-    another by the same per-rank drivers (buffer reuse and growth); the per-call results are then
-    returned.  configs: per-rank configs (default `config` everywhere)."""
-    lw = NativeLocalWorld(world)
+    """The native driver for `world` logical ranks on ONE device (LocalNativeRunner).  shards[g] =
+    (rk, rp, sk, sp) CUDA tensors of rank g; returns the per-rank JoinResults of the last of
+    `repeat` calls (rank order).  calls: a list of such shard lists, joined one after another by the
+    same per-rank drivers (buffer reuse and growth); the per-call results are then returned.
+    configs: per-rank configs (default `config` everywhere)."""
     seq = list(calls) if calls is not None else [shards] * repeat
     dev = torch.device(device) if device is not None else seq[0][0][0].device
-    res: list = [[None] * world for _ in seq]
-    err: list = []
-
-    def worker(g):
-        drv = None
-        comm = lw.comm(g)
-        try:
-            with torch.cuda.device(dev):
-                s = torch.cuda.Stream(dev)
-                with torch.cuda.stream(s):
-                    drv = ShardedJoin(comm, dev)
-                    out = (torch.empty((out_capacity, 2), dtype=torch.int32, device=dev)
-                           if mode == "materialize" else None)
-                    cfg = configs[g] if configs is not None else config
-                    for i, sh in enumerate(seq):
-                        res[i][g] = drv.join(*sh[g], config=cfg, mode=mode, out=out, exchange=exchange)
-                s.synchronize()
-        except BaseException as e:  # the library aborted the world (or we do): the other ranks return too
-            err.append((g, e))
-            comm.abort()
-        finally:
-            if drv is not None:
-                drv.close()
-
-    th = [threading.Thread(target=worker, args=(g,)) for g in range(world)]
-    for t in th:
-        t.start()
-    for t in th:
-        t.join()
-    lw.close()
-    if err:
-        err.sort(key=lambda x: "peer rank failed" in str(x[1]))   # the root cause first
-        raise err[0][1]
-    return res if calls is not None else res[-1]
+    runner = LocalNativeRunner(world, dev)
+    try:
+        outs = ([torch.empty((out_capacity, 2), dtype=torch.int32, device=dev) for _ in range(world)]
+                if mode == "materialize" else None)
+        got = [runner.run(sh, config=config, mode=mode, outs=outs, exchange=exchange, configs=configs) for sh in seq]
+    finally:
+        runner.close()
+    return got if calls is not None else got[-1]
 
 
 class _DevBytes:
