@@ -66,6 +66,10 @@ def parse():
     ap.add_argument("--mode", default="count", choices=["count", "materialize"])
     ap.add_argument("--detect", default="exact", choices=["exact", "sampled"],
                     help="skew detection: exact counts (default) or the paper's 1%% sample + top-3 (L107, L112)")
+    ap.add_argument("--gbase-sweep", action="store_true",
+                    help="GSH vs the Gbase-style join (NEXT-4) at the paper's Table I size (2^25 per side), one JSON line")
+    ap.add_argument("--hybrid", action="store_true",
+                    help="CSH's hybrid partition (gsh_config.hybrid, SURVEY NEXT-1): sampled skewed keys routed in pass 1")
     ap.add_argument("--out-cap", type=int, default=1 << 30, help="MATERIALIZE output capacity (pairs)")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -297,10 +301,8 @@ def theta_sweep(gsh, dev, seed, steps=3):
     3e15 pairs), plus the skewed-key phase's pairs/s at the largest sizes that finish in seconds."""
     import datagen
     out = {"points": [], "dense": []}
-    for theta, n, inp in SWEEP:
-        rk, rp, sk, sp = datagen.make_workload("zipf", n, theta, seed=seed, device=dev)
-        cfg = gsh.make_config(timing=True, input_side_only=inp)
-        ws = torch.empty(gsh.workspace_bytes(n, n, cfg), dtype=torch.uint8, device=dev)
+
+    def timed(rk, rp, sk, sp, cfg, ws):
         r = gsh.join(rk, rp, sk, sp, config=cfg, workspace=ws)
         ph = {}
         for _ in range(steps):
@@ -308,6 +310,13 @@ def theta_sweep(gsh, dev, seed, steps=3):
             for k, v in r.stats.items():
                 if k.startswith("ms_"):
                     ph[k] = ph.get(k, 0.0) + v / steps
+        return r, ph
+
+    for theta, n, inp in SWEEP:
+        rk, rp, sk, sp = datagen.make_workload("zipf", n, theta, seed=seed, device=dev)
+        cfg = gsh.make_config(timing=True, input_side_only=inp)
+        ws = torch.empty(gsh.workspace_bytes(n, n, gsh.make_config(hybrid=True)), dtype=torch.uint8, device=dev)
+        r, ph = timed(rk, rp, sk, sp, cfg, ws)
         st = dict(r.stats)
         pt = {"theta": theta, "n_per_side": n, "input_side_only": inp, "phases_ms": ph,
               "n_large": st["n_large"], "n_heavy": st["n_heavy"],
@@ -317,6 +326,11 @@ def theta_sweep(gsh, dev, seed, steps=3):
             pt["count"] = r.count
             pt["input_tuples_per_s"] = 2 * n / (ph["ms_total"] / 1e3)
             pt["output_tuples_per_s"] = r.count / (ph["ms_total"] / 1e3)
+        # the same point with CSH's hybrid partition (NEXT-1): sampled keys skip pass 2, detect, split
+        rh, phh = timed(rk, rp, sk, sp, gsh.make_config(timing=True, input_side_only=inp, hybrid=True), ws)
+        assert inp or (rh.count, rh.checksum) == (r.count, r.checksum), "hybrid result differs"
+        pt["hybrid"] = {"phases_ms": phh, "n_hybrid": rh.stats["n_hybrid"], "n_heavy": rh.stats["n_heavy"],
+                        "n_large": rh.stats["n_large"], "large_tuples": rh.stats["large_tuples"]}
         out["points"].append(pt)
         del rk, rp, sk, sp, ws
     for theta, n in DENSE:
@@ -330,6 +344,57 @@ def theta_sweep(gsh, dev, seed, steps=3):
                              "output_tuples_per_s": r.count / (st["ms_total"] / 1e3)})
         del rk, rp, sk, sp
     torch.cuda.empty_cache()
+    return out
+
+
+GBASE_THETAS = [0.0, 0.25, 0.5, 0.6, 0.7, 0.8, 0.9, 1.0]
+
+
+def gbase_sweep(gsh, dev, seed, n=1 << 25, budget_s=8.0):
+    """PAPER.md Table I (L157-L160) re-measured on this GPU: |R| = |S| = 2^25 (the paper's 32M) Zipf
+    tuples, both sides, COUNT.  GSH (and its hybrid variant) vs the Gbase-style comparison join
+    (gsh_join_gbase) per theta: partition ms and join ms as the paper splits them, the same count /
+    checksum required of both.  Gbase is skipped at a theta once its previous point exceeded
+    budget_s (its join time grows ~10x per 0.1 of theta, L158)."""
+    import datagen
+    out = []
+    gb_last = 0.0
+    cfg = gsh.make_config(timing=True)
+    cfgh = gsh.make_config(timing=True, hybrid=True)
+    ws = torch.empty(gsh.workspace_bytes(n, n, cfgh), dtype=torch.uint8, device=dev)
+
+    def run(impl, c, reps):
+        r = gsh.join(rk, rp, sk, sp, config=c, workspace=ws, impl=impl)
+        ph = {}
+        for _ in range(reps):
+            r = gsh.join(rk, rp, sk, sp, config=c, workspace=ws, impl=impl)
+            for k, v in r.stats.items():
+                if k.startswith("ms_"):
+                    ph[k] = ph.get(k, 0.0) + v / reps
+        return r, ph
+
+    for theta in GBASE_THETAS:
+        rk, rp, sk, sp = datagen.make_workload("zipf", n, theta, seed=seed, device=dev)
+        r, ph = run("gsh", cfg, 3 if theta < 0.9 else 1)
+        part = ph["ms_hist"] + ph["ms_pass1"] + ph["ms_pass2"]
+        pt = {"theta": theta, "n_per_side": n, "count": r.count,
+              "gsh": {"partition_ms": part, "all_other_ms": ph["ms_total"] - part, "total_ms": ph["ms_total"],
+                      "n_heavy": r.stats["n_heavy"]}}
+        rh, phh = run("gsh", cfgh, 3 if theta < 0.9 else 1)
+        assert (rh.count, rh.checksum) == (r.count, r.checksum), "hybrid result differs"
+        pt["gsh_hybrid"] = {"total_ms": phh["ms_total"], "n_hybrid": rh.stats["n_hybrid"]}
+        if gb_last <= budget_s:
+            g, pg = run("gbase", cfg, 1 if theta >= 0.6 else 3)
+            assert (g.count, g.checksum) == (r.count, r.checksum), "Gbase result differs"
+            gpart = pg["ms_hist"] + pg["ms_pass1"] + pg["ms_pass2"]
+            pt["gbase"] = {"partition_ms": gpart, "join_ms": pg["ms_nmjoin"], "total_ms": pg["ms_total"]}
+            pt["speedup_gsh_over_gbase"] = pg["ms_total"] / ph["ms_total"]
+            gb_last = pg["ms_total"] / 1e3
+        else:
+            pt["gbase"] = None
+        out.append(pt)
+        print(json.dumps(pt), file=sys.stderr, flush=True)
+        del rk, rp, sk, sp
     return out
 
 
@@ -419,6 +484,12 @@ def main():
 
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
+    if args.gbase_sweep:
+        pts = gbase_sweep(gsh, dev, args.seed)
+        print(json.dumps({"metric": "GSH vs Gbase-style join, PAPER.md Table I shape (ms per join)",
+                          "config": {"workload": "|R|=|S|=2^25 Zipf both sides, COUNT, 1 B200"},
+                          "impl": "gsh+gbase", "points": pts}))
+        return
     kind, n, theta, desc = WORKLOADS[args.workload]
     if args.mode == "materialize":
         desc = desc.replace("COUNT", "MATERIALIZE")
@@ -432,6 +503,8 @@ def main():
     extra = json.loads(os.environ.get("GSH_BENCH_CFG", "{}"))  # experiments only
     if args.detect == "sampled":
         extra["detect_mode"] = 1
+    if args.hybrid:
+        extra["hybrid"] = True
     # per-phase CUDA events stay on inside the timed region (the roofline's kernel time is
     # measured live there); they cost ~30 us of host time per call, included in the step time
     if args.input_side:

@@ -121,6 +121,20 @@ typedef struct {
                                   detect, split) and stop before the NM-join and the skewed-key
                                   join; count / checksum / written are then 0.  Used to time the
                                   partition passes on inputs whose output takes minutes. */
+    int32_t hybrid;            /* CSH's hybrid partition on the GPU (§IV-A;
+                                  SURVEY §8(f) NEXT-1): 1 = before partitioning, every
+                                  hybrid_stride-th key of R and of S is sampled into a
+                                  linear-probing table; keys sampled more than hybrid_min - 1 times
+                                  (L89: "exceeds the pre-defined threshold (e.g., 2)"), at most the
+                                  512 most frequent, are skewed up front.  The histogram pass counts
+                                  them exactly and pass 1 writes their R AND S tuples straight into
+                                  the per-key arrays R_k / S_k (payloads), so they skip pass 2,
+                                  detection and the split.  Skew left in the partitions is still
+                                  detected after partitioning as usual.  0 = off (GSH, L104).
+                                  Ignored with force_all_normal / force_all_heavy.  The result never
+                                  depends on it. */
+    uint32_t hybrid_stride;    /* hybrid: 1 key in hybrid_stride is sampled.  0 = 100 (1 %, L89) */
+    uint32_t hybrid_min;       /* hybrid: sampled count a key needs.  0 = 3 (L89: "exceeds ... 2") */
 } gsh_config;
 
 /* Per-call result (host struct). */
@@ -147,6 +161,9 @@ typedef struct {
     uint32_t prepass_bits;     /* pre-partition bits actually used (0 = none) */
     float ms_prepass;          /* pre-partition pass (count + scatter), included in ms_total */
     uint64_t large_tuples;     /* R + S tuples in large partitions (read by detect and split) */
+    uint32_t n_hybrid;         /* skewed keys found by the hybrid sample (gsh_config.hybrid), the
+                                  first n_hybrid of the n_heavy */
+    float ms_sample;           /* hybrid sample + selection, included in ms_total */
 } gsh_result;
 
 /* Fill *cfg with defaults (all auto, no hooks, timing off). */
@@ -178,6 +195,21 @@ GSH_API size_t gsh_workspace_bytes(uint64_t n_r, uint64_t n_s, const gsh_config 
 GSH_API gsh_status gsh_join(const gsh_relation *R, const gsh_relation *S, gsh_out_mode mode,
                     const gsh_output *out, void *workspace, size_t workspace_bytes,
                     const gsh_config *cfg, void *stream, gsh_result *res);
+
+/*
+ * gsh_join_gbase -- the paper's GPU comparison system "Gbase" (§II-B, §III
+ * L78-L80), re-implemented on this GPU for the GSH-vs-Gbase measurement
+ * (Table I): no skew detection; after the same two partition passes, one thread block
+ * per (partition, R sub-list of <= 4096 tuples) builds a chained shared-memory table and probes it
+ * with the FULL S partition (L71-L72's sub lists), all threads advancing one chain element per
+ * round with a write bitmap and a block barrier per round (L79-L80).  Arguments, workspace
+ * (gsh_workspace_bytes), errors and result semantics as gsh_join: identical count, checksum and
+ * pair multiset.  res: ms_hist / ms_pass1 / ms_pass2 = the partition phase, ms_nmjoin = the Gbase
+ * join phase, ms_total; skew fields 0.  At most 2^28 tuples per side (GSH_ERR_INVALID beyond).
+ */
+GSH_API gsh_status gsh_join_gbase(const gsh_relation *R, const gsh_relation *S, gsh_out_mode mode,
+                                  const gsh_output *out, void *workspace, size_t workspace_bytes,
+                                  const gsh_config *cfg, void *stream, gsh_result *res);
 
 /* Device workspace for gsh_join_host: gsh_workspace_bytes + device staging for the inputs
  * (8 B per tuple) and, for MATERIALIZE, for out_capacity pairs (8 B per pair). */

@@ -51,6 +51,9 @@ class GshConfig(ctypes.Structure):
         ("prepass_bits", i32),
         ("heavy_detail", i32),
         ("input_side_only", i32),
+        ("hybrid", i32),
+        ("hybrid_stride", u32),
+        ("hybrid_min", u32),
     ]
 
 
@@ -85,6 +88,8 @@ class GshResult(ctypes.Structure):
         ("prepass_bits", u32),
         ("ms_prepass", ctypes.c_float),
         ("large_tuples", u64),
+        ("n_hybrid", u32),
+        ("ms_sample", ctypes.c_float),
     ]
 
     def as_dict(self) -> dict:
@@ -145,6 +150,9 @@ _PROTOS = [
     ("gsh_join", ctypes.c_int, [ctypes.POINTER(GshRelation), ctypes.POINTER(GshRelation), ctypes.c_int,
                                 ctypes.POINTER(GshOutput), vp, ctypes.c_size_t, ctypes.POINTER(GshConfig), vp,
                                 ctypes.POINTER(GshResult)]),
+    ("gsh_join_gbase", ctypes.c_int, [ctypes.POINTER(GshRelation), ctypes.POINTER(GshRelation), ctypes.c_int,
+                                      ctypes.POINTER(GshOutput), vp, ctypes.c_size_t, ctypes.POINTER(GshConfig), vp,
+                                      ctypes.POINTER(GshResult)]),
     ("gsh_host_workspace_bytes", ctypes.c_size_t, [u64, u64, ctypes.c_int, u64, ctypes.POINTER(GshConfig)]),
     ("gsh_join_host", ctypes.c_int, [ctypes.POINTER(GshRelation), ctypes.POINTER(GshRelation), ctypes.c_int,
                                      ctypes.POINTER(GshOutput), vp, ctypes.c_size_t, ctypes.POINTER(GshConfig), vp,

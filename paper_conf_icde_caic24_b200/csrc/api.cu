@@ -132,6 +132,10 @@ bool plan_build(Plan& p, uint64_t nR, uint64_t nS, const gsh_config* cfg_in, voi
     p.top_k = cfg.top_k ? cfg.top_k : 3;
     if (p.top_k > 32) return false;
     if (p.force_normal && p.force_heavy) return false;
+    if (cfg.hybrid < 0 || cfg.hybrid > 1) return false;
+    p.hybrid = cfg.hybrid && !p.force_normal && !p.force_heavy;
+    p.hyb_stride = cfg.hybrid_stride ? cfg.hybrid_stride : 100;
+    p.hyb_min = cfg.hybrid_min ? cfg.hybrid_min : 3;
     p.hist_grid = num_sms;  // one 1024-thread CTA (128 KB of counters) per SM
     uint64_t t = next_pow2_u64(2 * (nR + nS));
     if (t < 1024) t = 1024;
@@ -146,6 +150,7 @@ bool plan_build(Plan& p, uint64_t nR, uint64_t nS, const gsh_config* cfg_in, voi
         if (p.detect_mode == 1 && uint64_t(p.F) * p.top_k > hm) hm = uint64_t(p.F) * p.top_k;
         p.h_max = hm < p.gt_cap_alloc ? hm : p.gt_cap_alloc;
     }
+    if (p.hybrid) p.h_max += kHybMaxKeys;   // the sampled keys come first in H
     // pass-1 units (= histogram slices): whole 16K-key chunks, about one unit per scatter CTA
     // (2 per SM) and at most kHistMaxUnitChunks chunks.  Pass-2 units: ranges of consecutive
     // slices of one pass-1 partition holding >= T tuples (planned on the device from the
@@ -220,6 +225,9 @@ bool plan_build(Plan& p, uint64_t nR, uint64_t nS, const gsh_config* cfg_in, voi
     p.nm = c.take<NmPart>(F);
     p.nm_prefix = c.take<uint64_t>(F + 1);
     p.scan_scratch = c.take<uint64_t>(p.scan_scratch_elems);
+    p.hyb_tab = c.take<unsigned long long>(kHybSlots);
+    p.hyb_list = c.take<uint32_t>(kHybMaxKeys);
+    p.hyb_cnt = c.take<uint32_t>(2 * kHybMaxKeys);
     p.bytes = c.off;
     return true;
 }
@@ -443,8 +451,26 @@ static gsh_status join_direct(const gsh_relation* R, const gsh_relation* S, gsh_
     int launches = 0;
     cudaMemsetAsync(p.st, 0, sizeof(DevState), s);
     const int e0 = tm.mark();
+    int es = e0;
+    cudaError_t ce;
+    if (p.hybrid) {   // CSH's sampling before partitioning (hybrid.cu): which keys pass 1 routes
+        launches += launch_hybrid_sample(p, R->keys, S->keys, s);
+        if ((st = check_launch("hybrid sample")) != GSH_OK) return st;
+        uint32_t nh0 = 0;
+        ce = cudaMemcpyAsync(&nh0, &p.st->n_h0, sizeof(nh0), cudaMemcpyDeviceToHost, s);
+        if (ce == cudaSuccess) ce = cudaStreamSynchronize(s);
+        if (ce != cudaSuccess) return cuda_fail(ce, "hybrid sample sync");
+        if (nh0 > kHybMaxKeys) return fail(GSH_ERR_INTERNAL, "hybrid key list overflow");
+        p.n_h0 = nh0;
+        es = tm.mark();
+    }
     launches += launch_hist(p, R->keys, S->keys, s);
     launches += launch_hist_reduce_scan(p, s);
+    if (p.n_h0) {   // H's first entries with their exact counts; R_k / S_k offsets for pass 1
+        launches += launch_hybrid_fill(p, s);
+        launches += launch_heavy_offsets(p, p.n_h0, s);
+        cudaMemsetAsync(p.h_cur, 0, size_t(2) * p.h_max * sizeof(uint32_t), s);
+    }
     const int e1 = tm.mark();
     {
         const uint32_t* keys[2] = {R->keys, S->keys};
@@ -458,13 +484,13 @@ static gsh_status join_direct(const gsh_relation* R, const gsh_relation* S, gsh_
     if ((st = check_launch("partition")) != GSH_OK) return st;
 
     DevState hs;
-    cudaError_t ce = cudaMemcpyAsync(&hs, p.st, sizeof(DevState), cudaMemcpyDeviceToHost, s);
+    ce = cudaMemcpyAsync(&hs, p.st, sizeof(DevState), cudaMemcpyDeviceToHost, s);
     if (ce == cudaSuccess) ce = cudaStreamSynchronize(s);
     if (ce != cudaSuccess) return cuda_fail(ce, "classify sync");
     if (hs.route_mismatch)
         return fail(GSH_ERR_INVALID, "gsh_config.route_bits: the tuples do not all share the top route_bits of h");
     const uint32_t n_large = hs.n_large;
-    uint32_t n_heavy = 0;
+    uint32_t n_heavy = p.n_h0;   // hybrid keys first; the detection below appends
     p.nm_slots = nm_table_slots(hs.max_rlen < p.C ? (hs.max_rlen ? hs.max_rlen : 1) : p.C);
     int e4 = e3, e5 = e3;
     if (n_large > 0) {
@@ -480,7 +506,6 @@ static gsh_status join_direct(const gsh_relation* R, const gsh_relation* S, gsh_
         n_heavy = hs.n_heavy;
         if (hs.heavy_overflow || n_heavy > p.h_max) return fail(GSH_ERR_INTERNAL, "skewed-key list overflow");
         launches += launch_heavy_prefix(p, n_heavy, n_large, s);
-        if (p.detail && n_heavy) cudaMemsetAsync(p.h_chk, 0, size_t(n_heavy) * 8, s);
         launches += launch_split(p, n_large, (uint32_t)gcap, s);
         e5 = tm.mark();
     }
@@ -496,8 +521,10 @@ static gsh_status join_direct(const gsh_relation* R, const gsh_relation* S, gsh_
         res->n_large = n_large;
         res->detect_overflow = hs.detect_overflow;
         res->launches = (uint32_t)launches;
+        res->n_hybrid = p.n_h0;
         if (p.timing) {
-            res->ms_hist = tm.ms(e0, e1);
+            res->ms_sample = tm.ms(e0, es);
+            res->ms_hist = tm.ms(es, e1);
             res->ms_pass1 = tm.ms(e1, e2);
             res->ms_pass2 = tm.ms(e2, e3);
             res->ms_detect = n_large ? tm.ms(e3, e4) : 0.f;
@@ -511,6 +538,7 @@ static gsh_status join_direct(const gsh_relation* R, const gsh_relation* S, gsh_
     // serialise a chain walk; the CSR table flattens those across the warp).
     p.nm_chain = (p.route_bits + p.b1 + p.b2 >= 16) && p.nm_table != 1 && (p.nm_table == 2 || n_large == 0);
     res->nm_table = p.nm_chain ? 2 : 1;
+    if (p.detail && n_heavy) cudaMemsetAsync(p.h_chk, 0, size_t(n_heavy) * 8, s);
     launches += launch_nm_setup(p, n_large, s);
     launches += launch_nmjoin(p, mat ? 1 : 0, pairs, cap, s);
     const int e6 = tm.mark();
@@ -535,8 +563,10 @@ static gsh_status join_direct(const gsh_relation* R, const gsh_relation* S, gsh_
     res->n_large = n_large;
     res->detect_overflow = hs.detect_overflow;
     res->launches = (uint32_t)launches;
+    res->n_hybrid = p.n_h0;
     if (p.timing) {
-        res->ms_hist = tm.ms(e0, e1);
+        res->ms_sample = tm.ms(e0, es);
+        res->ms_hist = tm.ms(es, e1);
         res->ms_pass1 = tm.ms(e1, e2);
         res->ms_pass2 = tm.ms(e2, e3);
         res->ms_detect = n_large ? tm.ms(e3, e4) : 0.f;
@@ -642,6 +672,8 @@ gsh_status gsh_join(const gsh_relation* R, const gsh_relation* S, gsh_out_mode m
         acc.large_tuples += sr.large_tuples;
         acc.n_heavy += sr.n_heavy;
         acc.n_large += sr.n_large;
+        acc.n_hybrid += sr.n_hybrid;
+        acc.ms_sample += sr.ms_sample;
         acc.detect_overflow |= sr.detect_overflow;
         acc.launches += sr.launches;
         if (sR.n && sS.n) {   // parameters of a non-empty sub-problem

@@ -80,6 +80,12 @@ constexpr uint32_t kDetectChunk = 2048;         // tuples per split (and sampled
 constexpr uint32_t kDetectItem = 16384;         // tuples per exact-detect work item
 constexpr uint32_t kNoHeavy = 0xffffffffu;
 constexpr int kDetectMaxProbe = 64;   // a full table degrades to "normal", never to a long probe
+// Hybrid partition (gsh_config.hybrid, hybrid.cu): at most kHybMaxKeys sampled skewed keys, looked
+// up in a kHybSlots-slot shared-memory copy of the table ((hid + 1) << 32 | h, 0 = empty; load <= 1/2)
+constexpr uint32_t kHybMaxKeys = 512;
+constexpr uint32_t kHybSlots = 1024;
+constexpr uint32_t kHybLogSlots = 10;
+constexpr int kScatterIptHyb = 16;               // pass-1 tile with the hybrid tables (two CTAs per SM)
 
 // Device-resident counters and accumulators, zeroed once per call.
 struct DevState {
@@ -96,6 +102,8 @@ struct DevState {
     unsigned int route_mismatch;                   // route_bits > 0: tuples differ in the top route bits
     unsigned int u2_front, u2_back;                // pass-2 units at the front / back of the list
     unsigned int heavy_overflow;                   // more skewed keys than the list H holds
+    unsigned int n_h0;                             // hybrid: sampled skewed keys selected
+    unsigned int hyb_bins[33];                     // hybrid: sampled keys per floor(log2 count)
 };
 
 // Per-(call site, device) one-time setup (kernel attributes): concurrent host threads wait until
@@ -135,6 +143,9 @@ struct Plan {
     int nm_chain = 0;               // chosen for this call (nm_ring.cu)
     int detect_mode = 0;            // 0 exact counts, 1 sampled top-k (L107, L112)
     uint32_t sample_stride = 100, top_k = 3;
+    int hybrid = 0;                 // CSH-style hybrid partition (hybrid.cu)
+    uint32_t hyb_stride = 100, hyb_min = 3;
+    uint32_t n_h0 = 0;              // hybrid keys selected (host copy, set after the sample)
     int num_sms = 148;
     int hist_grid = 148;            // histogram CTAs (1 per SM)
     uint32_t unit_chunks = 1;       // chunks per pass-1 unit (= histogram slice)
@@ -182,12 +193,16 @@ struct Plan {
     NmPart* nm = nullptr;                     // [F]
     uint64_t* nm_prefix = nullptr;            // [F + 1]
     uint64_t* scan_scratch = nullptr;         // block sums for the generic scan
+    unsigned long long* hyb_tab = nullptr;    // [kHybSlots] hybrid lookup table
+    uint32_t* hyb_list = nullptr;             // [kHybMaxKeys] h of hybrid key hid
+    uint32_t* hyb_cnt = nullptr;              // [2][kHybMaxKeys] exact counts (histogram pass)
     size_t bytes = 0;
 };
 
 // Computes parameters and carves `ws` (may be nullptr to only size it).  Returns false on
 // invalid configuration.
 bool plan_build(Plan& p, uint64_t nR, uint64_t nS, const gsh_config* cfg, void* ws, int num_sms);
+gsh_status api_fail(gsh_status st, const char* msg);   // api.cu: sets the thread-local message
 
 // ------------------------------------------------------------------ launchers --
 // Every launcher enqueues on `s` and returns the number of kernels it launched.
@@ -202,6 +217,11 @@ int launch_detect(const Plan& p, uint32_t n_large, uint32_t gt_cap, cudaStream_t
 int launch_sample_topk(const Plan& p, uint32_t n_large, uint32_t gt_cap, cudaStream_t s);
 int launch_select(const Plan& p, uint32_t gt_cap, cudaStream_t s);
 int launch_heavy_prefix(const Plan& p, uint32_t n_heavy, uint32_t n_large, cudaStream_t s);
+int launch_heavy_offsets(const Plan& p, uint32_t n_heavy, cudaStream_t s);   // h_off / h_tiles only
+// hybrid.cu: sample + select (n_h0 and hyb_tab on the device), then after the histogram pass the
+// first n_h0 entries of H with their exact counts
+int launch_hybrid_sample(const Plan& p, const uint32_t* k0, const uint32_t* k1, cudaStream_t s);
+int launch_hybrid_fill(const Plan& p, cudaStream_t s);
 int launch_split(const Plan& p, uint32_t n_large, uint32_t gt_cap, cudaStream_t s);
 int launch_nm_setup(const Plan& p, uint32_t n_large, cudaStream_t s);
 int launch_nmjoin(const Plan& p, int materialize, uint32_t* pairs, uint64_t cap, cudaStream_t s);

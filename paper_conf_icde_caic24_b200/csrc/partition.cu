@@ -59,15 +59,36 @@ constexpr uint32_t kHistMaxEvents = 128;
 static_assert(kScatterChunk == 16 * kHistBlock, "a full chunk is 4 uint4 per histogram thread");
 static_assert(3 * ((uint64_t(kHistMaxUnitChunks) * kScatterChunk) >> 16) <= kHistMaxEvents, "wrap events of a slice");
 
+// Hybrid partition (hybrid.cu): the sampled skewed keys' table, (hid + 1) << 32 | h, 0 = empty.
+__device__ __forceinline__ uint32_t hyb_find(const unsigned long long* tab, uint32_t h) {
+    uint32_t s = (h * 0x9E3779B1u) >> (32 - kHybLogSlots);
+    for (;;) {   // load <= 1/2: an empty slot ends every probe
+        const unsigned long long e = tab[s];
+        if (e == 0) return kNoHeavy;
+        if ((uint32_t)e == h) return (uint32_t)(e >> 32) - 1;
+        s = (s + 1) & (kHybSlots - 1);
+    }
+}
+
 // CHECK (route_bits > 0): also verify the caller's gsh_config.route_bits assertion -- every tuple
 // shares the top route_bits of h -- by OR-ing t and ~t over all keys (t = those bits): they are all
 // equal iff (OR t) & (OR ~t) has no bit set.  The NM-join's chained table relies on it.
-template <bool FAST16, bool CHECK>
+// HYB (gsh_config.hybrid): a key of the sampled skewed set is counted per (side, key) -- hyb_cnt,
+// the sizes of R_k / S_k -- instead of in its digit bins, so every later offset covers the
+// partitioned (normal) tuples only.
+template <bool FAST16, bool CHECK, bool HYB>
 __global__ void __launch_bounds__(kHistBlock, 1)
 k_hist2d(const uint32_t* __restrict__ k0, uint64_t n0, const uint32_t* __restrict__ k1, uint64_t n1,
          uint32_t shift, uint32_t nbits, uint32_t b2, uint32_t* __restrict__ partial, uint32_t* __restrict__ c1cnt,
          uint32_t nu0, uint32_t nu1, uint32_t unit_chunks, uint32_t rshift, DevState* st,
-         uint32_t* __restrict__ slice_dom) {
+         uint32_t* __restrict__ slice_dom, const unsigned long long* __restrict__ hyb_tab, uint32_t n_h0,
+         uint32_t* __restrict__ hyb_cnt) {
+    __shared__ unsigned long long s_htab[HYB ? kHybSlots : 1];
+    __shared__ uint32_t s_hc[HYB ? kHybMaxKeys : 1];
+    if (HYB) {
+        for (uint32_t i = threadIdx.x; i < kHybSlots; i += blockDim.x) s_htab[i] = hyb_tab[i];
+        for (uint32_t i = threadIdx.x; i < kHybMaxKeys; i += blockDim.x) s_hc[i] = 0;
+    }
     uint32_t r_or = 0, r_nor = 0;
     __shared__ uint32_t s_dom;
     extern __shared__ uint32_t cnt[];
@@ -106,7 +127,21 @@ k_hist2d(const uint32_t* __restrict__ k0, uint64_t n0, const uint32_t* __restric
         }
     };
     auto count_key = [&](uint32_t key) {
-        if (FAST16) {
+        if (HYB) {
+            const uint32_t hk = hash32(key);
+            if (CHECK) {
+                const uint32_t t = hk >> rshift;
+                r_or |= t;
+                r_nor |= ~t;
+            }
+            const uint32_t hid = hyb_find(s_htab, hk);
+            if (hid != kNoHeavy) {
+                atomicAdd(&s_hc[hid], 1u);
+                return;
+            }
+            const uint32_t bin = (hk >> shift) & mask;
+            if (packed) count_exact(bin); else atomicAdd(&cnt[bin], 1u);
+        } else if (FAST16) {
             count_exact(hash32_top(key) >> 16);
         } else {
             const uint32_t hk = top16 ? hash32_top(key) : hash32(key);
@@ -174,6 +209,12 @@ k_hist2d(const uint32_t* __restrict__ k0, uint64_t n0, const uint32_t* __restric
             }
         }
         __syncthreads();
+        if (HYB)   // the slice's skewed-key counts (every slice belongs to one side)
+            for (uint32_t i = threadIdx.x; i < n_h0; i += blockDim.x)
+                if (s_hc[i]) {
+                    atomicAdd(&hyb_cnt[side * kHybMaxKeys + i], s_hc[i]);
+                    s_hc[i] = 0;
+                }
         // flush this slice's joint counts (and their per-d1 sums) and reset
         uint32_t* row = partial + (size_t(side ? nu0 : 0) + sl) * F;
         for (uint32_t w = threadIdx.x; w < nwords; w += blockDim.x) {
@@ -233,27 +274,32 @@ int launch_hist(const Plan& p, const uint32_t* k0, const uint32_t* k1, cudaStrea
     const size_t smem = size_t(F > (1u << 15) ? F / 2 : F) * 4;
     static std::once_flag attr_once[kMaxDevices];
     once_per_device(attr_once, [] {
-        cudaFuncSetAttribute(k_hist2d<false, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, 128 * 1024);
-        cudaFuncSetAttribute(k_hist2d<false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, 128 * 1024);
-        cudaFuncSetAttribute(k_hist2d<true, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, 128 * 1024);
+        cudaFuncSetAttribute(k_hist2d<false, false, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, 128 * 1024);
+        cudaFuncSetAttribute(k_hist2d<false, true, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, 128 * 1024);
+        cudaFuncSetAttribute(k_hist2d<true, false, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, 128 * 1024);
+        cudaFuncSetAttribute(k_hist2d<false, false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, 128 * 1024);
+        cudaFuncSetAttribute(k_hist2d<false, true, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, 128 * 1024);
     });
     const bool fast16 = nbits == 16 && p.route_bits == 0 && p.b2 == 8;
     const uint32_t rshift = 32 - p.route_bits;
     // (Rejected, kept in history: CTA pairs each counting one half of 2^16 u32 bins -- every key
     // hashed twice, ALU-bound at 0.76 ms for 2^28 keys; a cluster pair exchanging bins through
     // DSMEM atomics, 3.6 ms, or DSMEM loads, 1.0 ms.)
-    if (fast16)
-        k_hist2d<true, false><<<p.hist_grid, kHistBlock, smem, s>>>(k0, p.n[0], k1, p.n[1], shift, nbits, p.b2,
-                                                                    p.hist_partial, p.c1cnt, p.nu1[0], p.nu1[1],
-                                                                    p.unit_chunks, rshift, p.st, p.slice_dom);
-    else if (p.route_bits)
-        k_hist2d<false, true><<<p.hist_grid, kHistBlock, smem, s>>>(k0, p.n[0], k1, p.n[1], shift, nbits, p.b2,
-                                                                    p.hist_partial, p.c1cnt, p.nu1[0], p.nu1[1],
-                                                                    p.unit_chunks, rshift, p.st, p.slice_dom);
-    else
-        k_hist2d<false, false><<<p.hist_grid, kHistBlock, smem, s>>>(k0, p.n[0], k1, p.n[1], shift, nbits, p.b2,
-                                                                     p.hist_partial, p.c1cnt, p.nu1[0], p.nu1[1],
-                                                                     p.unit_chunks, rshift, p.st, p.slice_dom);
+    auto go = [&](auto kern) {
+        kern<<<p.hist_grid, kHistBlock, smem, s>>>(k0, p.n[0], k1, p.n[1], shift, nbits, p.b2, p.hist_partial,
+                                                   p.c1cnt, p.nu1[0], p.nu1[1], p.unit_chunks, rshift, p.st,
+                                                   p.slice_dom, p.hyb_tab, p.n_h0, p.hyb_cnt);
+    };
+    if (p.n_h0) {
+        if (p.route_bits) go(k_hist2d<false, true, true>);
+        else go(k_hist2d<false, false, true>);
+    } else if (fast16) {
+        go(k_hist2d<true, false, false>);
+    } else if (p.route_bits) {
+        go(k_hist2d<false, true, false>);
+    } else {
+        go(k_hist2d<false, false, false>);
+    }
     return 1;
 }
 
@@ -423,6 +469,12 @@ struct ScatterArgs {
     uint32_t unit_len;         // tuples per pass-1 unit
     uint32_t pass, b1, b2, route_bits;
     unsigned int* unit_ctr;
+    // hybrid pass 1 (HYB): sampled skewed keys' table, their count, R_k / S_k offsets, cursors, arrays
+    const unsigned long long* hyb_tab;
+    uint32_t n_h0;
+    const uint64_t* h_off[2];
+    uint32_t* h_cur[2];
+    uint32_t* heavy_pay[2];
 };
 
 struct ScatterSmem {
@@ -558,7 +610,11 @@ __device__ __forceinline__ void tile_issue(const ScatterArgs& a, int side, const
 
 // TMAST: whole-sector bucket runs leave the staging buffer as TMA bulk stores (one per bucket
 // and tile, issued by the bucket's thread) instead of per-tuple stores.
-template <int BLOCK, int IPT, int PASS, bool TMAST>
+// HYB (pass 1, gsh_config.hybrid -- CSH's hybrid partition, L90-L91, L100): a tuple of a sampled
+// skewed key is ranked per key in the tile (rank | 0x4000), one global atomic per (tile, key)
+// reserves its run in R_k / S_k, and its payload is stored there instead of being staged: it never
+// reaches a partition.
+template <int BLOCK, int IPT, int PASS, bool TMAST, bool HYB = false>
 __global__ void __launch_bounds__(BLOCK, 2) k_scatter(ScatterArgs a) {
     constexpr int TILE = BLOCK * IPT;
     static_assert(TILE < 0x7fff, "ranks are packed as u16: bit 15 = dominant bucket, 0xffff = masked");
@@ -569,6 +625,12 @@ __global__ void __launch_bounds__(BLOCK, 2) k_scatter(ScatterArgs a) {
     uint32_t* op = ok + TILE + 4;                       // pass 1: payloads
     uint2* o2 = reinterpret_cast<uint2*>(buf0);         // pass 2: (h, payload)
     uint2* stage = reinterpret_cast<uint2*>(buf0 + (size_t(TILE) + 4) * 8);
+    unsigned char* hyb0 = buf0 + (size_t(TILE) + 4) * 8 + (size_t(TILE) + 4 * 256 + 4) * 8;
+    unsigned long long* htab = reinterpret_cast<unsigned long long*>(hyb0);    // [kHybSlots]
+    uint32_t* hcnt = reinterpret_cast<uint32_t*>(hyb0 + kHybSlots * 8);        // [kHybMaxKeys] tile ranks
+    uint32_t* hbase = hcnt + kHybMaxKeys;                                       // [kHybMaxKeys] run starts
+    static_assert(!HYB || PASS == 1, "hybrid routing happens in pass 1");
+    static_assert(!HYB || BLOCK * IPT < 0x4000, "hybrid ranks are tagged 0x4000 | rank");
 
     const uint32_t tid = threadIdx.x;
     constexpr bool p1 = (PASS == 1);
@@ -583,6 +645,10 @@ __global__ void __launch_bounds__(BLOCK, 2) k_scatter(ScatterArgs a) {
     const uint64_t rpol = policy_evict_first(), wpol = policy_evict_first();
 
     if (tid < 256) S.tcnt[tid] = 0;
+    if (HYB) {
+        for (uint32_t i = tid; i < kHybSlots; i += BLOCK) htab[i] = a.hyb_tab[i];
+        for (uint32_t i = tid; i < kHybMaxKeys; i += BLOCK) hcnt[i] = 0;
+    }
     if (tid == 0) {
         mbar_init(&S.mbar, 1);
         S.claim = atomicAdd(a.unit_ctr, 1u);
@@ -671,16 +737,26 @@ __global__ void __launch_bounds__(BLOCK, 2) k_scatter(ScatterArgs a) {
                     }
                 };
                 if (p1) {    // uint4 = 4 keys; slot 4 * v + c of element 4 * (v * BLOCK + tid) + c
+                    // a sampled skewed key's tuple: ranked among its key's tuples in the tile
+                    auto rank1 = [&](uint32_t h) -> uint32_t {
+                        if constexpr (HYB) {
+                            const uint32_t hid = hyb_find(htab, h);
+                            const uint32_t r = rank_of(hid == kNoHeavy, (h >> dshift) & dmask);
+                            return hid == kNoHeavy ? r : (0x4000u | atomicAdd(&hcnt[hid], 1u));
+                        } else {
+                            return rank_of(true, (h >> dshift) & dmask);
+                        }
+                    };
 #pragma unroll
                     for (int v = 0; v < NV; ++v) {
                         uint4 x = reinterpret_cast<const uint4*>(ok)[v * BLOCK + tid];
                         xb[v] = reinterpret_cast<const uint4*>(op)[v * BLOCK + tid];
                         x.x = hash32(x.x); x.y = hash32(x.y); x.z = hash32(x.z); x.w = hash32(x.w);
                         xa[v] = x;
-                        const uint32_t r0 = rank_of(true, (x.x >> dshift) & dmask);
-                        const uint32_t r1 = rank_of(true, (x.y >> dshift) & dmask);
-                        const uint32_t r2 = rank_of(true, (x.z >> dshift) & dmask);
-                        const uint32_t r3 = rank_of(true, (x.w >> dshift) & dmask);
+                        const uint32_t r0 = rank1(x.x);
+                        const uint32_t r1 = rank1(x.y);
+                        const uint32_t r2 = rank1(x.z);
+                        const uint32_t r3 = rank1(x.w);
                         rk[2 * v] = r0 | (r1 << 16);
                         rk[2 * v + 1] = r2 | (r3 << 16);
                     }
@@ -728,7 +804,10 @@ __global__ void __launch_bounds__(BLOCK, 2) k_scatter(ScatterArgs a) {
                                 h = e.x;
                             }
                         }
-                        r = atomicAdd(&S.tcnt[(h >> dshift) & dmask], 1u);
+                        uint32_t hid = kNoHeavy;
+                        if constexpr (HYB) hid = hyb_find(htab, h);
+                        r = hid == kNoHeavy ? atomicAdd(&S.tcnt[(h >> dshift) & dmask], 1u)
+                                            : (0x4000u | atomicAdd(&hcnt[hid], 1u));
                     }
                     if (jj & 1) rk[jj >> 1] |= r << 16; else rk[jj >> 1] = r;
                 }
@@ -743,6 +822,15 @@ __global__ void __launch_bounds__(BLOCK, 2) k_scatter(ScatterArgs a) {
             // Write combining: bucket b's staged run = [carry from the previous tile | this tile's
             // tuples]; only whole 32-byte sectors are written, the < 4-tuple remainder carries
             // over (the unit's last tile flushes everything).  u32 offsets (n < 2^32).
+            if constexpr (HYB) {   // reserve this tile's run of every skewed key it holds
+                for (uint32_t i = tid; i < a.n_h0; i += BLOCK) {
+                    const uint32_t c = hcnt[i];
+                    if (c) {
+                        hbase[i] = (uint32_t)a.h_off[ui.side][i] + atomicAdd(&a.h_cur[ui.side][i], c);
+                        hcnt[i] = 0;
+                    }
+                }
+            }
             uint32_t tc = (tid < nb) ? S.tcnt[tid] : 0u;
             if (dom_on) {
                 constexpr uint32_t NW = BLOCK / 32;
@@ -790,13 +878,20 @@ __global__ void __launch_bounds__(BLOCK, 2) k_scatter(ScatterArgs a) {
                     return (r & 0x8000u) ? dbase + (r & 0x7fffu) : S.local_start[b] + r;
                 };
                 if (p1) {
+                    // staged, or (hybrid: rank tagged 0x4000, dominant bit clear) stored into R_k / S_k
+                    auto put = [&](uint32_t h, uint32_t pay, uint32_t r) {
+                        if (HYB && (r & 0xc000u) == 0x4000u)
+                            a.heavy_pay[ui.side][hbase[hyb_find(htab, h)] + (r & 0x3fffu)] = pay;
+                        else
+                            stage[spos((h >> dshift) & dmask, r)] = make_uint2(h, pay);
+                    };
 #pragma unroll
                     for (int v = 0; v < NV; ++v) {
                         const uint4 h4 = xa[v], p4 = xb[v];
-                        stage[spos((h4.x >> dshift) & dmask, rk[2 * v] & 0xffffu)] = make_uint2(h4.x, p4.x);
-                        stage[spos((h4.y >> dshift) & dmask, rk[2 * v] >> 16)] = make_uint2(h4.y, p4.y);
-                        stage[spos((h4.z >> dshift) & dmask, rk[2 * v + 1] & 0xffffu)] = make_uint2(h4.z, p4.z);
-                        stage[spos((h4.w >> dshift) & dmask, rk[2 * v + 1] >> 16)] = make_uint2(h4.w, p4.w);
+                        put(h4.x, p4.x, rk[2 * v] & 0xffffu);
+                        put(h4.y, p4.y, rk[2 * v] >> 16);
+                        put(h4.z, p4.z, rk[2 * v + 1] & 0xffffu);
+                        put(h4.w, p4.w, rk[2 * v + 1] >> 16);
                     }
                 } else {   // ranks < TILE <= 0x7fff, so 0xffff marks a masked slot
 #pragma unroll
@@ -814,7 +909,10 @@ __global__ void __launch_bounds__(BLOCK, 2) k_scatter(ScatterArgs a) {
                     if (i < ql) {
                         const uint2 e = p1 ? make_uint2(ok[i], op[i]) : o2[i + lp.shift];
                         const uint32_t r = (jj & 1) ? (rk[jj >> 1] >> 16) : (rk[jj >> 1] & 0xffffu);
-                        stage[S.local_start[(e.x >> dshift) & dmask] + r] = e;
+                        if (HYB && (r & 0xc000u) == 0x4000u)
+                            a.heavy_pay[ui.side][hbase[hyb_find(htab, e.x)] + (r & 0x3fffu)] = e.y;
+                        else
+                            stage[S.local_start[(e.x >> dshift) & dmask] + r] = e;
                     }
                 }
                 fence_proxy_async_smem();  // reads of the input tile precede the next TMA writes
@@ -858,17 +956,19 @@ __global__ void __launch_bounds__(BLOCK, 2) k_scatter(ScatterArgs a) {
     if (TMAST && tid < nb) bulk_wait0();  // shared memory must outlive the bulk stores' reads
 }
 
-size_t scatter_smem_bytes(int tile) {
-    // input tile (+4 slack) and staging = tile + up to 3 carried tuples per bucket
-    return ((sizeof(ScatterSmem) + 127) & ~size_t(127)) + (size_t(tile) + 4) * 8 + (size_t(tile) + 4 * 256 + 4) * 8;
+size_t scatter_smem_bytes(int tile, bool hyb = false) {
+    // input tile (+4 slack) and staging = tile + up to 3 carried tuples per bucket (+ the hybrid
+    // table, tile ranks and run starts)
+    return ((sizeof(ScatterSmem) + 127) & ~size_t(127)) + (size_t(tile) + 4) * 8 + (size_t(tile) + 4 * 256 + 4) * 8 +
+           (hyb ? size_t(kHybSlots) * 8 + size_t(kHybMaxKeys) * 8 : 0);
 }
 
-template <int BLOCK, int IPT, int PASS, bool TMAST>
+template <int BLOCK, int IPT, int PASS, bool TMAST, bool HYB = false>
 int launch_scatter_pass(const Plan& p, const ScatterArgs& a, cudaStream_t s) {
-    const size_t smem = scatter_smem_bytes(BLOCK * IPT);
+    const size_t smem = scatter_smem_bytes(BLOCK * IPT, HYB);
     static std::once_flag attr_once[kMaxDevices];   // > 48 KB of dynamic shared memory: opt in once per device
     once_per_device(attr_once, [&] {
-        cudaFuncSetAttribute(k_scatter<BLOCK, IPT, PASS, TMAST>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+        cudaFuncSetAttribute(k_scatter<BLOCK, IPT, PASS, TMAST, HYB>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                              (int)smem);
     });
     static int occ_dev[kMaxDevices] = {0};   // per kernel instance and device: query once
@@ -877,10 +977,10 @@ int launch_scatter_pass(const Plan& p, const ScatterArgs& a, cudaStream_t s) {
     int& occ = occ_dev[dev >= 0 && dev < kMaxDevices ? dev : 0];
     if (occ < 1) {
         int o = 0;
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, k_scatter<BLOCK, IPT, PASS, TMAST>, BLOCK, smem);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, k_scatter<BLOCK, IPT, PASS, TMAST, HYB>, BLOCK, smem);
         occ = o < 1 ? 1 : o;
     }
-    k_scatter<BLOCK, IPT, PASS, TMAST><<<(unsigned)(p.num_sms * occ), BLOCK, smem, s>>>(a);
+    k_scatter<BLOCK, IPT, PASS, TMAST, HYB><<<(unsigned)(p.num_sms * occ), BLOCK, smem, s>>>(a);
     return 1;
 }
 template <int BLOCK, int IPT, bool TMAST>
@@ -915,6 +1015,13 @@ int launch_scatter(const Plan& p, int pass, const uint32_t* const keys[2], const
     a.b2 = p.b2;
     a.route_bits = p.route_bits;
     a.unit_ctr = &p.st->claim[pass - 1];
+    a.hyb_tab = p.hyb_tab;
+    a.n_h0 = p.n_h0;
+    for (int side = 0; side < 2; ++side) {
+        a.h_off[side] = p.h_off + size_t(side) * (p.h_max + 1);
+        a.h_cur[side] = p.h_cur + size_t(side) * p.h_max;
+        a.heavy_pay[side] = p.heavy_pay[side];
+    }
     static int cfg = -1;
     if (cfg < 0) {
         const char* e = getenv("GSH_SCATTER_CFG");  // experiments only
@@ -928,6 +1035,7 @@ int launch_scatter(const Plan& p, int pass, const uint32_t* const keys[2], const
     // 448 x 12 = 5376 tuples (0.976 ms; 512 x 8: 1.032, 384 x 12: 1.011, 512 x 12: 1.187).
     // Tiles need not divide a unit: a unit's ragged last tile takes the scalar path.
     if (cfg == 1) return launch_scatter_cfg<kScatterBlock, kScatterIpt, true>(p, a, s);
+    if (pass == 1 && p.n_h0) return launch_scatter_pass<kScatterBlock1, kScatterIptHyb, 1, false, true>(p, a, s);
     return pass == 1 ? launch_scatter_pass<kScatterBlock1, kScatterIpt1, 1, false>(p, a, s)
                      : launch_scatter_pass<kScatterBlock2, kScatterIpt, 2, false>(p, a, s);
 }

@@ -496,11 +496,18 @@ struct NormalRemainder {
     }
 };
 
-int launch_heavy_prefix(const Plan& p, uint32_t n_heavy, uint32_t n_large, cudaStream_t s) {
+// Per-key array offsets (R_k, S_k) and dense-tile prefix over H[0, n_heavy).  Entries keep their
+// offsets when more are appended (hybrid keys first, then the residual detection's).
+int launch_heavy_offsets(const Plan& p, uint32_t n_heavy, cudaStream_t s) {
     int l = 0;
     l += launch_scan(HeavyCount{p.H, 0}, n_heavy, p.h_off, p.scan_scratch, s);
     l += launch_scan(HeavyCount{p.H, 1}, n_heavy, p.h_off + (p.h_max + 1), p.scan_scratch, s);
     l += launch_scan(HeavyTiles{p.H}, n_heavy, p.h_tiles, p.scan_scratch, s);
+    return l;
+}
+
+int launch_heavy_prefix(const Plan& p, uint32_t n_heavy, uint32_t n_large, cudaStream_t s) {
+    int l = launch_heavy_offsets(p, n_heavy, s);
     l += launch_scan(NormalRemainder{p.cnt, p.part_heavy, p.large_list, p.F, 0}, n_large, p.nrm_off,
                      p.scan_scratch, s);
     l += launch_scan(NormalRemainder{p.cnt, p.part_heavy, p.large_list, p.F, 1}, n_large, p.nrm_off + (p.F + 1),

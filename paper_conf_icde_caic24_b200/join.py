@@ -20,7 +20,8 @@ def make_config(capacity: int = 0, pass_bits=None, heavy_threshold: int = 0, rou
                 force_all_normal: bool = False, force_all_heavy: bool = False, timing: bool = False,
                 large_threshold: int = 0, nm_table: int = 0, detect_mode: int = 0, sample_stride: int = 0,
                 top_k: int = 0, prepass_bits: int = 0, input_side_only: bool = False,
-                heavy_detail: bool = False) -> GshConfig:
+                heavy_detail: bool = False, hybrid: bool = False, hybrid_stride: int = 0,
+                hybrid_min: int = 0) -> GshConfig:
     """Build a gsh_config (see include/gsh.h for each field's meaning)."""
     cfg = _lib.default_config()
     cfg.capacity = int(capacity)
@@ -40,6 +41,9 @@ def make_config(capacity: int = 0, pass_bits=None, heavy_threshold: int = 0, rou
     cfg.prepass_bits = int(prepass_bits)
     cfg.input_side_only = int(bool(input_side_only))
     cfg.heavy_detail = int(bool(heavy_detail))
+    cfg.hybrid = int(bool(hybrid))
+    cfg.hybrid_stride = int(hybrid_stride)
+    cfg.hybrid_min = int(hybrid_min)
     return cfg
 
 
@@ -126,12 +130,17 @@ def workspace_bytes(n_r: int, n_s: int, config: GshConfig | None = None) -> int:
 
 def join(r_keys: torch.Tensor, r_payloads: torch.Tensor, s_keys: torch.Tensor, s_payloads: torch.Tensor,
          mode: str = "count", out: torch.Tensor | None = None, out_capacity: int | None = None,
-         config: GshConfig | None = None, stream=None, workspace: torch.Tensor | None = None) -> JoinResult:
+         config: GshConfig | None = None, stream=None, workspace: torch.Tensor | None = None,
+         impl: str = "gsh") -> JoinResult:
     """GSH equi-join of device-resident R and S (gsh_join, include/gsh.h).
 
     mode: "count" (count + checksum) or "materialize" (also (payload_R, payload_S) pairs into
     `out`, an int32 CUDA tensor of shape (capacity, 2), or a fresh one of out_capacity rows).
+    impl: "gsh" (gsh_join) or "gbase" (gsh_join_gbase: the paper's skew-unaware comparison system,
+    same result, for the GSH-vs-Gbase measurement).
     """
+    if impl not in ("gsh", "gbase"):
+        raise ValueError("impl must be 'gsh' or 'gbase'")
     lib = load()
     rk, rp = _check_dev(r_keys, "r_keys"), _check_dev(r_payloads, "r_payloads")
     sk, sp = _check_dev(s_keys, "s_keys"), _check_dev(s_payloads, "s_payloads")
@@ -159,12 +168,13 @@ def join(r_keys: torch.Tensor, r_payloads: torch.Tensor, s_keys: torch.Tensor, s
     args = (ctypes.byref(R), ctypes.byref(S), _lib.GSH_OUT_MATERIALIZE if mat else _lib.GSH_OUT_COUNT,
             ctypes.byref(outp) if outp is not None else None, ws.data_ptr(), ws.numel(),
             ctypes.byref(config) if config is not None else None, _stream_handle(stream, dev), ctypes.byref(res))
+    fn = lib.gsh_join if impl == "gsh" else lib.gsh_join_gbase
     if dev.index == torch.cuda.current_device():
-        st = lib.gsh_join(*args)
+        st = fn(*args)
     else:
         with torch.cuda.device(dev):
-            st = lib.gsh_join(*args)
-    check(st, "gsh_join")
+            st = fn(*args)
+    check(st, "gsh_join" if impl == "gsh" else "gsh_join_gbase")
     return JoinResult(count=int(res.count), checksum=int(res.checksum), written=int(res.written),
                       overflow=bool(res.overflow), pairs=(out[: res.written] if mat else None), raw=res)
 

@@ -31,6 +31,11 @@ CASES = [  # kind, n, theta, config
     ("graph", 1 << 16, 0.909, {}),
     ("zipf", 1 << 16, 1.0, {"prepass_bits": 2}),
     ("pkfk_zipf", 1 << 16, 1.0, {"heavy_detail": True}),
+    ("zipf", 1 << 17, 1.0, {"hybrid": True}),
+    ("zipf", 1 << 15, 1.5, {"hybrid": True, "hybrid_stride": 1}),
+    ("pkfk_zipf", 1 << 16, 1.0, {"hybrid": True}),
+    ("zipf", (1 << 15) + 3, 1.0, {"impl": "gbase"}),
+    ("graph", 1 << 15, 0.909, {"impl": "gbase"}),
 ]
 
 
@@ -42,16 +47,18 @@ def main():
     dev = torch.device("cuda", 0)
     tool = os.environ.get("SAN_TOOL", "?")
     for kind, n, theta, kw in CASES:
+        kw = dict(kw)
+        impl = kw.pop("impl", "gsh")
         rk, rp, sk, sp = datagen.make_workload(kind, n, theta, seed=3)
         on, oc, _ = oracle.join(u(rk), u(rp), u(sk), u(sp))
         d = [t.to(dev) for t in (rk, rp, sk, sp)]
         cfg = gsh.make_config(**kw)
-        r = gsh.join(*d, config=cfg)
+        r = gsh.join(*d, config=cfg, impl=impl)
         assert (r.count, r.checksum) == (on, oc), (kind, n, theta, kw)
         if on <= (1 << 22) and not kw.get("heavy_detail"):
-            m = gsh.join(*d, mode="materialize", out_capacity=on, config=gsh.make_config(**kw))
+            m = gsh.join(*d, mode="materialize", out_capacity=on, config=gsh.make_config(**kw), impl=impl)
             assert (m.count, m.checksum, m.written) == (on, oc, on)
-        print(f"[{tool}] ok {kind} n={n} theta={theta} {kw} count={on}", flush=True)
+        print(f"[{tool}] ok {impl} {kind} n={n} theta={theta} {kw} count={on}", flush=True)
     full = [t.to(dev) for t in datagen.make_workload("zipf", 1 << 15, 1.0, seed=5)]
     on, oc, _ = oracle.join(*(u(t) for t in full))
     shards = [tuple(t[g * (1 << 14):(g + 1) * (1 << 14)] for t in full) for g in range(2)]

@@ -113,6 +113,31 @@ def test_argument_errors_before_any_launch():
     assert st == _lib.GSH_ERR_INVALID  # n >= 2^32
 
 
+def test_gbase_argument_errors_before_any_launch():
+    lib = _lib.load()
+    res = _lib.GshResult()
+    R = _lib.GshRelation(None, None, 10)
+    S = _lib.GshRelation(None, None, 0)
+    assert lib.gsh_join_gbase(ctypes.byref(R), ctypes.byref(S), 0, None, None, 0, None, None,
+                              ctypes.byref(res)) == _lib.GSH_ERR_INVALID
+    R = _lib.GshRelation(None, None, 0)
+    assert lib.gsh_join_gbase(ctypes.byref(R), ctypes.byref(S), 1, None, None, 0, None, None,
+                              ctypes.byref(res)) == _lib.GSH_ERR_INVALID   # MATERIALIZE without output
+    big = _lib.GshRelation(1, 1, (1 << 28) + 1)   # never dereferenced: refused first
+    assert lib.gsh_join_gbase(ctypes.byref(big), ctypes.byref(S), 0, None, None, 0, None, None,
+                              ctypes.byref(res)) == _lib.GSH_ERR_INVALID
+    assert b"2^28" in lib.gsh_last_error()
+
+
+def test_hybrid_config_validation():
+    lib = _lib.load()
+    assert gsh.workspace_bytes(1 << 20, 1 << 20, gsh.make_config(hybrid=True)) > \
+        gsh.workspace_bytes(1 << 20, 1 << 20)
+    cfg = gsh.make_config()
+    cfg.hybrid = 2
+    assert lib.gsh_workspace_bytes(1000, 1000, ctypes.byref(cfg)) == 0
+
+
 def test_product_path_refuses_cpu_tensors():
     import torch
     k = torch.zeros(4, dtype=torch.int32)
