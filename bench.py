@@ -47,6 +47,7 @@ WORKLOADS = {
     "zipf10s": ("zipf", 1 << 24, 1.0, "cfg3-shaped (scaled): |R|=|S|=2^24 Zipf theta=1.0 both sides, COUNT"),
     "zipf15s": ("zipf", 1 << 22, 1.5, "cfg3-shaped (scaled): |R|=|S|=2^22 Zipf theta=1.5 both sides, COUNT"),
     "graph": ("graph", 1 << 26, 0.909, "cfg4-shaped (scaled): 2^26-edge power-law graph self-join (dst, src), COUNT"),
+    "graph28": ("graph", 1 << 28, 0.909, "cfg4: 2^28-edge power-law graph self-join (dst, src), V = 2^24, COUNT (~8.6e13 pairs)"),
     "pkfk28": ("pkfk", 1 << 28, 0.0, "scale point: |R|=|S|=2^28 uniform 1:1 PK-FK (cfg5's per-GPU share at G=8), COUNT"),
     "pkfk29": ("pkfk", 1 << 29, 0.0, "scale point: |R|=|S|=2^29 uniform 1:1 PK-FK (4x cfg2; 2^30 input tuples), COUNT"),
     "pkfk30": ("pkfk", 1 << 30, 0.0, "scale point: |R|=|S|=2^30 uniform 1:1 PK-FK (8x cfg2; 2^31 input tuples), COUNT"),

@@ -225,7 +225,7 @@ bool plan_build(Plan& p, uint64_t nR, uint64_t nS, const gsh_config* cfg_in, voi
     p.nm = c.take<NmPart>(F);
     p.nm_prefix = c.take<uint64_t>(F + 1);
     p.scan_scratch = c.take<uint64_t>(p.scan_scratch_elems);
-    p.hyb_tab = c.take<unsigned long long>(kHybSlots);
+    p.hyb_tab = reinterpret_cast<uint32_t*>(c.take<unsigned char>(kHybTabBytes));
     p.hyb_list = c.take<uint32_t>(kHybMaxKeys);
     p.hyb_cnt = c.take<uint32_t>(2 * kHybMaxKeys);
     p.bytes = c.off;
@@ -778,7 +778,7 @@ gsh_status gsh_heavy_detail(uint64_t n_r, uint64_t n_s, const gsh_config* cfg, v
     cudaError_t ce = cudaMemcpyAsync(&hs, p.st, sizeof(DevState), cudaMemcpyDeviceToHost, s);
     if (ce == cudaSuccess) ce = cudaStreamSynchronize(s);
     if (ce != cudaSuccess) return cuda_fail(ce, "detail sync");
-    const uint32_t nh = hs.n_large ? hs.n_heavy : 0u;
+    const uint32_t nh = hs.n_heavy;   // hybrid keys (gsh_config.hybrid) + detected ones
     *h_n = nh;
     if (nh > cap) return fail(GSH_ERR_INVALID, "capacity too small (see *h_n)");
     if (nh) {

@@ -81,10 +81,14 @@ constexpr uint32_t kDetectItem = 16384;         // tuples per exact-detect work 
 constexpr uint32_t kNoHeavy = 0xffffffffu;
 constexpr int kDetectMaxProbe = 64;   // a full table degrades to "normal", never to a long probe
 // Hybrid partition (gsh_config.hybrid, hybrid.cu): at most kHybMaxKeys sampled skewed keys, looked
-// up in a kHybSlots-slot shared-memory copy of the table ((hid + 1) << 32 | h, 0 = empty; load <= 1/2)
+// up in a kHybSlots-slot shared-memory copy of the table: u32 h per slot (kHybEmpty = empty; a key
+// whose h is kHybEmpty is never chosen), then u16 key ids; load <= 1/4, so a miss usually ends at
+// its first slot.
 constexpr uint32_t kHybMaxKeys = 512;
-constexpr uint32_t kHybSlots = 1024;
-constexpr uint32_t kHybLogSlots = 10;
+constexpr uint32_t kHybSlots = 2048;
+constexpr uint32_t kHybLogSlots = 11;
+constexpr uint32_t kHybEmpty = 0xffffffffu;
+constexpr size_t kHybTabBytes = size_t(kHybSlots) * 6;   // keys, then ids
 constexpr int kScatterIptHyb = 16;               // pass-1 tile with the hybrid tables (two CTAs per SM)
 
 // Device-resident counters and accumulators, zeroed once per call.
@@ -193,7 +197,7 @@ struct Plan {
     NmPart* nm = nullptr;                     // [F]
     uint64_t* nm_prefix = nullptr;            // [F + 1]
     uint64_t* scan_scratch = nullptr;         // block sums for the generic scan
-    unsigned long long* hyb_tab = nullptr;    // [kHybSlots] hybrid lookup table
+    uint32_t* hyb_tab = nullptr;              // hybrid lookup table: u32 h [kHybSlots], u16 id [kHybSlots]
     uint32_t* hyb_list = nullptr;             // [kHybMaxKeys] h of hybrid key hid
     uint32_t* hyb_cnt = nullptr;              // [2][kHybMaxKeys] exact counts (histogram pass)
     size_t bytes = 0;

@@ -59,15 +59,34 @@ constexpr uint32_t kHistMaxEvents = 128;
 static_assert(kScatterChunk == 16 * kHistBlock, "a full chunk is 4 uint4 per histogram thread");
 static_assert(3 * ((uint64_t(kHistMaxUnitChunks) * kScatterChunk) >> 16) <= kHistMaxEvents, "wrap events of a slice");
 
-// Hybrid partition (hybrid.cu): the sampled skewed keys' table, (hid + 1) << 32 | h, 0 = empty.
-__device__ __forceinline__ uint32_t hyb_find(const unsigned long long* tab, uint32_t h) {
+// Hybrid partition (hybrid.cu): the sampled skewed keys' table (u32 h per slot, kHybEmpty = empty,
+// then u16 ids); load <= 1/4, so most misses end at their first slot.
+__device__ __forceinline__ uint32_t hyb_find(const uint32_t* key, const uint16_t* id, uint32_t h) {
+    if (h == kHybEmpty) return kNoHeavy;   // never chosen (it marks empty slots)
     uint32_t s = (h * 0x9E3779B1u) >> (32 - kHybLogSlots);
-    for (;;) {   // load <= 1/2: an empty slot ends every probe
-        const unsigned long long e = tab[s];
-        if (e == 0) return kNoHeavy;
-        if ((uint32_t)e == h) return (uint32_t)(e >> 32) - 1;
+    for (;;) {
+        const uint32_t k = key[s];
+        if (k == h) return id[s];
+        if (k == kHybEmpty) return kNoHeavy;
         s = (s + 1) & (kHybSlots - 1);
     }
+}
+
+// Rank / count aggregation over the lanes of `am` holding the same skewed key as the first such
+// lane (the warp's reference key): one shared atomic for all of them.  Returns the lane's rank
+// among its key's tuples (0x4000-tagged by the caller) when it is heavy.
+__device__ __forceinline__ uint32_t hyb_rank(uint32_t am, uint32_t hid, uint32_t* cnt) {
+    const bool heavy = hid != kNoHeavy;
+    const uint32_t hm = __ballot_sync(am, heavy);
+    if (!hm) return 0;
+    const uint32_t ref = __shfl_sync(am, hid, __ffs(hm) - 1);
+    const uint32_t mr = __ballot_sync(am, heavy && hid == ref);
+    const uint32_t lead = __ffs(mr) - 1;
+    uint32_t base = 0;
+    if (lane_id() == lead) base = atomicAdd(&cnt[ref], (uint32_t)__popc(mr));
+    base = __shfl_sync(am, base, lead);
+    if (!heavy) return 0;
+    return hid == ref ? base + __popc(mr & lanemask_lt()) : atomicAdd(&cnt[hid], 1u);
 }
 
 // CHECK (route_bits > 0): also verify the caller's gsh_config.route_bits assertion -- every tuple
@@ -81,12 +100,16 @@ __global__ void __launch_bounds__(kHistBlock, 1)
 k_hist2d(const uint32_t* __restrict__ k0, uint64_t n0, const uint32_t* __restrict__ k1, uint64_t n1,
          uint32_t shift, uint32_t nbits, uint32_t b2, uint32_t* __restrict__ partial, uint32_t* __restrict__ c1cnt,
          uint32_t nu0, uint32_t nu1, uint32_t unit_chunks, uint32_t rshift, DevState* st,
-         uint32_t* __restrict__ slice_dom, const unsigned long long* __restrict__ hyb_tab, uint32_t n_h0,
+         uint32_t* __restrict__ slice_dom, const uint32_t* __restrict__ hyb_tab, uint32_t n_h0,
          uint32_t* __restrict__ hyb_cnt) {
-    __shared__ unsigned long long s_htab[HYB ? kHybSlots : 1];
+    __shared__ uint32_t s_hkey[HYB ? kHybSlots : 1];
+    __shared__ uint16_t s_hid[HYB ? kHybSlots : 1];
     __shared__ uint32_t s_hc[HYB ? kHybMaxKeys : 1];
     if (HYB) {
-        for (uint32_t i = threadIdx.x; i < kHybSlots; i += blockDim.x) s_htab[i] = hyb_tab[i];
+        for (uint32_t i = threadIdx.x; i < kHybSlots; i += blockDim.x) {
+            s_hkey[i] = hyb_tab[i];
+            s_hid[i] = reinterpret_cast<const uint16_t*>(hyb_tab + kHybSlots)[i];
+        }
         for (uint32_t i = threadIdx.x; i < kHybMaxKeys; i += blockDim.x) s_hc[i] = 0;
     }
     uint32_t r_or = 0, r_nor = 0;
@@ -134,11 +157,9 @@ k_hist2d(const uint32_t* __restrict__ k0, uint64_t n0, const uint32_t* __restric
                 r_or |= t;
                 r_nor |= ~t;
             }
-            const uint32_t hid = hyb_find(s_htab, hk);
-            if (hid != kNoHeavy) {
-                atomicAdd(&s_hc[hid], 1u);
-                return;
-            }
+            const uint32_t hid = hyb_find(s_hkey, s_hid, hk);
+            hyb_rank(__activemask(), hid, s_hc);   // counts only (the rank is not needed)
+            if (hid != kNoHeavy) return;
             const uint32_t bin = (hk >> shift) & mask;
             if (packed) count_exact(bin); else atomicAdd(&cnt[bin], 1u);
         } else if (FAST16) {
@@ -470,7 +491,7 @@ struct ScatterArgs {
     uint32_t pass, b1, b2, route_bits;
     unsigned int* unit_ctr;
     // hybrid pass 1 (HYB): sampled skewed keys' table, their count, R_k / S_k offsets, cursors, arrays
-    const unsigned long long* hyb_tab;
+    const uint32_t* hyb_tab;
     uint32_t n_h0;
     const uint64_t* h_off[2];
     uint32_t* h_cur[2];
@@ -614,7 +635,10 @@ __device__ __forceinline__ void tile_issue(const ScatterArgs& a, int side, const
 // skewed key is ranked per key in the tile (rank | 0x4000), one global atomic per (tile, key)
 // reserves its run in R_k / S_k, and its payload is stored there instead of being staged: it never
 // reaches a partition.
-template <int BLOCK, int IPT, int PASS, bool TMAST, bool HYB = false>
+// WOB: the write-out walks buckets (one warp per bucket run: the run's description is a broadcast
+// load, its stage reads and global stores are contiguous) instead of staged positions (one thread
+// per position: a random 8-byte shared load of the position's bucket descriptor).
+template <int BLOCK, int IPT, int PASS, bool TMAST, bool HYB = false, bool WOB = false>
 __global__ void __launch_bounds__(BLOCK, 2) k_scatter(ScatterArgs a) {
     constexpr int TILE = BLOCK * IPT;
     static_assert(TILE < 0x7fff, "ranks are packed as u16: bit 15 = dominant bucket, 0xffff = masked");
@@ -626,9 +650,10 @@ __global__ void __launch_bounds__(BLOCK, 2) k_scatter(ScatterArgs a) {
     uint2* o2 = reinterpret_cast<uint2*>(buf0);         // pass 2: (h, payload)
     uint2* stage = reinterpret_cast<uint2*>(buf0 + (size_t(TILE) + 4) * 8);
     unsigned char* hyb0 = buf0 + (size_t(TILE) + 4) * 8 + (size_t(TILE) + 4 * 256 + 4) * 8;
-    unsigned long long* htab = reinterpret_cast<unsigned long long*>(hyb0);    // [kHybSlots]
-    uint32_t* hcnt = reinterpret_cast<uint32_t*>(hyb0 + kHybSlots * 8);        // [kHybMaxKeys] tile ranks
+    uint32_t* hkey = reinterpret_cast<uint32_t*>(hyb0);                        // [kHybSlots]
+    uint32_t* hcnt = hkey + kHybSlots;                                          // [kHybMaxKeys] tile ranks
     uint32_t* hbase = hcnt + kHybMaxKeys;                                       // [kHybMaxKeys] run starts
+    uint16_t* hid16 = reinterpret_cast<uint16_t*>(hbase + kHybMaxKeys);         // [kHybSlots]
     static_assert(!HYB || PASS == 1, "hybrid routing happens in pass 1");
     static_assert(!HYB || BLOCK * IPT < 0x4000, "hybrid ranks are tagged 0x4000 | rank");
 
@@ -646,7 +671,10 @@ __global__ void __launch_bounds__(BLOCK, 2) k_scatter(ScatterArgs a) {
 
     if (tid < 256) S.tcnt[tid] = 0;
     if (HYB) {
-        for (uint32_t i = tid; i < kHybSlots; i += BLOCK) htab[i] = a.hyb_tab[i];
+        for (uint32_t i = tid; i < kHybSlots; i += BLOCK) {
+            hkey[i] = a.hyb_tab[i];
+            hid16[i] = reinterpret_cast<const uint16_t*>(a.hyb_tab + kHybSlots)[i];
+        }
         for (uint32_t i = tid; i < kHybMaxKeys; i += BLOCK) hcnt[i] = 0;
     }
     if (tid == 0) {
@@ -740,9 +768,10 @@ __global__ void __launch_bounds__(BLOCK, 2) k_scatter(ScatterArgs a) {
                     // a sampled skewed key's tuple: ranked among its key's tuples in the tile
                     auto rank1 = [&](uint32_t h) -> uint32_t {
                         if constexpr (HYB) {
-                            const uint32_t hid = hyb_find(htab, h);
+                            const uint32_t hid = hyb_find(hkey, hid16, h);
                             const uint32_t r = rank_of(hid == kNoHeavy, (h >> dshift) & dmask);
-                            return hid == kNoHeavy ? r : (0x4000u | atomicAdd(&hcnt[hid], 1u));
+                            const uint32_t hr = hyb_rank(kFull, hid, hcnt);
+                            return hid == kNoHeavy ? r : (0x4000u | hr);
                         } else {
                             return rank_of(true, (h >> dshift) & dmask);
                         }
@@ -805,7 +834,7 @@ __global__ void __launch_bounds__(BLOCK, 2) k_scatter(ScatterArgs a) {
                             }
                         }
                         uint32_t hid = kNoHeavy;
-                        if constexpr (HYB) hid = hyb_find(htab, h);
+                        if constexpr (HYB) hid = hyb_find(hkey, hid16, h);
                         r = hid == kNoHeavy ? atomicAdd(&S.tcnt[(h >> dshift) & dmask], 1u)
                                             : (0x4000u | atomicAdd(&hcnt[hid], 1u));
                     }
@@ -862,7 +891,8 @@ __global__ void __launch_bounds__(BLOCK, 2) k_scatter(ScatterArgs a) {
                 my_w0 = w0;
                 my_ew = ew;
                 S.local_start[tid] = lstart + cin;
-                S.gw[tid] = make_uint2(w0 - lstart, ew);
+                // WOB: (stage start, output start) of the run; its length is tailpos - stage start
+                S.gw[tid] = WOB ? make_uint2(lstart, w0) : make_uint2(w0 - lstart, ew);
                 S.tailpos[tid] = lstart + (ew - w0);
                 for (uint32_t k = 0; k < cin; ++k) stage[lstart + k] = S.cbuf[tid][k];
                 S.wpos[tid] = ew;
@@ -881,7 +911,7 @@ __global__ void __launch_bounds__(BLOCK, 2) k_scatter(ScatterArgs a) {
                     // staged, or (hybrid: rank tagged 0x4000, dominant bit clear) stored into R_k / S_k
                     auto put = [&](uint32_t h, uint32_t pay, uint32_t r) {
                         if (HYB && (r & 0xc000u) == 0x4000u)
-                            a.heavy_pay[ui.side][hbase[hyb_find(htab, h)] + (r & 0x3fffu)] = pay;
+                            a.heavy_pay[ui.side][hbase[hyb_find(hkey, hid16, h)] + (r & 0x3fffu)] = pay;
                         else
                             stage[spos((h >> dshift) & dmask, r)] = make_uint2(h, pay);
                     };
@@ -910,7 +940,7 @@ __global__ void __launch_bounds__(BLOCK, 2) k_scatter(ScatterArgs a) {
                         const uint2 e = p1 ? make_uint2(ok[i], op[i]) : o2[i + lp.shift];
                         const uint32_t r = (jj & 1) ? (rk[jj >> 1] >> 16) : (rk[jj >> 1] & 0xffffu);
                         if (HYB && (r & 0xc000u) == 0x4000u)
-                            a.heavy_pay[ui.side][hbase[hyb_find(htab, e.x)] + (r & 0x3fffu)] = e.y;
+                            a.heavy_pay[ui.side][hbase[hyb_find(hkey, hid16, e.x)] + (r & 0x3fffu)] = e.y;
                         else
                             stage[S.local_start[(e.x >> dshift) & dmask] + r] = e;
                     }
@@ -936,6 +966,14 @@ __global__ void __launch_bounds__(BLOCK, 2) k_scatter(ScatterArgs a) {
                     if (a0 + n2 < my_ew) st_stream_u2(out + (my_ew - 1), stage[lstart + (my_ew - 1 - my_w0)], wpol);
                     bulk_commit();
                 }
+            } else if (WOB) {
+                constexpr uint32_t NW = BLOCK / 32;
+                const uint32_t lane = tid & 31u;
+                for (uint32_t b = tid >> 5; b < nb; b += NW) {
+                    const uint2 wo = S.gw[b];
+                    const uint32_t len = S.tailpos[b] - wo.x;
+                    for (uint32_t k = lane; k < len; k += 32) st_stream_u2(out + wo.y + k, stage[wo.x + k], wpol);
+                }
             } else {
 #pragma unroll 4
                 for (uint32_t i = tid; i < all; i += BLOCK) {
@@ -960,15 +998,15 @@ size_t scatter_smem_bytes(int tile, bool hyb = false) {
     // input tile (+4 slack) and staging = tile + up to 3 carried tuples per bucket (+ the hybrid
     // table, tile ranks and run starts)
     return ((sizeof(ScatterSmem) + 127) & ~size_t(127)) + (size_t(tile) + 4) * 8 + (size_t(tile) + 4 * 256 + 4) * 8 +
-           (hyb ? size_t(kHybSlots) * 8 + size_t(kHybMaxKeys) * 8 : 0);
+           (hyb ? size_t(kHybSlots) * 6 + size_t(kHybMaxKeys) * 8 : 0);
 }
 
-template <int BLOCK, int IPT, int PASS, bool TMAST, bool HYB = false>
+template <int BLOCK, int IPT, int PASS, bool TMAST, bool HYB = false, bool WOB = false>
 int launch_scatter_pass(const Plan& p, const ScatterArgs& a, cudaStream_t s) {
     const size_t smem = scatter_smem_bytes(BLOCK * IPT, HYB);
     static std::once_flag attr_once[kMaxDevices];   // > 48 KB of dynamic shared memory: opt in once per device
     once_per_device(attr_once, [&] {
-        cudaFuncSetAttribute(k_scatter<BLOCK, IPT, PASS, TMAST, HYB>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+        cudaFuncSetAttribute(k_scatter<BLOCK, IPT, PASS, TMAST, HYB, WOB>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                              (int)smem);
     });
     static int occ_dev[kMaxDevices] = {0};   // per kernel instance and device: query once
@@ -977,10 +1015,10 @@ int launch_scatter_pass(const Plan& p, const ScatterArgs& a, cudaStream_t s) {
     int& occ = occ_dev[dev >= 0 && dev < kMaxDevices ? dev : 0];
     if (occ < 1) {
         int o = 0;
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, k_scatter<BLOCK, IPT, PASS, TMAST, HYB>, BLOCK, smem);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, k_scatter<BLOCK, IPT, PASS, TMAST, HYB, WOB>, BLOCK, smem);
         occ = o < 1 ? 1 : o;
     }
-    k_scatter<BLOCK, IPT, PASS, TMAST, HYB><<<(unsigned)(p.num_sms * occ), BLOCK, smem, s>>>(a);
+    k_scatter<BLOCK, IPT, PASS, TMAST, HYB, WOB><<<(unsigned)(p.num_sms * occ), BLOCK, smem, s>>>(a);
     return 1;
 }
 template <int BLOCK, int IPT, bool TMAST>
@@ -1035,6 +1073,11 @@ int launch_scatter(const Plan& p, int pass, const uint32_t* const keys[2], const
     // 448 x 12 = 5376 tuples (0.976 ms; 512 x 8: 1.032, 384 x 12: 1.011, 512 x 12: 1.187).
     // Tiles need not divide a unit: a unit's ragged last tile takes the scalar path.
     if (cfg == 1) return launch_scatter_cfg<kScatterBlock, kScatterIpt, true>(p, a, s);
+    if (cfg == 2)   // write-out by bucket run (experiment)
+        return pass == 1 ? launch_scatter_pass<kScatterBlock1, kScatterIpt1, 1, false, false, true>(p, a, s)
+                         : launch_scatter_pass<kScatterBlock2, kScatterIpt, 2, false, false, true>(p, a, s);
+    if (cfg == 3)   // pass 2 only
+        if (pass == 2) return launch_scatter_pass<kScatterBlock2, kScatterIpt, 2, false, false, true>(p, a, s);
     if (pass == 1 && p.n_h0) return launch_scatter_pass<kScatterBlock1, kScatterIptHyb, 1, false, true>(p, a, s);
     return pass == 1 ? launch_scatter_pass<kScatterBlock1, kScatterIpt1, 1, false>(p, a, s)
                      : launch_scatter_pass<kScatterBlock2, kScatterIpt, 2, false>(p, a, s);
