@@ -34,7 +34,7 @@ import torch  # noqa: E402
 MEASURED_PEAKS = os.path.join(ROOT, "MEASURED_PEAKS.json")
 PROFILE_SUMMARY = os.path.join(ROOT, "profiles", "ncu_traffic.json")
 FALLBACK_HBM_GBS = 6650.0  # /opt/skills/guides/B200_PROFILING.md fallback
-DEVSTATE_BYTES = 168        # sizeof(gsh::DevState): D2H'd twice per step (classify + final)
+DEVSTATE_BYTES = 568        # sizeof(gsh::DevState): D2H'd twice per step (classify + final)
 
 WORKLOADS = {
     # name: (kind, n per side (per rank), theta, description)

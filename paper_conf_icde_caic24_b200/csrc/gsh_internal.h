@@ -108,6 +108,7 @@ struct DevState {
     unsigned int heavy_overflow;                   // more skewed keys than the list H holds
     unsigned int n_h0;                             // hybrid: sampled skewed keys selected
     unsigned int hyb_bins[33];                     // hybrid: sampled keys per floor(log2 count)
+    unsigned long long hyb_mass[33];               // hybrid: their summed sample counts
 };
 
 // Per-(call site, device) one-time setup (kernel attributes): concurrent host threads wait until

@@ -61,15 +61,22 @@ static_assert(3 * ((uint64_t(kHistMaxUnitChunks) * kScatterChunk) >> 16) <= kHis
 
 // Hybrid partition (hybrid.cu): the sampled skewed keys' table (u32 h per slot, kHybEmpty = empty,
 // then u16 ids); load <= 1/4, so most misses end at their first slot.
-__device__ __forceinline__ uint32_t hyb_find(const uint32_t* key, const uint16_t* id, uint32_t h) {
-    if (h == kHybEmpty) return kNoHeavy;   // never chosen (it marks empty slots)
-    uint32_t s = (h * 0x9E3779B1u) >> (32 - kHybLogSlots);
+__device__ __forceinline__ uint32_t hyb_slot(uint32_t h) { return (h * 0x9E3779B1u) >> (32 - kHybLogSlots); }
+// The lookup of h whose first slot's key k0 = key[hyb_slot(h)] is already loaded (callers issue all
+// their first probes before resolving any: independent shared loads instead of a dependent chain).
+__device__ __forceinline__ uint32_t hyb_resolve(const uint32_t* key, const uint16_t* id, uint32_t h, uint32_t k0) {
+    if (h == kHybEmpty || k0 == kHybEmpty) return kNoHeavy;   // kHybEmpty is never chosen
+    uint32_t s = hyb_slot(h);
+    if (k0 == h) return id[s];
     for (;;) {
+        s = (s + 1) & (kHybSlots - 1);
         const uint32_t k = key[s];
         if (k == h) return id[s];
         if (k == kHybEmpty) return kNoHeavy;
-        s = (s + 1) & (kHybSlots - 1);
     }
+}
+__device__ __forceinline__ uint32_t hyb_find(const uint32_t* key, const uint16_t* id, uint32_t h) {
+    return hyb_resolve(key, id, h, key[hyb_slot(h)]);
 }
 
 // Rank / count aggregation over the lanes of `am` holding the same skewed key as the first such
@@ -207,11 +214,38 @@ k_hist2d(const uint32_t* __restrict__ k0, uint64_t n0, const uint32_t* __restric
 #pragma unroll
                 for (int u = 0; u < 4; ++u) cur[u] = v[u];
                 if (c + 1 < cend && chunk_full(c + 1)) load_chunk(c + 1);
+                if constexpr (HYB) {   // all 16 first probes in flight before any is resolved
+                    uint32_t hk[16], k0[16];
 #pragma unroll
-                for (int u = 0; u < 4; ++u) {
-                    const uint32_t kk[4] = {cur[u].x, cur[u].y, cur[u].z, cur[u].w};
+                    for (int u = 0; u < 4; ++u) {
+                        hk[4 * u] = hash32(cur[u].x);
+                        hk[4 * u + 1] = hash32(cur[u].y);
+                        hk[4 * u + 2] = hash32(cur[u].z);
+                        hk[4 * u + 3] = hash32(cur[u].w);
+                    }
 #pragma unroll
-                    for (int q = 0; q < 4; ++q) count_key(kk[q]);
+                    for (int q = 0; q < 16; ++q) k0[q] = s_hkey[hyb_slot(hk[q])];
+#pragma unroll
+                    for (int q = 0; q < 16; ++q) {
+                        if (CHECK) {
+                            const uint32_t t = hk[q] >> rshift;
+                            r_or |= t;
+                            r_nor |= ~t;
+                        }
+                        const uint32_t hid = hyb_resolve(s_hkey, s_hid, hk[q], k0[q]);
+                        hyb_rank(kFull, hid, s_hc);
+                        if (hid == kNoHeavy) {
+                            const uint32_t bin = (hk[q] >> shift) & mask;
+                            if (packed) count_exact(bin); else atomicAdd(&cnt[bin], 1u);
+                        }
+                    }
+                } else {
+#pragma unroll
+                    for (int u = 0; u < 4; ++u) {
+                        const uint32_t kk[4] = {cur[u].x, cur[u].y, cur[u].z, cur[u].w};
+#pragma unroll
+                        for (int q = 0; q < 4; ++q) count_key(kk[q]);
+                    }
                 }
             } else {  // the ragged last chunk, or keys not 16-byte aligned
                 uint64_t done = cb;
@@ -635,10 +669,7 @@ __device__ __forceinline__ void tile_issue(const ScatterArgs& a, int side, const
 // skewed key is ranked per key in the tile (rank | 0x4000), one global atomic per (tile, key)
 // reserves its run in R_k / S_k, and its payload is stored there instead of being staged: it never
 // reaches a partition.
-// WOB: the write-out walks buckets (one warp per bucket run: the run's description is a broadcast
-// load, its stage reads and global stores are contiguous) instead of staged positions (one thread
-// per position: a random 8-byte shared load of the position's bucket descriptor).
-template <int BLOCK, int IPT, int PASS, bool TMAST, bool HYB = false, bool WOB = false>
+template <int BLOCK, int IPT, int PASS, bool TMAST, bool HYB = false>
 __global__ void __launch_bounds__(BLOCK, 2) k_scatter(ScatterArgs a) {
     constexpr int TILE = BLOCK * IPT;
     static_assert(TILE < 0x7fff, "ranks are packed as u16: bit 15 = dominant bucket, 0xffff = masked");
@@ -776,6 +807,38 @@ __global__ void __launch_bounds__(BLOCK, 2) k_scatter(ScatterArgs a) {
                             return rank_of(true, (h >> dshift) & dmask);
                         }
                     };
+                    if constexpr (HYB) {   // hashes and first probes of the whole tile row, then ranks
+                        uint32_t k0[4 * NV];
+#pragma unroll
+                        for (int v = 0; v < NV; ++v) {
+                            uint4 x = reinterpret_cast<const uint4*>(ok)[v * BLOCK + tid];
+                            xb[v] = reinterpret_cast<const uint4*>(op)[v * BLOCK + tid];
+                            x.x = hash32(x.x); x.y = hash32(x.y); x.z = hash32(x.z); x.w = hash32(x.w);
+                            xa[v] = x;
+                        }
+#pragma unroll
+                        for (int v = 0; v < NV; ++v) {
+                            k0[4 * v] = hkey[hyb_slot(xa[v].x)];
+                            k0[4 * v + 1] = hkey[hyb_slot(xa[v].y)];
+                            k0[4 * v + 2] = hkey[hyb_slot(xa[v].z)];
+                            k0[4 * v + 3] = hkey[hyb_slot(xa[v].w)];
+                        }
+                        auto rank2 = [&](uint32_t h, uint32_t kz) -> uint32_t {
+                            const uint32_t hid = hyb_resolve(hkey, hid16, h, kz);
+                            const uint32_t r = rank_of(hid == kNoHeavy, (h >> dshift) & dmask);
+                            const uint32_t hr = hyb_rank(kFull, hid, hcnt);
+                            return hid == kNoHeavy ? r : (0x4000u | hr);
+                        };
+#pragma unroll
+                        for (int v = 0; v < NV; ++v) {
+                            const uint32_t r0 = rank2(xa[v].x, k0[4 * v]);
+                            const uint32_t r1 = rank2(xa[v].y, k0[4 * v + 1]);
+                            const uint32_t r2 = rank2(xa[v].z, k0[4 * v + 2]);
+                            const uint32_t r3 = rank2(xa[v].w, k0[4 * v + 3]);
+                            rk[2 * v] = r0 | (r1 << 16);
+                            rk[2 * v + 1] = r2 | (r3 << 16);
+                        }
+                    } else {
 #pragma unroll
                     for (int v = 0; v < NV; ++v) {
                         uint4 x = reinterpret_cast<const uint4*>(ok)[v * BLOCK + tid];
@@ -788,6 +851,7 @@ __global__ void __launch_bounds__(BLOCK, 2) k_scatter(ScatterArgs a) {
                         const uint32_t r3 = rank1(x.w);
                         rk[2 * v] = r0 | (r1 << 16);
                         rk[2 * v + 1] = r2 | (r3 << 16);
+                    }
                     }
                 } else {     // uint4 = 2 AoS tuples: shared slots 2u, 2u + 1 = tile elements 2u - off, ...
 #pragma unroll
@@ -891,8 +955,7 @@ __global__ void __launch_bounds__(BLOCK, 2) k_scatter(ScatterArgs a) {
                 my_w0 = w0;
                 my_ew = ew;
                 S.local_start[tid] = lstart + cin;
-                // WOB: (stage start, output start) of the run; its length is tailpos - stage start
-                S.gw[tid] = WOB ? make_uint2(lstart, w0) : make_uint2(w0 - lstart, ew);
+                S.gw[tid] = make_uint2(w0 - lstart, ew);
                 S.tailpos[tid] = lstart + (ew - w0);
                 for (uint32_t k = 0; k < cin; ++k) stage[lstart + k] = S.cbuf[tid][k];
                 S.wpos[tid] = ew;
@@ -966,14 +1029,6 @@ __global__ void __launch_bounds__(BLOCK, 2) k_scatter(ScatterArgs a) {
                     if (a0 + n2 < my_ew) st_stream_u2(out + (my_ew - 1), stage[lstart + (my_ew - 1 - my_w0)], wpol);
                     bulk_commit();
                 }
-            } else if (WOB) {
-                constexpr uint32_t NW = BLOCK / 32;
-                const uint32_t lane = tid & 31u;
-                for (uint32_t b = tid >> 5; b < nb; b += NW) {
-                    const uint2 wo = S.gw[b];
-                    const uint32_t len = S.tailpos[b] - wo.x;
-                    for (uint32_t k = lane; k < len; k += 32) st_stream_u2(out + wo.y + k, stage[wo.x + k], wpol);
-                }
             } else {
 #pragma unroll 4
                 for (uint32_t i = tid; i < all; i += BLOCK) {
@@ -1001,12 +1056,12 @@ size_t scatter_smem_bytes(int tile, bool hyb = false) {
            (hyb ? size_t(kHybSlots) * 6 + size_t(kHybMaxKeys) * 8 : 0);
 }
 
-template <int BLOCK, int IPT, int PASS, bool TMAST, bool HYB = false, bool WOB = false>
+template <int BLOCK, int IPT, int PASS, bool TMAST, bool HYB = false>
 int launch_scatter_pass(const Plan& p, const ScatterArgs& a, cudaStream_t s) {
     const size_t smem = scatter_smem_bytes(BLOCK * IPT, HYB);
     static std::once_flag attr_once[kMaxDevices];   // > 48 KB of dynamic shared memory: opt in once per device
     once_per_device(attr_once, [&] {
-        cudaFuncSetAttribute(k_scatter<BLOCK, IPT, PASS, TMAST, HYB, WOB>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+        cudaFuncSetAttribute(k_scatter<BLOCK, IPT, PASS, TMAST, HYB>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                              (int)smem);
     });
     static int occ_dev[kMaxDevices] = {0};   // per kernel instance and device: query once
@@ -1015,10 +1070,10 @@ int launch_scatter_pass(const Plan& p, const ScatterArgs& a, cudaStream_t s) {
     int& occ = occ_dev[dev >= 0 && dev < kMaxDevices ? dev : 0];
     if (occ < 1) {
         int o = 0;
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, k_scatter<BLOCK, IPT, PASS, TMAST, HYB, WOB>, BLOCK, smem);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, k_scatter<BLOCK, IPT, PASS, TMAST, HYB>, BLOCK, smem);
         occ = o < 1 ? 1 : o;
     }
-    k_scatter<BLOCK, IPT, PASS, TMAST, HYB, WOB><<<(unsigned)(p.num_sms * occ), BLOCK, smem, s>>>(a);
+    k_scatter<BLOCK, IPT, PASS, TMAST, HYB><<<(unsigned)(p.num_sms * occ), BLOCK, smem, s>>>(a);
     return 1;
 }
 template <int BLOCK, int IPT, bool TMAST>
@@ -1073,11 +1128,6 @@ int launch_scatter(const Plan& p, int pass, const uint32_t* const keys[2], const
     // 448 x 12 = 5376 tuples (0.976 ms; 512 x 8: 1.032, 384 x 12: 1.011, 512 x 12: 1.187).
     // Tiles need not divide a unit: a unit's ragged last tile takes the scalar path.
     if (cfg == 1) return launch_scatter_cfg<kScatterBlock, kScatterIpt, true>(p, a, s);
-    if (cfg == 2)   // write-out by bucket run (experiment)
-        return pass == 1 ? launch_scatter_pass<kScatterBlock1, kScatterIpt1, 1, false, false, true>(p, a, s)
-                         : launch_scatter_pass<kScatterBlock2, kScatterIpt, 2, false, false, true>(p, a, s);
-    if (cfg == 3)   // pass 2 only
-        if (pass == 2) return launch_scatter_pass<kScatterBlock2, kScatterIpt, 2, false, false, true>(p, a, s);
     if (pass == 1 && p.n_h0) return launch_scatter_pass<kScatterBlock1, kScatterIptHyb, 1, false, true>(p, a, s);
     return pass == 1 ? launch_scatter_pass<kScatterBlock1, kScatterIpt1, 1, false>(p, a, s)
                      : launch_scatter_pass<kScatterBlock2, kScatterIpt, 2, false>(p, a, s);

@@ -119,11 +119,17 @@ def test_hybrid_edge_cases():
     z = torch.zeros
     cases = [
         # one giant key on both sides (every sample hits it)
-        (z(30000, dtype=torch.int32), torch.arange(30000, dtype=torch.int32),
-         z(20000, dtype=torch.int32), torch.arange(20000, dtype=torch.int32)),
-        # the giant key only in S (R unique: PK-FK), all-ones key
+        (z(3000, dtype=torch.int32), torch.arange(3000, dtype=torch.int32),
+         z(2000, dtype=torch.int32), torch.arange(2000, dtype=torch.int32)),
+        # the giant key only in S (R unique: PK-FK), all-ones key (h = fmix32(~0) != the table's empty mark)
         (torch.arange(-5, 5000, dtype=torch.int32), torch.arange(5005, dtype=torch.int32),
          torch.full((50000,), -1, dtype=torch.int32), torch.arange(50000, dtype=torch.int32)),
+        # a giant key whose h = fmix32(0x331da083) = 0xffffffff, the lookup table's empty mark: never
+        # routed by the hybrid pass (detected after partitioning instead), still joined
+        (torch.cat([torch.full((4000,), 0x331da083, dtype=torch.int32), torch.arange(100, dtype=torch.int32)]),
+         torch.arange(4100, dtype=torch.int32),
+         torch.cat([torch.full((3000,), 0x331da083, dtype=torch.int32), torch.arange(50, 150, dtype=torch.int32)]),
+         torch.arange(3100, dtype=torch.int32)),
         # fewer tuples than the sample stride, empty side
         (torch.tensor([7, 7, 7], dtype=torch.int32), torch.arange(3, dtype=torch.int32),
          torch.tensor([7], dtype=torch.int32), torch.arange(1, dtype=torch.int32)),
