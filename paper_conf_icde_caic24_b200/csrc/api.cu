@@ -180,6 +180,10 @@ bool plan_build(Plan& p, uint64_t nR, uint64_t nS, const gsh_config* cfg_in, voi
                              (uint64_t(p.nu1[1]) * 256 + 4095)) / 4096 + 8;
         if (m4 > p.scan_scratch_elems) p.scan_scratch_elems = m4;
     }
+    if (p.hybrid) {   // the hybrid key-major scans (kHybMaxKeys x slices per side)
+        const uint64_t m = uint64_t(kHybMaxKeys) * (p.nu1[0] > p.nu1[1] ? p.nu1[0] : p.nu1[1]) + 1;
+        if (m / 4096 + 2 > p.scan_scratch_elems) p.scan_scratch_elems = m / 4096 + 2;
+    }
 
     Carver c{reinterpret_cast<unsigned char*>(ws)};
     const size_t F = p.F;
@@ -228,6 +232,11 @@ bool plan_build(Plan& p, uint64_t nR, uint64_t nS, const gsh_config* cfg_in, voi
     p.hyb_tab = reinterpret_cast<uint32_t*>(c.take<unsigned char>(kHybTabBytes));
     p.hyb_list = c.take<uint32_t>(kHybMaxKeys);
     p.hyb_cnt = c.take<uint32_t>(2 * kHybMaxKeys);
+    {
+        const size_t hs = p.hybrid ? (size_t(p.nu1[0]) + p.nu1[1]) * kHybMaxKeys : 0;
+        p.hyb_slice = c.take<uint32_t>(hs);
+        p.hyb_off = c.take<uint64_t>(hs + 2);
+    }
     p.bytes = c.off;
     return true;
 }
@@ -466,10 +475,9 @@ static gsh_status join_direct(const gsh_relation* R, const gsh_relation* S, gsh_
     }
     launches += launch_hist(p, R->keys, S->keys, s);
     launches += launch_hist_reduce_scan(p, s);
-    if (p.n_h0) {   // H's first entries with their exact counts; R_k / S_k offsets for pass 1
+    if (p.n_h0) {   // H's first entries with their exact counts; (key, unit) offsets for pass 1
         launches += launch_hybrid_fill(p, s);
         launches += launch_heavy_offsets(p, p.n_h0, s);
-        cudaMemsetAsync(p.h_cur, 0, size_t(2) * p.h_max * sizeof(uint32_t), s);
     }
     const int e1 = tm.mark();
     {

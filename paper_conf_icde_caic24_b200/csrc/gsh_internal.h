@@ -201,6 +201,9 @@ struct Plan {
     uint32_t* hyb_tab = nullptr;              // hybrid lookup table: u32 h [kHybSlots], u16 id [kHybSlots]
     uint32_t* hyb_list = nullptr;             // [kHybMaxKeys] h of hybrid key hid
     uint32_t* hyb_cnt = nullptr;              // [2][kHybMaxKeys] exact counts (histogram pass)
+    uint32_t* hyb_slice = nullptr;            // [nu1[0] + nu1[1]][kHybMaxKeys] counts per histogram slice
+    uint64_t* hyb_off = nullptr;              // per side [kHybMaxKeys][nu1]: pass-1 unit's write offset
+                                              // in heavy_pay (key-major scan of hyb_slice)
     size_t bytes = 0;
 };
 
@@ -226,7 +229,7 @@ int launch_heavy_offsets(const Plan& p, uint32_t n_heavy, cudaStream_t s);   // 
 // hybrid.cu: sample + select (n_h0 and hyb_tab on the device), then after the histogram pass the
 // first n_h0 entries of H with their exact counts
 int launch_hybrid_sample(const Plan& p, const uint32_t* k0, const uint32_t* k1, cudaStream_t s);
-int launch_hybrid_fill(const Plan& p, cudaStream_t s);
+int launch_hybrid_fill(const Plan& p, cudaStream_t s);   // + the per-(key, unit) offsets
 int launch_split(const Plan& p, uint32_t n_large, uint32_t gt_cap, cudaStream_t s);
 int launch_nm_setup(const Plan& p, uint32_t n_large, cudaStream_t s);
 int launch_nmjoin(const Plan& p, int materialize, uint32_t* pairs, uint64_t cap, cudaStream_t s);

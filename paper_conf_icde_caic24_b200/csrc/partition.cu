@@ -108,7 +108,7 @@ k_hist2d(const uint32_t* __restrict__ k0, uint64_t n0, const uint32_t* __restric
          uint32_t shift, uint32_t nbits, uint32_t b2, uint32_t* __restrict__ partial, uint32_t* __restrict__ c1cnt,
          uint32_t nu0, uint32_t nu1, uint32_t unit_chunks, uint32_t rshift, DevState* st,
          uint32_t* __restrict__ slice_dom, const uint32_t* __restrict__ hyb_tab, uint32_t n_h0,
-         uint32_t* __restrict__ hyb_cnt) {
+         uint32_t* __restrict__ hyb_cnt, uint32_t* __restrict__ hyb_slice) {
     __shared__ uint32_t s_hkey[HYB ? kHybSlots : 1];
     __shared__ uint16_t s_hid[HYB ? kHybSlots : 1];
     __shared__ uint32_t s_hc[HYB ? kHybMaxKeys : 1];
@@ -214,38 +214,11 @@ k_hist2d(const uint32_t* __restrict__ k0, uint64_t n0, const uint32_t* __restric
 #pragma unroll
                 for (int u = 0; u < 4; ++u) cur[u] = v[u];
                 if (c + 1 < cend && chunk_full(c + 1)) load_chunk(c + 1);
-                if constexpr (HYB) {   // all 16 first probes in flight before any is resolved
-                    uint32_t hk[16], k0[16];
 #pragma unroll
-                    for (int u = 0; u < 4; ++u) {
-                        hk[4 * u] = hash32(cur[u].x);
-                        hk[4 * u + 1] = hash32(cur[u].y);
-                        hk[4 * u + 2] = hash32(cur[u].z);
-                        hk[4 * u + 3] = hash32(cur[u].w);
-                    }
+                for (int u = 0; u < 4; ++u) {
+                    const uint32_t kk[4] = {cur[u].x, cur[u].y, cur[u].z, cur[u].w};
 #pragma unroll
-                    for (int q = 0; q < 16; ++q) k0[q] = s_hkey[hyb_slot(hk[q])];
-#pragma unroll
-                    for (int q = 0; q < 16; ++q) {
-                        if (CHECK) {
-                            const uint32_t t = hk[q] >> rshift;
-                            r_or |= t;
-                            r_nor |= ~t;
-                        }
-                        const uint32_t hid = hyb_resolve(s_hkey, s_hid, hk[q], k0[q]);
-                        hyb_rank(kFull, hid, s_hc);
-                        if (hid == kNoHeavy) {
-                            const uint32_t bin = (hk[q] >> shift) & mask;
-                            if (packed) count_exact(bin); else atomicAdd(&cnt[bin], 1u);
-                        }
-                    }
-                } else {
-#pragma unroll
-                    for (int u = 0; u < 4; ++u) {
-                        const uint32_t kk[4] = {cur[u].x, cur[u].y, cur[u].z, cur[u].w};
-#pragma unroll
-                        for (int q = 0; q < 4; ++q) count_key(kk[q]);
-                    }
+                    for (int q = 0; q < 4; ++q) count_key(kk[q]);
                 }
             } else {  // the ragged last chunk, or keys not 16-byte aligned
                 uint64_t done = cb;
@@ -264,12 +237,15 @@ k_hist2d(const uint32_t* __restrict__ k0, uint64_t n0, const uint32_t* __restric
             }
         }
         __syncthreads();
-        if (HYB)   // the slice's skewed-key counts (every slice belongs to one side)
-            for (uint32_t i = threadIdx.x; i < n_h0; i += blockDim.x)
-                if (s_hc[i]) {
-                    atomicAdd(&hyb_cnt[side * kHybMaxKeys + i], s_hc[i]);
+        if (HYB)   // the slice's skewed-key counts (every slice belongs to one side) and their totals
+            for (uint32_t i = threadIdx.x; i < n_h0; i += blockDim.x) {
+                const uint32_t c = s_hc[i];
+                hyb_slice[(size_t(side ? nu0 : 0) + sl) * kHybMaxKeys + i] = c;
+                if (c) {
+                    atomicAdd(&hyb_cnt[side * kHybMaxKeys + i], c);
                     s_hc[i] = 0;
                 }
+            }
         // flush this slice's joint counts (and their per-d1 sums) and reset
         uint32_t* row = partial + (size_t(side ? nu0 : 0) + sl) * F;
         for (uint32_t w = threadIdx.x; w < nwords; w += blockDim.x) {
@@ -343,7 +319,7 @@ int launch_hist(const Plan& p, const uint32_t* k0, const uint32_t* k1, cudaStrea
     auto go = [&](auto kern) {
         kern<<<p.hist_grid, kHistBlock, smem, s>>>(k0, p.n[0], k1, p.n[1], shift, nbits, p.b2, p.hist_partial,
                                                    p.c1cnt, p.nu1[0], p.nu1[1], p.unit_chunks, rshift, p.st,
-                                                   p.slice_dom, p.hyb_tab, p.n_h0, p.hyb_cnt);
+                                                   p.slice_dom, p.hyb_tab, p.n_h0, p.hyb_cnt, p.hyb_slice);
     };
     if (p.n_h0) {
         if (p.route_bits) go(k_hist2d<false, true, true>);
@@ -527,8 +503,7 @@ struct ScatterArgs {
     // hybrid pass 1 (HYB): sampled skewed keys' table, their count, R_k / S_k offsets, cursors, arrays
     const uint32_t* hyb_tab;
     uint32_t n_h0;
-    const uint64_t* h_off[2];
-    uint32_t* h_cur[2];
+    const uint64_t* hyb_off[2];   // per side [kHybMaxKeys][nu1]: (key, unit) write offsets
     uint32_t* heavy_pay[2];
 };
 
@@ -666,9 +641,9 @@ __device__ __forceinline__ void tile_issue(const ScatterArgs& a, int side, const
 // TMAST: whole-sector bucket runs leave the staging buffer as TMA bulk stores (one per bucket
 // and tile, issued by the bucket's thread) instead of per-tuple stores.
 // HYB (pass 1, gsh_config.hybrid -- CSH's hybrid partition, L90-L91, L100): a tuple of a sampled
-// skewed key is ranked per key in the tile (rank | 0x4000), one global atomic per (tile, key)
-// reserves its run in R_k / S_k, and its payload is stored there instead of being staged: it never
-// reaches a partition.
+// skewed key is ranked per key in the tile (rank | 0x4000), the unit's running offset of the key
+// (from the histogram pass: no atomics) places the tile's run in R_k / S_k, and its payload is
+// stored there instead of being staged: it never reaches a partition.
 template <int BLOCK, int IPT, int PASS, bool TMAST, bool HYB = false>
 __global__ void __launch_bounds__(BLOCK, 2) k_scatter(ScatterArgs a) {
     constexpr int TILE = BLOCK * IPT;
@@ -684,7 +659,8 @@ __global__ void __launch_bounds__(BLOCK, 2) k_scatter(ScatterArgs a) {
     uint32_t* hkey = reinterpret_cast<uint32_t*>(hyb0);                        // [kHybSlots]
     uint32_t* hcnt = hkey + kHybSlots;                                          // [kHybMaxKeys] tile ranks
     uint32_t* hbase = hcnt + kHybMaxKeys;                                       // [kHybMaxKeys] run starts
-    uint16_t* hid16 = reinterpret_cast<uint16_t*>(hbase + kHybMaxKeys);         // [kHybSlots]
+    uint32_t* hrun = hbase + kHybMaxKeys;                                       // [kHybMaxKeys] unit cursors
+    uint16_t* hid16 = reinterpret_cast<uint16_t*>(hrun + kHybMaxKeys);          // [kHybSlots]
     static_assert(!HYB || PASS == 1, "hybrid routing happens in pass 1");
     static_assert(!HYB || BLOCK * IPT < 0x4000, "hybrid ranks are tagged 0x4000 | rank");
 
@@ -738,6 +714,9 @@ __global__ void __launch_bounds__(BLOCK, 2) k_scatter(ScatterArgs a) {
             S.wpos[tid] = r0;
             S.carry[tid] = 0;
         }
+        if constexpr (HYB)   // the unit's offset of every skewed key (read after the first barrier)
+            for (uint32_t i = tid; i < a.n_h0; i += BLOCK)
+                hrun[i] = (uint32_t)a.hyb_off[ui.side][size_t(i) * a.nu1[ui.side] + ui.grp];
         // Dominant bucket (skewed data: one key's bucket holds >= 1/8 of the slice / pass-1
         // partition, from the histogram pass): its tuples are ranked with warp ballots and per-warp
         // register counters instead of shared-memory atomics, which serialise when most lanes of
@@ -807,38 +786,6 @@ __global__ void __launch_bounds__(BLOCK, 2) k_scatter(ScatterArgs a) {
                             return rank_of(true, (h >> dshift) & dmask);
                         }
                     };
-                    if constexpr (HYB) {   // hashes and first probes of the whole tile row, then ranks
-                        uint32_t k0[4 * NV];
-#pragma unroll
-                        for (int v = 0; v < NV; ++v) {
-                            uint4 x = reinterpret_cast<const uint4*>(ok)[v * BLOCK + tid];
-                            xb[v] = reinterpret_cast<const uint4*>(op)[v * BLOCK + tid];
-                            x.x = hash32(x.x); x.y = hash32(x.y); x.z = hash32(x.z); x.w = hash32(x.w);
-                            xa[v] = x;
-                        }
-#pragma unroll
-                        for (int v = 0; v < NV; ++v) {
-                            k0[4 * v] = hkey[hyb_slot(xa[v].x)];
-                            k0[4 * v + 1] = hkey[hyb_slot(xa[v].y)];
-                            k0[4 * v + 2] = hkey[hyb_slot(xa[v].z)];
-                            k0[4 * v + 3] = hkey[hyb_slot(xa[v].w)];
-                        }
-                        auto rank2 = [&](uint32_t h, uint32_t kz) -> uint32_t {
-                            const uint32_t hid = hyb_resolve(hkey, hid16, h, kz);
-                            const uint32_t r = rank_of(hid == kNoHeavy, (h >> dshift) & dmask);
-                            const uint32_t hr = hyb_rank(kFull, hid, hcnt);
-                            return hid == kNoHeavy ? r : (0x4000u | hr);
-                        };
-#pragma unroll
-                        for (int v = 0; v < NV; ++v) {
-                            const uint32_t r0 = rank2(xa[v].x, k0[4 * v]);
-                            const uint32_t r1 = rank2(xa[v].y, k0[4 * v + 1]);
-                            const uint32_t r2 = rank2(xa[v].z, k0[4 * v + 2]);
-                            const uint32_t r3 = rank2(xa[v].w, k0[4 * v + 3]);
-                            rk[2 * v] = r0 | (r1 << 16);
-                            rk[2 * v + 1] = r2 | (r3 << 16);
-                        }
-                    } else {
 #pragma unroll
                     for (int v = 0; v < NV; ++v) {
                         uint4 x = reinterpret_cast<const uint4*>(ok)[v * BLOCK + tid];
@@ -851,7 +798,6 @@ __global__ void __launch_bounds__(BLOCK, 2) k_scatter(ScatterArgs a) {
                         const uint32_t r3 = rank1(x.w);
                         rk[2 * v] = r0 | (r1 << 16);
                         rk[2 * v + 1] = r2 | (r3 << 16);
-                    }
                     }
                 } else {     // uint4 = 2 AoS tuples: shared slots 2u, 2u + 1 = tile elements 2u - off, ...
 #pragma unroll
@@ -919,7 +865,8 @@ __global__ void __launch_bounds__(BLOCK, 2) k_scatter(ScatterArgs a) {
                 for (uint32_t i = tid; i < a.n_h0; i += BLOCK) {
                     const uint32_t c = hcnt[i];
                     if (c) {
-                        hbase[i] = (uint32_t)a.h_off[ui.side][i] + atomicAdd(&a.h_cur[ui.side][i], c);
+                        hbase[i] = hrun[i];
+                        hrun[i] += c;
                         hcnt[i] = 0;
                     }
                 }
@@ -1053,7 +1000,7 @@ size_t scatter_smem_bytes(int tile, bool hyb = false) {
     // input tile (+4 slack) and staging = tile + up to 3 carried tuples per bucket (+ the hybrid
     // table, tile ranks and run starts)
     return ((sizeof(ScatterSmem) + 127) & ~size_t(127)) + (size_t(tile) + 4) * 8 + (size_t(tile) + 4 * 256 + 4) * 8 +
-           (hyb ? size_t(kHybSlots) * 6 + size_t(kHybMaxKeys) * 8 : 0);
+           (hyb ? size_t(kHybSlots) * 6 + size_t(kHybMaxKeys) * 12 : 0);
 }
 
 template <int BLOCK, int IPT, int PASS, bool TMAST, bool HYB = false>
@@ -1111,8 +1058,7 @@ int launch_scatter(const Plan& p, int pass, const uint32_t* const keys[2], const
     a.hyb_tab = p.hyb_tab;
     a.n_h0 = p.n_h0;
     for (int side = 0; side < 2; ++side) {
-        a.h_off[side] = p.h_off + size_t(side) * (p.h_max + 1);
-        a.h_cur[side] = p.h_cur + size_t(side) * p.h_max;
+        a.hyb_off[side] = p.hyb_off + (side ? size_t(p.nu1[0]) * kHybMaxKeys + 1 : 0);
         a.heavy_pay[side] = p.heavy_pay[side];
     }
     static int cfg = -1;
