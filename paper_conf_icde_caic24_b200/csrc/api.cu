@@ -236,6 +236,7 @@ bool plan_build(Plan& p, uint64_t nR, uint64_t nS, const gsh_config* cfg_in, voi
         const size_t hs = p.hybrid ? (size_t(p.nu1[0]) + p.nu1[1]) * kHybMaxKeys : 0;
         p.hyb_slice = c.take<uint32_t>(hs);
         p.hyb_off = c.take<uint64_t>(hs + 2);
+        p.hyb_ref = c.take<uint32_t>(p.hybrid ? size_t(p.nu1[0]) + p.nu1[1] : 0);
     }
     p.bytes = c.off;
     return true;

@@ -204,6 +204,7 @@ struct Plan {
     uint32_t* hyb_slice = nullptr;            // [nu1[0] + nu1[1]][kHybMaxKeys] counts per histogram slice
     uint64_t* hyb_off = nullptr;              // per side [kHybMaxKeys][nu1]: pass-1 unit's write offset
                                               // in heavy_pay (key-major scan of hyb_slice)
+    uint32_t* hyb_ref = nullptr;              // [nu1[0] + nu1[1]] the slice's most frequent hybrid key or ~0
     size_t bytes = 0;
 };
 

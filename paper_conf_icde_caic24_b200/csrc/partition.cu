@@ -79,23 +79,6 @@ __device__ __forceinline__ uint32_t hyb_find(const uint32_t* key, const uint16_t
     return hyb_resolve(key, id, h, key[hyb_slot(h)]);
 }
 
-// Rank / count aggregation over the lanes of `am` holding the same skewed key as the first such
-// lane (the warp's reference key): one shared atomic for all of them.  Returns the lane's rank
-// among its key's tuples (0x4000-tagged by the caller) when it is heavy.
-__device__ __forceinline__ uint32_t hyb_rank(uint32_t am, uint32_t hid, uint32_t* cnt) {
-    const bool heavy = hid != kNoHeavy;
-    const uint32_t hm = __ballot_sync(am, heavy);
-    if (!hm) return 0;
-    const uint32_t ref = __shfl_sync(am, hid, __ffs(hm) - 1);
-    const uint32_t mr = __ballot_sync(am, heavy && hid == ref);
-    const uint32_t lead = __ffs(mr) - 1;
-    uint32_t base = 0;
-    if (lane_id() == lead) base = atomicAdd(&cnt[ref], (uint32_t)__popc(mr));
-    base = __shfl_sync(am, base, lead);
-    if (!heavy) return 0;
-    return hid == ref ? base + __popc(mr & lanemask_lt()) : atomicAdd(&cnt[hid], 1u);
-}
-
 // CHECK (route_bits > 0): also verify the caller's gsh_config.route_bits assertion -- every tuple
 // shares the top route_bits of h -- by OR-ing t and ~t over all keys (t = those bits): they are all
 // equal iff (OR t) & (OR ~t) has no bit set.  The NM-join's chained table relies on it.
@@ -108,7 +91,8 @@ k_hist2d(const uint32_t* __restrict__ k0, uint64_t n0, const uint32_t* __restric
          uint32_t shift, uint32_t nbits, uint32_t b2, uint32_t* __restrict__ partial, uint32_t* __restrict__ c1cnt,
          uint32_t nu0, uint32_t nu1, uint32_t unit_chunks, uint32_t rshift, DevState* st,
          uint32_t* __restrict__ slice_dom, const uint32_t* __restrict__ hyb_tab, uint32_t n_h0,
-         uint32_t* __restrict__ hyb_cnt, uint32_t* __restrict__ hyb_slice) {
+         uint32_t* __restrict__ hyb_cnt, uint32_t* __restrict__ hyb_slice, uint32_t* __restrict__ hyb_ref) {
+    __shared__ uint32_t s_href;   // HYB: max over the slice's keys of (count << 9 | id)
     __shared__ uint32_t s_hkey[HYB ? kHybSlots : 1];
     __shared__ uint16_t s_hid[HYB ? kHybSlots : 1];
     __shared__ uint32_t s_hc[HYB ? kHybMaxKeys : 1];
@@ -118,7 +102,9 @@ k_hist2d(const uint32_t* __restrict__ k0, uint64_t n0, const uint32_t* __restric
             s_hid[i] = reinterpret_cast<const uint16_t*>(hyb_tab + kHybSlots)[i];
         }
         for (uint32_t i = threadIdx.x; i < kHybMaxKeys; i += blockDim.x) s_hc[i] = 0;
+        if (threadIdx.x == 0) s_href = 0;
     }
+    static_assert(kHybMaxKeys <= 512 && kHistMaxUnitChunks * kScatterChunk <= (1u << 22), "(count << 9 | id) fits");
     uint32_t r_or = 0, r_nor = 0;
     __shared__ uint32_t s_dom;
     extern __shared__ uint32_t cnt[];
@@ -165,8 +151,10 @@ k_hist2d(const uint32_t* __restrict__ k0, uint64_t n0, const uint32_t* __restric
                 r_nor |= ~t;
             }
             const uint32_t hid = hyb_find(s_hkey, s_hid, hk);
-            hyb_rank(__activemask(), hid, s_hc);   // counts only (the rank is not needed)
-            if (hid != kNoHeavy) return;
+            if (hid != kNoHeavy) {
+                atomicAdd(&s_hc[hid], 1u);   // no return value: warp-aggregated in hardware
+                return;
+            }
             const uint32_t bin = (hk >> shift) & mask;
             if (packed) count_exact(bin); else atomicAdd(&cnt[bin], 1u);
         } else if (FAST16) {
@@ -243,6 +231,7 @@ k_hist2d(const uint32_t* __restrict__ k0, uint64_t n0, const uint32_t* __restric
                 hyb_slice[(size_t(side ? nu0 : 0) + sl) * kHybMaxKeys + i] = c;
                 if (c) {
                     atomicAdd(&hyb_cnt[side * kHybMaxKeys + i], c);
+                    atomicMax(&s_href, c << 9 | i);
                     s_hc[i] = 0;
                 }
             }
@@ -290,6 +279,10 @@ k_hist2d(const uint32_t* __restrict__ k0, uint64_t n0, const uint32_t* __restric
         }
         __syncthreads();
         if (threadIdx.x == 0) slice_dom[(side ? nu0 : 0) + sl] = (s_dom >> 8) >= 32 ? (s_dom & 255u) : 0xffffffffu;
+        if (HYB && threadIdx.x == 0) {   // the slice's reference skewed key (pass 1 ranks it by ballot)
+            hyb_ref[(side ? nu0 : 0) + sl] = (s_href >> 9) >= 64 ? (s_href & 511u) : kNoHeavy;
+            s_href = 0;
+        }
     }
     if (CHECK) {
         r_or = __reduce_or_sync(kFull, r_or);
@@ -319,7 +312,8 @@ int launch_hist(const Plan& p, const uint32_t* k0, const uint32_t* k1, cudaStrea
     auto go = [&](auto kern) {
         kern<<<p.hist_grid, kHistBlock, smem, s>>>(k0, p.n[0], k1, p.n[1], shift, nbits, p.b2, p.hist_partial,
                                                    p.c1cnt, p.nu1[0], p.nu1[1], p.unit_chunks, rshift, p.st,
-                                                   p.slice_dom, p.hyb_tab, p.n_h0, p.hyb_cnt, p.hyb_slice);
+                                                   p.slice_dom, p.hyb_tab, p.n_h0, p.hyb_cnt, p.hyb_slice,
+                                                   p.hyb_ref);
     };
     if (p.n_h0) {
         if (p.route_bits) go(k_hist2d<false, true, true>);
@@ -504,6 +498,7 @@ struct ScatterArgs {
     const uint32_t* hyb_tab;
     uint32_t n_h0;
     const uint64_t* hyb_off[2];   // per side [kHybMaxKeys][nu1]: (key, unit) write offsets
+    const uint32_t* hyb_ref;      // per pass-1 unit: its most frequent skewed key (ballot-ranked) or ~0
     uint32_t* heavy_pay[2];
 };
 
@@ -660,9 +655,11 @@ __global__ void __launch_bounds__(BLOCK, 2) k_scatter(ScatterArgs a) {
     uint32_t* hcnt = hkey + kHybSlots;                                          // [kHybMaxKeys] tile ranks
     uint32_t* hbase = hcnt + kHybMaxKeys;                                       // [kHybMaxKeys] run starts
     uint32_t* hrun = hbase + kHybMaxKeys;                                       // [kHybMaxKeys] unit cursors
-    uint16_t* hid16 = reinterpret_cast<uint16_t*>(hrun + kHybMaxKeys);          // [kHybSlots]
+    uint32_t* hwref = hrun + kHybMaxKeys;                                       // [32] per warp: ref-key tuples
+    uint32_t* hwoff = hwref + 32;                                               // [32] their prefix over warps
+    uint16_t* hid16 = reinterpret_cast<uint16_t*>(hwoff + 32);                  // [kHybSlots]
     static_assert(!HYB || PASS == 1, "hybrid routing happens in pass 1");
-    static_assert(!HYB || BLOCK * IPT < 0x4000, "hybrid ranks are tagged 0x4000 | rank");
+    static_assert(!HYB || BLOCK * IPT < 0x2000, "hybrid ranks are tagged 0x4000 | [0x2000 ref |] rank");
 
     const uint32_t tid = threadIdx.x;
     constexpr bool p1 = (PASS == 1);
@@ -717,6 +714,7 @@ __global__ void __launch_bounds__(BLOCK, 2) k_scatter(ScatterArgs a) {
         if constexpr (HYB)   // the unit's offset of every skewed key (read after the first barrier)
             for (uint32_t i = tid; i < a.n_h0; i += BLOCK)
                 hrun[i] = (uint32_t)a.hyb_off[ui.side][size_t(i) * a.nu1[ui.side] + ui.grp];
+        const uint32_t href = HYB ? a.hyb_ref[u] : kNoHeavy;   // pass 1: u indexes the slices
         // Dominant bucket (skewed data: one key's bucket holds >= 1/8 of the slice / pass-1
         // partition, from the histogram pass): its tuples are ranked with warp ballots and per-warp
         // register counters instead of shared-memory atomics, which serialise when most lanes of
@@ -753,6 +751,7 @@ __global__ void __launch_bounds__(BLOCK, 2) k_scatter(ScatterArgs a) {
             par ^= 1;
             uint32_t rk[IPT / 2];  // ranks, packed 2 x u16 (bit 15: dominant-bucket rank; 0xffff: masked)
             uint32_t wrun = 0;     // this warp's dominant-bucket tuples so far in this tile
+            uint32_t wref = 0;     // HYB: this warp's tuples of the unit's reference skewed key
             // rank of one tuple of bucket b: dominant bucket by ballot, others by shared atomics
             // full tile: the input stays in registers from the ranking to the staging step, so
             // the input buffer is free (and the next tile's TMA issued) after the first barrier
@@ -778,9 +777,16 @@ __global__ void __launch_bounds__(BLOCK, 2) k_scatter(ScatterArgs a) {
                     // a sampled skewed key's tuple: ranked among its key's tuples in the tile
                     auto rank1 = [&](uint32_t h) -> uint32_t {
                         if constexpr (HYB) {
+                            // the reference key by ballot (0x2000 | rank in the warp's run), other
+                            // skewed keys by shared atomics
                             const uint32_t hid = hyb_find(hkey, hid16, h);
                             const uint32_t r = rank_of(hid == kNoHeavy, (h >> dshift) & dmask);
-                            const uint32_t hr = hyb_rank(kFull, hid, hcnt);
+                            const bool isref = hid != kNoHeavy && hid == href;
+                            const uint32_t m = __ballot_sync(kFull, isref);
+                            uint32_t hr = 0;
+                            if (isref) hr = 0x2000u | (wref + __popc(m & lanemask_lt()));
+                            else if (hid != kNoHeavy) hr = atomicAdd(&hcnt[hid], 1u);
+                            wref += __popc(m);
                             return hid == kNoHeavy ? r : (0x4000u | hr);
                         } else {
                             return rank_of(true, (h >> dshift) & dmask);
@@ -852,6 +858,7 @@ __global__ void __launch_bounds__(BLOCK, 2) k_scatter(ScatterArgs a) {
                 }
             }
             if ((tid & 31) == 0) S.wdom[tid >> 5] = wrun;
+            if (HYB && (tid & 31) == 0) hwref[tid >> 5] = wref;
             // the previous tile's bulk stores must have read the staging buffer before any thread
             // writes it again (after the barrier below)
             if (TMAST && tid < nb) bulk_wait_read0();
@@ -861,13 +868,30 @@ __global__ void __launch_bounds__(BLOCK, 2) k_scatter(ScatterArgs a) {
             // Write combining: bucket b's staged run = [carry from the previous tile | this tile's
             // tuples]; only whole 32-byte sectors are written, the < 4-tuple remainder carries
             // over (the unit's last tile flushes everything).  u32 offsets (n < 2^32).
-            if constexpr (HYB) {   // reserve this tile's run of every skewed key it holds
+            if constexpr (HYB) {   // place this tile's run of every skewed key it holds
                 for (uint32_t i = tid; i < a.n_h0; i += BLOCK) {
                     const uint32_t c = hcnt[i];
-                    if (c) {
+                    if (c && i != href) {
                         hbase[i] = hrun[i];
                         hrun[i] += c;
                         hcnt[i] = 0;
+                    }
+                }
+                if (href != kNoHeavy && tid < 32) {   // the reference key: ballot ranks (full tiles)
+                    constexpr uint32_t NW = BLOCK / 32;   // + atomic ranks (ragged tiles), never both
+                    const uint32_t c = tid < NW ? hwref[tid] : 0u;
+                    uint32_t x = c;
+#pragma unroll
+                    for (int o = 1; o < 32; o <<= 1) {
+                        const uint32_t y = __shfl_up_sync(kFull, x, o);
+                        if (tid >= (uint32_t)o) x += y;
+                    }
+                    if (tid < NW) hwoff[tid] = x - c;
+                    const uint32_t tot = __shfl_sync(kFull, x, 31) + hcnt[href];
+                    if (tid == 0) {
+                        hbase[href] = hrun[href];
+                        hrun[href] += tot;
+                        hcnt[href] = 0;
                     }
                 }
             }
@@ -920,9 +944,11 @@ __global__ void __launch_bounds__(BLOCK, 2) k_scatter(ScatterArgs a) {
                 if (p1) {
                     // staged, or (hybrid: rank tagged 0x4000, dominant bit clear) stored into R_k / S_k
                     auto put = [&](uint32_t h, uint32_t pay, uint32_t r) {
-                        if (HYB && (r & 0xc000u) == 0x4000u)
-                            a.heavy_pay[ui.side][hbase[hyb_find(hkey, hid16, h)] + (r & 0x3fffu)] = pay;
-                        else
+                        if (HYB && (r & 0xc000u) == 0x4000u) {
+                            const uint32_t pos = (r & 0x2000u) ? hbase[href] + hwoff[tid >> 5] + (r & 0x1fffu)
+                                                               : hbase[hyb_find(hkey, hid16, h)] + (r & 0x1fffu);
+                            a.heavy_pay[ui.side][pos] = pay;
+                        } else
                             stage[spos((h >> dshift) & dmask, r)] = make_uint2(h, pay);
                     };
 #pragma unroll
@@ -950,7 +976,7 @@ __global__ void __launch_bounds__(BLOCK, 2) k_scatter(ScatterArgs a) {
                         const uint2 e = p1 ? make_uint2(ok[i], op[i]) : o2[i + lp.shift];
                         const uint32_t r = (jj & 1) ? (rk[jj >> 1] >> 16) : (rk[jj >> 1] & 0xffffu);
                         if (HYB && (r & 0xc000u) == 0x4000u)
-                            a.heavy_pay[ui.side][hbase[hyb_find(hkey, hid16, e.x)] + (r & 0x3fffu)] = e.y;
+                            a.heavy_pay[ui.side][hbase[hyb_find(hkey, hid16, e.x)] + (r & 0x1fffu)] = e.y;
                         else
                             stage[S.local_start[(e.x >> dshift) & dmask] + r] = e;
                     }
@@ -1000,7 +1026,7 @@ size_t scatter_smem_bytes(int tile, bool hyb = false) {
     // input tile (+4 slack) and staging = tile + up to 3 carried tuples per bucket (+ the hybrid
     // table, tile ranks and run starts)
     return ((sizeof(ScatterSmem) + 127) & ~size_t(127)) + (size_t(tile) + 4) * 8 + (size_t(tile) + 4 * 256 + 4) * 8 +
-           (hyb ? size_t(kHybSlots) * 6 + size_t(kHybMaxKeys) * 12 : 0);
+           (hyb ? size_t(kHybSlots) * 6 + size_t(kHybMaxKeys) * 12 + 64 * 4 : 0);
 }
 
 template <int BLOCK, int IPT, int PASS, bool TMAST, bool HYB = false>
@@ -1056,6 +1082,7 @@ int launch_scatter(const Plan& p, int pass, const uint32_t* const keys[2], const
     a.route_bits = p.route_bits;
     a.unit_ctr = &p.st->claim[pass - 1];
     a.hyb_tab = p.hyb_tab;
+    a.hyb_ref = p.hyb_ref;
     a.n_h0 = p.n_h0;
     for (int side = 0; side < 2; ++side) {
         a.hyb_off[side] = p.hyb_off + (side ? size_t(p.nu1[0]) * kHybMaxKeys + 1 : 0);
