@@ -3,6 +3,7 @@
 // Nothing here is shared with oracle/ (the oracle carries its own hashes).
 #pragma once
 #include <cstdint>
+#include <cstdio>
 #include <cuda_runtime.h>
 
 namespace gsh {
@@ -12,6 +13,24 @@ __host__ __device__ __forceinline__ uint32_t umin32(uint32_t a, uint32_t b) { re
 __host__ __device__ __forceinline__ uint32_t umax32(uint32_t a, uint32_t b) { return a > b ? a : b; }
 
 constexpr uint32_t kFull = 0xffffffffu;
+
+// Bounds checks of computed indices, compiled in only for the checking build
+// (scripts/build_variant.sh bounds "-DGSH_CHECK_BOUNDS"; compute-sanitizer is not available on the
+// GPU pool): a violation prints its site and traps, so the calling test fails with a CUDA error.
+#ifdef GSH_CHECK_BOUNDS
+#define GSH_BOUNDS(cond, what)                                                                       \
+    do {                                                                                             \
+        if (!(cond)) {                                                                               \
+            printf("GSH_BOUNDS violated: %s (%s:%d) block %d thread %d\n", what, __FILE__, __LINE__,  \
+                   (int)blockIdx.x, (int)threadIdx.x);                                              \
+            __trap();                                                                                \
+        }                                                                                            \
+    } while (0)
+#else
+#define GSH_BOUNDS(cond, what) \
+    do {                       \
+    } while (0)
+#endif
 
 // h = fmix32(key): the MurmurHash3 32-bit finalizer, a bijection on u32, so equality of h
 // is equality of keys.  Partition digits are taken from h, most significant bits first

@@ -712,8 +712,10 @@ __global__ void __launch_bounds__(BLOCK, 2) k_scatter(ScatterArgs a) {
             S.carry[tid] = 0;
         }
         if constexpr (HYB)   // the unit's offset of every skewed key (read after the first barrier)
-            for (uint32_t i = tid; i < a.n_h0; i += BLOCK)
+            for (uint32_t i = tid; i < a.n_h0; i += BLOCK) {
+                GSH_BOUNDS(ui.grp < a.nu1[ui.side], "hybrid pass 1: unit index");
                 hrun[i] = (uint32_t)a.hyb_off[ui.side][size_t(i) * a.nu1[ui.side] + ui.grp];
+            }
         const uint32_t href = HYB ? a.hyb_ref[u] : kNoHeavy;   // pass 1: u indexes the slices
         // Dominant bucket (skewed data: one key's bucket holds >= 1/8 of the slice / pass-1
         // partition, from the histogram pass): its tuples are ranked with warp ballots and per-warp
@@ -947,6 +949,7 @@ __global__ void __launch_bounds__(BLOCK, 2) k_scatter(ScatterArgs a) {
                         if (HYB && (r & 0xc000u) == 0x4000u) {
                             const uint32_t pos = (r & 0x2000u) ? hbase[href] + hwoff[tid >> 5] + (r & 0x1fffu)
                                                                : hbase[hyb_find(hkey, hid16, h)] + (r & 0x1fffu);
+                            GSH_BOUNDS(pos < a.n[ui.side], "hybrid pass 1: skewed payload position");
                             a.heavy_pay[ui.side][pos] = pay;
                         } else
                             stage[spos((h >> dshift) & dmask, r)] = make_uint2(h, pay);
@@ -975,8 +978,11 @@ __global__ void __launch_bounds__(BLOCK, 2) k_scatter(ScatterArgs a) {
                     if (i < ql) {
                         const uint2 e = p1 ? make_uint2(ok[i], op[i]) : o2[i + lp.shift];
                         const uint32_t r = (jj & 1) ? (rk[jj >> 1] >> 16) : (rk[jj >> 1] & 0xffffu);
-                        if (HYB && (r & 0xc000u) == 0x4000u)
-                            a.heavy_pay[ui.side][hbase[hyb_find(hkey, hid16, e.x)] + (r & 0x1fffu)] = e.y;
+                        if (HYB && (r & 0xc000u) == 0x4000u) {
+                            const uint32_t pos = hbase[hyb_find(hkey, hid16, e.x)] + (r & 0x1fffu);
+                            GSH_BOUNDS(pos < a.n[ui.side], "hybrid pass 1 (ragged tile): skewed payload position");
+                            a.heavy_pay[ui.side][pos] = e.y;
+                        }
                         else
                             stage[S.local_start[(e.x >> dshift) & dmask] + r] = e;
                     }
@@ -1008,6 +1014,7 @@ __global__ void __launch_bounds__(BLOCK, 2) k_scatter(ScatterArgs a) {
                     const uint2 e = stage[i];
                     const uint2 ge = S.gw[(e.x >> dshift) & dmask];
                     const uint32_t g = ge.x + i;
+                    GSH_BOUNDS(g >= ge.y || g < a.n[ui.side], "scatter: output position");
                     if (g < ge.y) st_stream_u2(out + g, e, wpol);
                 }
             }
