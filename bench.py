@@ -625,7 +625,22 @@ def main():
         assert rr.count == r.count and rr.checksum == r.checksum
         e2e = {"value": 2 * n * world * ke / (ems / 1e3), "unit": "input tuples/s", "h2d_bytes_per_step": 16 * n,
                "d2h_bytes_per_step": d2h, "steps": ke, "ms_per_step": ems / ke, "api": api}
-        del hk
+        # the bound of this number: the same bytes as plain pinned-memory H2D copies (PCIe), timed alike
+        dst = [torch.empty_like(h, device=dev) for h in hk]
+        for _ in range(2):
+            for dd, hh in zip(dst, hk):
+                dd.copy_(hh, non_blocking=True)
+        torch.cuda.synchronize()
+        h0.record(stream)
+        for _ in range(ke):
+            for dd, hh in zip(dst, hk):
+                dd.copy_(hh, non_blocking=True)
+        h1.record(stream)
+        torch.cuda.synchronize()
+        cms = h0.elapsed_time(h1) / ke
+        e2e["h2d_copy"] = {"ms_per_step": cms, "gbs": 16 * n / (cms * 1e6),
+                           "e2e_frac": cms / (ems / ke)}   # share of the e2e step that is the bare copy
+        del hk, dst
 
     sweep = None
     if not multi and not args.no_sweep and args.workload == "cfg2" and args.mode == "count":

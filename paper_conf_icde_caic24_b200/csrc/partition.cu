@@ -127,20 +127,47 @@ k_hist2d(const uint32_t* __restrict__ k0, uint64_t n0, const uint32_t* __restric
             ev_delta[e] = d;
         }
     };
+    // inc = 1 << (16 * (bin & 1)) and m = its half's mask, without variable shifts (the
+    // histogram is ALU-bound): a wrap is old's half == 0xffff, i.e. (~old & m) == 0
+    auto wrap_events = [&](uint32_t bin, uint32_t old) {   // rare: a u16 wrapped
+        const uint32_t s16 = (bin & 1u) << 4;
+        event(bin, 65536);
+        if (s16 == 0) {
+            event(bin | 1u, -1);
+            if ((old >> 16) == 0xffffu) event(bin | 1u, 65536);
+        }
+    };
     auto count_exact = [&](uint32_t bin) {
-        // inc = 1 << (16 * (bin & 1)) and m = its half's mask, without variable shifts (the
-        // histogram is ALU-bound): a wrap is old's half == 0xffff, i.e. (~old & m) == 0
         const uint32_t inc = umax32((bin & 1u) << 16, 1u);
         const uint32_t m = inc * 0xffffu;
         const uint32_t old = atomicAdd(&cnt[bin >> 1], inc);
-        if (__builtin_expect((~old & m) == 0, 0)) {  // a u16 wrapped
-            const uint32_t s16 = (bin & 1u) << 4;
-            event(bin, 65536);
-            if (s16 == 0) {
-                event(bin | 1u, -1);
-                if ((old >> 16) == 0xffffu) event(bin | 1u, 65536);
-            }
+        if (__builtin_expect((~old & m) == 0, 0)) wrap_events(bin, old);
+    };
+    // Packed counters, a batch of keys: every atomic is issued before any returned value is
+    // tested, so their shared-memory round trips overlap (one per key otherwise: the wrap test
+    // of key i would hold back the atomic of key i + 1).
+    auto count_exact_batch = [&](const uint32_t (&bins)[8]) {
+        uint32_t old[8];
+#pragma unroll
+        for (int q = 0; q < 8; ++q) old[q] = atomicAdd(&cnt[bins[q] >> 1], umax32((bins[q] & 1u) << 16, 1u));
+        auto rest = [&](int q) { return ~old[q] & (umax32((bins[q] & 1u) << 16, 1u) * 0xffffu); };   // 0: wrapped
+        uint32_t mn = rest(0);
+#pragma unroll
+        for (int q = 1; q < 8; ++q) mn = umin32(mn, rest(q));
+        if (__builtin_expect(mn == 0, 0))
+#pragma unroll
+            for (int q = 0; q < 8; ++q)
+                if (rest(q) == 0) wrap_events(bins[q], old[q]);
+    };
+    auto bin_of = [&](uint32_t key) -> uint32_t {
+        if (FAST16) return hash32_top(key) >> 16;
+        const uint32_t hk = top16 ? hash32_top(key) : hash32(key);
+        if (CHECK) {
+            const uint32_t t = hk >> rshift;
+            r_or |= t;
+            r_nor |= ~t;
         }
+        return (hk >> shift) & mask;
     };
     auto count_key = [&](uint32_t key) {
         if (HYB) {
@@ -202,11 +229,22 @@ k_hist2d(const uint32_t* __restrict__ k0, uint64_t n0, const uint32_t* __restric
 #pragma unroll
                 for (int u = 0; u < 4; ++u) cur[u] = v[u];
                 if (c + 1 < cend && chunk_full(c + 1)) load_chunk(c + 1);
+                if (!HYB && packed) {
 #pragma unroll
-                for (int u = 0; u < 4; ++u) {
-                    const uint32_t kk[4] = {cur[u].x, cur[u].y, cur[u].z, cur[u].w};
+                    for (int h2 = 0; h2 < 2; ++h2) {
+                        const uint32_t bins[8] = {bin_of(cur[2 * h2].x), bin_of(cur[2 * h2].y),
+                                                  bin_of(cur[2 * h2].z), bin_of(cur[2 * h2].w),
+                                                  bin_of(cur[2 * h2 + 1].x), bin_of(cur[2 * h2 + 1].y),
+                                                  bin_of(cur[2 * h2 + 1].z), bin_of(cur[2 * h2 + 1].w)};
+                        count_exact_batch(bins);
+                    }
+                } else {
 #pragma unroll
-                    for (int q = 0; q < 4; ++q) count_key(kk[q]);
+                    for (int u = 0; u < 4; ++u) {
+                        const uint32_t kk[4] = {cur[u].x, cur[u].y, cur[u].z, cur[u].w};
+#pragma unroll
+                        for (int q = 0; q < 4; ++q) count_key(kk[q]);
+                    }
                 }
             } else {  // the ragged last chunk, or keys not 16-byte aligned
                 uint64_t done = cb;
