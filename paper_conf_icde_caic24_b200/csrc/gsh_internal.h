@@ -32,6 +32,10 @@ constexpr int kScatterChunk = 16384;               // keys: the histogram's load
 #define GSH_SCATTER_BLOCK1 256
 #endif
 constexpr int kScatterBlock1 = GSH_SCATTER_BLOCK1;  // pass 1: threads per CTA
+#ifndef GSH_SCATTER_MINB
+#define GSH_SCATTER_MINB 2
+#endif
+constexpr int kScatterMinBlocks = GSH_SCATTER_MINB;  // resident scatter CTAs per SM the register budget targets
 static_assert(kScatterIpt1 % 4 == 0 && kScatterIpt % 2 == 0, "vector tile loads: uint4 = 4 keys / 2 tuples");
 static_assert(kScatterBlock1 >= 256 && kScatterBlock2 >= 256 && kScatterBlock >= 256,
               "scatter CTAs keep one thread per bucket (2^kMaxDigitBits = 256)");

@@ -678,7 +678,7 @@ __device__ __forceinline__ void tile_issue(const ScatterArgs& a, int side, const
 // (from the histogram pass: no atomics) places the tile's run in R_k / S_k, and its payload is
 // stored there instead of being staged: it never reaches a partition.
 template <int BLOCK, int IPT, int PASS, bool TMAST, bool HYB = false>
-__global__ void __launch_bounds__(BLOCK, 2) k_scatter(ScatterArgs a) {
+__global__ void __launch_bounds__(BLOCK, kScatterMinBlocks) k_scatter(ScatterArgs a) {
     constexpr int TILE = BLOCK * IPT;
     static_assert(TILE < 0x7fff, "ranks are packed as u16: bit 15 = dominant bucket, 0xffff = masked");
     extern __shared__ __align__(128) unsigned char smem_raw[];
