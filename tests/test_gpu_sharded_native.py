@@ -227,3 +227,19 @@ def test_native_two_processes_gloo_ipc():
     on, oc, _ = oracle.join(*(t.numpy().view(np.uint32) for t in full))
     for _, res in out:
         assert res == [(on, oc)] * 3
+
+
+@pytest.mark.parametrize("exchange", ["a2a", "p2p"])
+@pytest.mark.parametrize("world,theta", [(2, 1.0), (4, 1.5)])
+def test_native_with_hybrid_local_joins(world, theta, exchange):
+    """gsh_config.hybrid reaches the ranks' local joins (the routed normal shard keeps route_bits =
+    log2 G): the global result is unchanged."""
+    from paper_conf_icde_caic24_b200 import make_config, sharded
+    dev = torch.device("cuda", 0)
+    full = datagen.make_workload("zipf", 1 << 18, theta, seed=31)
+    on, oc, _ = oracle.join(*(t.numpy().view(np.uint32) for t in full))
+    shards = [tuple(_shard(t, g, world).to(dev) for t in full) for g in range(world)]
+    res = sharded.run_local_native(world, shards, config=make_config(hybrid=True, hybrid_stride=10),
+                                   exchange=exchange)
+    for r in res:
+        assert (r.count, r.checksum) == (on, oc), (r.stats, on, oc)
