@@ -78,6 +78,17 @@ __device__ __forceinline__ uint32_t hyb_resolve(const uint32_t* key, const uint1
 __device__ __forceinline__ uint32_t hyb_find(const uint32_t* key, const uint16_t* id, uint32_t h) {
     return hyb_resolve(key, id, h, key[hyb_slot(h)]);
 }
+// Both first slots loaded unconditionally, resolved with selects; the probe loop runs only when
+// both hold other keys (rare at load <= 1/4), so the common case has no divergent path.
+__device__ __forceinline__ uint32_t hyb_find2(const uint32_t* key, const uint16_t* id, uint32_t h) {
+    const uint32_t s0 = hyb_slot(h), s1 = (s0 + 1) & (kHybSlots - 1);
+    const uint32_t ka = key[s0], kb = key[s1];
+    if (h == kHybEmpty || ka == kHybEmpty) return kNoHeavy;
+    if (ka == h) return id[s0];
+    if (kb == h) return id[s1];
+    if (kb == kHybEmpty) return kNoHeavy;
+    return hyb_find(key, id, h);
+}
 
 // CHECK (route_bits > 0): also verify the caller's gsh_config.route_bits assertion -- every tuple
 // shares the top route_bits of h -- by OR-ing t and ~t over all keys (t = those bits): they are all
@@ -229,7 +240,62 @@ k_hist2d(const uint32_t* __restrict__ k0, uint64_t n0, const uint32_t* __restric
 #pragma unroll
                 for (int u = 0; u < 4; ++u) cur[u] = v[u];
                 if (c + 1 < cend && chunk_full(c + 1)) load_chunk(c + 1);
-                if (!HYB && packed) {
+                if (HYB && packed) {
+                    // four keys at a time, no divergent path in the common case: both first probe
+                    // slots of every key loaded up front (load <= 1/4: a third is rarely needed),
+                    // then predicated atomics -- the bin counter of a normal key, the per-key
+                    // counter of a sampled skewed one -- and one batched wrap test
+#pragma unroll
+                    for (int u = 0; u < 4; ++u) {
+                        const uint32_t kk[4] = {cur[u].x, cur[u].y, cur[u].z, cur[u].w};
+                        uint32_t hk[4], ka[4], kb[4], hid[4];
+#pragma unroll
+                        for (int q = 0; q < 4; ++q) {
+                            hk[q] = hash32(kk[q]);
+                            if (CHECK) {
+                                const uint32_t t = hk[q] >> rshift;
+                                r_or |= t;
+                                r_nor |= ~t;
+                            }
+                            const uint32_t s0 = hyb_slot(hk[q]);
+                            ka[q] = s_hkey[s0];
+                            kb[q] = s_hkey[(s0 + 1) & (kHybSlots - 1)];
+                        }
+#pragma unroll
+                        for (int q = 0; q < 4; ++q) {
+                            const uint32_t s0 = hyb_slot(hk[q]);
+                            uint32_t id = kNoHeavy;
+                            if (hk[q] != kHybEmpty && ka[q] != kHybEmpty) {
+                                if (ka[q] == hk[q]) id = s_hid[s0];
+                                else if (kb[q] == hk[q]) id = s_hid[(s0 + 1) & (kHybSlots - 1)];
+                                else if (kb[q] != kHybEmpty) id = hyb_find(s_hkey, s_hid, hk[q]);   // rare
+                            }
+                            hid[q] = id;
+                        }
+                        uint32_t old[4], rest = 0xffffffffu;
+#pragma unroll
+                        for (int q = 0; q < 4; ++q) {
+                            const uint32_t bin = (hk[q] >> shift) & mask;
+                            const uint32_t inc = umax32((bin & 1u) << 16, 1u);
+                            old[q] = 0;
+                            if (hid[q] == kNoHeavy) old[q] = atomicAdd(&cnt[bin >> 1], inc);
+                            else atomicAdd(&s_hc[hid[q]], 1u);
+                        }
+#pragma unroll
+                        for (int q = 0; q < 4; ++q) {
+                            const uint32_t bin = (hk[q] >> shift) & mask;
+                            const uint32_t m = umax32((bin & 1u) << 16, 1u) * 0xffffu;
+                            rest = umin32(rest, hid[q] == kNoHeavy ? (~old[q] & m) : 1u);
+                        }
+                        if (__builtin_expect(rest == 0, 0))
+#pragma unroll
+                            for (int q = 0; q < 4; ++q) {
+                                const uint32_t bin = (hk[q] >> shift) & mask;
+                                const uint32_t m = umax32((bin & 1u) << 16, 1u) * 0xffffu;
+                                if (hid[q] == kNoHeavy && (~old[q] & m) == 0) wrap_events(bin, old[q]);
+                            }
+                    }
+                } else if (!HYB && packed) {
 #pragma unroll
                     for (int h2 = 0; h2 < 2; ++h2) {
                         const uint32_t bins[8] = {bin_of(cur[2 * h2].x), bin_of(cur[2 * h2].y),
@@ -819,7 +885,7 @@ __global__ void __launch_bounds__(BLOCK, kScatterMinBlocks) k_scatter(ScatterArg
                         if constexpr (HYB) {
                             // the reference key by ballot (0x2000 | rank in the warp's run), other
                             // skewed keys by shared atomics
-                            const uint32_t hid = hyb_find(hkey, hid16, h);
+                            const uint32_t hid = hyb_find2(hkey, hid16, h);
                             const uint32_t r = rank_of(hid == kNoHeavy, (h >> dshift) & dmask);
                             const bool isref = hid != kNoHeavy && hid == href;
                             const uint32_t m = __ballot_sync(kFull, isref);
@@ -890,7 +956,7 @@ __global__ void __launch_bounds__(BLOCK, kScatterMinBlocks) k_scatter(ScatterArg
                             }
                         }
                         uint32_t hid = kNoHeavy;
-                        if constexpr (HYB) hid = hyb_find(hkey, hid16, h);
+                        if constexpr (HYB) hid = hyb_find2(hkey, hid16, h);
                         r = hid == kNoHeavy ? atomicAdd(&S.tcnt[(h >> dshift) & dmask], 1u)
                                             : (0x4000u | atomicAdd(&hcnt[hid], 1u));
                     }
@@ -986,7 +1052,7 @@ __global__ void __launch_bounds__(BLOCK, kScatterMinBlocks) k_scatter(ScatterArg
                     auto put = [&](uint32_t h, uint32_t pay, uint32_t r) {
                         if (HYB && (r & 0xc000u) == 0x4000u) {
                             const uint32_t pos = (r & 0x2000u) ? hbase[href] + hwoff[tid >> 5] + (r & 0x1fffu)
-                                                               : hbase[hyb_find(hkey, hid16, h)] + (r & 0x1fffu);
+                                                               : hbase[hyb_find2(hkey, hid16, h)] + (r & 0x1fffu);
                             GSH_BOUNDS(pos < a.n[ui.side], "hybrid pass 1: skewed payload position");
                             a.heavy_pay[ui.side][pos] = pay;
                         } else
@@ -1017,7 +1083,7 @@ __global__ void __launch_bounds__(BLOCK, kScatterMinBlocks) k_scatter(ScatterArg
                         const uint2 e = p1 ? make_uint2(ok[i], op[i]) : o2[i + lp.shift];
                         const uint32_t r = (jj & 1) ? (rk[jj >> 1] >> 16) : (rk[jj >> 1] & 0xffffu);
                         if (HYB && (r & 0xc000u) == 0x4000u) {
-                            const uint32_t pos = hbase[hyb_find(hkey, hid16, e.x)] + (r & 0x1fffu);
+                            const uint32_t pos = hbase[hyb_find2(hkey, hid16, e.x)] + (r & 0x1fffu);
                             GSH_BOUNDS(pos < a.n[ui.side], "hybrid pass 1 (ragged tile): skewed payload position");
                             a.heavy_pay[ui.side][pos] = e.y;
                         }
