@@ -199,14 +199,20 @@ GSH_API gsh_status gsh_join(const gsh_relation *R, const gsh_relation *S, gsh_ou
 /*
  * gsh_join_gbase -- the paper's GPU comparison system "Gbase" (§II-B, §III
  * L78-L80), re-implemented on this GPU for the GSH-vs-Gbase measurement
- * (Table I): no skew detection; after the same two partition passes, one thread block
- * per (partition, R sub-list of <= 4096 tuples) builds a chained shared-memory table and probes it
- * with the FULL S partition (L71-L72's sub lists), all threads advancing one chain element per
- * round with a write bitmap and a block barrier per round (L79-L80).  Arguments, workspace
- * (gsh_workspace_bytes), errors and result semantics as gsh_join: identical count, checksum and
- * pair multiset.  res: ms_hist / ms_pass1 / ms_pass2 = the partition phase, ms_nmjoin = the Gbase
- * join phase, ms_total; skew fields 0.  At most 2^28 tuples per side (GSH_ERR_INVALID beyond).
+ * (Table I), with no skew detection:
+ *   partition: two passes into bucket-chained partitions (2048-tuple buckets allocated from a pool
+ *   as partitions fill, linked per partition; tiles of 4 tuples per thread reordered in shared
+ *   memory and written as coalesced runs, L70) -- GSH's fanout (R7);
+ *   join: one thread block per (partition, R sub-list of two buckets) builds a chained
+ *   shared-memory table and probes it with ALL of S's buckets of that partition (L71-L72), every
+ *   thread advancing one chain element per round with a write bitmap and a block barrier per round
+ *   (L79-L80).
+ * Arguments, errors and result semantics as gsh_join (identical count, checksum and pair multiset);
+ * the workspace is gsh_gbase_workspace_bytes (bucket pools: ~4x gsh_join's at 2^27 per side).
+ * res: ms_pass1 / ms_pass2 = the partition passes, ms_nmjoin = the join phase, ms_total; skew
+ * fields 0.  At most 2^28 tuples per side (GSH_ERR_INVALID beyond).
  */
+GSH_API size_t gsh_gbase_workspace_bytes(uint64_t n_r, uint64_t n_s, const gsh_config *cfg);   /* 0: invalid */
 GSH_API gsh_status gsh_join_gbase(const gsh_relation *R, const gsh_relation *S, gsh_out_mode mode,
                                   const gsh_output *out, void *workspace, size_t workspace_bytes,
                                   const gsh_config *cfg, void *stream, gsh_result *res);

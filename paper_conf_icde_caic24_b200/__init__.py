@@ -2,6 +2,7 @@
 
 Public API (all GPU work runs in libgsh.so, include/gsh.h):
   join(...)            device-resident equi-join -> count, checksum, optional pairs
+                       (impl="gbase": the paper's skew-unaware comparison system, same result)
   join_host(...)       end-to-end variant over host tensors
   make_config(...)     tuning / test hooks
   hash_keys, radix_histogram, partition, detect   -- single phases (parity tests)
@@ -12,6 +13,7 @@ from .join import (  # noqa: F401
     JoinResult,
     Workspace,
     detect,
+    gbase_workspace_bytes,
     hash_keys,
     join,
     join_detail,

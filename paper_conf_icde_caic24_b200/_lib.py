@@ -150,6 +150,7 @@ _PROTOS = [
     ("gsh_join", ctypes.c_int, [ctypes.POINTER(GshRelation), ctypes.POINTER(GshRelation), ctypes.c_int,
                                 ctypes.POINTER(GshOutput), vp, ctypes.c_size_t, ctypes.POINTER(GshConfig), vp,
                                 ctypes.POINTER(GshResult)]),
+    ("gsh_gbase_workspace_bytes", ctypes.c_size_t, [u64, u64, ctypes.POINTER(GshConfig)]),
     ("gsh_join_gbase", ctypes.c_int, [ctypes.POINTER(GshRelation), ctypes.POINTER(GshRelation), ctypes.c_int,
                                       ctypes.POINTER(GshOutput), vp, ctypes.c_size_t, ctypes.POINTER(GshConfig), vp,
                                       ctypes.POINTER(GshResult)]),

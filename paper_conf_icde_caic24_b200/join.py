@@ -128,6 +128,14 @@ def workspace_bytes(n_r: int, n_s: int, config: GshConfig | None = None) -> int:
     return int(nb)
 
 
+def gbase_workspace_bytes(n_r: int, n_s: int, config: GshConfig | None = None) -> int:
+    """Device workspace of the Gbase-style join (gsh_gbase_workspace_bytes: its bucket pools)."""
+    nb = load().gsh_gbase_workspace_bytes(n_r, n_s, ctypes.byref(config) if config is not None else None)
+    if nb == 0:
+        raise ValueError("invalid gsh_config or more than 2^28 tuples per side")
+    return int(nb)
+
+
 def join(r_keys: torch.Tensor, r_payloads: torch.Tensor, s_keys: torch.Tensor, s_payloads: torch.Tensor,
          mode: str = "count", out: torch.Tensor | None = None, out_capacity: int | None = None,
          config: GshConfig | None = None, stream=None, workspace: torch.Tensor | None = None,
@@ -163,7 +171,8 @@ def join(r_keys: torch.Tensor, r_payloads: torch.Tensor, s_keys: torch.Tensor, s
     if workspace is not None:   # gsh_join itself rejects a too-small workspace (GSH_ERR_INVALID)
         ws = workspace
     else:
-        ws = _default_ws.get(workspace_bytes(R.n, S.n, config), dev)
+        nb = workspace_bytes(R.n, S.n, config) if impl == "gsh" else gbase_workspace_bytes(R.n, S.n, config)
+        ws = _default_ws.get(nb, dev)
     res = GshResult()
     args = (ctypes.byref(R), ctypes.byref(S), _lib.GSH_OUT_MATERIALIZE if mat else _lib.GSH_OUT_COUNT,
             ctypes.byref(outp) if outp is not None else None, ws.data_ptr(), ws.numel(),
