@@ -200,10 +200,10 @@ GSH_API gsh_status gsh_join(const gsh_relation *R, const gsh_relation *S, gsh_ou
  * gsh_join_gbase -- the paper's GPU comparison system "Gbase" (§II-B, §III
  * L78-L80), re-implemented on this GPU for the GSH-vs-Gbase measurement
  * (Table I), with no skew detection:
- *   partition: two passes into bucket-chained partitions (2048-tuple buckets allocated from a pool
+ *   partition: two passes into bucket-chained partitions (4096-tuple buckets allocated from a pool
  *   as partitions fill, linked per partition; tiles of 4 tuples per thread reordered in shared
  *   memory and written as coalesced runs, L70) -- GSH's fanout (R7);
- *   join: one thread block per (partition, R sub-list of two buckets) builds a chained
+ *   join: one thread block per (partition, R sub-list = one bucket) builds a chained
  *   shared-memory table and probes it with ALL of S's buckets of that partition (L71-L72), every
  *   thread advancing one chain element per round with a write bitmap and a block barrier per round
  *   (L79-L80).
