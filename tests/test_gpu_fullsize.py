@@ -152,6 +152,25 @@ def test_cfg3_theta075_count_fullsize():
     assert r.stats["n_heavy"] > 0 and r.stats["n_large"] > 0
     r2 = gsh.join(rk, rp, sk, sp, config=gsh.make_config(force_all_normal=True))
     assert (r2.count, r2.checksum) == (r.count, r.checksum)
+    # CSH's hybrid partition (NEXT-1) at full size: the sampled keys leave in pass 1, the same pairs
+    r3 = gsh.join(rk, rp, sk, sp, config=gsh.make_config(hybrid=True))
+    assert (r3.count, r3.checksum) == (r.count, r.checksum) and r3.stats["n_hybrid"] > 0
+
+
+@pytest.mark.parametrize("theta", [1.0, 1.5])
+def test_hybrid_fullsize_input_side(theta):
+    """The hybrid partition at 2^27 per side, theta = 1.0 / 1.5 (8e13 / 3e15 pairs: input side only,
+    the per-key counts are pinned by the P5 hook at the ladder size, tests/test_gpu_hybrid.py): the
+    sampled keys plus the keys detected after partitioning must still send (nearly) all of the output
+    to the dense skewed-key phase, as GSH's detection alone does."""
+    n = N2
+    rk, rp, sk, sp = datagen.zipf_pair(n, n, theta, seed=0x6A5, device="cuda")
+    r = gsh.join(rk, rp, sk, sp, config=gsh.make_config(hybrid=True, input_side_only=True))
+    st = r.stats
+    assert st["n_hybrid"] > 0
+    g = gsh.join(rk, rp, sk, sp, config=gsh.make_config(input_side_only=True))
+    assert st["skew_pairs"] > 0.99 * g.stats["skew_pairs"]
+    assert st["heavy_tuples_r"] <= n and st["heavy_tuples_s"] <= n
 
 
 def _closed_form_gpu(rk, sk):
