@@ -226,6 +226,13 @@ bool plan_build(Plan& p, uint64_t nR, uint64_t nS, const gsh_config* cfg_in, voi
     p.h_tiles = c.take<uint64_t>(p.h_max + 1);
     p.h_chk = c.take<unsigned long long>(p.detail ? p.h_max : 0);
     p.h_cur = c.take<uint32_t>(2 * p.h_max);
+    {   // the split's compact skewed-key table: load <= 1/2 at the list's capacity
+        uint64_t hc = next_pow2_u64(2 * p.h_max);
+        if (hc < 1024) hc = 1024;
+        if (hc > (1ull << 26)) hc = 1ull << 26;
+        p.htab_cap = (uint32_t)hc;
+        p.htab = c.take<unsigned long long>(hc);
+    }
     p.nm = c.take<NmPart>(F);
     p.nm_prefix = c.take<uint64_t>(F + 1);
     p.scan_scratch = c.take<uint64_t>(p.scan_scratch_elems);
@@ -515,7 +522,7 @@ static gsh_status join_direct(const gsh_relation* R, const gsh_relation* S, gsh_
         n_heavy = hs.n_heavy;
         if (hs.heavy_overflow || n_heavy > p.h_max) return fail(GSH_ERR_INTERNAL, "skewed-key list overflow");
         launches += launch_heavy_prefix(p, n_heavy, n_large, s);
-        launches += launch_split(p, n_large, (uint32_t)gcap, s);
+        launches += launch_split(p, n_large, n_heavy, s);
         e5 = tm.mark();
     }
     if (p.input_only) {   // measurement hook: stop after the input side

@@ -198,6 +198,9 @@ struct Plan {
     uint64_t* h_tiles = nullptr;              // [h_max + 1]
     unsigned long long* h_chk = nullptr;      // [h_max] per skewed key checksum share (heavy_detail)
     uint32_t* h_cur = nullptr;                // [2][h_max] split cursors
+    unsigned long long* htab = nullptr;       // [htab_cap] compact skewed-key table for the split:
+                                              // (hid + 1) << 32 | h, 0 = empty (L2-resident size)
+    uint32_t htab_cap = 0;
     uint32_t* nrm_cur = nullptr;              // [2][F]     split cursors (normal)
     NmPart* nm = nullptr;                     // [F]
     uint64_t* nm_prefix = nullptr;            // [F + 1]
@@ -235,7 +238,7 @@ int launch_heavy_offsets(const Plan& p, uint32_t n_heavy, cudaStream_t s);   // 
 // first n_h0 entries of H with their exact counts
 int launch_hybrid_sample(const Plan& p, const uint32_t* k0, const uint32_t* k1, cudaStream_t s);
 int launch_hybrid_fill(const Plan& p, cudaStream_t s);   // + the per-(key, unit) offsets
-int launch_split(const Plan& p, uint32_t n_large, uint32_t gt_cap, cudaStream_t s);
+int launch_split(const Plan& p, uint32_t n_large, uint32_t n_heavy, cudaStream_t s);
 int launch_nm_setup(const Plan& p, uint32_t n_large, cudaStream_t s);
 int launch_nmjoin(const Plan& p, int materialize, uint32_t* pairs, uint64_t cap, cudaStream_t s);
 int launch_nmjoin_ring(const Plan& p, int materialize, uint32_t* pairs, uint64_t cap, cudaStream_t s);

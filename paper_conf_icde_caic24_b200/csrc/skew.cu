@@ -533,8 +533,33 @@ constexpr size_t kSplitSmemBytes = size_t(kSplitHidSlots) * 8;
 static_assert(kSplitIpt * kDetBlock == kDetectChunk, "split item = 8 tuples per thread");
 static_assert(kSplitHidSlots == 4096, "slot hash below takes 12 bits");
 
-__global__ void __launch_bounds__(kDetBlock, 4) k_split(LargeView v, const unsigned long long* __restrict__ gt_key,
-                                                    const uint32_t* __restrict__ gt_hid, uint32_t logcap,
+// The split's skewed-key lookups go to a compact table of H only ((hid + 1) << 32 | h, 0 = empty,
+// 2 slots per key: a few hundred KB, L2-resident) instead of the detection table (one slot per
+// counted key, up to 256 MB: one DRAM sector per first probe of every tuple of a large partition).
+__global__ void k_htab_build(const HeavyKey* __restrict__ H, uint32_t n_heavy, unsigned long long* htab,
+                             uint32_t logcap) {
+    const uint32_t mask = (1u << logcap) - 1;
+    for (uint32_t hid = blockIdx.x * blockDim.x + threadIdx.x; hid < n_heavy; hid += gridDim.x * blockDim.x) {
+        const uint32_t h = H[hid].h;
+        const unsigned long long e = (uint64_t(hid + 1) << 32) | h;
+        uint32_t s = gt_slot0(h, logcap);
+        while (atomicCAS(&htab[s], 0ull, e) != 0ull) s = (s + 1) & mask;   // load <= 1/2: terminates
+    }
+}
+
+__device__ __forceinline__ uint32_t htab_find(const unsigned long long* __restrict__ htab, uint32_t h,
+                                              uint32_t logcap, uint32_t s) {
+    const uint32_t mask = (1u << logcap) - 1;
+    for (;;) {
+        const unsigned long long e = htab[s];
+        if (e == 0) return kNoHeavy;
+        if ((uint32_t)e == h) return (uint32_t)(e >> 32) - 1;
+        s = (s + 1) & mask;
+    }
+}
+
+__global__ void __launch_bounds__(kDetBlock, 4) k_split(LargeView v, const unsigned long long* __restrict__ htab,
+                                                    uint32_t logcap,
                                                     const uint64_t* __restrict__ h_off, uint64_t h_stride,
                                                     uint32_t* h_cur, uint32_t h_max, uint32_t* heavy_pay_r,
                                                     uint32_t* heavy_pay_s, const uint64_t* __restrict__ nrm_off,
@@ -568,17 +593,17 @@ __global__ void __launch_bounds__(kDetBlock, 4) k_split(LargeView v, const unsig
             t[j] = e < r.e1 ? (e < r.cr ? pr[e] : ps[e - r.cr]) : make_uint2(0, 0);
         }
         // skewed-key ids: the first probe of every tuple is issued before any is resolved (the
-        // table holds only possible skewed keys, so most first probes find an empty slot)
-        uint32_t probe0 = 0;   // 2 bits per tuple: 0 = first slot empty (normal), 1 = found there, 2 = probe on
+        // table holds only the skewed keys, so most first probes of normal tuples find an empty slot)
+        uint32_t ids[kSplitIpt];
         {
             unsigned long long w0[kSplitIpt];
 #pragma unroll
-            for (int j = 0; j < kSplitIpt; ++j) w0[j] = gt_key[gt_slot0(t[j].x, logcap)];
+            for (int j = 0; j < kSplitIpt; ++j) w0[j] = htab[gt_slot0(t[j].x, logcap)];
 #pragma unroll
-            for (int j = 0; j < kSplitIpt; ++j) {
-                const uint32_t st2 = w0[j] == ((1ull << 32) | t[j].x) ? 1u : (w0[j] == 0 ? 0u : 2u);
-                probe0 |= st2 << (2 * j);
-            }
+            for (int j = 0; j < kSplitIpt; ++j)
+                ids[j] = w0[j] == 0 ? kNoHeavy
+                       : (uint32_t)w0[j] == t[j].x ? (uint32_t)(w0[j] >> 32) - 1
+                       : htab_find(htab, t[j].x, logcap, (gt_slot0(t[j].x, logcap) + 1) & ((1u << logcap) - 1));
         }
         // Ranks: normal tuples by one shared atomic per (warp, side); skewed tuples of the warp's
         // reference key by one shared atomic per warp (lanes ranked by ballot prefix); other skewed
@@ -591,10 +616,7 @@ __global__ void __launch_bounds__(kDetBlock, 4) k_split(LargeView v, const unsig
             const uint64_t e = r.e0 + uint64_t(j) * kDetBlock + threadIdx.x;
             const bool valid = e < r.e1;
             const uint32_t side = e >= r.cr;
-            const uint32_t st2 = (probe0 >> (2 * j)) & 3u;
-            uint32_t g = kNoHeavy;
-            if (valid && st2) g = st2 == 1 ? gt_slot0(t[j].x, logcap) : gt_find(gt_key, t[j].x, logcap);
-            const uint32_t id = g == kNoHeavy ? kNoHeavy : gt_hid[g];
+            const uint32_t id = ids[j];
             const bool heavy = valid && id != kNoHeavy;
             const uint32_t key = heavy ? ((id << 1 | side) + 1) : 0u;
             uint32_t rr = 0xffffffffu;
@@ -679,21 +701,26 @@ __global__ void __launch_bounds__(kDetBlock, 4) k_split(LargeView v, const unsig
     }
 }
 
-int launch_split(const Plan& p, uint32_t n_large, uint32_t gt_cap, cudaStream_t s) {
+int launch_split(const Plan& p, uint32_t n_large, uint32_t n_heavy, cudaStream_t s) {
     if (n_large == 0) return 0;
-    uint32_t logcap = 0;
-    while ((1u << logcap) < gt_cap) ++logcap;
+    uint64_t hc = 1024;
+    while (hc < 2 * uint64_t(n_heavy) && hc < p.htab_cap) hc <<= 1;
+    const uint32_t logcap = log2_pow2(hc);
+    cudaMemsetAsync(p.htab, 0, hc * sizeof(unsigned long long), s);
+    if (n_heavy)
+        k_htab_build<<<(unsigned)umin64((n_heavy + 255) / 256, uint64_t(p.num_sms) * 8), 256, 0, s>>>(p.H, n_heavy,
+                                                                                                p.htab, logcap);
     static std::once_flag attr_once[kMaxDevices];
     once_per_device(attr_once, [] {
         cudaFuncSetAttribute(k_split, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSplitSmemBytes);
     });
     LargeView v{{p.bufB[0], p.bufB[1]}, p.start, p.cnt, p.large_list, p.det_prefix, p.F, n_large, kDetectChunk,
                 p.item_li};
-    k_split<<<p.num_sms * 4, kDetBlock, kSplitSmemBytes, s>>>(v, p.gt_key, p.gt_hid, logcap, p.h_off, p.h_max + 1,
+    k_split<<<p.num_sms * 4, kDetBlock, kSplitSmemBytes, s>>>(v, p.htab, logcap, p.h_off, p.h_max + 1,
                                                              p.h_cur, (uint32_t)p.h_max, p.heavy_pay[0],
                                                              p.heavy_pay[1], p.nrm_off, p.nrm_cur, p.bufA[0],
                                                              p.bufA[1], &p.st->claim[3]);
-    return 1;
+    return n_heavy ? 2 : 1;
 }
 
 // --------------------------------------------------------------- NM descriptors --
