@@ -569,12 +569,15 @@ __global__ void __launch_bounds__(kDetBlock, 4) k_split(LargeView v, const unsig
     uint32_t* s_key = split_dyn;                    // (hid << 1 | side) + 1, 0 = empty
     uint32_t* s_cnt = split_dyn + kSplitHidSlots;   // count, then the item's run base
     __shared__ uint32_t s_nrm[2], s_nbase[2];
+    __shared__ uint32_t s_used[kSplitHidSlots];   // the item's claimed slots (the reservation walks only these)
+    __shared__ uint32_t s_nused;
     __shared__ unsigned int s_it;
     for (uint32_t i = threadIdx.x; i < kSplitHidSlots; i += kDetBlock) {
         s_key[i] = 0;
         s_cnt[i] = 0;
     }
     if (threadIdx.x < 2) s_nrm[threadIdx.x] = 0;
+    if (threadIdx.x == 0) s_nused = 0;
     const uint64_t total = v.det_prefix[v.n_large];
     for (;;) {
         if (threadIdx.x == 0) s_it = atomicAdd(claim, 1u);
@@ -647,7 +650,11 @@ __global__ void __launch_bounds__(kDetBlock, 4) k_split(LargeView v, const unsig
                     if (cur == key) break;
                     if (cur == 0) {
                         const uint32_t prev = atomicCAS(&s_key[slot], 0u, key);
-                        if (prev == 0 || prev == key) break;
+                        if (prev == 0) {
+                            s_used[atomicAdd(&s_nused, 1u)] = slot;
+                            break;
+                        }
+                        if (prev == key) break;
                     }
                     slot = (slot + 1) & (kSplitHidSlots - 1);
                 }
@@ -663,12 +670,11 @@ __global__ void __launch_bounds__(kDetBlock, 4) k_split(LargeView v, const unsig
         }
         __syncthreads();
         // reserve this item's runs: one global atomic per distinct (side, key) and per side
-        for (uint32_t i = threadIdx.x; i < kSplitHidSlots; i += kDetBlock) {
+        for (uint32_t u = threadIdx.x; u < s_nused; u += kDetBlock) {
+            const uint32_t i = s_used[u];
             const uint32_t key = s_key[i];
-            if (key) {
-                const uint32_t id = (key - 1) >> 1, side = (key - 1) & 1u;
-                s_cnt[i] = atomicAdd(&h_cur[size_t(side) * h_max + id], s_cnt[i]);
-            }
+            const uint32_t id = (key - 1) >> 1, side = (key - 1) & 1u;
+            s_cnt[i] = atomicAdd(&h_cur[size_t(side) * h_max + id], s_cnt[i]);
         }
         if (threadIdx.x < 2 && s_nrm[threadIdx.x])
             s_nbase[threadIdx.x] = atomicAdd(&nrm_cur[size_t(threadIdx.x) * v.F + r.li], s_nrm[threadIdx.x]);
@@ -698,6 +704,7 @@ __global__ void __launch_bounds__(kDetBlock, 4) k_split(LargeView v, const unsig
             }
         }
         if (threadIdx.x < 2) s_nrm[threadIdx.x] = 0;
+        if (threadIdx.x == 0) s_nused = 0;
     }
 }
 
