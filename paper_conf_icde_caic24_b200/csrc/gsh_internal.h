@@ -80,7 +80,11 @@ constexpr int kSkewBlock = 256;                 // skewed-key join CTA
 constexpr int kSkewSpt = 4;                     // S payloads per thread (registers)
 constexpr int kSkewTileS = kSkewBlock * kSkewSpt;  // 1024
 constexpr int kSkewTileR = 64;                  // R payloads per tile (shared memory)
-constexpr uint32_t kDetectChunk = 2048;         // tuples per split (and sampled-detect) work item
+#ifndef GSH_SKEWSPLIT_BLOCK
+#define GSH_SKEWSPLIT_BLOCK 256
+#endif
+constexpr int kSkewSplitBlock = GSH_SKEWSPLIT_BLOCK;   // split CTA (8 tuples per thread in registers)
+constexpr uint32_t kDetectChunk = 8 * kSkewSplitBlock;   // tuples per split (and sampled-detect) work item
 constexpr uint32_t kDetectItem = 16384;         // tuples per exact-detect work item
 constexpr uint32_t kNoHeavy = 0xffffffffu;
 constexpr int kDetectMaxProbe = 64;   // a full table degrades to "normal", never to a long probe

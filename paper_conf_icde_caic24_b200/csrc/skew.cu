@@ -528,10 +528,11 @@ int launch_heavy_prefix(const Plan& p, uint32_t n_heavy, uint32_t n_large, cudaS
 // (2) one global atomic per distinct (side, key) and per side reserves the item's runs, and the
 // tuples are written at base + rank (consecutive for runs of one key: coalesced).
 constexpr uint32_t kSplitHidSlots = 2 * kDetectChunk;   // an item's distinct (side, key) always fit
-constexpr int kSplitIpt = kDetectChunk / kDetBlock;
+constexpr int kSplitIpt = kDetectChunk / kSkewSplitBlock;
+constexpr uint32_t kSplitSlotBits = kSplitHidSlots == 4096 ? 12 : kSplitHidSlots == 8192 ? 13 : 14;
 constexpr size_t kSplitSmemBytes = size_t(kSplitHidSlots) * 8;
-static_assert(kSplitIpt * kDetBlock == kDetectChunk, "split item = 8 tuples per thread");
-static_assert(kSplitHidSlots == 4096, "slot hash below takes 12 bits");
+static_assert(kSplitIpt * kSkewSplitBlock == kDetectChunk, "split item = 8 tuples per thread");
+static_assert((1u << kSplitSlotBits) == kSplitHidSlots, "slot hash bits");
 
 // The split's skewed-key lookups go to a compact table of H only ((hid + 1) << 32 | h, 0 = empty,
 // 2 slots per key: a few hundred KB, L2-resident) instead of the detection table (one slot per
@@ -558,7 +559,7 @@ __device__ __forceinline__ uint32_t htab_find(const unsigned long long* __restri
     }
 }
 
-__global__ void __launch_bounds__(kDetBlock, 4) k_split(LargeView v, const unsigned long long* __restrict__ htab,
+__global__ void __launch_bounds__(kSkewSplitBlock, 1024 / kSkewSplitBlock) k_split(LargeView v, const unsigned long long* __restrict__ htab,
                                                     uint32_t logcap,
                                                     const uint64_t* __restrict__ h_off, uint64_t h_stride,
                                                     uint32_t* h_cur, uint32_t h_max, uint32_t* heavy_pay_r,
@@ -572,7 +573,7 @@ __global__ void __launch_bounds__(kDetBlock, 4) k_split(LargeView v, const unsig
     __shared__ uint32_t s_used[kSplitHidSlots];   // the item's claimed slots (the reservation walks only these)
     __shared__ uint32_t s_nused;
     __shared__ unsigned int s_it;
-    for (uint32_t i = threadIdx.x; i < kSplitHidSlots; i += kDetBlock) {
+    for (uint32_t i = threadIdx.x; i < kSplitHidSlots; i += kSkewSplitBlock) {
         s_key[i] = 0;
         s_cnt[i] = 0;
     }
@@ -592,7 +593,7 @@ __global__ void __launch_bounds__(kDetBlock, 4) k_split(LargeView v, const unsig
         uint32_t rk[kSplitIpt];
 #pragma unroll
         for (int j = 0; j < kSplitIpt; ++j) {
-            const uint64_t e = r.e0 + uint64_t(j) * kDetBlock + threadIdx.x;
+            const uint64_t e = r.e0 + uint64_t(j) * kSkewSplitBlock + threadIdx.x;
             t[j] = e < r.e1 ? (e < r.cr ? pr[e] : ps[e - r.cr]) : make_uint2(0, 0);
         }
         // skewed-key ids: the first probe of every tuple is issued before any is resolved (the
@@ -616,7 +617,7 @@ __global__ void __launch_bounds__(kDetBlock, 4) k_split(LargeView v, const unsig
         const uint32_t lane = lane_id(), ltm = lanemask_lt();
 #pragma unroll
         for (int j = 0; j < kSplitIpt; ++j) {
-            const uint64_t e = r.e0 + uint64_t(j) * kDetBlock + threadIdx.x;
+            const uint64_t e = r.e0 + uint64_t(j) * kSkewSplitBlock + threadIdx.x;
             const bool valid = e < r.e1;
             const uint32_t side = e >= r.cr;
             const uint32_t id = ids[j];
@@ -644,7 +645,7 @@ __global__ void __launch_bounds__(kDetBlock, 4) k_split(LargeView v, const unsig
             }
             const bool other = heavy && key != ref;
             if (other) {
-                uint32_t slot = (key * 0x9E3779B1u) >> (32 - 12);   // kSplitHidSlots = 2^12
+                uint32_t slot = (key * 0x9E3779B1u) >> (32 - kSplitSlotBits);
                 for (;;) {   // an item has <= kDetectChunk distinct keys: a free slot always exists
                     const uint32_t cur = s_key[slot];
                     if (cur == key) break;
@@ -670,7 +671,7 @@ __global__ void __launch_bounds__(kDetBlock, 4) k_split(LargeView v, const unsig
         }
         __syncthreads();
         // reserve this item's runs: one global atomic per distinct (side, key) and per side
-        for (uint32_t u = threadIdx.x; u < s_nused; u += kDetBlock) {
+        for (uint32_t u = threadIdx.x; u < s_nused; u += kSkewSplitBlock) {
             const uint32_t i = s_used[u];
             const uint32_t key = s_key[i];
             const uint32_t id = (key - 1) >> 1, side = (key - 1) & 1u;
@@ -723,7 +724,7 @@ int launch_split(const Plan& p, uint32_t n_large, uint32_t n_heavy, cudaStream_t
     });
     LargeView v{{p.bufB[0], p.bufB[1]}, p.start, p.cnt, p.large_list, p.det_prefix, p.F, n_large, kDetectChunk,
                 p.item_li};
-    k_split<<<p.num_sms * 4, kDetBlock, kSplitSmemBytes, s>>>(v, p.htab, logcap, p.h_off, p.h_max + 1,
+    k_split<<<p.num_sms * (1024 / kSkewSplitBlock), kSkewSplitBlock, kSplitSmemBytes, s>>>(v, p.htab, logcap, p.h_off, p.h_max + 1,
                                                              p.h_cur, (uint32_t)p.h_max, p.heavy_pay[0],
                                                              p.heavy_pay[1], p.nrm_off, p.nrm_cur, p.bufA[0],
                                                              p.bufA[1], &p.st->claim[3]);
