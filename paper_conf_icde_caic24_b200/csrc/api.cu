@@ -209,7 +209,6 @@ bool plan_build(Plan& p, uint64_t nR, uint64_t nS, const gsh_config* cfg_in, voi
     p.start = c.take<uint64_t>(2 * (F + 1));
     p.gt_key = c.take<unsigned long long>(p.gt_cap_alloc);
     p.gt_cnt = c.take<uint32_t>(size_t(2) * p.gt_cap_alloc);
-    p.gt_hid = c.take<uint32_t>(p.gt_cap_alloc);
     p.large_list = c.take<uint32_t>(F);
     p.large_idx = c.take<uint32_t>(F);
     p.part_heavy = c.take<uint32_t>(2 * F);

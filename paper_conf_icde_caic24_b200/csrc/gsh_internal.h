@@ -187,7 +187,6 @@ struct Plan {
     DevState* st = nullptr;
     unsigned long long* gt_key = nullptr;     // [gt_cap_alloc]  (1 << 32 | h), 0 = empty
     uint32_t* gt_cnt = nullptr;               // [2][gt_cap_alloc]
-    uint32_t* gt_hid = nullptr;               // [gt_cap_alloc]
     uint32_t* large_list = nullptr;           // [F]
     uint32_t* large_idx = nullptr;            // [F] partition -> large index or kNoHeavy
     uint32_t* part_heavy = nullptr;           // [2][F]  skewed tuples per partition

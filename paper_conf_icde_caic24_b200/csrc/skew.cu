@@ -430,7 +430,7 @@ int launch_sample_topk(const Plan& p, uint32_t n_large, uint32_t gt_cap, cudaStr
 
 // ------------------------------------------------------------------- a6: select --
 __global__ void k_select(const unsigned long long* __restrict__ gt_key, const uint32_t* __restrict__ gt_cnt,
-                         uint32_t* __restrict__ gt_hid, uint32_t cap, uint32_t cap_alloc, uint32_t Th,
+                         uint32_t cap, uint32_t cap_alloc, uint32_t Th,
                          int force_heavy, uint32_t pshift, uint32_t pmask, uint32_t F, HeavyKey* __restrict__ H,
                          uint64_t h_max, uint32_t* __restrict__ part_heavy, DevState* st) {
     for (uint32_t slot = blockIdx.x * blockDim.x + threadIdx.x; slot < cap; slot += gridDim.x * blockDim.x) {
@@ -439,13 +439,11 @@ __global__ void k_select(const unsigned long long* __restrict__ gt_key, const ui
         const uint32_t h = (uint32_t)kw;
         const uint32_t cr = gt_cnt[slot], cs = gt_cnt[cap_alloc + slot];
         const bool heavy = force_heavy || max(cr, cs) >= Th;
-        uint32_t hid = kNoHeavy;
         if (heavy) {
             const uint32_t p = part_of(h, pshift, pmask);
-            hid = atomicAdd(&st->n_heavy, 1u);
+            const uint32_t hid = atomicAdd(&st->n_heavy, 1u);
             if (hid >= h_max) {   // the side list is full: the call fails (GSH_ERR_INTERNAL)
                 st->heavy_overflow = 1;
-                gt_hid[slot] = kNoHeavy;
                 continue;
             }
             H[hid] = HeavyKey{h, cr, cs, p};
@@ -455,7 +453,6 @@ __global__ void k_select(const unsigned long long* __restrict__ gt_key, const ui
             atomicAdd(&st->heavy_tuples[1], (unsigned long long)cs);
             atomicAdd(&st->skew_pairs, (unsigned long long)cr * cs);
         }
-        gt_hid[slot] = hid;
     }
 }
 
@@ -465,7 +462,7 @@ int launch_select(const Plan& p, uint32_t gt_cap, cudaStream_t s) {
     unsigned grid = (unsigned)umin64((gt_cap + 255) / 256, uint64_t(p.num_sms) * 16);
     // detect_mode 1: the table holds exactly the sampled top-k keys, all skewed
     const uint32_t th = p.detect_mode == 1 ? 1u : p.Th;
-    k_select<<<grid, 256, 0, s>>>(p.gt_key, p.gt_cnt, p.gt_hid, gt_cap, p.gt_cap_alloc, th, p.force_heavy, pshift,
+    k_select<<<grid, 256, 0, s>>>(p.gt_key, p.gt_cnt, gt_cap, p.gt_cap_alloc, th, p.force_heavy, pshift,
                                   p.F - 1, p.F, p.H, p.h_max, p.part_heavy, p.st);
     return 1;
 }
