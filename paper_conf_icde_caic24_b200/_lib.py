@@ -54,6 +54,7 @@ class GshConfig(ctypes.Structure):
         ("hybrid", i32),
         ("hybrid_stride", u32),
         ("hybrid_min", u32),
+        ("hybrid_share", u32),
     ]
 
 

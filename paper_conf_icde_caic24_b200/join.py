@@ -21,7 +21,7 @@ def make_config(capacity: int = 0, pass_bits=None, heavy_threshold: int = 0, rou
                 large_threshold: int = 0, nm_table: int = 0, detect_mode: int = 0, sample_stride: int = 0,
                 top_k: int = 0, prepass_bits: int = 0, input_side_only: bool = False,
                 heavy_detail: bool = False, hybrid: bool = False, hybrid_stride: int = 0,
-                hybrid_min: int = 0) -> GshConfig:
+                hybrid_min: int = 0, hybrid_share: int = 0) -> GshConfig:
     """Build a gsh_config (see include/gsh.h for each field's meaning)."""
     cfg = _lib.default_config()
     cfg.capacity = int(capacity)
@@ -44,6 +44,7 @@ def make_config(capacity: int = 0, pass_bits=None, heavy_threshold: int = 0, rou
     cfg.hybrid = int(bool(hybrid))
     cfg.hybrid_stride = int(hybrid_stride)
     cfg.hybrid_min = int(hybrid_min)
+    cfg.hybrid_share = int(hybrid_share)
     return cfg
 
 

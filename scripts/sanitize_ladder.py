@@ -31,9 +31,9 @@ CASES = [  # kind, n, theta, config
     ("graph", 1 << 16, 0.909, {}),
     ("zipf", 1 << 16, 1.0, {"prepass_bits": 2}),
     ("pkfk_zipf", 1 << 16, 1.0, {"heavy_detail": True}),
-    ("zipf", 1 << 17, 1.0, {"hybrid": True}),
-    ("zipf", 1 << 15, 1.5, {"hybrid": True, "hybrid_stride": 1}),
-    ("pkfk_zipf", 1 << 16, 1.0, {"hybrid": True}),
+    ("zipf", 1 << 17, 1.0, {"hybrid": True, "hybrid_share": 1}),
+    ("zipf", 1 << 15, 1.5, {"hybrid": True, "hybrid_stride": 1, "hybrid_share": 1}),
+    ("pkfk_zipf", 1 << 16, 1.0, {"hybrid": True, "hybrid_share": 1}),
     ("zipf", (1 << 15) + 3, 1.0, {"impl": "gbase"}),
     ("graph", 1 << 15, 0.909, {"impl": "gbase"}),
 ]

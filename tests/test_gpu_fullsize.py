@@ -167,7 +167,7 @@ def test_hybrid_fullsize_input_side(theta):
     to the dense skewed-key phase, as GSH's detection alone does."""
     n = N2
     rk, rp, sk, sp = datagen.zipf_pair(n, n, theta, seed=0x6A5, device="cuda")
-    r = gsh.join(rk, rp, sk, sp, config=gsh.make_config(hybrid=True, input_side_only=True))
+    r = gsh.join(rk, rp, sk, sp, config=gsh.make_config(hybrid=True, input_side_only=True, hybrid_share=1))
     st = r.stats
     assert st["n_hybrid"] > 0
     g = gsh.join(rk, rp, sk, sp, config=gsh.make_config(input_side_only=True))

@@ -29,7 +29,9 @@ def _sorted_pairs(p):
     return a[np.lexsort((a[:, 1], a[:, 0]))]
 
 
-HYB = dict(hybrid=True, timing=True)
+# hybrid_share=1: engage whenever the sample chose keys (the default 1/4 gate would keep GSH's passes
+# on several of these inputs); the gate itself: test_hybrid_share_gate
+HYB = dict(hybrid=True, timing=True, hybrid_share=1)
 
 # skewed: the sample must choose keys (True), must not (False: chance triples of a skew-free input
 # hold < 1/64 of the sample), or either (None: theta = 0.5, little mass in the top keys)
@@ -71,7 +73,7 @@ def test_hybrid_decomposition_exact_counts(kind, n, theta):
     histogram pass's), the parts add up, the NM share is the oracle join without every skewed key,
     and C_k equals brute force for the keys whose product is small enough."""
     rk, rp, sk, sp = datagen.make_workload(kind, n, theta, seed=17)
-    r, det = gsh.join_detail(*_dev(rk, rp, sk, sp), config=gsh.make_config(hybrid=True, heavy_detail=True))
+    r, det = gsh.join_detail(*_dev(rk, rp, sk, sp), config=gsh.make_config(hybrid=True, heavy_detail=True, hybrid_share=1))
     st = r.stats
     nh = st["n_hybrid"]
     assert 0 < nh <= det["h"].numel() == st["n_heavy"]
@@ -107,7 +109,7 @@ def test_hybrid_invariant_under_config(cfg):
     rk, rp, sk, sp = datagen.zipf_pair(1 << 16, (1 << 16) + 9, 1.0, seed=21)
     on, oc, op = oracle.join_sorted_pairs(_np(rk), _np(rp), _np(sk), _np(sp))
     d = _dev(rk, rp, sk, sp)
-    c = gsh.make_config(hybrid=True, **cfg)
+    c = gsh.make_config(hybrid=True, hybrid_share=1, **cfg)
     r = gsh.join(*d, config=c)
     assert (r.count, r.checksum) == (on, oc)
     if cfg.get("hybrid_min") == 1:
@@ -141,7 +143,7 @@ def test_hybrid_edge_cases():
     for rk, rp, sk, sp in cases:
         on, oc, op = oracle.join_sorted_pairs(_np(rk), _np(rp), _np(sk), _np(sp))
         for stride in (0, 1):
-            c = gsh.make_config(hybrid=True, hybrid_stride=stride)
+            c = gsh.make_config(hybrid=True, hybrid_stride=stride, hybrid_share=1)
             r = gsh.join(*_dev(rk, rp, sk, sp), config=c)
             assert (r.count, r.checksum) == (on, oc)
             m = gsh.join(*_dev(rk, rp, sk, sp), mode="materialize", out_capacity=on, config=c)
@@ -154,19 +156,35 @@ def test_hybrid_unaligned_views_and_routing_bits():
     rk, rp, sk, sp = datagen.zipf_pair(90_001, 70_003, 1.0, seed=3)
     d = _dev(rk, rp, sk, sp)
     on, oc, _ = oracle.join(_np(rk[1:]), _np(rp[1:]), _np(sk[3:]), _np(sp[2:-1]))
-    r = gsh.join(d[0][1:], d[1][1:], d[2][3:], d[3][2:-1], config=gsh.make_config(hybrid=True))
+    r = gsh.join(d[0][1:], d[1][1:], d[2][3:], d[3][2:-1], config=gsh.make_config(hybrid=True, hybrid_share=1))
     assert (r.count, r.checksum) == (on, oc) and r.stats["n_hybrid"] > 0
     kr = (oracle.fmix32(_np(rk)) >> 30) == 1
     ks = (oracle.fmix32(_np(sk)) >> 30) == 1
     sh = [t[torch.from_numpy(m)] for t, m in ((rk, kr), (rp, kr), (sk, ks), (sp, ks))]
     on2, oc2, _ = oracle.join(*(_np(t) for t in sh))
-    r2 = gsh.join(*_dev(*sh), config=gsh.make_config(hybrid=True, route_bits=2))
+    r2 = gsh.join(*_dev(*sh), config=gsh.make_config(hybrid=True, route_bits=2, hybrid_share=1))
     assert (r2.count, r2.checksum) == (on2, oc2)
 
 
 def test_hybrid_repeatable():
     rk, rp, sk, sp = _dev(*datagen.zipf_pair(1 << 18, 1 << 18, 1.25, seed=2))
-    c = gsh.make_config(hybrid=True)
+    c = gsh.make_config(hybrid=True, hybrid_share=1)
     a = gsh.join(rk, rp, sk, sp, config=c)
     b = gsh.join(rk, rp, sk, sp, config=c)
     assert (a.count, a.checksum, a.stats["n_heavy"]) == (b.count, b.checksum, b.stats["n_heavy"])
+
+
+def test_hybrid_share_gate():
+    """gsh_config.hybrid_share: the hybrid passes run only when the chosen keys hold at least that share
+    of the sample.  Zipf 1.5 (the top keys hold most of the input) passes the default 1/4; theta 0.75 does
+    not (GSH's passes run, the same result); any sampled skew passes 1/256."""
+    for theta, engaged_default in ((1.5, True), (0.75, False)):
+        rk, rp, sk, sp = _dev(*datagen.zipf_pair(1 << 18, 1 << 18, theta, seed=4))
+        on, oc, _ = oracle.join(*(_np(t) for t in (rk, rp, sk, sp)))
+        r = gsh.join(rk, rp, sk, sp, config=gsh.make_config(hybrid=True))
+        assert (r.count, r.checksum) == (on, oc)
+        assert (r.stats["n_hybrid"] > 0) == engaged_default, (theta, r.stats["n_hybrid"])
+        r1 = gsh.join(rk, rp, sk, sp, config=gsh.make_config(hybrid=True, hybrid_share=1))
+        assert (r1.count, r1.checksum) == (on, oc) and r1.stats["n_hybrid"] > 0
+        r2 = gsh.join(rk, rp, sk, sp, config=gsh.make_config(hybrid=True, hybrid_share=256))
+        assert (r2.count, r2.checksum) == (on, oc) and r2.stats["n_hybrid"] == 0

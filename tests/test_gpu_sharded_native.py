@@ -239,7 +239,7 @@ def test_native_with_hybrid_local_joins(world, theta, exchange):
     full = datagen.make_workload("zipf", 1 << 18, theta, seed=31)
     on, oc, _ = oracle.join(*(t.numpy().view(np.uint32) for t in full))
     shards = [tuple(_shard(t, g, world).to(dev) for t in full) for g in range(world)]
-    res = sharded.run_local_native(world, shards, config=make_config(hybrid=True, hybrid_stride=10),
+    res = sharded.run_local_native(world, shards, config=make_config(hybrid=True, hybrid_stride=10, hybrid_share=1),
                                    exchange=exchange)
     for r in res:
         assert (r.count, r.checksum) == (on, oc), (r.stats, on, oc)
