@@ -136,8 +136,9 @@ typedef struct {
     uint32_t hybrid_stride;    /* hybrid: 1 key in hybrid_stride is sampled.  0 = 100 (1 %, L89) */
     uint32_t hybrid_min;       /* hybrid: sampled count a key needs.  0 = 3 (L89: "exceeds ... 2") */
     uint32_t hybrid_share;     /* hybrid: the chosen keys must hold >= hybrid_share / 256 of the sample,
-                                  else the partition passes run without them (GSH).  0 = 64 (1/4: the
-                                  measured break-even on a B200, R22). */
+                                  else the partition passes run without them (GSH).  0 = 128 (1/2: the
+                                  hybrid passes pay off where the sampled keys hold most of the input,
+                                  DESIGN.md R22). */
 } gsh_config;
 
 /* Per-call result (host struct). */

@@ -137,7 +137,7 @@ bool plan_build(Plan& p, uint64_t nR, uint64_t nS, const gsh_config* cfg_in, voi
     p.hyb_stride = cfg.hybrid_stride ? cfg.hybrid_stride : 100;
     p.hyb_min = cfg.hybrid_min ? cfg.hybrid_min : 3;
     if (cfg.hybrid_share > 256) return false;
-    p.hyb_share = cfg.hybrid_share ? cfg.hybrid_share : 64;
+    p.hyb_share = cfg.hybrid_share ? cfg.hybrid_share : 128;
     p.hist_grid = num_sms;  // one 1024-thread CTA (128 KB of counters) per SM
     uint64_t t = next_pow2_u64(2 * (nR + nS));
     if (t < 1024) t = 1024;

@@ -157,7 +157,7 @@ struct Plan {
     int detect_mode = 0;            // 0 exact counts, 1 sampled top-k (L107, L112)
     uint32_t sample_stride = 100, top_k = 3;
     int hybrid = 0;                 // CSH-style hybrid partition (hybrid.cu)
-    uint32_t hyb_stride = 100, hyb_min = 3, hyb_share = 64;
+    uint32_t hyb_stride = 100, hyb_min = 3, hyb_share = 128;
     uint32_t n_h0 = 0;              // hybrid keys selected (host copy, set after the sample)
     int num_sms = 148;
     int hist_grid = 148;            // histogram CTAs (1 per SM)

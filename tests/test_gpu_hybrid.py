@@ -29,7 +29,7 @@ def _sorted_pairs(p):
     return a[np.lexsort((a[:, 1], a[:, 0]))]
 
 
-# hybrid_share=1: engage whenever the sample chose keys (the default 1/4 gate would keep GSH's passes
+# hybrid_share=1: engage whenever the sample chose keys (the default 1/2 gate would keep GSH's passes
 # on several of these inputs); the gate itself: test_hybrid_share_gate
 HYB = dict(hybrid=True, timing=True, hybrid_share=1)
 
@@ -176,7 +176,7 @@ def test_hybrid_repeatable():
 
 def test_hybrid_share_gate():
     """gsh_config.hybrid_share: the hybrid passes run only when the chosen keys hold at least that share
-    of the sample.  Zipf 1.5 (the top keys hold most of the input) passes the default 1/4; theta 0.75 does
+    of the sample.  Zipf 1.5 (the top keys hold ~90 % of the input) passes the default 1/2; theta 0.75 does
     not (GSH's passes run, the same result); any sampled skew passes 1/256."""
     for theta, engaged_default in ((1.5, True), (0.75, False)):
         rk, rp, sk, sp = _dev(*datagen.zipf_pair(1 << 18, 1 << 18, theta, seed=4))
