@@ -454,9 +454,10 @@ def roofline_of(phases, st, n_tot, clocks, workload):
             "algorithmic_bytes_per_launch": algo[dom]}
 
 
-def sharded_summary(phases, st, world):
+def sharded_summary(phases, st, world, one_gpu=False):
     """Multi-GPU step: protocol phase times and the exchange's bytes against NVLink 5
-    (900 GB/s per direction per GPU)."""
+    (900 GB/s per direction per GPU).  one_gpu (--fake-ranks): the "exchange" is device copies inside
+    one GPU's HBM, so no NVLink fraction is reported."""
     keys = ("ms_agree", "ms_route", "ms_exchange", "ms_broadcast", "ms_join_normal", "ms_join_heavy", "ms_reduce")
     out = {k: phases.get(k) for k in keys}
     xb = st.get("exchange_send_bytes", st.get("exchange_bytes", 0))
@@ -466,8 +467,10 @@ def sharded_summary(phases, st, world):
         gbs = nb / (ms * 1e6) if ms > 0 else None
         out[f"{name}_bytes_per_rank"] = nb
         out[f"{name}_GBps"] = gbs
-        out[f"{name}_nvlink_frac"] = gbs / 900.0 if gbs else None
-    out["nvlink_peak_GBps"] = 900.0
+        out[f"{name}_nvlink_frac"] = gbs / 900.0 if gbs and not one_gpu else None
+    out["nvlink_peak_GBps"] = None if one_gpu else 900.0
+    if one_gpu:
+        out["note"] = "logical ranks on one GPU: exchanges are local HBM copies (code-path timing, not NVLink)"
     out["world"] = world
     return out
 
@@ -674,7 +677,7 @@ def main():
             "stats": {k: v for k, v in r.stats.items() if not k.startswith("ms_") and not isinstance(v, dict)},
         }
         if multi:
-            line["sharded"] = sharded_summary(phases, r.stats, fake or world)
+            line["sharded"] = sharded_summary(phases, r.stats, fake or world, one_gpu=fake >= 1)
         if sweep is not None:
             line["theta_sweep"] = sweep
         line["pass_fractions"] = pass_fractions(phases, jst, n_tot)
