@@ -129,12 +129,24 @@ def test_gbase_argument_errors_before_any_launch():
     assert b"2^28" in lib.gsh_last_error()
 
 
+def test_gbase_workspace_sizing():
+    # bucket pools: larger than GSH's workspace, growing with n; refused beyond 2^28 per side
+    lib = _lib.load()
+    a, b = gsh.gbase_workspace_bytes(1 << 20, 1 << 20), gsh.gbase_workspace_bytes(1 << 27, 1 << 27)
+    assert 0 < a < b and b > gsh.workspace_bytes(1 << 27, 1 << 27)
+    assert lib.gsh_gbase_workspace_bytes((1 << 28) + 1, 10, None) == 0
+    with pytest.raises(ValueError):
+        gsh.gbase_workspace_bytes((1 << 28) + 1, 10)
+
+
 def test_hybrid_config_validation():
     lib = _lib.load()
     assert gsh.workspace_bytes(1 << 20, 1 << 20, gsh.make_config(hybrid=True)) > \
         gsh.workspace_bytes(1 << 20, 1 << 20)
     cfg = gsh.make_config()
     cfg.hybrid = 2
+    assert lib.gsh_workspace_bytes(1000, 1000, ctypes.byref(cfg)) == 0
+    cfg = gsh.make_config(hybrid=True, hybrid_share=257)
     assert lib.gsh_workspace_bytes(1000, 1000, ctypes.byref(cfg)) == 0
 
 
